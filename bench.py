@@ -1,0 +1,315 @@
+#!/usr/bin/env python3
+"""Benchmark: deterministic Jacobi-SGR coloring GTEPS on B200 (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config 4] [--impl ours|reference]
+
+One "step" = one complete coloring (every round of the hot path: F_1, then fused
+assign/detect/compact passes until the worklist is empty) of the config's graph, resident in
+HBM. GTEPS = input nnz / step time; redundant rounds never inflate it.
+Rank 0 prints ONE JSON line. For N > 1 (torchrun) the graph is partitioned into nnz-balanced
+contiguous vertex ranges and colored by sgr_color_dist (NCCL exchange per round; strong
+scaling: the total work is fixed).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "coloring GTEPS at 1/2/4/8 B200 (% HBM roofline); colors used vs seq greedy"
+L2_BYTES = 126 * 1024 * 1024
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", type=int, default=4, help="BASELINE.json config (1-based)")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--tiebreak", default="lowid", choices=["lowid", "paper"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--loop-mode", default="auto")
+    return ap.parse_args()
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+
+    def __init__(self, gpu_index: int):
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--id={gpu_index}", f"--query-gpu={q}",
+                                       "--format=csv,noheader,nounits", "-lms", "200"],
+                                      stdout=self.f, stderr=subprocess.DEVNULL)
+        except FileNotFoundError:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        try:
+            self.p.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.p.kill()
+        self.f.seek(0)
+        rows = [r.split(",") for r in self.f.read().strip().splitlines() if r.strip()]
+        os.unlink(self.f.name)
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            try:
+                sm.append(float(r[1]))
+                mx = float(r[2])
+                for nm, val in zip(names, r[5:9]):
+                    if val.strip() == "Active":
+                        reasons.add(nm)
+            except (ValueError, IndexError):
+                continue
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def host_graph(cfg: int):
+    from paper_conf_ipps_licqfsty16_b200 import gen
+    t0 = time.time()
+    g = gen.config(cfg)
+    return g, time.time() - t0
+
+
+def workload_name(cfg):
+    from paper_conf_ipps_licqfsty16_b200 import gen
+    return gen.CONFIG_NAMES[cfg]
+
+
+# ------------------------------------------------------------------------ CPU oracle legs
+def oracle_run(g, tiebreak: int, edges_total: int | None, budget_s: float = 30.0):
+    """Time the oracle (as it stands) on the box's host cores. A full O2 run if it fits the
+    budget; else the first rounds, extrapolated by scanned CSR entries (the unit of work)."""
+    import oracle
+    cores = oracle.max_threads()
+    t0 = time.perf_counter()
+    probe = oracle.jacobi(g, tiebreak, nthreads=cores, max_rounds=4)
+    t_probe = time.perf_counter() - t0
+    if probe.converged:
+        return {"seconds": t_probe, "cores": cores, "sample": "full run", "result": probe}
+    total = edges_total
+    est = None if not total else t_probe * total / max(probe.edges_scanned, 1)
+    if est is not None and est <= budget_s:
+        t0 = time.perf_counter()
+        full = oracle.jacobi(g, tiebreak, nthreads=cores)
+        return {"seconds": time.perf_counter() - t0, "cores": cores, "sample": "full run",
+                "result": full}
+    return {"seconds": est if est is not None else float("nan"), "cores": cores,
+            "sample": (f"first {probe.rounds} Jacobi rounds ({probe.edges_scanned} of {total} "
+                       f"scanned CSR entries), time extrapolated by scanned entries"),
+            "result": None}
+
+
+def alg1_run(g):
+    import oracle
+    t0 = time.perf_counter()
+    c = oracle.alg1(g)
+    return int(c.max()), time.perf_counter() - t0
+
+
+# ------------------------------------------------------------------------ reference arm
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import oracle
+    tb = 0 if args.tiebreak == "lowid" else 1
+    g, _ = host_graph(args.config)
+    cores = oracle.max_threads()
+    times = []
+    edges_total = None
+    res = None
+    for i in range(args.warmup + args.steps):
+        r = oracle_run(g, tb, edges_total, budget_s=60.0)
+        if r["result"] is not None:
+            res = r["result"]
+            edges_total = res.edges_scanned
+        if i >= args.warmup:
+            times.append(r["seconds"])
+        if r["sample"] != "full run" and i + 1 >= args.warmup + 1:
+            break  # sampled: one timed sample is enough
+    t = statistics.mean(times)
+    value = g.nnz / t / 1e9
+    sample = "full oracle run per step" if res is not None else r["sample"]
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "GTEPS",
+            "n_gpus": 0, "steps": len(times), "warmup": args.warmup, "ms_per_step": t * 1e3,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": "int32", "data": "synthetic",
+            "config": {"workload": workload_name(args.config), "n": g.n, "nnz": g.nnz,
+                       "tiebreak": args.tiebreak},
+            "cpu_baseline": {"value": value, "unit": "GTEPS", "cores": cores, "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": value, "unit": "GTEPS", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    if res is not None:
+        line["rounds"] = res.rounds
+        line["num_colors"] = res.num_colors
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------------ our arm, 1 GPU
+def run_single(args):
+    import torch
+    import paper_conf_ipps_licqfsty16_b200 as sgr
+
+    dev = torch.device("cuda", 0)
+    torch.cuda.set_device(dev)
+    g, gen_s = host_graph(args.config)
+    rp_h = torch.from_numpy(g.row_ptr).pin_memory()
+    ci_h = torch.from_numpy(g.col_idx).pin_memory()
+    rp = rp_h.to(dev, non_blocking=True)
+    ci = ci_h.to(dev, non_blocking=True)
+    colors = torch.empty(g.n, dtype=torch.int32, device=dev)
+    ws = torch.empty(sgr.workspace_bytes(g.n, g.nnz), dtype=torch.uint8, device=dev)
+    flush = torch.empty(2 * L2_BYTES // 4, dtype=torch.int32, device=dev)
+    stream = torch.cuda.current_stream()
+    torch.cuda.synchronize()
+
+    def step(profile=False):
+        return sgr.color(rp, ci, args.tiebreak, out=colors, workspace=ws, profile=profile,
+                         loop_mode=args.loop_mode)
+
+    for _ in range(max(args.warmup, 3)):
+        res = step()
+    torch.cuda.synchronize()
+
+    # timed region: K complete colorings, L2 flushed between them (outside the events)
+    clocks = Clocks(0)
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+          for _ in range(args.steps)]
+    launches = 0
+    torch.cuda.synchronize()
+    wall0 = time.perf_counter()
+    for i in range(args.steps):
+        flush.fill_(i)
+        ev[i][0].record(stream)
+        res = step()
+        ev[i][1].record(stream)
+        launches += res.stats["launches"]
+    torch.cuda.synchronize()
+    wall = time.perf_counter() - wall0
+    clk = clocks.stop()
+    step_ms = [a.elapsed_time(b) for a, b in ev]
+    ms = statistics.mean(step_ms)
+    st = res.stats
+    value = g.nnz / (ms * 1e-3) / 1e9
+
+    # profiled region: same K steps, CUDA events around every kernel launch (host loop)
+    prof_ms, kms, kl, kb = [], {}, {}, {}
+    for i in range(args.steps):
+        flush.fill_(i)
+        r = step(profile=True)
+        prof_ms.append(r.stats["elapsed_ms"])
+        for k, v in r.stats["kernel_ms"].items():
+            kms[k] = kms.get(k, 0.0) + v
+            kl[k] = kl.get(k, 0) + r.stats["kernel_launches"][k]
+            kb[k] = kb.get(k, 0) + r.stats["kernel_bytes"][k]
+    torch.cuda.synchronize()
+    peak, peak_src = peaks()
+    dom = max((k for k in kms if k != "control"), key=lambda k: kms[k])
+    achieved = kb[dom] / (kms[dom] * 1e-3) / 1e9 if kms[dom] > 0 else 0.0
+    total_kernel_ms = sum(kms.values())
+    roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak,
+                "unit": "GB/s", "frac": achieved / peak, "traffic": None,
+                "peak_source": peak_src,
+                "launches_per_step": kl[dom] / args.steps,
+                "algorithmic_bytes_per_launch": kb[dom] / max(kl[dom], 1),
+                "avg_launch_us": kms[dom] * 1e3 / max(kl[dom], 1),
+                "share_of_kernel_time": kms[dom] / total_kernel_ms if total_kernel_ms else None,
+                "kernel_ms_per_step": {k: v / args.steps for k, v in kms.items()},
+                "whole_step": {"algorithmic_GBps": st["bytes_algorithmic"] / (ms * 1e-3) / 1e9,
+                               "frac": st["bytes_algorithmic"] / (ms * 1e-3) / 1e9 / peak},
+                "profiled_step_ms": statistics.mean(prof_ms)}
+
+    # e2e: the same coloring through sgr_color_host from pinned host buffers
+    e2e = None
+    if not args.no_e2e:
+        out_h = torch.empty(g.n, dtype=torch.int32).pin_memory()
+        sgr.color_host(rp_h, ci_h, args.tiebreak, out=out_h)
+        e_ms = []
+        for i in range(min(args.steps, 5)):
+            flush.fill_(i)
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            sgr.color_host(rp_h, ci_h, args.tiebreak, out=out_h)
+            e_ms.append((time.perf_counter() - t0) * 1e3)
+        assert torch.equal(out_h, colors.cpu()), "e2e colors differ from device-resident run"
+        e2e = {"value": g.nnz / (statistics.mean(e_ms) * 1e-3) / 1e9, "unit": "GTEPS",
+               "h2d_bytes_per_step": int((g.n + 1) * 8 + g.nnz * 4),
+               "d2h_bytes_per_step": int(g.n * 4), "ms_per_step": statistics.mean(e_ms)}
+
+    line = {"metric": METRIC, "value": value, "unit": "GTEPS", "n_gpus": 1,
+            "steps": args.steps, "warmup": max(args.warmup, 3), "ms_per_step": ms,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": "int32", "data": "synthetic",
+            "config": {"workload": workload_name(args.config), "n": g.n, "nnz": g.nnz,
+                       "tiebreak": args.tiebreak, "parallelism": "single GPU",
+                       "l2": "flushed between steps (256 MiB write, outside the step events); "
+                             "CSR inputs 1.2 GB > L2",
+                       "loop_mode": args.loop_mode},
+            "rounds": st["rounds"], "num_colors": st["num_colors"],
+            "A_scanned_per_nnz": st["edges_scanned"] / g.nnz,
+            "B_worklist_per_n": st["vertices_processed"] / g.n,
+            "vertices_per_s": g.n / (ms * 1e-3), "step_ms_min": min(step_ms),
+            "wall_s_timed_region": wall, "gpu_launches": launches,
+            "roofline": roofline, "clocks": clk, "e2e": e2e, "gen_s": gen_s}
+
+    if not args.no_cpu_baseline:
+        tb = 0 if args.tiebreak == "lowid" else 1
+        o = oracle_run(g, tb, st["edges_scanned"], budget_s=30.0)
+        a1_colors, a1_s = alg1_run(g)
+        line["cpu_baseline"] = {"value": g.nnz / o["seconds"] / 1e9, "unit": "GTEPS",
+                                "cores": o["cores"], "kind": "oracle", "sample": o["sample"]}
+        line["colors_vs_seq_greedy"] = {"ours": st["num_colors"], "alg1": a1_colors,
+                                        "ratio": st["num_colors"] / a1_colors,
+                                        "alg1_seconds_1core": a1_s,
+                                        "speedup_vs_alg1_1core": a1_s / (ms * 1e-3)}
+        if o["result"] is not None:
+            ok = bool(np.array_equal(o["result"].colors, colors.cpu().numpy()))
+            line["parity_vs_oracle_full"] = ok
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if world > 1 or args.gpus > 1:
+        from paper_conf_ipps_licqfsty16_b200 import benchdist
+        return benchdist.run(args)
+    return run_single(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,193 @@
+/*
+ * sgr.h — C ABI of the B200 (sm_100a) deterministic speculative-greedy (SGR) coloring
+ * library, libsgr.so. Every function is extern "C", never throws, and returns an
+ * sgr_status (0 = OK, < 0 = error; sgr_last_error() gives a thread-local message).
+ *
+ * What it computes (PAPER.md = /root/reference/PAPER.md, "P:N" = line N):
+ *   Vertex coloring: "assign colors to all the vertices of a graph such that no neighboring
+ *   vertices have the same color", by the data-driven speculative greedy
+ *   method, Algorithm 5: rounds of first-fit assignment over a worklist
+ *   (Alg. 5 l.4-10) followed by conflict detection that returns the losing endpoint of
+ *   every monochromatic edge to the next worklist (Alg. 5 l.12-18, pushed with a
+ *   prefix-sum / aggregated atomic), until the worklist is empty (l.3, l.19).
+ *   Rounds are Jacobi-style (reading C1): assignment in round r reads the
+ *   colors as they were when round r started, so the result is a deterministic function
+ *   of (graph, tie-break) only — independent of GPU count, launch shape, bins or timing —
+ *   and is bit-identical to the CPU oracle (oracle/, test infrastructure).
+ *
+ * Graph input: CSR "R" (row offsets, n+1) and "C" (column indices, nnz), stored
+ * "in the order they are defined" with no relabeling (reading C19). Contract:
+ *   - row_ptr is int64, row_ptr[0] = 0, nondecreasing, row_ptr[n] = nnz;
+ *   - col_idx is int32, 0 <= col_idx[e] < n, each row sorted ascending;
+ *   - the pattern is symmetric (w in adj(v) <=> v in adj(w)); asymmetric input is
+ *     undefined (conflicts may go unseen);
+ *   - self-loops and duplicate entries are allowed and provably never change the result;
+ *   - n < 2^31; n = 0 is OK (no kernels); nnz = 0 gives all colors 1 in one round.
+ * Output: colors_out[v] in [1, deg(v)+1] (colors are positive integers), a
+ *   proper coloring.
+ *
+ * Ownership: the caller owns every buffer passed in; the library never frees or retains
+ * caller memory after a call returns. Device scratch is either the caller's `workspace`
+ * (>= sgr_workspace_bytes()) or taken from the stream-ordered allocator and released
+ * before return.
+ * Synchronization: sgr_color / sgr_color_ex / sgr_color_host return when colors_out and
+ * *stats are valid (they synchronize opts->stream once at the end). The step entry points
+ * (sgr_assign, sgr_commit, sgr_detect, sgr_compact) are asynchronous on opts->stream.
+ * Errors: SGR_EINVAL for a null required pointer, n < 0, nnz < 0, n >= 2^31, aliasing
+ * that the operation forbids, or (with opts->validate) a CSR that breaks the contract;
+ * SGR_ECUDA for a CUDA error (message in sgr_last_error()); SGR_ENOCONV if opts->max_rounds
+ * was reached (cannot happen with the default cap n+1: |W| strictly shrinks every round).
+ */
+#ifndef SGR_H
+#define SGR_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  SGR_OK = 0,
+  SGR_EINVAL = -1,
+  SGR_ENOMEM = -2,
+  SGR_ECUDA = -3,
+  SGR_ENCCL = -4,
+  SGR_ENOCONV = -5,
+  SGR_EUNSUPPORTED = -6
+} sgr_status;
+
+/* Which endpoint of a conflicting edge (v, w), color[v] = color[w], goes back to the
+ * worklist (DESIGN.md §3 reading C4). */
+typedef enum {
+  SGR_TIEBREAK_LOWID_KEEPS = 0, /* the higher id recolors: lose(v,w) = v > w (default) */
+  SGR_TIEBREAK_PAPER = 1        /* Alg. 2 l.14 / Alg. 4 l.17 / Alg. 5 l.14: v < w -> v */
+} sgr_tiebreak;
+
+typedef enum {
+  SGR_LOOP_AUTO = 0,  /* = SGR_LOOP_GRAPH */
+  SGR_LOOP_GRAPH = 1, /* batches of rounds replayed as one CUDA graph */
+  SGR_LOOP_HOST = 3   /* batches of rounds launched kernel by kernel */
+} sgr_loop_mode;
+
+/* Device CSR (both pointers in device memory). */
+typedef struct {
+  const int64_t* row_ptr; /* n+1 */
+  const int32_t* col_idx; /* nnz */
+} sgr_csr;
+
+typedef struct {
+  int32_t tiebreak;      /* sgr_tiebreak; default LOWID_KEEPS */
+  int32_t max_rounds;    /* 0 = n+1 (never reached) */
+  int32_t loop_mode;     /* sgr_loop_mode */
+  int32_t block_size;    /* threads per block of the thread/warp-bin kernels; 0 = 256 */
+  int32_t bin_small_max; /* degree bins: d <= small -> thread per vertex (<= 62); 0 = 32 */
+  int32_t bin_med_max;   /* small < d <= med -> warp per vertex; d > med -> CTA; 0 = 4096 */
+  void* stream;          /* cudaStream_t; NULL = legacy default stream */
+  int32_t* round_sizes;  /* optional DEVICE buffer: |W_r| for r = 1..R (R capped by cap) */
+  int64_t* round_edges;  /* optional DEVICE buffer: sum of deg(v), v in W_r, r = 1..R   */
+  int32_t round_cap;     /* capacity of round_sizes / round_edges */
+  int32_t validate;      /* != 0: check the CSR contract on the device first (slow) */
+  int32_t rounds_per_batch; /* rounds issued between termination checks; 0 = 8 */
+  int32_t profile;       /* != 0: time every kernel launch with CUDA events (host loop) */
+} sgr_opts;
+
+/* Per-kernel-class device time, filled when opts->profile != 0. */
+enum { SGR_K_FIRST = 0, SGR_K_SMALL = 1, SGR_K_MED = 2, SGR_K_HUB = 3, SGR_K_CTRL = 4,
+       SGR_K_COUNT = 5 };
+
+typedef struct {
+  int32_t rounds;             /* R = number of assignment rounds (P4 path: 4)           */
+  int32_t num_colors;         /* max color                                               */
+  int64_t vertices_processed; /* sum over rounds of |W_r|                                */
+  int64_t edges_scanned;      /* sum over rounds of sum_{v in W_r} deg(v) (A * nnz)      */
+  int64_t bytes_algorithmic;  /* DESIGN.md §6 byte model, summed over all launches       */
+  float elapsed_ms;           /* device time from the first kernel to the final count   */
+  int32_t launches;           /* kernels launched by this call                           */
+  float kernel_ms[SGR_K_COUNT];      /* opts->profile: device time per kernel class      */
+  int64_t kernel_launches[SGR_K_COUNT];
+  int64_t kernel_bytes[SGR_K_COUNT]; /* algorithmic bytes per kernel class             */
+} sgr_stats;
+
+void sgr_opts_default(sgr_opts* opts);
+
+/* Scratch the library needs for a graph of this size (device bytes). */
+size_t sgr_workspace_bytes(int64_t n, int64_t nnz, const sgr_opts* opts);
+
+/* Color the graph. csr and colors_out (n int32) are device pointers. stats: host, nullable. */
+sgr_status sgr_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* colors_out,
+                     sgr_stats* stats);
+
+/* Same, with options and optional caller workspace (device, >= sgr_workspace_bytes). */
+sgr_status sgr_color_ex(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* colors_out,
+                        sgr_stats* stats, const sgr_opts* opts, void* workspace,
+                        size_t workspace_bytes);
+
+/* End to end from HOST buffers: copies row_ptr/col_idx host->device, colors, copies the
+ * colors device->host. Host buffers should be pinned for full PCIe/C2C speed. */
+sgr_status sgr_color_host(const int64_t* row_ptr, const int32_t* col_idx, int64_t n,
+                          int64_t nnz, int32_t* colors_out, sgr_stats* stats,
+                          const sgr_opts* opts);
+
+/* ---- one-round step entry points: Algorithm 5 split line by line (all device pointers,
+ * asynchronous on opts->stream; opts may be NULL) ---------------------------------------- */
+
+/* Alg. 5 l.4-10 against a snapshot: tent_out[i] = min{c > 0 : c != colors_in[w] for all
+ * w in adj(wl[i])}. colors_in must not alias tent_out. */
+sgr_status sgr_assign(const sgr_csr* csr, int64_t n, const int32_t* wl, int64_t wl_len,
+                      const int32_t* colors_in, int32_t* tent_out, const sgr_opts* opts);
+
+/* Alg. 5 l.9 applied after the whole assignment step: colors[wl[i]] = tent[i]. */
+sgr_status sgr_commit(const int32_t* wl, const int32_t* tent, int64_t wl_len, int32_t* colors,
+                      const sgr_opts* opts);
+
+/* Alg. 5 l.13-14 for the listed vertices: conflict_out[i] = 1 iff some w in adj(v),
+ * v = wl[i], has colors[w] == colors[v] and v loses by opts->tiebreak; else 0. */
+sgr_status sgr_detect(const sgr_csr* csr, int64_t n, const int32_t* wl, int64_t wl_len,
+                      const int32_t* colors, uint8_t* conflict_out, const sgr_opts* opts);
+
+/* Alg. 5 l.15 / P:228-230: wl_out = [wl[i] : flags[i] != 0] in input order (block scan +
+ * one aggregated offset per block); *count_out (device int64) = its length. */
+sgr_status sgr_compact(const int32_t* wl, const uint8_t* flags, int64_t len, int32_t* wl_out,
+                       int64_t* count_out, const sgr_opts* opts);
+
+/* Device-side CSR contract check; *violations (host) gets the sgr_gen_validate-style
+ * bitmask (1 offsets, 2 range, 4 unsorted). Symmetry is not checked on the device. */
+sgr_status sgr_validate_csr(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* violations,
+                            void* stream);
+
+/* ---- multi-GPU: contiguous vertex ranges, one NCCL exchange per round -- */
+
+/* nnz-balanced contiguous ranges: ranges[p] = min{v : row_ptr[v] >= ceil(p*nnz/P)},
+ * ranges[0] = 0, ranges[P] = n. row_ptr is a HOST array here. */
+sgr_status sgr_partition(const int64_t* row_ptr, int64_t n, int32_t P, int64_t* ranges);
+
+/* NCCL communicator wrapper: nccl_unique_id is the 128-byte ncclUniqueId that rank 0
+ * created (sgr_nccl_unique_id) and every rank received out of band. */
+sgr_status sgr_nccl_unique_id(void* id_out_128B);
+sgr_status sgr_comm_init(void** comm, int32_t rank, int32_t world, const void* nccl_unique_id,
+                         int32_t device);
+sgr_status sgr_comm_destroy(void* comm);
+
+/* One call per rank, collective over comm. `local` holds the rank's OWNED rows
+ * [v_begin, v_end) with local row offsets (local.row_ptr[0] = 0, length v_end-v_begin+1)
+ * and GLOBAL column ids. colors_out: device, n_global int32, filled on every rank. */
+sgr_status sgr_color_dist(void* comm, const sgr_csr* local, int64_t n_global, int64_t v_begin,
+                          int64_t v_end, int64_t nnz_local, int32_t* colors_out,
+                          sgr_stats* stats, const sgr_opts* opts);
+
+/* P logical partitions on ONE device: same per-rank kernels, exchange and commit as
+ * sgr_color_dist, with the all-gather done by device copies (for testing the distributed
+ * path bit-exactly on a single GPU). csr is the full device CSR; ranges: host, P+1. */
+sgr_status sgr_color_partitioned(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t P,
+                                 const int64_t* ranges, int32_t* colors_out, sgr_stats* stats,
+                                 const sgr_opts* opts);
+
+const char* sgr_strerror(sgr_status s);
+const char* sgr_last_error(void);
+const char* sgr_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

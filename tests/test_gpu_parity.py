@@ -1,0 +1,264 @@
+"""Parity of the CUDA path (libsgr.so through its C ABI) against the CPU oracle (-m gpu).
+
+Bar: everything here is integer work, so colors, the round count R and the
+per-round worklist sizes |W_r| must be BIT-EXACT; the worklists' order is unspecified, so
+step-level compaction is compared as ordered output (sgr_compact is order-preserving) and
+the fused path's worklists through their sizes and the final colors.
+"""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_ipps_licqfsty16_b200 import gen
+from tests._inputs import random_graph, raw_csr, with_loops_and_dups
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+if not torch.cuda.is_available():  # the marker keeps these off the CPU suite
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+import paper_conf_ipps_licqfsty16_b200 as sgr  # noqa: E402
+
+LOW, PAP = oracle.TIEBREAK_LOWID_KEEPS, oracle.TIEBREAK_PAPER
+RULE = {LOW: "lowid", PAP: "paper"}
+
+
+def dev(g):
+    return (torch.from_numpy(np.ascontiguousarray(g.row_ptr)).cuda(),
+            torch.from_numpy(np.ascontiguousarray(g.col_idx)).cuda())
+
+
+def check_full(g, tb, **kw):
+    rp, ci = dev(g)
+    res = sgr.color(rp, ci, RULE[tb], trace=True, **kw)
+    ref = oracle.jacobi(g, tb, nthreads=oracle.max_threads())
+    got = res.colors.cpu().numpy()
+    assert res.stats["rounds"] == ref.rounds, (g.name, res.stats["rounds"], ref.rounds)
+    if not np.array_equal(got, ref.colors):
+        bad = np.nonzero(got != ref.colors)[0]
+        raise AssertionError(f"{g.name}: {len(bad)} colors differ, first {bad[:8]} "
+                             f"got {got[bad[:8]]} want {ref.colors[bad[:8]]}")
+    assert np.array_equal(res.round_sizes, ref.round_sizes), g.name
+    assert np.array_equal(res.round_edges, ref.trace["w_edges"]), g.name
+    assert res.stats["num_colors"] == ref.num_colors
+    assert res.stats["edges_scanned"] == ref.edges_scanned
+    assert res.stats["vertices_processed"] == ref.vertices_processed
+    return res, ref
+
+
+# ----------------------------------------------------------------------------- full path
+@pytest.mark.parametrize("seed", range(48))
+@pytest.mark.parametrize("tb", [LOW, PAP])
+def test_random_small_graphs(seed, tb):
+    check_full(random_graph(seed), tb)
+
+
+@pytest.mark.parametrize("tb", [LOW, PAP])
+def test_cfg1_rmat_s16_bit_exact(tb):
+    res, ref = check_full(gen.config(1), tb)
+    if tb == LOW:  # north_star quality target: within 10% of Algorithm 1
+        a1 = int(oracle.alg1(gen.config(1)).max())
+        assert abs(res.stats["num_colors"] - a1) <= 0.1 * a1
+
+
+@pytest.mark.parametrize("maker", [
+    lambda: gen.stencil3d(24, 24, 24, 27),
+    lambda: gen.stencil3d(13, 11, 9, 7),
+    lambda: gen.stencil2d(57, 31, 5),
+    lambda: gen.stencil2d(40, 40, 9),
+    lambda: gen.er(1 << 15, 8 << 15, seed=3),
+    lambda: gen.rmat(15, 8, 0.57, 0.19, 0.19, seed=4, permute=True),
+    lambda: gen.rmat(14, 10, 0.45, 0.15, 0.15, seed=2),   # rmat-g shape (Table I)
+    lambda: gen.rmat(14, 10, 0.25, 0.25, 0.25, seed=2),   # rmat-er shape (Table I)
+], ids=["s27-24", "s7", "s5", "s9", "er15", "rmat15-perm", "rmat-g14", "rmat-er14"])
+@pytest.mark.parametrize("tb", [LOW, PAP])
+def test_generator_families(maker, tb):
+    check_full(maker(), tb)
+
+
+def degree_boundary_graph():
+    """Stars whose centres have degrees at every bin boundary, plus cliques K_70 / K_300
+    (first-fit values above 64 and 256: window slides in the warp and CTA bins)."""
+    edges = []
+    n = 0
+    for d in [0, 1, 2, 31, 32, 33, 61, 62, 63, 64, 65, 2047, 2048, 2049, 4095, 4096, 4097, 9000]:
+        c = n
+        edges += [(c, c + 1 + i) for i in range(d)]
+        n += d + 1
+    for k in (70, 300):
+        base = n
+        edges += [(base + i, base + j) for i in range(k) for j in range(i + 1, k)]
+        n += k
+    # tie the pieces together so the stars' leaves also collide
+    edges += [(i, i + 7) for i in range(0, n - 7, 5)]
+    return gen.from_edges(n, np.asarray(edges, np.int64))
+
+
+@pytest.mark.parametrize("tb", [LOW, PAP])
+@pytest.mark.parametrize("bins", [(0, 0), (62, 62), (1, 1), (8, 64), (32, 2048), (62, 100000)])
+def test_degree_bins_and_windows(tb, bins):
+    check_full(degree_boundary_graph(), tb, bin_small_max=bins[0], bin_med_max=bins[1])
+
+
+@pytest.mark.parametrize("k", [64, 257, 520])
+def test_complete_graphs_large_mex(k):
+    g = gen.from_edges(k, [(i, j) for i in range(k) for j in range(i + 1, k)])
+    for bins in [(0, 0), (1, 1), (62, 100000)]:
+        res, _ = check_full(g, LOW, bin_small_max=bins[0], bin_med_max=bins[1])
+        assert res.colors.cpu().numpy().tolist() == list(range(1, k + 1))
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_self_loops_and_duplicates(seed):
+    g = random_graph(seed, n=200)
+    h = with_loops_and_dups(g, seed)
+    for tb in (LOW, PAP):
+        a = sgr.color(*dev(g), RULE[tb]).colors.cpu().numpy()
+        b = sgr.color(*dev(h), RULE[tb]).colors.cpu().numpy()
+        assert np.array_equal(a, b)
+        assert np.array_equal(b, oracle.jacobi(h, tb).colors)
+
+
+def test_edge_cases_n0_n1_nnz0():
+    g0 = gen.from_edges(0, np.zeros((0, 2), np.int64))
+    r0 = sgr.color(*dev(g0))
+    assert r0.stats["rounds"] == 0 and r0.colors.numel() == 0
+    g1 = gen.from_edges(1, np.zeros((0, 2), np.int64))
+    r1 = sgr.color(*dev(g1))
+    assert r1.stats["rounds"] == 1 and r1.colors.cpu().tolist() == [1]
+    g5 = gen.from_edges(5, np.zeros((0, 2), np.int64))
+    r5 = sgr.color(*dev(g5), trace=True)
+    assert r5.stats["rounds"] == 1 and r5.colors.cpu().tolist() == [1] * 5
+    assert r5.round_sizes.tolist() == [5]
+    loops = raw_csr(3, [(0, 0), (1, 1), (2, 2)])
+    assert sgr.color(*dev(loops)).colors.cpu().tolist() == [1, 1, 1]
+
+
+@pytest.mark.parametrize("mode", ["host", "graph"])
+@pytest.mark.parametrize("batch", [1, 3, 8, 32])
+def test_loop_modes_and_batches(mode, batch):
+    g = gen.config(1)
+    rp, ci = dev(g)
+    ref = sgr.color(rp, ci).colors
+    res = sgr.color(rp, ci, loop_mode=mode, rounds_per_batch=batch)
+    assert torch.equal(res.colors, ref)
+
+
+def test_profile_mode_and_stats():
+    g = gen.config(1)
+    rp, ci = dev(g)
+    res = sgr.color(rp, ci, profile=True)
+    st = res.stats
+    assert st["kernel_launches"]["first"] == 1
+    assert st["kernel_launches"]["warp_bin"] >= st["rounds"] - 1
+    assert all(v >= 0 for v in st["kernel_ms"].values())
+    assert st["bytes_algorithmic"] == sum(st["kernel_bytes"].values())
+    ref = oracle.jacobi(g, LOW)
+    assert torch.equal(res.colors.cpu(), torch.from_numpy(ref.colors))
+
+
+def test_deterministic_repeats():
+    g = gen.rmat(16, 8, 0.57, 0.19, 0.19, seed=9, permute=True)
+    rp, ci = dev(g)
+    a = sgr.color(rp, ci).colors.clone()
+    for _ in range(3):
+        assert torch.equal(sgr.color(rp, ci).colors, a)
+
+
+def test_max_rounds_enoconv():
+    g = gen.from_edges(6, [(i, i + 1) for i in range(5)])  # path: R = 6
+    rp, ci = dev(g)
+    with pytest.raises(RuntimeError, match="max_rounds"):
+        sgr.color(rp, ci, max_rounds=3)
+    assert sgr.color(rp, ci, max_rounds=6).stats["rounds"] == 6
+
+
+def test_validate_rejects_bad_csr():
+    rp = torch.tensor([0, 2, 3, 4], dtype=torch.int64, device="cuda")
+    ci = torch.tensor([2, 1, 0, 0], dtype=torch.int32, device="cuda")  # row 0 unsorted
+    assert sgr.validate_csr(rp, ci) & 4
+    with pytest.raises(RuntimeError, match="invalid"):
+        sgr.color(rp, ci, validate=True)
+    g = gen.config(1)
+    assert sgr.validate_csr(*dev(g)) == 0
+
+
+def test_color_host_equals_device():
+    g = gen.rmat(14, 8, 0.57, 0.19, 0.19, seed=1)
+    a = sgr.color(*dev(g)).colors.cpu().numpy()
+    rp = torch.from_numpy(g.row_ptr).pin_memory()
+    ci = torch.from_numpy(g.col_idx).pin_memory()
+    out = torch.zeros(g.n, dtype=torch.int32).pin_memory()
+    res = sgr.color_host(rp, ci, out=out)
+    assert np.array_equal(out.numpy(), a)
+    assert res.stats["rounds"] > 1
+    b = sgr.color_host(g.row_ptr, g.col_idx).colors  # pageable numpy also works
+    assert np.array_equal(b, a)
+
+
+# ----------------------------------------------------------------------------- step API
+@pytest.mark.parametrize("seed", range(16))
+def test_step_entry_points(seed):
+    rng = np.random.default_rng(seed)
+    g = random_graph(seed, n=int(rng.integers(1, 400)))
+    rp, ci = dev(g)
+    snap = rng.integers(0, 9, g.n).astype(np.int32)
+    wl = np.sort(rng.choice(g.n, size=int(rng.integers(0, g.n + 1)), replace=False)).astype(np.int32)
+    twl = torch.from_numpy(wl).cuda()
+    tsnap = torch.from_numpy(snap).cuda()
+    tent = sgr.assign(rp, ci, twl, tsnap)
+    assert np.array_equal(tent.cpu().numpy(), oracle.assign(g, wl, snap))
+    for tb in (LOW, PAP):
+        fl = sgr.detect(rp, ci, twl, tsnap, RULE[tb])
+        ref = oracle.detect(g, wl, snap, tb)
+        assert np.array_equal(fl.cpu().numpy(), ref)
+        out = sgr.compact(twl, fl)
+        assert np.array_equal(out.cpu().numpy(), wl[ref.astype(bool)])
+    colors = tsnap.clone()
+    sgr.commit(twl, tent, colors)
+    exp = snap.copy()
+    exp[wl] = oracle.assign(g, wl, snap)
+    assert np.array_equal(colors.cpu().numpy(), exp)
+
+
+def test_step_loop_reproduces_algorithm5():
+    """Driving assign -> commit -> detect -> compact from Python = the fused library path."""
+    g = gen.rmat(13, 8, 0.57, 0.19, 0.19, seed=6)
+    rp, ci = dev(g)
+    colors = torch.zeros(g.n, dtype=torch.int32, device="cuda")
+    wl = torch.arange(g.n, dtype=torch.int32, device="cuda")
+    rounds = 0
+    while wl.numel():
+        rounds += 1
+        snapshot = colors.clone()
+        tent = sgr.assign(rp, ci, wl, snapshot)
+        sgr.commit(wl, tent, colors)
+        flags = sgr.detect(rp, ci, wl, colors)
+        wl = sgr.compact(wl, flags)
+    ref = oracle.jacobi(g, LOW)
+    assert rounds == ref.rounds
+    assert np.array_equal(colors.cpu().numpy(), ref.colors)
+    assert torch.equal(sgr.color(rp, ci).colors, colors)
+
+
+def test_compact_large_ragged():
+    rng = np.random.default_rng(0)
+    for L in (1, 1023, 1024, 1025, 300_001):
+        wl = rng.integers(0, 1 << 30, L).astype(np.int32)
+        fl = (rng.random(L) < 0.37).astype(np.uint8)
+        out = sgr.compact(torch.from_numpy(wl).cuda(), torch.from_numpy(fl).cuda())
+        assert np.array_equal(out.cpu().numpy(), wl[fl.astype(bool)])
+
+
+# ----------------------------------------------------------------------------- full size
+@pytest.mark.slow
+@pytest.mark.parametrize("cfg", [2, 3, 4])
+def test_full_size_configs_bit_exact(cfg):
+    """BASELINE.json configs 2-4 at full size, in the launch configuration bench.py times
+    (default options), against the full oracle (OpenMP over each round's independent
+    per-vertex loops; identical to the single-threaded oracle by construction)."""
+    g = gen.config(cfg)
+    check_full(g, LOW)
