@@ -18,7 +18,8 @@
  * Graph input: CSR "R" (row offsets, n+1) and "C" (column indices, nnz), stored
  * "in the order they are defined" with no relabeling (reading C19). Contract:
  *   - row_ptr is int64, row_ptr[0] = 0, nondecreasing, row_ptr[n] = nnz;
- *   - col_idx is int32, 0 <= col_idx[e] < n, each row sorted ascending;
+ *   - col_idx is int32, 0 <= col_idx[e] < n, each row sorted ascending, and the col_idx
+ *     pointer is 16-byte aligned (rows are read with 16-byte vector loads);
  *   - the pattern is symmetric (w in adj(v) <=> v in adj(w)); asymmetric input is
  *     undefined (conflicts may go unseen);
  *   - self-loops and duplicate entries are allowed and provably never change the result;
@@ -65,9 +66,10 @@ typedef enum {
 } sgr_tiebreak;
 
 typedef enum {
-  SGR_LOOP_AUTO = 0,  /* = SGR_LOOP_GRAPH */
-  SGR_LOOP_GRAPH = 1, /* batches of rounds replayed as one CUDA graph */
-  SGR_LOOP_HOST = 3   /* batches of rounds launched kernel by kernel */
+  SGR_LOOP_AUTO = 0,       /* = SGR_LOOP_PERSISTENT */
+  SGR_LOOP_GRAPH = 1,      /* one kernel per round, batches of rounds replayed as a CUDA graph */
+  SGR_LOOP_PERSISTENT = 2, /* all rounds in one cooperative kernel, grid barrier per round */
+  SGR_LOOP_HOST = 3        /* one kernel per round, launched from the host in batches */
 } sgr_loop_mode;
 
 /* Device CSR (both pointers in device memory). */
@@ -80,21 +82,25 @@ typedef struct {
   int32_t tiebreak;      /* sgr_tiebreak; default LOWID_KEEPS */
   int32_t max_rounds;    /* 0 = n+1 (never reached) */
   int32_t loop_mode;     /* sgr_loop_mode */
-  int32_t block_size;    /* threads per block of the thread/warp-bin kernels; 0 = 256 */
-  int32_t bin_small_max; /* degree bins: d <= small -> thread per vertex (<= 62); 0 = 32 */
-  int32_t bin_med_max;   /* small < d <= med -> warp per vertex; d > med -> CTA; 0 = 4096 */
+  int32_t color_bits;    /* width of the working color arrays: 16 (default; a first fit
+                            above 65535 triggers an automatic 32-bit rerun) or 32 */
+  int32_t bin_small_max; /* degree bins: d <= small -> 8 lanes/vertex, register mask (<= 62);
+                            0 = 32 */
+  int32_t bin_med_max;   /* small < d <= med -> 8 lanes/vertex, smem table (<= 256); 0 = 256;
+                            d > med -> one warp per 1024-entry aligned chunk of the row */
   void* stream;          /* cudaStream_t; NULL = legacy default stream */
   int32_t* round_sizes;  /* optional DEVICE buffer: |W_r| for r = 1..R (R capped by cap) */
   int64_t* round_edges;  /* optional DEVICE buffer: sum of deg(v), v in W_r, r = 1..R   */
   int32_t round_cap;     /* capacity of round_sizes / round_edges */
   int32_t validate;      /* != 0: check the CSR contract on the device first (slow) */
   int32_t rounds_per_batch; /* rounds issued between termination checks; 0 = 8 */
-  int32_t profile;       /* != 0: time every kernel launch with CUDA events (host loop) */
+  int32_t profile;       /* != 0: time every kernel launch with CUDA events */
+  float* round_ms;       /* optional HOST buffer (round_cap): with profile != 0 and the host
+                            loop, device time of each round pass k = 2, 3, ... */
 } sgr_opts;
 
-/* Per-kernel-class device time, filled when opts->profile != 0. */
-enum { SGR_K_FIRST = 0, SGR_K_SMALL = 1, SGR_K_MED = 2, SGR_K_HUB = 3, SGR_K_CTRL = 4,
-       SGR_K_COUNT = 5 };
+/* Kernel classes (stats->kernel_*): F_1, the fused round pass(es), loop control, final. */
+enum { SGR_K_FIRST = 0, SGR_K_ROUND = 1, SGR_K_CTRL = 2, SGR_K_FINAL = 3, SGR_K_COUNT = 4 };
 
 typedef struct {
   int32_t rounds;             /* R = number of assignment rounds (P4 path: 4)           */
@@ -107,6 +113,11 @@ typedef struct {
   float kernel_ms[SGR_K_COUNT];      /* opts->profile: device time per kernel class      */
   int64_t kernel_launches[SGR_K_COUNT];
   int64_t kernel_bytes[SGR_K_COUNT]; /* algorithmic bytes per kernel class             */
+  int64_t bin_vertices[3];           /* rounds >= 2, per degree bin (thread/group/chunk) */
+  int64_t bin_edges[3];
+  int64_t chunk_items;               /* warp work items processed in the chunk bin       */
+  int32_t grid_blocks;               /* blocks of the round kernel                        */
+  int32_t color_bits;                /* width the coloring finished with (16 or 32)       */
 } sgr_stats;
 
 void sgr_opts_default(sgr_opts* opts);

@@ -24,7 +24,7 @@ from . import gen  # noqa: F401  (seeded input generators; no coloring arithmeti
 from ._lib import Csr, Opts, Stats, check, load
 
 TIEBREAK = {"lowid": 0, "lowid_keeps": 0, "paper": 1}
-LOOP = {"auto": 0, "graph": 1, "host": 3}
+LOOP = {"auto": 0, "graph": 1, "persistent": 2, "host": 3}
 
 __all__ = ["color", "color_host", "color_partitioned", "color_dist", "assign", "commit",
            "detect", "compact", "validate_csr", "partition", "workspace_bytes", "gen",
@@ -65,15 +65,16 @@ def _check_csr(row_ptr, col_idx):
         raise TypeError("row_ptr must be int64 and col_idx int32")
 
 
-def make_opts(tiebreak="lowid", stream=None, max_rounds=0, loop_mode="auto", block_size=0,
+def make_opts(tiebreak="lowid", stream=None, max_rounds=0, loop_mode="auto", color_bits=0,
               bin_small_max=0, bin_med_max=0, validate=False, rounds_per_batch=0,
-              profile=False, round_sizes=None, round_edges=None, round_cap=0) -> Opts:
+              profile=False, round_sizes=None, round_edges=None, round_cap=0,
+              round_ms=None) -> Opts:
     o = Opts()
     load().sgr_opts_default(ctypes.byref(o))
     o.tiebreak = _tb(tiebreak)
     o.max_rounds = int(max_rounds)
     o.loop_mode = LOOP[loop_mode] if isinstance(loop_mode, str) else int(loop_mode)
-    o.block_size = int(block_size)
+    o.color_bits = int(color_bits)
     o.bin_small_max = int(bin_small_max)
     o.bin_med_max = int(bin_med_max)
     o.stream = _stream_ptr(stream)
@@ -83,6 +84,7 @@ def make_opts(tiebreak="lowid", stream=None, max_rounds=0, loop_mode="auto", blo
     o.round_sizes = round_sizes.data_ptr() if round_sizes is not None else None
     o.round_edges = round_edges.data_ptr() if round_edges is not None else None
     o.round_cap = int(round_cap)
+    o.round_ms = round_ms.ctypes.data if round_ms is not None else None
     return o
 
 
@@ -115,8 +117,9 @@ def color(row_ptr, col_idx, tiebreak="lowid", *, out=None, stream=None, trace=Fa
     if trace:
         rs = torch.zeros(n + 2, dtype=torch.int32, device=row_ptr.device)
         re = torch.zeros(n + 2, dtype=torch.int64, device=row_ptr.device)
+    rms = np.zeros(n + 2, np.float32) if trace else None
     opts = make_opts(tiebreak, stream, round_sizes=rs, round_edges=re,
-                     round_cap=(n + 2) if trace else 0, **opt_kw)
+                     round_cap=(n + 2) if trace else 0, round_ms=rms, **opt_kw)
     csr = Csr(row_ptr.data_ptr(), col_idx.data_ptr() if nnz else None)
     st = Stats()
     ws_ptr, ws_len = None, 0
@@ -130,6 +133,7 @@ def color(row_ptr, col_idx, tiebreak="lowid", *, out=None, stream=None, trace=Fa
         R = res.stats["rounds"]
         res.round_sizes = rs[:R].cpu().numpy()
         res.round_edges = re[:R].cpu().numpy()
+        res.extra["round_ms"] = rms[:R]
     return res
 
 

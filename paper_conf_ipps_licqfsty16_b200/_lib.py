@@ -9,8 +9,9 @@ from pathlib import Path
 
 LIBPATH = Path(__file__).resolve().parent / "lib" / "libsgr.so"
 
-SGR_K_COUNT = 5
-KERNEL_CLASSES = ("first", "thread_bin", "warp_bin", "cta_bin", "control")
+SGR_K_COUNT = 4
+KERNEL_CLASSES = ("first", "round", "control", "final")
+BINS = ("thread", "group", "chunk")
 
 
 class Csr(ctypes.Structure):
@@ -19,12 +20,12 @@ class Csr(ctypes.Structure):
 
 class Opts(ctypes.Structure):
     _fields_ = [("tiebreak", ctypes.c_int32), ("max_rounds", ctypes.c_int32),
-                ("loop_mode", ctypes.c_int32), ("block_size", ctypes.c_int32),
+                ("loop_mode", ctypes.c_int32), ("color_bits", ctypes.c_int32),
                 ("bin_small_max", ctypes.c_int32), ("bin_med_max", ctypes.c_int32),
                 ("stream", ctypes.c_void_p), ("round_sizes", ctypes.c_void_p),
                 ("round_edges", ctypes.c_void_p), ("round_cap", ctypes.c_int32),
                 ("validate", ctypes.c_int32), ("rounds_per_batch", ctypes.c_int32),
-                ("profile", ctypes.c_int32)]
+                ("profile", ctypes.c_int32), ("round_ms", ctypes.c_void_p)]
 
 
 class Stats(ctypes.Structure):
@@ -34,7 +35,10 @@ class Stats(ctypes.Structure):
                 ("launches", ctypes.c_int32),
                 ("kernel_ms", ctypes.c_float * SGR_K_COUNT),
                 ("kernel_launches", ctypes.c_int64 * SGR_K_COUNT),
-                ("kernel_bytes", ctypes.c_int64 * SGR_K_COUNT)]
+                ("kernel_bytes", ctypes.c_int64 * SGR_K_COUNT),
+                ("bin_vertices", ctypes.c_int64 * 3), ("bin_edges", ctypes.c_int64 * 3),
+                ("chunk_items", ctypes.c_int64), ("grid_blocks", ctypes.c_int32),
+                ("color_bits", ctypes.c_int32)]
 
     def as_dict(self) -> dict:
         d = {k: getattr(self, k) for k in ("rounds", "num_colors", "vertices_processed",
@@ -43,6 +47,11 @@ class Stats(ctypes.Structure):
         d["kernel_ms"] = dict(zip(KERNEL_CLASSES, list(self.kernel_ms)))
         d["kernel_launches"] = dict(zip(KERNEL_CLASSES, list(self.kernel_launches)))
         d["kernel_bytes"] = dict(zip(KERNEL_CLASSES, list(self.kernel_bytes)))
+        d["bin_vertices"] = dict(zip(BINS, list(self.bin_vertices)))
+        d["bin_edges"] = dict(zip(BINS, list(self.bin_edges)))
+        d["chunk_items"] = self.chunk_items
+        d["grid_blocks"] = self.grid_blocks
+        d["color_bits"] = self.color_bits
         return d
 
 

@@ -1,5 +1,5 @@
 // sgr.cu — host side of libsgr.so: the C ABI of include/sgr.h (single GPU + step entry
-// points). Multi-GPU lives in sgr_dist.cu. See DESIGN.md §5 for the round loop.
+// points). Multi-GPU lives in sgr_dist.cu. DESIGN.md §5 describes the round loop.
 #include <cuda_runtime.h>
 
 #include <cstdarg>
@@ -10,7 +10,8 @@
 
 #include "sgr.h"
 #include "sgr_internal.h"
-#include "sgr_kernels.cuh"
+#include "sgr_round.cuh"
+#include "sgr_step.cuh"
 
 namespace sgr {
 
@@ -31,8 +32,7 @@ sgr_status cuda_fail(cudaError_t e, const char* what, int line) {
 int num_sms() {
   static int sms[64] = {0};
   int dev = 0;
-  if (cudaGetDevice(&dev) != cudaSuccess) return 148;
-  if (dev < 0 || dev >= 64) return 148;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return 148;
   if (sms[dev] == 0) {
     int v = 0;
     if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || v <= 0)
@@ -51,11 +51,12 @@ Resolved resolve_opts(const sgr_opts* o, int64_t n) {
   if (!o) o = &d;
   r.tiebreak = o->tiebreak == SGR_TIEBREAK_PAPER ? 1 : 0;
   r.max_rounds = o->max_rounds > 0 ? o->max_rounds : (int32_t)std::min<int64_t>(n + 1, INT32_MAX);
-  r.loop_mode = o->loop_mode == SGR_LOOP_HOST ? SGR_LOOP_HOST : SGR_LOOP_GRAPH;
-  r.block = o->block_size > 0 ? o->block_size : 256;
-  r.block = std::max(32, std::min(1024, r.block / 32 * 32));
+  r.loop_mode = (o->loop_mode == SGR_LOOP_HOST || o->loop_mode == SGR_LOOP_GRAPH)
+                    ? o->loop_mode : SGR_LOOP_PERSISTENT;
+  r.color_bits = o->color_bits == 32 ? 32 : 16;
   r.small_max = o->bin_small_max > 0 ? std::min(o->bin_small_max, 62) : 32;
-  r.med_max = o->bin_med_max > 0 ? std::max(o->bin_med_max, r.small_max) : 4096;
+  r.med_max = o->bin_med_max > 0 ? std::min(o->bin_med_max, kMaxMed) : kMaxMed;
+  r.med_max = std::max(r.med_max, r.small_max);
   r.stream = (cudaStream_t)o->stream;
   r.round_sizes = o->round_sizes;
   r.round_edges = o->round_edges;
@@ -63,112 +64,129 @@ Resolved resolve_opts(const sgr_opts* o, int64_t n) {
   r.validate = o->validate;
   r.batch = o->rounds_per_batch > 0 ? o->rounds_per_batch : 8;
   r.profile = o->profile;
+  r.round_ms = o->round_ms;
   return r;
 }
 
-// Workspace layout: [Ctrl][Y: n int32][wl: 2 x kBins x n int32]
-size_t ws_bytes(int64_t n) {
-  size_t b = align_up(sizeof(Ctrl), 256);
-  b += align_up((size_t)n * 4, 256);
-  b += (size_t)2 * kBins * align_up((size_t)n * 4, 256);
-  return b;
-}
-
-struct Workspace {
-  Ctrl* ctrl;
-  int32_t* y;
-  int32_t* wl[2][kBins];
+// Workspace layout (bytes, each piece 256-aligned):
+//   Ctrl | X16, Y16: 2 x n u16 (16-bit mode) | Y32: n i32 | wl_t: 2 x n i32 |
+//   wl_m: 2 x cap_m i32 | wl_c: 2 x cap_c i64 | big_id: n i32 | acc_bits | acc_cnt
+// In 32-bit mode the caller's colors_out is C_k's ping-pong partner of Y32; in 16-bit mode
+// the two u16 buffers ping-pong and the result is widened into colors_out at the end.
+struct Layout {
+  int64_t cap_m, cap_c, cap_big;
+  size_t off_c16, off_y32, off_t, off_m, off_c, off_big, off_accb, off_accc, total;
 };
 
-static Workspace carve(void* base, int64_t n) {
-  Workspace w;
-  char* p = (char*)base;
-  w.ctrl = (Ctrl*)p;
-  p += align_up(sizeof(Ctrl), 256);
-  w.y = (int32_t*)p;
-  p += align_up((size_t)n * 4, 256);
-  for (int par = 0; par < 2; ++par)
-    for (int q = 0; q < kBins; ++q) {
-      w.wl[par][q] = (int32_t*)p;
-      p += align_up((size_t)n * 4, 256);
-    }
-  return w;
+static Layout layout(int64_t n, int64_t nnz, const Resolved& r) {
+  Layout L;
+  L.cap_m = std::min<int64_t>(n, nnz / (r.small_max + 1) + 1);
+  // each bin-2 vertex (deg > med_max) has <= deg / kChunk + 2 aligned chunks
+  L.cap_c = nnz / kChunk + 2 * (nnz / (r.med_max + 1)) + 2;
+  L.cap_big = nnz / (r.med_max + 1) + 1;
+  size_t o = align_up(sizeof(Ctrl), 256);
+  L.off_c16 = o;
+  o += 2 * align_up((size_t)n * 2, 256);
+  L.off_y32 = o;
+  o += align_up((size_t)n * 4, 256);
+  L.off_t = o;
+  o += 2 * align_up((size_t)n * 4, 256);
+  L.off_m = o;
+  o += 2 * align_up((size_t)L.cap_m * 4, 256);
+  L.off_c = o;
+  o += 2 * align_up((size_t)L.cap_c * 8, 256);
+  L.off_big = o;
+  o += align_up((size_t)n * 4, 256);
+  L.off_accb = o;
+  o += align_up((size_t)L.cap_big * 128, 256);
+  L.off_accc = o;
+  o += align_up((size_t)L.cap_big * 8, 256);
+  L.total = o;
+  return L;
+}
+
+size_t ws_bytes(int64_t n, int64_t nnz, const Resolved& r) { return layout(n, nnz, r).total; }
+
+template <class C>
+static void build_args(RoundArgs<C>& a, const sgr_csr* csr, int64_t n, int32_t* colors,
+                       void* ws, const Layout& L, const Resolved& r) {
+  memset(&a, 0, sizeof(a));
+  char* b = (char*)ws;
+  a.row_ptr = csr->row_ptr;
+  a.col_idx = csr->col_idx;
+  if constexpr (sizeof(C) == 2) {
+    a.col[0] = (C*)(b + L.off_c16);
+    a.col[1] = (C*)(b + L.off_c16 + align_up((size_t)n * 2, 256));
+  } else {
+    a.col[0] = (C*)colors;
+    a.col[1] = (C*)(b + L.off_y32);
+  }
+  const size_t st = align_up((size_t)n * 4, 256);
+  a.wl_t[0] = (int32_t*)(b + L.off_t);
+  a.wl_t[1] = (int32_t*)(b + L.off_t + st);
+  const size_t sm = align_up((size_t)L.cap_m * 4, 256);
+  a.wl_m[0] = (int32_t*)(b + L.off_m);
+  a.wl_m[1] = (int32_t*)(b + L.off_m + sm);
+  const size_t sc = align_up((size_t)L.cap_c * 8, 256);
+  a.wl_c[0] = (int64_t*)(b + L.off_c);
+  a.wl_c[1] = (int64_t*)(b + L.off_c + sc);
+  a.big_id = (int32_t*)(b + L.off_big);
+  a.acc_bits = (uint32_t*)(b + L.off_accb);
+  a.acc_cnt = (unsigned long long*)(b + L.off_accc);
+  a.ctrl = (Ctrl*)b;
+  a.n = (int32_t)n;
+  a.nnz = 0;
+  a.small_max = r.small_max;
+  a.med_max = r.med_max;
 }
 
 // Pinned host slots for termination flags (reused across calls on this thread).
 static int32_t* pinned_flags() {
   static thread_local int32_t* p = nullptr;
-  if (!p) {
-    if (cudaMallocHost(&p, 64 * sizeof(int32_t)) != cudaSuccess) p = nullptr;
-  }
+  if (!p && cudaMallocHost(&p, 64 * sizeof(int32_t)) != cudaSuccess) p = nullptr;
   return p;
 }
 
-// ----- per-launch grids ------------------------------------------------------------------
-struct Grids {
-  int first, thread_b, warp_b, cta_b, block, cta_threads;
-};
-
-static Grids make_grids(int64_t n, const Resolved& r) {
-  Grids g;
-  const int sms = num_sms();
-  g.block = r.block;
-  const int per_sm = std::max(1, 2048 / g.block);
-  g.first = (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, (int64_t)sms * 8));
-  g.thread_b = (int)std::max<int64_t>(1, std::min<int64_t>((n + g.block - 1) / g.block, (int64_t)sms * per_sm));
-  g.warp_b = (int)std::max<int64_t>(1, std::min<int64_t>((n * 32 + g.block - 1) / g.block, (int64_t)sms * per_sm));
-  g.cta_threads = 512;
-  g.cta_b = sms * 4;
-  return g;
+int first_grid(int64_t n) {
+  return (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, (int64_t)num_sms() * 8));
 }
 
-// ----- the round-pass launcher (shared by the host loop, graph capture and dist) --------
-template <int TB>
-static void launch_pass(const RoundArgs& a, const Grids& g, cudaStream_t s) {
-  k_round_cta<TB><<<g.cta_b, g.cta_threads, 0, s>>>(a);
-  k_round_warp<TB><<<g.warp_b, g.block, 0, s>>>(a);
-  k_round_thread<TB><<<g.thread_b, g.block, 0, s>>>(a);
-  k_advance<<<1, 32, 0, s>>>(a.ctrl, 0);
+// Blocks of the round kernels: as many as are co-resident (persistent: required).
+template <int TB, class C>
+static int round_grid(bool persistent) {
+  int per_sm = 0;
+  cudaError_t e = persistent
+      ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_persistent<TB, C>, kBlock, 0)
+      : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_round<TB, C>, kBlock, 0);
+  if (e != cudaSuccess || per_sm <= 0) per_sm = 1;
+  return per_sm * num_sms();
 }
 
-void launch_first(const RoundArgs& a, int tiebreak, bool sorted, int grid, cudaStream_t s) {
-  if (sorted) {
-    if (tiebreak) k_first<1><<<grid, 256, 0, s>>>(a);
-    else k_first<0><<<grid, 256, 0, s>>>(a);
-  } else {
-    if (tiebreak) k_first_unsorted<1><<<grid, 256, 0, s>>>(a);
-    else k_first_unsorted<0><<<grid, 256, 0, s>>>(a);
-  }
-}
-
-void launch_round_pass(const RoundArgs& a, int tiebreak, int64_t n, const Resolved& r,
-                       cudaStream_t s) {
-  Grids g = make_grids(n, r);
-  if (tiebreak) launch_pass<1>(a, g, s);
-  else launch_pass<0>(a, g, s);
-}
-
-// ----- CUDA-graph cache: one graph = `batch` fused passes ----------------------------------
+// ----- CUDA-graph cache: one graph = `batch` round passes -----------------------------------
 struct GraphKey {
-  RoundArgs a;
-  Grids g;
-  int tiebreak, batch, dev;
+  unsigned char args[sizeof(RoundArgs<int32_t>)];
+  int tiebreak, bits, batch, dev, grid;
   bool operator==(const GraphKey& o) const { return memcmp(this, &o, sizeof(GraphKey)) == 0; }
 };
 
-struct GraphEntry {
-  GraphKey key;
-  cudaGraphExec_t exec;
-};
-
 static std::mutex g_graph_mu;
-static std::vector<GraphEntry> g_graphs;
+static std::vector<std::pair<GraphKey, cudaGraphExec_t>> g_graphs;
 
-static sgr_status get_graph(const GraphKey& key, cudaGraphExec_t* out) {
+template <int TB, class C>
+static sgr_status get_graph(const RoundArgs<C>& a, int grid, int batch, cudaGraphExec_t* out) {
+  GraphKey key;
+  memset(&key, 0, sizeof(key));
+  static_assert(sizeof(RoundArgs<C>) <= sizeof(key.args), "graph key");
+  memcpy(key.args, &a, sizeof(a));
+  key.tiebreak = TB;
+  key.bits = 8 * (int)sizeof(C);
+  key.batch = batch;
+  key.grid = grid;
+  cudaGetDevice(&key.dev);
   std::lock_guard<std::mutex> lk(g_graph_mu);
   for (auto& e : g_graphs)
-    if (e.key == key) {
-      *out = e.exec;
+    if (e.first == key) {
+      *out = e.second;
       return SGR_OK;
     }
   cudaStream_t cs;
@@ -179,9 +197,9 @@ static sgr_status get_graph(const GraphKey& key, cudaGraphExec_t* out) {
     cudaStreamDestroy(cs);
     return cuda_fail(err, "cudaStreamBeginCapture", __LINE__);
   }
-  for (int b = 0; b < key.batch; ++b) {
-    if (key.tiebreak) launch_pass<1>(key.a, key.g, cs);
-    else launch_pass<0>(key.a, key.g, cs);
+  for (int b = 0; b < batch; ++b) {
+    k_round<TB, C><<<grid, kBlock, 0, cs>>>(a);
+    k_advance<<<1, 32, 0, cs>>>(a.ctrl, 0);
   }
   cudaGraph_t graph;
   err = cudaStreamEndCapture(cs, &graph);
@@ -192,7 +210,7 @@ static sgr_status get_graph(const GraphKey& key, cudaGraphExec_t* out) {
   cudaGraphDestroy(graph);
   if (err != cudaSuccess) return cuda_fail(err, "cudaGraphInstantiate", __LINE__);
   if (g_graphs.size() >= 8) {
-    cudaGraphExecDestroy(g_graphs.front().exec);
+    cudaGraphExecDestroy(g_graphs.front().second);
     g_graphs.erase(g_graphs.begin());
   }
   g_graphs.push_back({key, exec});
@@ -200,8 +218,9 @@ static sgr_status get_graph(const GraphKey& key, cudaGraphExec_t* out) {
   return SGR_OK;
 }
 
-// ----- profiling (opts->profile): CUDA events around every launch -----------------------
+// ----- profiling (opts->profile): CUDA events around launches ------------------------------
 struct Prof {
+  bool on = false;
   std::vector<cudaEvent_t> pool;
   std::vector<std::pair<int, std::pair<cudaEvent_t, cudaEvent_t>>> marks;
   size_t used = 0;
@@ -213,57 +232,224 @@ struct Prof {
     }
     return pool[used++];
   }
+  template <class F>
+  void timed(int cls, cudaStream_t s, F&& fn) {
+    if (!on) {
+      fn();
+      return;
+    }
+    cudaEvent_t e0 = get(), e1 = get();
+    cudaEventRecord(e0, s);
+    fn();
+    cudaEventRecord(e1, s);
+    marks.push_back({cls, {e0, e1}});
+  }
+  void reset() {
+    used = 0;
+    marks.clear();
+  }
   ~Prof() {
     for (auto e : pool) cudaEventDestroy(e);
   }
 };
 
-template <int TB>
-static void launch_pass_prof(const RoundArgs& a, const Grids& g, cudaStream_t s, Prof& pr) {
-  auto timed = [&](int cls, auto&& fn) {
-    cudaEvent_t e0 = pr.get(), e1 = pr.get();
-    cudaEventRecord(e0, s);
-    fn();
-    cudaEventRecord(e1, s);
-    pr.marks.push_back({cls, {e0, e1}});
-  };
-  timed(SGR_K_HUB, [&] { k_round_cta<TB><<<g.cta_b, g.cta_threads, 0, s>>>(a); });
-  timed(SGR_K_MED, [&] { k_round_warp<TB><<<g.warp_b, g.block, 0, s>>>(a); });
-  timed(SGR_K_SMALL, [&] { k_round_thread<TB><<<g.thread_b, g.block, 0, s>>>(a); });
-  timed(SGR_K_CTRL, [&] { k_advance<<<1, 32, 0, s>>>(a.ctrl, 0); });
-}
-
-// Fill the byte model and counters from the final Ctrl.
+// Byte model and counters from the final Ctrl.
 void fill_stats(const Ctrl& c, int64_t n, int64_t nnz, sgr_stats* st) {
-  const int64_t vpass = (int64_t)(c.verts_total[0] + c.verts_total[1] + c.verts_total[2]);
-  const int64_t epass = (int64_t)(c.edges_total[0] + c.edges_total[1] + c.edges_total[2]);
+  int64_t vpass = 0, epass = 0, b_round = 0;
+  for (int q = 0; q < kBins; ++q) {
+    vpass += (int64_t)c.verts_total[q];
+    epass += (int64_t)c.edges_total[q];
+    st->bin_vertices[q] = (int64_t)c.verts_total[q];
+    st->bin_edges[q] = (int64_t)c.edges_total[q];
+    // per worklist vertex: 4 B id + 16 B row pair + 4 B X[v] + 4 B Y[v]; 8 B per scanned
+    // entry (4 B col_idx + 4 B X[w]); 4 B per vertex pushed to W_{k+1}
+    b_round += 28 * (int64_t)c.verts_total[q] + 8 * (int64_t)c.edges_total[q] +
+               4 * (int64_t)c.pushes_total[q];
+  }
+  st->chunk_items = (int64_t)c.items_total;
   st->rounds = c.k - 1;
   st->num_colors = c.max_color;
-  st->vertices_processed = (n > 0 ? n : 0) + vpass;
-  st->edges_scanned = (n > 0 ? nnz : 0) + epass;
-  // F_1: 8 B row offset + 4 B first/last col entry + 8 B two color writes per vertex,
-  //      + 4 B per pushed vertex.
+  st->vertices_processed = n + vpass;
+  st->edges_scanned = nnz + epass;
+  // F_1 per vertex: 8 B row offset + 4 B first/last entry + 4 B + 4 B color writes; 4 B/push
   const int64_t b_first = 20 * n + 4 * (int64_t)c.pushes_total[kBins];
-  int64_t b_bins[kBins];
-  for (int q = 0; q < kBins; ++q)  // per vertex: 4 B id + 16 B row pair + 4 B X[v] + 4 B Y[v]
-    b_bins[q] = 28 * (int64_t)c.verts_total[q] + 8 * (int64_t)c.edges_total[q] +
-                4 * (int64_t)c.pushes_total[q];
-  st->bytes_algorithmic = b_first + b_bins[0] + b_bins[1] + b_bins[2];
+  const int64_t b_final = 4 * n;
+  st->bytes_algorithmic = b_first + b_round + b_final;
   st->kernel_bytes[SGR_K_FIRST] = b_first;
-  st->kernel_bytes[SGR_K_SMALL] = b_bins[0];
-  st->kernel_bytes[SGR_K_MED] = b_bins[1];
-  st->kernel_bytes[SGR_K_HUB] = b_bins[2];
+  st->kernel_bytes[SGR_K_ROUND] = b_round;
   st->kernel_bytes[SGR_K_CTRL] = 0;
+  st->kernel_bytes[SGR_K_FINAL] = b_final;
+}
+
+// One complete coloring with working color type C. *overflow_out = 1 if a u16 first fit
+// exceeded 65535 (the caller then reruns with 32-bit colors).
+template <int TB, class C>
+static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* colors_out,
+                            sgr_stats* stats, const Resolved& r, void* ws, const Layout& L,
+                            int* overflow_out) {
+  cudaStream_t s = r.stream;
+  RoundArgs<C> a;
+  build_args<C>(a, csr, n, colors_out, ws, L, r);
+  a.nnz = nnz;
+  Prof prof;
+  prof.on = r.profile != 0;
+  int32_t launches = 0;
+  const bool persistent = r.loop_mode == SGR_LOOP_PERSISTENT;
+  const int grid = round_grid<TB, C>(persistent);
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  sgr_status status = SGR_OK;
+  do {
+    Ctrl hc;
+    memset(&hc, 0, sizeof(hc));
+    hc.k = 1;
+    hc.max_rounds = r.max_rounds;
+    hc.round_cap = r.round_cap;
+    hc.round_sizes = r.round_sizes;
+    hc.round_edges = r.round_edges;
+    cudaError_t le = cudaMemcpyAsync(a.ctrl, &hc, sizeof(Ctrl), cudaMemcpyHostToDevice, s);
+    if (le == cudaSuccess) le = cudaMemsetAsync((char*)ws + L.off_accb, 0, L.total - L.off_accb, s);
+    if (le != cudaSuccess) {
+      status = cuda_fail(le, "workspace init", __LINE__);
+      break;
+    }
+    if (r.round_cap > 0) {  // round 1: |W_1| = n, sum of degrees = nnz
+      int32_t n32 = (int32_t)n;
+      int64_t nz = nnz;
+      if (r.round_sizes) cudaMemcpyAsync(r.round_sizes, &n32, 4, cudaMemcpyHostToDevice, s);
+      if (r.round_edges) cudaMemcpyAsync(r.round_edges, &nz, 8, cudaMemcpyHostToDevice, s);
+    }
+    cudaEventCreate(&ev0);
+    cudaEventCreate(&ev1);
+    cudaEventRecord(ev0, s);
+
+    prof.timed(SGR_K_FIRST, s, [&] { k_first<TB, C><<<first_grid(n), 256, 0, s>>>(a, 1); });
+    prof.timed(SGR_K_CTRL, s, [&] { k_advance<<<1, 32, 0, s>>>(a.ctrl, 1); });
+    launches += 2;
+    le = cudaGetLastError();
+    if (le != cudaSuccess) {
+      status = cuda_fail(le, "launch F_1", __LINE__);
+      break;
+    }
+
+    if (persistent) {
+      prof.timed(SGR_K_ROUND, s, [&] {
+        void* args[] = {(void*)&a};
+        le = cudaLaunchCooperativeKernel((const void*)k_persistent<TB, C>, grid, kBlock, args, 0, s);
+      });
+      launches += 1;
+      if (le != cudaSuccess) {
+        status = cuda_fail(le, "cooperative launch of k_persistent", __LINE__);
+        break;
+      }
+    } else {
+      int32_t* flags = pinned_flags();
+      if (!flags) {
+        status = cuda_fail(cudaErrorMemoryAllocation, "cudaMallocHost", __LINE__);
+        break;
+      }
+      cudaEvent_t done_ev[2];
+      cudaEventCreateWithFlags(&done_ev[0], cudaEventDisableTiming);
+      cudaEventCreateWithFlags(&done_ev[1], cudaEventDisableTiming);
+      const bool use_graph = r.loop_mode == SGR_LOOP_GRAPH && !prof.on;
+      cudaGraphExec_t gexec = nullptr;
+      if (use_graph) status = get_graph<TB, C>(a, grid, r.batch, &gexec);
+      // Pipelined termination test: batch b's `active` flag is read after batch b+1 is
+      // enqueued, so the GPU never waits for the host; surplus passes are no-ops.
+      int64_t batches = 0;
+      bool finished = status != SGR_OK;
+      while (!finished) {
+        if (use_graph) {
+          le = cudaGraphLaunch(gexec, s);
+        } else {
+          for (int b = 0; b < r.batch; ++b) {
+            prof.timed(SGR_K_ROUND, s, [&] { k_round<TB, C><<<grid, kBlock, 0, s>>>(a); });
+            prof.timed(SGR_K_CTRL, s, [&] { k_advance<<<1, 32, 0, s>>>(a.ctrl, 0); });
+          }
+          le = cudaGetLastError();
+        }
+        launches += 2 * r.batch;
+        if (le != cudaSuccess) {
+          status = cuda_fail(le, "launch round batch", __LINE__);
+          break;
+        }
+        const int slot = (int)(batches & 1);
+        cudaMemcpyAsync(&flags[slot], &a.ctrl->active, 4, cudaMemcpyDeviceToHost, s);
+        cudaEventRecord(done_ev[slot], s);
+        if (batches > 0) {
+          cudaEventSynchronize(done_ev[slot ^ 1]);
+          if (flags[slot ^ 1] == 0) finished = true;
+        }
+        ++batches;
+      }
+      cudaEventDestroy(done_ev[0]);
+      cudaEventDestroy(done_ev[1]);
+      if (status != SGR_OK) break;
+    }
+
+    prof.timed(SGR_K_FINAL, s, [&] {
+      if constexpr (sizeof(C) == 2) k_widen<<<first_grid(n), 256, 0, s>>>(a.col[0], colors_out, n);
+      k_max_color<<<first_grid(n), 256, 0, s>>>(colors_out, n, &a.ctrl->max_color);
+    });
+    launches += sizeof(C) == 2 ? 2 : 1;
+    cudaEventRecord(ev1, s);
+    Ctrl fin;
+    cudaMemcpyAsync(&fin, a.ctrl, sizeof(Ctrl), cudaMemcpyDeviceToHost, s);
+    le = cudaStreamSynchronize(s);
+    if (le != cudaSuccess) {
+      status = cuda_fail(le, "sgr_color", __LINE__);
+      break;
+    }
+    *overflow_out = fin.overflow;
+    if (stats) {
+      fill_stats(fin, n, nnz, stats);
+      cudaEventElapsedTime(&stats->elapsed_ms, ev0, ev1);
+      stats->launches = launches;
+      stats->grid_blocks = grid;
+      stats->color_bits = 8 * (int)sizeof(C);
+      int32_t ri = 0;
+      for (auto& m : prof.marks) {
+        float ms = 0.f;
+        cudaEventElapsedTime(&ms, m.second.first, m.second.second);
+        stats->kernel_ms[m.first] += ms;
+        stats->kernel_launches[m.first] += 1;
+        if (m.first == SGR_K_ROUND && r.round_ms && ri < r.round_cap) r.round_ms[ri++] = ms;
+      }
+    }
+    if (fin.status == 1) {
+      set_error("sgr_color: max_rounds (%d) reached", r.max_rounds);
+      status = SGR_ENOCONV;
+    }
+  } while (0);
+  if (ev0) cudaEventDestroy(ev0);
+  if (ev1) cudaEventDestroy(ev1);
+  return status;
+}
+
+template <int TB>
+static sgr_status run_any(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* colors_out,
+                          sgr_stats* stats, const Resolved& r, void* ws, const Layout& L) {
+  int overflow = 0;
+  if (r.color_bits == 16) {
+    const sgr_status st = run_color<TB, uint16_t>(csr, n, nnz, colors_out, stats, r, ws, L, &overflow);
+    if (st != SGR_OK || !overflow) return st;
+    // a first fit exceeded 65535: the 16-bit run is discarded and redone in 32 bits
+  }
+  const sgr_status st = run_color<TB, int32_t>(csr, n, nnz, colors_out, stats, r, ws, L, &overflow);
+  if (st == SGR_OK && overflow) {
+    set_error("sgr_color: 32-bit color overflow");
+    return SGR_EUNSUPPORTED;
+  }
+  return st;
 }
 
 }  // namespace sgr
 
 using namespace sgr;
 
-#define CK(call)                                                         \
-  do {                                                                   \
-    cudaError_t e_ = (call);                                             \
-    if (e_ != cudaSuccess) return cuda_fail(e_, #call, __LINE__);        \
+#define CK(call)                                                  \
+  do {                                                            \
+    cudaError_t e_ = (call);                                      \
+    if (e_ != cudaSuccess) return cuda_fail(e_, #call, __LINE__); \
   } while (0)
 
 extern "C" {
@@ -276,9 +462,8 @@ void sgr_opts_default(sgr_opts* o) {
 }
 
 size_t sgr_workspace_bytes(int64_t n, int64_t nnz, const sgr_opts* opts) {
-  (void)nnz;
-  (void)opts;
-  return n > 0 ? ws_bytes(n) : 0;
+  if (n <= 0) return 0;
+  return ws_bytes(n, nnz, resolve_opts(opts, n));
 }
 
 const char* sgr_strerror(sgr_status s) {
@@ -295,15 +480,15 @@ const char* sgr_strerror(sgr_status s) {
 }
 
 const char* sgr_last_error(void) { return g_err; }
-const char* sgr_version(void) { return "sgr-b200 0.1 (sm_100a)"; }
+const char* sgr_version(void) { return "sgr-b200 0.2 (sm_100a)"; }
 
-static sgr_status run_validate(const sgr_csr* csr, int64_t n, int64_t nnz, Ctrl* ctrl,
+static sgr_status run_validate(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* dviol,
                                cudaStream_t s, int32_t* viol_out) {
-  CK(cudaMemsetAsync(&ctrl->violations, 0, sizeof(int32_t), s));
-  k_validate<<<num_sms() * 4, 256, 0, s>>>(csr->row_ptr, csr->col_idx, n, nnz, ctrl);
+  CK(cudaMemsetAsync(dviol, 0, sizeof(int32_t), s));
+  k_validate<<<num_sms() * 4, 256, 0, s>>>(csr->row_ptr, csr->col_idx, n, nnz, dviol);
   CK(cudaGetLastError());
   int32_t v = 0;
-  CK(cudaMemcpyAsync(&v, &ctrl->violations, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+  CK(cudaMemcpyAsync(&v, dviol, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
   CK(cudaStreamSynchronize(s));
   *viol_out = v;
   return SGR_OK;
@@ -314,10 +499,10 @@ sgr_status sgr_validate_csr(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
   if (!csr || !csr->row_ptr || n < 0 || nnz < 0 || !violations || (nnz > 0 && !csr->col_idx))
     return SGR_EINVAL;
   cudaStream_t s = (cudaStream_t)stream;
-  Ctrl* ctrl;
-  CK(cudaMallocAsync((void**)&ctrl, sizeof(Ctrl), s));
-  sgr_status st = run_validate(csr, n, nnz, ctrl, s, violations);
-  cudaFreeAsync(ctrl, s);
+  int32_t* d;
+  CK(cudaMallocAsync((void**)&d, sizeof(int32_t), s));
+  sgr_status st = run_validate(csr, n, nnz, d, s, violations);
+  cudaFreeAsync(d, s);
   cudaStreamSynchronize(s);
   return st;
 }
@@ -335,179 +520,31 @@ sgr_status sgr_color_ex(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* col
     set_error("sgr_color: null pointer");
     return SGR_EINVAL;
   }
+  if (((uintptr_t)csr->col_idx & 15u) != 0) {
+    set_error("sgr_color: col_idx must be 16-byte aligned");
+    return SGR_EINVAL;
+  }
   const Resolved r = resolve_opts(opts, n);
   cudaStream_t s = r.stream;
-  const size_t need = ws_bytes(n);
+  const Layout L = layout(n, nnz, r);
   void* ws = workspace;
   bool own = false;
-  if (!ws || workspace_bytes < need) {
-    CK(cudaMallocAsync(&ws, need, s));
+  if (!ws || workspace_bytes < L.total) {
+    CK(cudaMallocAsync(&ws, L.total, s));
     own = true;
   }
-  Workspace w = carve(ws, n);
   sgr_status status = SGR_OK;
-  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
-  Prof prof;
-  int32_t launches = 0;
-  do {
-    if (r.validate) {
-      int32_t viol = 0;
-      status = run_validate(csr, n, nnz, w.ctrl, s, &viol);
-      if (status != SGR_OK) break;
-      if (viol) {
-        set_error("sgr_color: CSR contract violated (mask %d)", viol);
-        status = SGR_EINVAL;
-        break;
-      }
+  if (r.validate) {
+    int32_t viol = 0;
+    status = run_validate(csr, n, nnz, &((Ctrl*)ws)->violations, s, &viol);
+    if (status == SGR_OK && viol) {
+      set_error("sgr_color: invalid CSR (violation mask %d)", viol);
+      status = SGR_EINVAL;
     }
-    // Ctrl init (host image -> device)
-    Ctrl hc;
-    memset(&hc, 0, sizeof(hc));
-    hc.k = 1;
-    hc.max_rounds = r.max_rounds;
-    hc.round_cap = r.round_cap;
-    hc.round_sizes = r.round_sizes;
-    hc.round_edges = r.round_edges;
-    if (cudaMemcpyAsync(w.ctrl, &hc, sizeof(Ctrl), cudaMemcpyHostToDevice, s) != cudaSuccess) {
-      status = cuda_fail(cudaGetLastError(), "ctrl init", __LINE__);
-      break;
-    }
-    if (r.round_cap > 0) {  // round 1: |W_1| = n, sum deg = nnz
-      int32_t n32 = (int32_t)n;
-      int64_t nz = nnz;
-      if (r.round_sizes) cudaMemcpyAsync(r.round_sizes, &n32, 4, cudaMemcpyHostToDevice, s);
-      if (r.round_edges) cudaMemcpyAsync(r.round_edges, &nz, 8, cudaMemcpyHostToDevice, s);
-    }
-    cudaEventCreate(&ev0);
-    cudaEventCreate(&ev1);
-    cudaEventRecord(ev0, s);
-
-    RoundArgs a;
-    memset(&a, 0, sizeof(a));
-    a.row_ptr = csr->row_ptr;
-    a.col_idx = csr->col_idx;
-    a.col[0] = colors_out;
-    a.col[1] = w.y;
-    for (int par = 0; par < 2; ++par)
-      for (int q = 0; q < kBins; ++q) a.wl[par][q] = w.wl[par][q];
-    a.ctrl = w.ctrl;
-    a.n = (int32_t)n;
-    a.small_max = r.small_max;
-    a.med_max = r.med_max;
-    const Grids g = make_grids(n, r);
-
-    cudaEvent_t pf0 = nullptr, pf1 = nullptr;
-    if (r.profile) {
-      pf0 = prof.get();
-      pf1 = prof.get();
-      cudaEventRecord(pf0, s);
-    }
-    launch_first(a, r.tiebreak, true, g.first, s);
-    if (r.profile) {
-      cudaEventRecord(pf1, s);
-      prof.marks.push_back({SGR_K_FIRST, {pf0, pf1}});
-    }
-    k_advance<<<1, 32, 0, s>>>(w.ctrl, 1);
-    launches += 2;
-    cudaError_t le = cudaGetLastError();
-    if (le != cudaSuccess) {
-      status = cuda_fail(le, "launch F_1", __LINE__);
-      break;
-    }
-
-    int32_t* flags = pinned_flags();
-    if (!flags) {
-      status = cuda_fail(cudaErrorMemoryAllocation, "cudaMallocHost", __LINE__);
-      break;
-    }
-    cudaEvent_t done_ev[2];
-    cudaEventCreateWithFlags(&done_ev[0], cudaEventDisableTiming);
-    cudaEventCreateWithFlags(&done_ev[1], cudaEventDisableTiming);
-    const bool use_graph = r.loop_mode == SGR_LOOP_GRAPH && !r.profile;
-    cudaGraphExec_t gexec = nullptr;
-    if (use_graph) {
-      GraphKey key;
-      memset(&key, 0, sizeof(key));
-      key.a = a;
-      key.g = g;
-      key.tiebreak = r.tiebreak;
-      key.batch = r.batch;
-      cudaGetDevice(&key.dev);
-      status = get_graph(key, &gexec);
-      if (status != SGR_OK) break;
-    }
-    // Pipelined termination test: batch b's `active` flag is read only after batch b+1 is
-    // enqueued, so the GPU never idles waiting for the host; surplus passes are no-ops.
-    int64_t batches = 0;
-    bool finished = false;
-    while (!finished) {
-      if (use_graph) {
-        le = cudaGraphLaunch(gexec, s);
-        launches += 4 * r.batch;
-      } else {
-        for (int b = 0; b < r.batch; ++b) {
-          if (r.profile) {
-            if (r.tiebreak) launch_pass_prof<1>(a, g, s, prof);
-            else launch_pass_prof<0>(a, g, s, prof);
-          } else {
-            if (r.tiebreak) launch_pass<1>(a, g, s);
-            else launch_pass<0>(a, g, s);
-          }
-        }
-        launches += 4 * r.batch;
-        le = cudaGetLastError();
-      }
-      if (le != cudaSuccess) {
-        status = cuda_fail(le, "launch round batch", __LINE__);
-        break;
-      }
-      const int slot = (int)(batches & 1);
-      cudaMemcpyAsync(&flags[slot], &w.ctrl->active, 4, cudaMemcpyDeviceToHost, s);
-      cudaEventRecord(done_ev[slot], s);
-      if (batches > 0) {
-        cudaEventSynchronize(done_ev[slot ^ 1]);
-        if (flags[slot ^ 1] == 0) finished = true;
-      }
-      ++batches;
-      if (batches > ((int64_t)r.max_rounds / r.batch) + 4) {  // defensive: cannot happen
-        cudaEventSynchronize(done_ev[slot]);
-        if (flags[slot] == 0) finished = true;
-      }
-    }
-    cudaEventDestroy(done_ev[0]);
-    cudaEventDestroy(done_ev[1]);
-    if (status != SGR_OK) break;
-
-    k_max_color<<<g.first, 256, 0, s>>>(colors_out, n, w.ctrl);
-    launches += 1;
-    cudaEventRecord(ev1, s);
-    Ctrl fin;
-    cudaMemcpyAsync(&fin, w.ctrl, sizeof(Ctrl), cudaMemcpyDeviceToHost, s);
-    le = cudaStreamSynchronize(s);
-    if (le != cudaSuccess) {
-      status = cuda_fail(le, "sgr_color", __LINE__);
-      break;
-    }
-    if (stats) {
-      fill_stats(fin, n, nnz, stats);
-      cudaEventElapsedTime(&stats->elapsed_ms, ev0, ev1);
-      stats->launches = launches;
-      if (r.profile) {
-        for (auto& m : prof.marks) {
-          float ms = 0.f;
-          cudaEventElapsedTime(&ms, m.second.first, m.second.second);
-          stats->kernel_ms[m.first] += ms;
-          stats->kernel_launches[m.first] += 1;
-        }
-      }
-    }
-    if (fin.status == 1) {
-      set_error("sgr_color: max_rounds (%d) reached", r.max_rounds);
-      status = SGR_ENOCONV;
-    }
-  } while (0);
-  if (ev0) cudaEventDestroy(ev0);
-  if (ev1) cudaEventDestroy(ev1);
+  }
+  if (status == SGR_OK)
+    status = r.tiebreak ? run_any<1>(csr, n, nnz, colors_out, stats, r, ws, L)
+                        : run_any<0>(csr, n, nnz, colors_out, stats, r, ws, L);
   if (own) {
     cudaFreeAsync(ws, s);
     cudaStreamSynchronize(s);
@@ -539,9 +576,7 @@ sgr_status sgr_color_host(const int64_t* row_ptr, const int32_t* col_idx, int64_
   if (nnz > 0) CK(cudaMemcpyAsync(d_ci, col_idx, (size_t)nnz * 4, cudaMemcpyHostToDevice, s));
   sgr_csr csr{d_rp, d_ci};
   sgr_status st = sgr_color_ex(&csr, n, nnz, d_col, stats, opts, nullptr, 0);
-  if (st == SGR_OK) {
-    CK(cudaMemcpyAsync(colors_out, d_col, (size_t)n * 4, cudaMemcpyDeviceToHost, s));
-  }
+  if (st == SGR_OK) CK(cudaMemcpyAsync(colors_out, d_col, (size_t)n * 4, cudaMemcpyDeviceToHost, s));
   cudaFreeAsync(d_rp, s);
   cudaFreeAsync(d_ci, s);
   cudaFreeAsync(d_col, s);
@@ -559,7 +594,7 @@ sgr_status sgr_assign(const sgr_csr* csr, int64_t n, const int32_t* wl, int64_t 
                       const int32_t* colors_in, int32_t* tent_out, const sgr_opts* opts) {
   if (!csr || n < 0 || wl_len < 0) return SGR_EINVAL;
   if (wl_len == 0) return SGR_OK;
-  if (!csr->row_ptr || !csr->col_idx || !wl || !colors_in || !tent_out ||
+  if (!csr->row_ptr || !wl || !colors_in || !tent_out ||
       (const void*)colors_in == (const void*)tent_out) {
     set_error("sgr_assign: null or aliased pointer");
     return SGR_EINVAL;
@@ -586,7 +621,7 @@ sgr_status sgr_detect(const sgr_csr* csr, int64_t n, const int32_t* wl, int64_t 
                       const int32_t* colors, uint8_t* conflict_out, const sgr_opts* opts) {
   if (!csr || n < 0 || wl_len < 0) return SGR_EINVAL;
   if (wl_len == 0) return SGR_OK;
-  if (!csr->row_ptr || !csr->col_idx || !wl || !colors || !conflict_out) return SGR_EINVAL;
+  if (!csr->row_ptr || !wl || !colors || !conflict_out) return SGR_EINVAL;
   const Resolved r = resolve_opts(opts, n);
   if (r.tiebreak)
     k_detect_step<1><<<grid_for(wl_len, 8), 256, 0, r.stream>>>(csr->row_ptr, csr->col_idx, wl,

@@ -9,14 +9,13 @@
 
 namespace sgr {
 
-struct RoundArgs;
 struct Ctrl;
 
 struct Resolved {
   int tiebreak;
   int32_t max_rounds;
   int loop_mode;
-  int block;
+  int color_bits;
   int small_max;
   int med_max;
   cudaStream_t stream;
@@ -26,16 +25,15 @@ struct Resolved {
   int validate;
   int batch;
   int profile;
+  float* round_ms;
 };
 
 void set_error(const char* fmt, ...);
 sgr_status cuda_fail(cudaError_t e, const char* what, int line);
 int num_sms();
 Resolved resolve_opts(const sgr_opts* o, int64_t n);
-size_t ws_bytes(int64_t n);
-void launch_first(const RoundArgs& a, int tiebreak, bool sorted, int grid, cudaStream_t s);
-void launch_round_pass(const RoundArgs& a, int tiebreak, int64_t n, const Resolved& r,
-                       cudaStream_t s);
+size_t ws_bytes(int64_t n, int64_t nnz, const Resolved& r);
+int first_grid(int64_t n);
 void fill_stats(const Ctrl& c, int64_t n, int64_t nnz, sgr_stats* st);
 
 }  // namespace sgr

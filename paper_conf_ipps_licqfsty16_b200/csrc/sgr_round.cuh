@@ -1,0 +1,694 @@
+// sgr_round.cuh — sm_100a kernels of the deterministic SGR round.
+//
+// One fused pass F_k per round k >= 2 computes, for every v in W_k (Alg. 5):
+//   conflict(v) = exists w in adj(v): X[w] == X[v] and lose(v, w)     (Alg. 5 l.12-15)
+//   tent(v)     = min{c > 0 : c not in {X[w] : w in adj(v)}}            (Alg. 5 l.4-8)
+//   Y[v]        = conflict(v) ? tent(v) : X[v];  v joins W_{k+1} iff conflict(v)
+// X = C_k is round k's color snapshot and Y the ping-pong buffer: it holds C_{k-1}, which
+// differs from C_{k+1} only inside W_k, exactly the set the pass writes (DESIGN.md §3,
+// proof (iv)). Detection of round k and assignment of round k+1 read the same snapshot, so
+// one adjacency scan serves both. F_1 needs no color gathers (every color is 1).
+//
+// The pass is bound by the rate of scattered color gathers (one L1TEX wavefront per
+// distinct 128-byte line, ~1 line / SM-cycle measured by tools/gather_bench.cu) and by
+// load latency, so every work item issues ALL its loads up front: the CSR entries, then
+// all color gathers, then the mask / conflict arithmetic. Work binning is static (degrees
+// never change and W only shrinks):
+//   bin 0  deg <= small_max (<= 62): 8 lanes per vertex (coalesced row reads), up to 8
+//          entries per lane, forbidden set in a u64 register per lane, OR-reduced in-group
+//   bin 1  deg <= med_max (<= 256):  8 lanes per vertex, up to 32 entries per lane,
+//          512-byte forbidden table (one byte per color) in shared memory
+//   bin 2  larger: one warp per CHUNK of `chunk` CSR entries on a grid aligned to
+//          `chunk` (16-byte vector loads), 1024-byte table; a vertex with several chunks
+//          merges the chunks' 1024-bit partial sets with atomicOr and the last chunk to
+//          finish (atomic ticket) decides conflict and tent. No row is ever scanned
+//          serially by one worker, so a round's critical path is one chunk.
+// Colors are stored as C = uint16_t (default; half the gather footprint, more lines shared
+// by sorted neighbours) or int32_t; a tent above 65535 sets an overflow flag and the host
+// reruns the coloring with 32-bit colors, so the result is identical either way.
+// Worklist pushes: warp ballot + popc + one atomicAdd per warp.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "sgr_common.cuh"
+
+namespace sgr {
+
+constexpr int kBins = 3;
+constexpr int kBlock = 256;             // threads per block (8 warps)
+constexpr int kGroup = 8;               // lanes per vertex in bins 0 and 1
+constexpr int kK0 = 8;                  // entries per lane, bin 0 (8 x 8 = 64 >= 62)
+constexpr int kK1 = 32;                 // entries per lane, bin 1 (8 x 32 = 256)
+constexpr int kMaxMed = kGroup * kK1;   // 256
+constexpr int kMedTbl = 512;            // bin-1 table bytes (colors < 512 > 257)
+constexpr int kBigTbl = 1024;           // bin-2 table bytes (colors < 1024)
+constexpr int kWarpTbl = 2048;          // per-warp smem: 4 x 512 (bin 1) or 1 x 1024 (bin 2)
+constexpr int kChunk = 1020;            // bin-2 chunk: entries per warp item, chosen so the
+                                        // 16-byte-aligned window (1024 = 32 lanes x 8 int4)
+                                        // always covers the chunk
+
+// Device-resident loop state (in the workspace).
+struct Ctrl {
+  int32_t k;                 // index of the next fused pass F_k (k = 2 after F_1)
+  int32_t active;            // 1 while W_k is non-empty
+  int32_t status;            // 0 ok, 1 = max_rounds reached with W non-empty
+  int32_t max_rounds;
+  int32_t cnt[2][kBins];     // work items per parity (k & 1) and bin
+  int32_t vcnt2[2];          // bin-2 worklist VERTICES per parity (items are chunks)
+  int32_t overflow;          // a first fit exceeded the color type (u16 -> rerun in i32)
+  int32_t round_cap;
+  uint32_t bar_count;        // grid barrier (persistent kernel)
+  uint32_t bar_gen;
+  int32_t big_count;         // slots handed to multi-chunk vertices by F_1
+  int32_t max_color;
+  int32_t violations;
+  int32_t pad[3];
+  unsigned long long edges_acc[kBins];
+  unsigned long long verts_total[kBins + 1];   // [kBins] = F_1
+  unsigned long long edges_total[kBins + 1];
+  unsigned long long pushes_total[kBins + 1];
+  unsigned long long items_total;
+  int32_t* round_sizes;
+  int64_t* round_edges;
+};
+
+template <class C>
+struct RoundArgs {
+  const int64_t* row_ptr;
+  const int32_t* col_idx;
+  C* col[2];                  // color ping-pong: C_k lives in col[(k - 1) & 1]
+  int32_t* wl_t[2];           // bin 0 vertex lists, W_k in [k & 1]
+  int32_t* wl_m[2];           // bin 1 vertex lists
+  int64_t* wl_c[2];           // bin 2 chunk items: (v << 32) | chunk
+  int32_t* big_id;            // slot of each multi-chunk vertex (F_1)
+  uint32_t* acc_bits;         // [slot][32] partial forbidden sets
+  unsigned long long* acc_cnt;  // [slot] chunks finished | conflicts << 32
+  Ctrl* ctrl;
+  int64_t nnz;
+  int32_t n;
+  int32_t small_max;
+  int32_t med_max;
+  int32_t pad;
+};
+
+// Parameter-struct selects without dynamic indexing (which would spill it to the stack).
+template <class T>
+__device__ __forceinline__ T sel(int par, T a0, T a1) { return par ? a1 : a0; }
+
+__device__ __forceinline__ int32_t ld_cg(const int32_t* p) { return __ldcg(p); }
+__device__ __forceinline__ uint32_t ld_cg(const uint32_t* p) { return __ldcg(p); }
+
+template <bool Persist, class C>
+__device__ __forceinline__ int32_t ldc(const C* p) {
+  if constexpr (Persist) return (int32_t)__ldcg(p);
+  else return (int32_t)__ldg(p);
+}
+
+template <class C>
+__device__ __forceinline__ C store_color(int32_t c, Ctrl* ctrl) {
+  if constexpr (sizeof(C) == 2) {
+    if (c > 65535) {
+      ctrl->overflow = 1;
+      return (C)65535;
+    }
+  }
+  return (C)c;
+}
+
+__device__ __forceinline__ int bin_of(int64_t d, int small_max, int med_max) {
+  return d <= small_max ? 0 : (d <= med_max ? 1 : 2);
+}
+
+// Chunks of a bin-2 row [s, e): [s + c * kChunk, s + (c + 1) * kChunk), c < ceil(deg / kChunk).
+__device__ __forceinline__ int32_t num_chunks(int64_t s, int64_t e) {
+  return (int32_t)((e - s + kChunk - 1) / kChunk);
+}
+
+__device__ __forceinline__ void prefetch_l2(const void* p) {
+  asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
+}
+
+// Release / acquire fences at GPU scope (lighter than the sequentially consistent
+// fence.sc.gpu that __threadfence() emits).
+__device__ __forceinline__ void fence_acq_rel_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+
+__device__ __forceinline__ int64_t make_item(int32_t v, int32_t c) {
+  return (int64_t)(((uint64_t)(uint32_t)v << 32) | (uint32_t)c);
+}
+
+// ---------------------------------------------------------------------------------------
+// F_1: round-1 detection + round-2 assignment without color gathers. After round 1 every
+// color is 1 (first fit against an all-zero snapshot), so with rows sorted ascending
+//   LOWID: conflict(v) <=> first entry < v ;  PAPER: conflict(v) <=> last entry > v
+// (a self-loop can never satisfy the strict inequality); tent(v) = mex({1}) = 2.
+// Writes col[0] = C_1 (all 1), col[1] = C_2, and W_2 into the bins' lists [0].
+template <int TB, class C>
+__global__ void __launch_bounds__(256) k_first(RoundArgs<C> a, int sorted) {
+  Ctrl* ctrl = a.ctrl;
+  C* __restrict__ X = a.col[0];
+  C* __restrict__ Y = a.col[1];
+  const int lane = threadIdx.x & 31;
+  const int64_t n = a.n;
+  for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < n;
+       base += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t vi = base + threadIdx.x;
+    bool conflict = false;
+    int64_t s = 0, e = 0;
+    const int32_t v = (int32_t)vi;
+    if (vi < n) {
+      s = ldg_i64(a.row_ptr + v);
+      e = ldg_i64(a.row_ptr + v + 1);
+      if (e > s) {
+        if (sorted) {
+          if constexpr (TB == 1) conflict = ldg_i32(a.col_idx + e - 1) > v;
+          else conflict = ldg_i32(a.col_idx + s) < v;
+        } else {
+          for (int64_t j = s; j < e && !conflict; ++j) conflict = lose<TB>(v, ldg_i32(a.col_idx + j));
+        }
+      }
+      X[v] = (C)1;
+      Y[v] = (C)(conflict ? 2 : 1);
+    }
+    const int b = bin_of(e - s, a.small_max, a.med_max);
+    warp_push(conflict && b == 0, v, a.wl_t[0], &ctrl->cnt[0][0]);
+    warp_push(conflict && b == 1, v, a.wl_m[0], &ctrl->cnt[0][1]);
+    // bin 2: one item per aligned chunk; multi-chunk vertices get an accumulator slot
+    const bool big = conflict && b == 2;
+    const int32_t nch = big ? num_chunks(s, e) : 0;
+    const unsigned mb = __ballot_sync(0xffffffffu, big);
+    if (mb) {
+      const unsigned mm = __ballot_sync(0xffffffffu, nch > 1);
+      if (mm) {
+        int sb = 0;
+        if (lane == __ffs(mm) - 1) sb = atomicAdd(&ctrl->big_count, __popc(mm));
+        sb = __shfl_sync(0xffffffffu, sb, __ffs(mm) - 1);
+        if (nch > 1) a.big_id[v] = sb + __popc(mm & ((1u << lane) - 1u));
+      }
+      int incl = nch;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int t = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += t;
+      }
+      const int total = __shfl_sync(0xffffffffu, incl, 31);
+      int ib = 0;
+      if (lane == 0) {
+        ib = atomicAdd(&ctrl->cnt[0][2], total);
+        atomicAdd(&ctrl->vcnt2[0], __popc(mb));
+      }
+      ib = __shfl_sync(0xffffffffu, ib, 0) + incl - nch;
+      for (int32_t t = 0; t < nch; ++t) a.wl_c[0][ib + t] = make_item(v, t);
+    }
+  }
+}
+
+// ---------------------------------------------------------------------------------------
+// Forbidden-table helpers (bytes in shared memory, one per color).
+
+// First free color >= 1 of a warp-owned table of N bytes (N multiple of 128); -1 if full.
+template <int N>
+__device__ __forceinline__ int32_t tbl_first_free_warp(const uint8_t* tbl, int lane) {
+  const uint32_t* t32 = reinterpret_cast<const uint32_t*>(tbl);
+#pragma unroll 1
+  for (int it = 0; it < N / 128; ++it) {
+    uint32_t word = t32[it * 32 + lane];
+    if (it == 0 && lane == 0) word |= 0xffu;  // color 0 is never a candidate
+    const uint32_t z = __vcmpeq4(word, 0u);
+    const unsigned b = __ballot_sync(0xffffffffu, z != 0u);
+    if (b) {
+      const int fl = __ffs(b) - 1;
+      const uint32_t zz = __shfl_sync(0xffffffffu, z, fl);
+      return (it * 32 + fl) * 4 + (__ffs(zz) - 1) / 8;
+    }
+  }
+  return -1;
+}
+
+// 32 bits = nonzero-ness of bytes [32 * lane, 32 * lane + 32) of a 1024-byte table.
+__device__ __forceinline__ uint32_t tbl_bits32(const uint8_t* tbl, int lane) {
+  const uint4* t = reinterpret_cast<const uint4*>(tbl) + lane * 2;
+  const uint4 a = t[0], b = t[1];
+  const uint32_t w[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
+  uint32_t bits = 0;
+#pragma unroll
+  for (int q = 0; q < 8; ++q) {
+    const uint32_t z = __vcmpne4(w[q], 0u);  // 0xff per nonzero byte
+    const uint32_t nib = ((z >> 7) & 1u) | ((z >> 14) & 2u) | ((z >> 21) & 4u) | ((z >> 28) & 8u);
+    bits |= nib << (4 * q);
+  }
+  return bits;
+}
+
+// Exact warp first fit from `base` (all colors in [1, base) forbidden) — rare fallback.
+template <bool Persist, class C>
+__device__ __noinline__ int32_t warp_first_fit_rescan(const int32_t* __restrict__ col_idx,
+                                                      const C* X, int64_t s, int64_t e,
+                                                      int32_t base, int lane) {
+  for (;;) {
+    uint64_t m0 = 0, m1 = 0, m2 = 0, m3 = 0;
+    if (base == 0) m0 = 1;
+    for (int64_t j = s + lane; j < e; j += 32) {
+      const uint32_t idx = (uint32_t)(ldc<Persist>(X + __ldg(col_idx + j)) - base);
+      if (idx < 256u) {
+        const uint64_t bit = 1ull << (idx & 63);
+        const uint32_t q = idx >> 6;
+        m0 |= q == 0 ? bit : 0ull;
+        m1 |= q == 1 ? bit : 0ull;
+        m2 |= q == 2 ? bit : 0ull;
+        m3 |= q == 3 ? bit : 0ull;
+      }
+    }
+    m0 = warp_or64(m0);
+    m1 = warp_or64(m1);
+    m2 = warp_or64(m2);
+    m3 = warp_or64(m3);
+    if (~m0) return base + __ffsll((long long)~m0) - 1;
+    if (~m1) return base + 64 + __ffsll((long long)~m1) - 1;
+    if (~m2) return base + 128 + __ffsll((long long)~m2) - 1;
+    if (~m3) return base + 192 + __ffsll((long long)~m3) - 1;
+    base += 256;
+  }
+}
+
+// ---------------------------------------------------------------------------------------
+// Bin 2: one warp processes one chunk item [cs, ce) of row [s, e). Entries are read as int4
+// from the 16-byte-aligned window starting at cs rounded down to a multiple of 4 (1024
+// entries >= kChunk + 3); positions outside [cs, ce) are masked.
+template <int TB, bool Persist, class C>
+__device__ __forceinline__ void process_chunk(const RoundArgs<C>& a, int32_t v, int32_t c,
+                                              int64_t s, int64_t e, const C* X, C* Y,
+                                              int64_t* out, int32_t* out_cnt,
+                                              int32_t* out_vcnt, uint8_t* tbl, int lane,
+                                              unsigned long long& edges) {
+  const int64_t cs = s + (int64_t)c * kChunk, ce = min(e, cs + kChunk);
+  const int64_t wbase = cs & ~(int64_t)3;  // 16-byte aligned window start
+  const int32_t nch = num_chunks(s, e);
+  const int4* col4 = reinterpret_cast<const int4*>(a.col_idx + wbase);
+  int32_t w[32];
+#pragma unroll
+  for (int q = 0; q < 8; ++q) {
+    const int64_t p0 = wbase + 4 * (lane + 32 * q);
+    int4 t = make_int4(-1, -1, -1, -1);
+    if (p0 + 3 >= cs && p0 < ce) {
+      if (p0 + 4 <= a.nnz) {
+        t = __ldg(col4 + lane + 32 * q);
+      } else {  // the array's last, partial 16-byte group: never read past nnz
+        t.x = __ldg(a.col_idx + p0);
+        if (p0 + 1 < a.nnz) t.y = __ldg(a.col_idx + p0 + 1);
+        if (p0 + 2 < a.nnz) t.z = __ldg(a.col_idx + p0 + 2);
+      }
+    }
+    w[4 * q + 0] = (p0 + 0 >= cs && p0 + 0 < ce) ? t.x : -1;
+    w[4 * q + 1] = (p0 + 1 >= cs && p0 + 1 < ce) ? t.y : -1;
+    w[4 * q + 2] = (p0 + 2 >= cs && p0 + 2 < ce) ? t.z : -1;
+    w[4 * q + 3] = (p0 + 3 >= cs && p0 + 3 < ce) ? t.w : -1;
+  }
+  const int32_t xv = ldc<Persist>(X + v);
+  uint32_t lb = 0;  // lose(v, w) bits
+#pragma unroll
+  for (int u = 0; u < 32; ++u) lb |= (w[u] >= 0 && lose<TB>(v, w[u])) ? (1u << u) : 0u;
+#pragma unroll
+  for (int u = 0; u < 32; ++u) w[u] = (w[u] >= 0) ? ldc<Persist>(X + w[u]) : 0;  // now colors
+  bool conf = false;
+#pragma unroll
+  for (int u = 0; u < 32; ++u) {
+    if ((uint32_t)w[u] < (uint32_t)kBigTbl) tbl[w[u]] = 1;
+    conf |= (w[u] == xv) & ((lb >> u) & 1u);
+  }
+  if (lane == 0) edges += (unsigned long long)(ce - cs);
+  __syncwarp();
+  const bool any = __any_sync(0xffffffffu, conf);
+  if (nch == 1) {
+    int32_t tent = 0;
+    if (any) {
+      tent = tbl_first_free_warp<kBigTbl>(tbl, lane);
+      if (tent < 0) tent = warp_first_fit_rescan<Persist>(a.col_idx, X, s, e, kBigTbl, lane);
+    }
+    if (lane == 0) {
+      Y[v] = any ? store_color<C>(tent, a.ctrl) : (C)xv;
+      if (any) {
+        out[atomicAdd(out_cnt, 1)] = make_item(v, 0);
+        atomicAdd(out_vcnt, 1);
+      }
+    }
+  } else {
+    const int32_t slot = __ldg(a.big_id + v);
+    uint32_t* accb = a.acc_bits + (int64_t)slot * 32;
+    const uint32_t bits = tbl_bits32(tbl, lane);
+    if (bits) atomicOr(accb + lane, bits);
+    __syncwarp();  // orders every lane's atomicOr before lane 0's release below
+    unsigned long long old = 0;
+    if (lane == 0) {
+      fence_acq_rel_gpu();  // release: every lane's partial set before the ticket
+      old = atomicAdd(a.acc_cnt + slot, 1ull | ((unsigned long long)any << 32));
+    }
+    old = __shfl_sync(0xffffffffu, old, 0);
+    if ((uint32_t)old == (uint32_t)(nch - 1)) {  // this warp finished the vertex's last chunk
+      fence_acq_rel_gpu();  // acquire: the other chunks' partial sets
+      uint32_t word = ld_cg(accb + lane);
+      accb[lane] = 0u;
+      if (lane == 0) a.acc_cnt[slot] = 0ull;
+      const bool conf_all = ((old >> 32) + (any ? 1ull : 0ull)) != 0ull;
+      int32_t tent = 0;
+      if (conf_all) {
+        if (lane == 0) word |= 1u;  // color 0
+        const unsigned fb = __ballot_sync(0xffffffffu, word != 0xffffffffu);
+        if (fb) {
+          const int fl = __ffs(fb) - 1;
+          const uint32_t w2 = __shfl_sync(0xffffffffu, word, fl);
+          tent = fl * 32 + __ffs(~w2) - 1;
+        } else {
+          tent = warp_first_fit_rescan<Persist>(a.col_idx, X, s, e, kBigTbl, lane);
+        }
+      }
+      int32_t ob = 0;
+      if (lane == 0) {
+        Y[v] = conf_all ? store_color<C>(tent, a.ctrl) : (C)xv;
+        if (conf_all) {
+          ob = atomicAdd(out_cnt, nch);
+          atomicAdd(out_vcnt, 1);
+        }
+      }
+      if (conf_all) {
+        ob = __shfl_sync(0xffffffffu, ob, 0);
+        for (int32_t t = lane; t < nch; t += 32) out[ob + t] = make_item(v, t);
+      }
+    }
+  }
+  // clear the table for the next item (32 bytes per lane)
+  uint4* t4 = reinterpret_cast<uint4*>(tbl) + lane * 2;
+  t4[0] = make_uint4(0, 0, 0, 0);
+  t4[1] = make_uint4(0, 0, 0, 0);
+  __syncwarp();
+}
+
+// Bins 0 and 1: each 8-lane group of the warp processes one vertex (v < 0: idle group).
+// All loads of the row are issued up front (K per lane, group lanes interleaved so a
+// group's reads of a row are contiguous), then all color gathers.
+template <int TB, bool Persist, class C, int K, bool Table>
+__device__ __forceinline__ void process_group(const RoundArgs<C>& a, int32_t v, int64_t s,
+                                              int64_t e, const C* X, C* Y, uint8_t* gtbl,
+                                              int gl, unsigned gmask, bool& push,
+                                              unsigned long long& edges) {
+  int32_t w[K];
+#pragma unroll
+  for (int u = 0; u < K; ++u) {
+    const int64_t j = s + gl + kGroup * u;
+    w[u] = (v >= 0 && j < e) ? __ldg(a.col_idx + j) : -1;
+  }
+  const int32_t xv = v >= 0 ? ldc<Persist>(X + v) : 0;
+  uint32_t lb = 0;
+#pragma unroll
+  for (int u = 0; u < K; ++u) lb |= (w[u] >= 0 && lose<TB>(v, w[u])) ? (1u << u) : 0u;
+#pragma unroll
+  for (int u = 0; u < K; ++u) w[u] = (w[u] >= 0) ? ldc<Persist>(X + w[u]) : 0;  // colors
+  bool conf = false;
+  uint64_t mask = 1ull;  // bit 0 = color 0, never a candidate
+#pragma unroll
+  for (int u = 0; u < K; ++u) {
+    if constexpr (Table) {
+      if ((uint32_t)w[u] < (uint32_t)kMedTbl) gtbl[w[u]] = 1;
+    } else {
+      mask |= ((uint32_t)w[u] < 64u) ? (1ull << w[u]) : 0ull;
+    }
+    conf |= (w[u] == xv) & ((lb >> u) & 1u);
+  }
+  if (v >= 0 && gl == 0) edges += (unsigned long long)(e - s);
+  const bool any = (__ballot_sync(0xffffffffu, conf) & gmask) != 0u;
+  int32_t tent = 0;
+  if constexpr (Table) {
+    __syncwarp();
+    if (v >= 0 && any) {  // the group scans its table 32 bytes (8 words) per step
+      const uint32_t* t32 = reinterpret_cast<const uint32_t*>(gtbl);
+      for (int it = 0; it < kMedTbl / 32; ++it) {
+        uint32_t word = t32[it * 8 + gl];
+        if (it == 0 && gl == 0) word |= 0xffu;
+        const uint32_t z = __vcmpeq4(word, 0u);
+        const unsigned b = __ballot_sync(gmask, z != 0u) & gmask;
+        if (b) {
+          const int fl = __ffs(b) - 1;  // absolute lane
+          const uint32_t zz = __shfl_sync(gmask, z, fl);
+          tent = (it * 8 + (fl & 7)) * 4 + (__ffs(zz) - 1) / 8;
+          break;
+        }
+      }
+      // deg <= 256 => first fit <= 257 < kMedTbl: the table always has a free slot
+    }
+    // clear the group's table (64 bytes per lane)
+    uint4* t4 = reinterpret_cast<uint4*>(gtbl) + gl * 4;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) t4[q] = make_uint4(0, 0, 0, 0);
+    __syncwarp();
+  } else {
+#pragma unroll
+    for (int o = 4; o > 0; o >>= 1) mask |= __shfl_xor_sync(0xffffffffu, mask, o);
+    tent = __ffsll((long long)~mask) - 1;  // deg <= 62 => first fit <= 63
+  }
+  if (v >= 0 && gl == 0) Y[v] = any ? store_color<C>(tent, a.ctrl) : (C)xv;
+  push = (v >= 0) && any && gl == 0;
+}
+
+// One fused pass F_k over all three bins; every warp of the grid calls it. Static
+// round-robin assignment (warp w takes items w, w + NW, ...), with the next item's list
+// entry and row offsets prefetched while the current one is processed.
+template <int TB, bool Persist, class C>
+__device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, uint8_t* wtbl,
+                                           unsigned long long (&edges)[kBins]) {
+  Ctrl* ctrl = a.ctrl;
+  const int p = k & 1;
+  const int lane = threadIdx.x & 31;
+  const int gw = (int)((blockIdx.x * blockDim.x + threadIdx.x) >> 5);
+  const int NW = (int)((gridDim.x * blockDim.x) >> 5);
+  const C* X = sel((k - 1) & 1, (const C*)a.col[0], (const C*)a.col[1]);
+  C* Y = sel(k & 1, a.col[0], a.col[1]);
+  // ---- bin 2: chunk items, one per warp
+  {
+    const int nC = ld_cg(&ctrl->cnt[p][2]);
+    const int64_t* items = sel(p, (const int64_t*)a.wl_c[0], (const int64_t*)a.wl_c[1]);
+    int64_t* out = sel(p ^ 1, a.wl_c[0], a.wl_c[1]);
+    int i = gw;
+    int64_t it = i < nC ? __ldcg(items + i) : 0;
+    int32_t v = (int32_t)((uint64_t)it >> 32);
+    int64_t s = i < nC ? ldg_i64(a.row_ptr + v) : 0, e = i < nC ? ldg_i64(a.row_ptr + v + 1) : 0;
+    while (i < nC) {
+      const int in = i + NW;
+      const int64_t itn = in < nC ? __ldcg(items + in) : 0;
+      const int32_t vn = (int32_t)((uint64_t)itn >> 32);
+      const int64_t sn = in < nC ? ldg_i64(a.row_ptr + vn) : 0;
+      const int64_t en = in < nC ? ldg_i64(a.row_ptr + vn + 1) : 0;
+      if (in < nC) {  // warm L2 with the next item's 4 KB window (one 128-byte line per lane)
+        const int64_t csn = sn + (int64_t)(int32_t)(uint32_t)itn * kChunk;
+        const int64_t ln = (csn & ~(int64_t)3) + 32 * lane;
+        if (ln < en) prefetch_l2(a.col_idx + ln);
+      }
+      process_chunk<TB, Persist, C>(a, v, (int32_t)(uint32_t)it, s, e, X, Y, out,
+                                    &ctrl->cnt[p ^ 1][2], &ctrl->vcnt2[p ^ 1], wtbl, lane,
+                                    edges[2]);
+      i = in;
+      it = itn;
+      v = vn;
+      s = sn;
+      e = en;
+    }
+  }
+  const int g = lane >> 3, gl = lane & 7;
+  const unsigned gmask = 0xffu << (g * 8);
+  // ---- bin 1: four vertices per warp (one per 8-lane group), 512-byte tables
+  {
+    const int nM = ld_cg(&ctrl->cnt[p][1]);
+    const int32_t* list = sel(p, (const int32_t*)a.wl_m[0], (const int32_t*)a.wl_m[1]);
+    int32_t* out = sel(p ^ 1, a.wl_m[0], a.wl_m[1]);
+    int i = gw * 4 + g;
+    int32_t v = i < nM ? ld_cg(list + i) : -1;
+    int64_t s = v >= 0 ? ldg_i64(a.row_ptr + v) : 0, e = v >= 0 ? ldg_i64(a.row_ptr + v + 1) : 0;
+    for (int base = gw * 4; base < nM; base += NW * 4) {
+      const int in = i + NW * 4;
+      const int32_t vn = in < nM ? ld_cg(list + in) : -1;
+      const int64_t sn = vn >= 0 ? ldg_i64(a.row_ptr + vn) : 0;
+      const int64_t en = vn >= 0 ? ldg_i64(a.row_ptr + vn + 1) : 0;
+      if (sn + 32 * gl < en) prefetch_l2(a.col_idx + sn + 32 * gl);  // next row, 1 line / lane
+      bool push = false;
+      process_group<TB, Persist, C, kK1, true>(a, v, s, e, X, Y, wtbl + g * kMedTbl, gl, gmask,
+                                               push, edges[1]);
+      warp_push(push, v, out, &ctrl->cnt[p ^ 1][1]);
+      i = in;
+      v = vn;
+      s = sn;
+      e = en;
+    }
+  }
+  // ---- bin 0: four vertices per warp, register masks
+  {
+    const int nT = ld_cg(&ctrl->cnt[p][0]);
+    const int32_t* list = sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]);
+    int32_t* out = sel(p ^ 1, a.wl_t[0], a.wl_t[1]);
+    int i = gw * 4 + g;
+    int32_t v = i < nT ? ld_cg(list + i) : -1;
+    int64_t s = v >= 0 ? ldg_i64(a.row_ptr + v) : 0, e = v >= 0 ? ldg_i64(a.row_ptr + v + 1) : 0;
+    for (int base = gw * 4; base < nT; base += NW * 4) {
+      const int in = i + NW * 4;
+      const int32_t vn = in < nT ? ld_cg(list + in) : -1;
+      const int64_t sn = vn >= 0 ? ldg_i64(a.row_ptr + vn) : 0;
+      const int64_t en = vn >= 0 ? ldg_i64(a.row_ptr + vn + 1) : 0;
+      bool push = false;
+      process_group<TB, Persist, C, kK0, false>(a, v, s, e, X, Y, nullptr, gl, gmask, push,
+                                                edges[0]);
+      warp_push(push, v, out, &ctrl->cnt[p ^ 1][0]);
+      i = in;
+      v = vn;
+      s = sn;
+      e = en;
+    }
+  }
+}
+
+// Block reduction of the three per-thread edge counters, one atomicAdd each per block.
+__device__ __forceinline__ void block_add3(unsigned long long (&x)[kBins], Ctrl* ctrl) {
+  __shared__ unsigned long long red[kBins][kBlock / 32];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+#pragma unroll
+  for (int q = 0; q < kBins; ++q) {
+    unsigned long long y = x[q];
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) y += __shfl_xor_sync(0xffffffffu, y, o);
+    if (lane == 0) red[q][wid] = y;
+  }
+  __syncthreads();
+  if (wid == 0) {
+#pragma unroll
+    for (int q = 0; q < kBins; ++q) {
+      unsigned long long y = lane < (kBlock / 32) ? red[q][lane] : 0ull;
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) y += __shfl_xor_sync(0xffffffffu, y, o);
+      if (lane == 0 && y) atomicAdd(&ctrl->edges_acc[q], y);
+    }
+  }
+}
+
+// End of pass F_k (one thread, after every block of the pass is done): fold the pass's
+// counters into totals and the trace, consume W_k, advance k and decide whether W_{k+1}
+// is non-empty. A pass over an empty W_k changes nothing, so any surplus pass a host loop
+// issues before it sees `active == 0` is a no-op.
+__device__ __forceinline__ void advance_body(Ctrl* ctrl, bool first) {
+  volatile Ctrl* c = ctrl;
+  if (first) {  // after F_1: W_2 is in parity 0
+    int tot = 0;
+    for (int q = 0; q < kBins; ++q) tot += c->cnt[0][q];
+    c->pushes_total[kBins] = (unsigned long long)(c->cnt[0][0] + c->cnt[0][1] + c->vcnt2[0]);
+    c->k = 2;
+    c->active = tot > 0;
+    if (c->active && c->max_rounds < 2) {
+      c->status = 1;
+      c->active = 0;
+      for (int q = 0; q < kBins; ++q) c->cnt[0][q] = 0;
+    }
+    return;
+  }
+  const int k = c->k;
+  const int p = k & 1;
+  const int items_in = c->cnt[p][0] + c->cnt[p][1] + c->cnt[p][2];
+  if (items_in == 0) {
+    c->active = 0;
+    return;
+  }
+  const int vin[kBins] = {c->cnt[p][0], c->cnt[p][1], c->vcnt2[p]};
+  const int vout[kBins] = {c->cnt[p ^ 1][0], c->cnt[p ^ 1][1], c->vcnt2[p ^ 1]};
+  unsigned long long e_all = 0;
+  int tot_in = 0;
+  for (int q = 0; q < kBins; ++q) {
+    c->verts_total[q] += (unsigned long long)vin[q];
+    c->edges_total[q] += c->edges_acc[q];
+    c->pushes_total[q] += (unsigned long long)vout[q];
+    e_all += c->edges_acc[q];
+    c->edges_acc[q] = 0;
+    tot_in += vin[q];
+  }
+  c->items_total += (unsigned long long)c->cnt[p][2];
+  for (int q = 0; q < kBins; ++q) c->cnt[p][q] = 0;
+  c->vcnt2[p] = 0;
+  if (k - 1 < c->round_cap) {
+    if (c->round_sizes) c->round_sizes[k - 1] = tot_in;
+    if (c->round_edges) c->round_edges[k - 1] = (int64_t)e_all;
+  }
+  c->k = k + 1;
+  const int items_out = c->cnt[p ^ 1][0] + c->cnt[p ^ 1][1] + c->cnt[p ^ 1][2];
+  c->active = items_out > 0;
+  if (c->active && k + 1 > c->max_rounds) {  // W_{k+1} non-empty beyond the cap
+    c->status = 1;
+    c->active = 0;
+    for (int q = 0; q < kBins; ++q) c->cnt[p ^ 1][q] = 0;
+    c->vcnt2[p ^ 1] = 0;
+  }
+}
+
+__global__ void k_advance(Ctrl* ctrl, int first) {
+  if (threadIdx.x == 0 && blockIdx.x == 0) advance_body(ctrl, first != 0);
+}
+
+__device__ __forceinline__ void zero_smem(uint8_t* p, int bytes) {
+  uint4* q = reinterpret_cast<uint4*>(p);
+  for (int i = threadIdx.x; i < bytes / 16; i += blockDim.x) q[i] = make_uint4(0, 0, 0, 0);
+}
+
+// One pass per launch (host / graph loop modes); k_advance follows it on the stream.
+template <int TB, class C>
+__global__ void __launch_bounds__(kBlock, 3) k_round(RoundArgs<C> a) {
+  __shared__ __align__(16) uint8_t tbl[kBlock / 32][kWarpTbl];
+  Ctrl* ctrl = a.ctrl;
+  if (!ctrl->active) return;  // uniform across the grid
+  zero_smem(&tbl[0][0], sizeof(tbl));
+  __syncthreads();
+  unsigned long long edges[kBins] = {0, 0, 0};
+  round_body<TB, false, C>(a, ctrl->k, tbl[threadIdx.x >> 5], edges);
+  block_add3(edges, ctrl);
+}
+
+// Grid-wide barrier whose last arriving block runs advance_body (persistent kernel).
+__device__ __forceinline__ void grid_sync_advance(Ctrl* ctrl) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    volatile uint32_t* gen_p = &ctrl->bar_gen;
+    const uint32_t gen = *gen_p;
+    __threadfence();
+    const uint32_t arrived = atomicAdd(&ctrl->bar_count, 1u);
+    if (arrived == gridDim.x - 1) {
+      __threadfence();
+      advance_body(ctrl, false);
+      *(volatile uint32_t*)&ctrl->bar_count = 0u;
+      __threadfence();
+      atomicAdd(&ctrl->bar_gen, 1u);
+    } else {
+      while (*gen_p == gen) __nanosleep(32);
+    }
+    __threadfence();
+  }
+  __syncthreads();
+}
+
+// All rounds in one cooperative launch (every block resident): pass, barrier+advance, ...
+template <int TB, class C>
+__global__ void __launch_bounds__(kBlock, 3) k_persistent(RoundArgs<C> a) {
+  __shared__ __align__(16) uint8_t tbl[kBlock / 32][kWarpTbl];
+  Ctrl* ctrl = a.ctrl;
+  zero_smem(&tbl[0][0], sizeof(tbl));
+  __syncthreads();
+  for (;;) {
+    const int active = ld_cg(&ctrl->active);
+    const int k = ld_cg(&ctrl->k);
+    if (!active) break;  // uniform: read after the barrier by every thread
+    unsigned long long edges[kBins] = {0, 0, 0};
+    round_body<TB, true, C>(a, k, tbl[threadIdx.x >> 5], edges);
+    block_add3(edges, ctrl);
+    grid_sync_advance(ctrl);
+  }
+}
+
+// Widen the final u16 colors into the caller's int32 output.
+__global__ void k_widen(const uint16_t* __restrict__ src, int32_t* __restrict__ dst, int64_t n) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x)
+    dst[i] = (int32_t)src[i];
+}
+
+}  // namespace sgr

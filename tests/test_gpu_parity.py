@@ -81,10 +81,11 @@ def test_generator_families(maker, tb):
 
 def degree_boundary_graph():
     """Stars whose centres have degrees at every bin boundary, plus cliques K_70 / K_300
-    (first-fit values above 64 and 256: window slides in the warp and CTA bins)."""
+    (first fits above 64 and 256; K_300 rows straddle 1024-aligned chunk boundaries)."""
     edges = []
     n = 0
-    for d in [0, 1, 2, 31, 32, 33, 61, 62, 63, 64, 65, 2047, 2048, 2049, 4095, 4096, 4097, 9000]:
+    for d in [0, 1, 2, 31, 32, 33, 61, 62, 63, 64, 65, 255, 256, 257, 1019, 1020, 1021, 2040,
+              2041, 2047, 2048, 2049, 4095, 4096, 4097, 9000]:
         c = n
         edges += [(c, c + 1 + i) for i in range(d)]
         n += d + 1
@@ -98,15 +99,18 @@ def degree_boundary_graph():
 
 
 @pytest.mark.parametrize("tb", [LOW, PAP])
-@pytest.mark.parametrize("bins", [(0, 0), (62, 62), (1, 1), (8, 64), (32, 2048), (62, 100000)])
-def test_degree_bins_and_windows(tb, bins):
-    check_full(degree_boundary_graph(), tb, bin_small_max=bins[0], bin_med_max=bins[1])
+@pytest.mark.parametrize("bins", [(0, 0), (62, 62), (1, 1), (8, 64), (32, 256), (62, 256), (1, 2)])
+@pytest.mark.parametrize("mode", ["persistent", "host"])
+@pytest.mark.parametrize("bits", [16, 32])
+def test_degree_bins_and_windows(tb, bins, mode, bits):
+    check_full(degree_boundary_graph(), tb, bin_small_max=bins[0], bin_med_max=bins[1],
+               loop_mode=mode, color_bits=bits)
 
 
 @pytest.mark.parametrize("k", [64, 257, 520])
 def test_complete_graphs_large_mex(k):
     g = gen.from_edges(k, [(i, j) for i in range(k) for j in range(i + 1, k)])
-    for bins in [(0, 0), (1, 1), (62, 100000)]:
+    for bins in [(0, 0), (1, 1), (62, 256), (1, 2)]:
         res, _ = check_full(g, LOW, bin_small_max=bins[0], bin_med_max=bins[1])
         assert res.colors.cpu().numpy().tolist() == list(range(1, k + 1))
 
@@ -137,7 +141,7 @@ def test_edge_cases_n0_n1_nnz0():
     assert sgr.color(*dev(loops)).colors.cpu().tolist() == [1, 1, 1]
 
 
-@pytest.mark.parametrize("mode", ["host", "graph"])
+@pytest.mark.parametrize("mode", ["host", "graph", "persistent"])
 @pytest.mark.parametrize("batch", [1, 3, 8, 32])
 def test_loop_modes_and_batches(mode, batch):
     g = gen.config(1)
@@ -153,7 +157,9 @@ def test_profile_mode_and_stats():
     res = sgr.color(rp, ci, profile=True)
     st = res.stats
     assert st["kernel_launches"]["first"] == 1
-    assert st["kernel_launches"]["warp_bin"] >= st["rounds"] - 1
+    assert st["kernel_launches"]["round"] == 1  # persistent: every round in one launch
+    assert st["kernel_ms"]["round"] > 0
+    assert sum(st["bin_edges"].values()) + g.nnz == st["edges_scanned"]
     assert all(v >= 0 for v in st["kernel_ms"].values())
     assert st["bytes_algorithmic"] == sum(st["kernel_bytes"].values())
     ref = oracle.jacobi(g, LOW)
