@@ -82,8 +82,10 @@ typedef struct {
   int32_t tiebreak;      /* sgr_tiebreak; default LOWID_KEEPS */
   int32_t max_rounds;    /* 0 = n+1 (never reached) */
   int32_t loop_mode;     /* sgr_loop_mode */
-  int32_t color_bits;    /* width of the working color arrays: 16 (default; a first fit
-                            above 65535 triggers an automatic 32-bit rerun) or 32 */
+  int32_t color_bits;    /* 16 (default): packed 16-bit color + 16-bit round words, with
+                            live-neighbour trimming of high-degree rows; a color or round
+                            above 65535 triggers an automatic 32-bit rerun. 32: plain int32
+                            colors, full rows every round */
   int32_t bin_small_max; /* degree bins: d <= small -> 8 lanes/vertex, register mask (<= 62);
                             0 = 32 */
   int32_t bin_med_max;   /* small < d <= med -> 8 lanes/vertex, smem table (<= 256); 0 = 256;
@@ -107,6 +109,8 @@ typedef struct {
   int32_t num_colors;         /* max color                                               */
   int64_t vertices_processed; /* sum over rounds of |W_r|                                */
   int64_t edges_scanned;      /* sum over rounds of sum_{v in W_r} deg(v) (A * nnz)      */
+  int64_t entries_read;       /* adjacency entries the passes actually read (rounds >= 2;
+                                 < edges_scanned - nnz when neighbour lists are trimmed) */
   int64_t bytes_algorithmic;  /* DESIGN.md §6 byte model, summed over all launches       */
   float elapsed_ms;           /* device time from the first kernel to the final count   */
   int32_t launches;           /* kernels launched by this call                           */

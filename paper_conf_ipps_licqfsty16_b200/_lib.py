@@ -31,6 +31,7 @@ class Opts(ctypes.Structure):
 class Stats(ctypes.Structure):
     _fields_ = [("rounds", ctypes.c_int32), ("num_colors", ctypes.c_int32),
                 ("vertices_processed", ctypes.c_int64), ("edges_scanned", ctypes.c_int64),
+                ("entries_read", ctypes.c_int64),
                 ("bytes_algorithmic", ctypes.c_int64), ("elapsed_ms", ctypes.c_float),
                 ("launches", ctypes.c_int32),
                 ("kernel_ms", ctypes.c_float * SGR_K_COUNT),
@@ -42,7 +43,7 @@ class Stats(ctypes.Structure):
 
     def as_dict(self) -> dict:
         d = {k: getattr(self, k) for k in ("rounds", "num_colors", "vertices_processed",
-                                             "edges_scanned", "bytes_algorithmic",
+                                             "edges_scanned", "entries_read", "bytes_algorithmic",
                                              "elapsed_ms", "launches")}
         d["kernel_ms"] = dict(zip(KERNEL_CLASSES, list(self.kernel_ms)))
         d["kernel_launches"] = dict(zip(KERNEL_CLASSES, list(self.kernel_launches)))

@@ -69,38 +69,54 @@ Resolved resolve_opts(const sgr_opts* o, int64_t n) {
 }
 
 // Workspace layout (bytes, each piece 256-aligned):
-//   Ctrl | X16, Y16: 2 x n u16 (16-bit mode) | Y32: n i32 | wl_t: 2 x n i32 |
-//   wl_m: 2 x cap_m i32 | wl_c: 2 x cap_c i64 | big_id: n i32 | acc_bits | acc_cnt
-// In 32-bit mode the caller's colors_out is C_k's ping-pong partner of Y32; in 16-bit mode
-// the two u16 buffers ping-pong and the result is widened into colors_out at the end.
+//   Ctrl | colors: 2 x n words | wl_t: 2 x n i32 | wl_m: 2 x cap_m i32 | wl_c: 2 x cap_c i64 |
+//   big_id: n i32 | acc_bits: cap_big x 32 u32 | acc_cnt: cap_big u64 |
+//   (packed mode) fixed: cap_big x 32 u32 | len: 2 x n i32 | adj: 2 x (nnz + 16) i32
+// 32-bit mode: the caller's colors_out is one of the two ping-pong buffers. Packed mode
+// (16-bit color + 16-bit round, trimming) uses two workspace buffers and unpacks at the end.
 struct Layout {
+  bool packed;
   int64_t cap_m, cap_c, cap_big;
-  size_t off_c16, off_y32, off_t, off_m, off_c, off_big, off_accb, off_accc, total;
+  size_t off_col, off_t, off_m, off_c, off_big, off_accb, off_accc, off_fixed, off_len, off_adj;
+  size_t zero_begin, zero_end, total;
 };
 
 static Layout layout(int64_t n, int64_t nnz, const Resolved& r) {
   Layout L;
+  L.packed = r.color_bits == 16;
   L.cap_m = std::min<int64_t>(n, nnz / (r.small_max + 1) + 1);
-  // each bin-2 vertex (deg > med_max) has <= deg / kChunk + 2 aligned chunks
-  L.cap_c = nnz / kChunk + 2 * (nnz / (r.med_max + 1)) + 2;
+  // each bin-2 vertex (deg > med_max) has <= deg / kChunk + 1 chunks
+  L.cap_c = nnz / kChunk + nnz / (r.med_max + 1) + 2;
   L.cap_big = nnz / (r.med_max + 1) + 1;
+  const size_t nb = align_up((size_t)n * 4, 256);
   size_t o = align_up(sizeof(Ctrl), 256);
-  L.off_c16 = o;
-  o += 2 * align_up((size_t)n * 2, 256);
-  L.off_y32 = o;
-  o += align_up((size_t)n * 4, 256);
+  L.off_col = o;
+  o += 2 * nb;
   L.off_t = o;
-  o += 2 * align_up((size_t)n * 4, 256);
+  o += 2 * nb;
   L.off_m = o;
   o += 2 * align_up((size_t)L.cap_m * 4, 256);
   L.off_c = o;
   o += 2 * align_up((size_t)L.cap_c * 8, 256);
   L.off_big = o;
-  o += align_up((size_t)n * 4, 256);
+  o += nb;
   L.off_accb = o;
+  L.zero_begin = o;
   o += align_up((size_t)L.cap_big * 128, 256);
   L.off_accc = o;
   o += align_up((size_t)L.cap_big * 8, 256);
+  L.off_fixed = L.off_len = L.off_adj = o;
+  if (L.packed) {
+    L.off_fixed = o;
+    o += align_up((size_t)L.cap_big * 128, 256);
+    L.off_len = o;
+    o += 2 * nb;
+  }
+  L.zero_end = o;  // accumulators, fixed sets and list lengths start at zero
+  if (L.packed) {
+    L.off_adj = o;
+    o += 2 * align_up((size_t)(nnz + 16) * 4, 256);
+  }
   L.total = o;
   return L;
 }
@@ -108,22 +124,28 @@ static Layout layout(int64_t n, int64_t nnz, const Resolved& r) {
 size_t ws_bytes(int64_t n, int64_t nnz, const Resolved& r) { return layout(n, nnz, r).total; }
 
 template <class C>
-static void build_args(RoundArgs<C>& a, const sgr_csr* csr, int64_t n, int32_t* colors,
-                       void* ws, const Layout& L, const Resolved& r) {
+static void build_args(RoundArgs<C>& a, const sgr_csr* csr, int64_t n, int64_t nnz,
+                       int32_t* colors, void* ws, const Layout& L, const Resolved& r) {
   memset(&a, 0, sizeof(a));
   char* b = (char*)ws;
+  const size_t nb = align_up((size_t)n * 4, 256);
   a.row_ptr = csr->row_ptr;
   a.col_idx = csr->col_idx;
-  if constexpr (sizeof(C) == 2) {
-    a.col[0] = (C*)(b + L.off_c16);
-    a.col[1] = (C*)(b + L.off_c16 + align_up((size_t)n * 2, 256));
+  if constexpr (packed<C>()) {
+    a.col[0] = (C*)(b + L.off_col);
+    a.col[1] = (C*)(b + L.off_col + nb);
+    a.fixed = (uint32_t*)(b + L.off_fixed);
+    a.len[0] = (int32_t*)(b + L.off_len);
+    a.len[1] = (int32_t*)(b + L.off_len + nb);
+    const size_t ab = align_up((size_t)(nnz + 16) * 4, 256);
+    a.adj[0] = (int32_t*)(b + L.off_adj);
+    a.adj[1] = (int32_t*)(b + L.off_adj + ab);
   } else {
     a.col[0] = (C*)colors;
-    a.col[1] = (C*)(b + L.off_y32);
+    a.col[1] = (C*)(b + L.off_col);
   }
-  const size_t st = align_up((size_t)n * 4, 256);
   a.wl_t[0] = (int32_t*)(b + L.off_t);
-  a.wl_t[1] = (int32_t*)(b + L.off_t + st);
+  a.wl_t[1] = (int32_t*)(b + L.off_t + nb);
   const size_t sm = align_up((size_t)L.cap_m * 4, 256);
   a.wl_m[0] = (int32_t*)(b + L.off_m);
   a.wl_m[1] = (int32_t*)(b + L.off_m + sm);
@@ -135,7 +157,7 @@ static void build_args(RoundArgs<C>& a, const sgr_csr* csr, int64_t n, int32_t* 
   a.acc_cnt = (unsigned long long*)(b + L.off_accc);
   a.ctrl = (Ctrl*)b;
   a.n = (int32_t)n;
-  a.nnz = 0;
+  a.nnz = nnz;
   a.small_max = r.small_max;
   a.med_max = r.med_max;
 }
@@ -151,13 +173,26 @@ int first_grid(int64_t n) {
   return (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, (int64_t)num_sms() * 8));
 }
 
+template <class C>
+static constexpr size_t round_smem() { return (size_t)kWarps * WarpSmem<C>::kBytes; }
+
 // Blocks of the round kernels: as many as are co-resident (persistent: required).
 template <int TB, class C>
 static int round_grid(bool persistent) {
+  static bool attr_set = false;
+  if (!attr_set) {  // opt in to > 48 KB of dynamic shared memory
+    cudaFuncSetAttribute(k_persistent<TB, C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)round_smem<C>());
+    cudaFuncSetAttribute(k_round<TB, C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)round_smem<C>());
+    attr_set = true;
+  }
   int per_sm = 0;
   cudaError_t e = persistent
-      ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_persistent<TB, C>, kBlock, 0)
-      : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_round<TB, C>, kBlock, 0);
+      ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_persistent<TB, C>, kBlock,
+                                                      round_smem<C>())
+      : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_round<TB, C>, kBlock,
+                                                      round_smem<C>());
   if (e != cudaSuccess || per_sm <= 0) per_sm = 1;
   return per_sm * num_sms();
 }
@@ -179,7 +214,7 @@ static sgr_status get_graph(const RoundArgs<C>& a, int grid, int batch, cudaGrap
   static_assert(sizeof(RoundArgs<C>) <= sizeof(key.args), "graph key");
   memcpy(key.args, &a, sizeof(a));
   key.tiebreak = TB;
-  key.bits = 8 * (int)sizeof(C);
+  key.bits = packed<C>() ? 16 : 32;
   key.batch = batch;
   key.grid = grid;
   cudaGetDevice(&key.dev);
@@ -198,7 +233,7 @@ static sgr_status get_graph(const RoundArgs<C>& a, int grid, int batch, cudaGrap
     return cuda_fail(err, "cudaStreamBeginCapture", __LINE__);
   }
   for (int b = 0; b < batch; ++b) {
-    k_round<TB, C><<<grid, kBlock, 0, cs>>>(a);
+    k_round<TB, C><<<grid, kBlock, round_smem<C>(), cs>>>(a);
     k_advance<<<1, 32, 0, cs>>>(a.ctrl, 0);
   }
   cudaGraph_t graph;
@@ -262,9 +297,10 @@ void fill_stats(const Ctrl& c, int64_t n, int64_t nnz, sgr_stats* st) {
     st->bin_vertices[q] = (int64_t)c.verts_total[q];
     st->bin_edges[q] = (int64_t)c.edges_total[q];
     // per worklist vertex: 4 B id + 16 B row pair + 4 B X[v] + 4 B Y[v]; 8 B per scanned
-    // entry (4 B col_idx + 4 B X[w]); 4 B per vertex pushed to W_{k+1}
-    b_round += 28 * (int64_t)c.verts_total[q] + 8 * (int64_t)c.edges_total[q] +
+    // entry actually read (4 B list entry + 4 B X[w]); 4 B per vertex pushed to W_{k+1}
+    b_round += 28 * (int64_t)c.verts_total[q] + 8 * (int64_t)c.entries_total[q] +
                4 * (int64_t)c.pushes_total[q];
+    st->entries_read += (int64_t)c.entries_total[q];
   }
   st->chunk_items = (int64_t)c.items_total;
   st->rounds = c.k - 1;
@@ -289,8 +325,7 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
                             int* overflow_out) {
   cudaStream_t s = r.stream;
   RoundArgs<C> a;
-  build_args<C>(a, csr, n, colors_out, ws, L, r);
-  a.nnz = nnz;
+  build_args<C>(a, csr, n, nnz, colors_out, ws, L, r);
   Prof prof;
   prof.on = r.profile != 0;
   int32_t launches = 0;
@@ -307,7 +342,12 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
     hc.round_sizes = r.round_sizes;
     hc.round_edges = r.round_edges;
     cudaError_t le = cudaMemcpyAsync(a.ctrl, &hc, sizeof(Ctrl), cudaMemcpyHostToDevice, s);
-    if (le == cudaSuccess) le = cudaMemsetAsync((char*)ws + L.off_accb, 0, L.total - L.off_accb, s);
+    if (le == cudaSuccess)
+      le = cudaMemsetAsync((char*)ws + L.zero_begin, 0, L.zero_end - L.zero_begin, s);
+    if constexpr (packed<C>()) {  // the bin-2 lists start as the full rows
+      if (le == cudaSuccess && nnz > 0)
+        le = cudaMemcpyAsync(a.adj[0], csr->col_idx, (size_t)nnz * 4, cudaMemcpyDeviceToDevice, s);
+    }
     if (le != cudaSuccess) {
       status = cuda_fail(le, "workspace init", __LINE__);
       break;
@@ -334,7 +374,8 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
     if (persistent) {
       prof.timed(SGR_K_ROUND, s, [&] {
         void* args[] = {(void*)&a};
-        le = cudaLaunchCooperativeKernel((const void*)k_persistent<TB, C>, grid, kBlock, args, 0, s);
+        le = cudaLaunchCooperativeKernel((const void*)k_persistent<TB, C>, grid, kBlock, args,
+                                         round_smem<C>(), s);
       });
       launches += 1;
       if (le != cudaSuccess) {
@@ -362,7 +403,7 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
           le = cudaGraphLaunch(gexec, s);
         } else {
           for (int b = 0; b < r.batch; ++b) {
-            prof.timed(SGR_K_ROUND, s, [&] { k_round<TB, C><<<grid, kBlock, 0, s>>>(a); });
+            prof.timed(SGR_K_ROUND, s, [&] { k_round<TB, C><<<grid, kBlock, round_smem<C>(), s>>>(a); });
             prof.timed(SGR_K_CTRL, s, [&] { k_advance<<<1, 32, 0, s>>>(a.ctrl, 0); });
           }
           le = cudaGetLastError();
@@ -387,10 +428,10 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
     }
 
     prof.timed(SGR_K_FINAL, s, [&] {
-      if constexpr (sizeof(C) == 2) k_widen<<<first_grid(n), 256, 0, s>>>(a.col[0], colors_out, n);
+      if constexpr (packed<C>()) k_unpack<<<first_grid(n), 256, 0, s>>>(a.col[0], colors_out, n);
       k_max_color<<<first_grid(n), 256, 0, s>>>(colors_out, n, &a.ctrl->max_color);
     });
-    launches += sizeof(C) == 2 ? 2 : 1;
+    launches += packed<C>() ? 2 : 1;
     cudaEventRecord(ev1, s);
     Ctrl fin;
     cudaMemcpyAsync(&fin, a.ctrl, sizeof(Ctrl), cudaMemcpyDeviceToHost, s);
@@ -405,7 +446,7 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
       cudaEventElapsedTime(&stats->elapsed_ms, ev0, ev1);
       stats->launches = launches;
       stats->grid_blocks = grid;
-      stats->color_bits = 8 * (int)sizeof(C);
+      stats->color_bits = packed<C>() ? 16 : 32;
       int32_t ri = 0;
       for (auto& m : prof.marks) {
         float ms = 0.f;
@@ -430,11 +471,15 @@ static sgr_status run_any(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* c
                           sgr_stats* stats, const Resolved& r, void* ws, const Layout& L) {
   int overflow = 0;
   if (r.color_bits == 16) {
-    const sgr_status st = run_color<TB, uint16_t>(csr, n, nnz, colors_out, stats, r, ws, L, &overflow);
+    const sgr_status st = run_color<TB, uint32_t>(csr, n, nnz, colors_out, stats, r, ws, L, &overflow);
     if (st != SGR_OK || !overflow) return st;
-    // a first fit exceeded 65535: the 16-bit run is discarded and redone in 32 bits
+    // a color or round number exceeded 16 bits: the packed run is discarded and redone
+    // with plain 32-bit colors (no trimming)
   }
-  const sgr_status st = run_color<TB, int32_t>(csr, n, nnz, colors_out, stats, r, ws, L, &overflow);
+  Resolved r32 = r;
+  r32.color_bits = 32;
+  const Layout L32 = layout(n, nnz, r32);
+  const sgr_status st = run_color<TB, int32_t>(csr, n, nnz, colors_out, stats, r32, ws, L32, &overflow);
   if (st == SGR_OK && overflow) {
     set_error("sgr_color: 32-bit color overflow");
     return SGR_EUNSUPPORTED;

@@ -9,23 +9,28 @@
 // proof (iv)). Detection of round k and assignment of round k+1 read the same snapshot, so
 // one adjacency scan serves both. F_1 needs no color gathers (every color is 1).
 //
-// The pass is bound by the rate of scattered color gathers (one L1TEX wavefront per
-// distinct 128-byte line, ~1 line / SM-cycle measured by tools/gather_bench.cu) and by
-// load latency, so every work item issues ALL its loads up front: the CSR entries, then
-// all color gathers, then the mask / conflict arithmetic. Work binning is static (degrees
-// never change and W only shrinks):
-//   bin 0  deg <= small_max (<= 62): 8 lanes per vertex (coalesced row reads), up to 8
-//          entries per lane, forbidden set in a u64 register per lane, OR-reduced in-group
-//   bin 1  deg <= med_max (<= 256):  8 lanes per vertex, up to 32 entries per lane,
-//          512-byte forbidden table (one byte per color) in shared memory
-//   bin 2  larger: one warp per CHUNK of `chunk` CSR entries on a grid aligned to
-//          `chunk` (16-byte vector loads), 1024-byte table; a vertex with several chunks
-//          merges the chunks' 1024-bit partial sets with atomicOr and the last chunk to
-//          finish (atomic ticket) decides conflict and tent. No row is ever scanned
-//          serially by one worker, so a round's critical path is one chunk.
-// Colors are stored as C = uint16_t (default; half the gather footprint, more lines shared
-// by sorted neighbours) or int32_t; a tent above 65535 sets an overflow flag and the host
-// reruns the coloring with 32-bit colors, so the result is identical either way.
+// The pass is bound by the rate of scattered color gathers (~1 distinct 128-byte line per
+// SM-cycle, tools/gather_bench.cu) and by load latency. Work binning is static:
+//   bin 0  deg <= small_max (<= 62): 8 lanes per vertex (coalesced row reads), <= 8 entries
+//          per lane, all loads issued first, u64 register mask per lane, OR-reduced in-group
+//   bin 1  deg <= med_max (<= 256): 8 lanes per vertex, <= 32 entries per lane, 512-byte
+//          forbidden table (one byte per color) in shared memory
+//   bin 2  larger rows, one warp per chunk of <= kChunk entries. A vertex with several
+//          chunks merges the chunks' 1024-bit partial sets with atomicOr and the last chunk
+//          to finish (atomic ticket) decides conflict and first fit.
+//
+// Live-neighbour trimming (bin 2, packed colors; DESIGN.md §3 proof (vii)): a neighbour
+// that has left the worklist never changes color again. Colors are stored packed as
+// (last round the vertex was in W) << 16 | color, so one gather also says whether the
+// neighbour is still live (last >= k). Each bin-2 vertex keeps its adjacency list in a
+// double-buffered copy adj[2] (same offsets as col_idx) and a 1024-bit set F of the colors
+// of the neighbours it has dropped; every pass reads the current list, drops the neighbours
+// that are no longer live (their colors go to F), and writes the compacted list for the
+// next round. Conflict and first fit are computed from F ∪ {colors of the listed
+// neighbours}, exactly the colors of all neighbours. The chunk windows of the lists are
+// staged into shared memory with TMA bulk copies (cp.async.bulk, mbarrier completion),
+// double-buffered per warp so the next chunk streams in while the current chunk's gathers
+// are in flight.
 // Worklist pushes: warp ballot + popc + one atomicAdd per warp.
 #pragma once
 #include <cstdint>
@@ -37,16 +42,31 @@ namespace sgr {
 
 constexpr int kBins = 3;
 constexpr int kBlock = 256;             // threads per block (8 warps)
+constexpr int kWarps = kBlock / 32;
 constexpr int kGroup = 8;               // lanes per vertex in bins 0 and 1
 constexpr int kK0 = 8;                  // entries per lane, bin 0 (8 x 8 = 64 >= 62)
 constexpr int kK1 = 32;                 // entries per lane, bin 1 (8 x 32 = 256)
 constexpr int kMaxMed = kGroup * kK1;   // 256
 constexpr int kMedTbl = 512;            // bin-1 table bytes (colors < 512 > 257)
 constexpr int kBigTbl = 1024;           // bin-2 table bytes (colors < 1024)
-constexpr int kWarpTbl = 2048;          // per-warp smem: 4 x 512 (bin 1) or 1 x 1024 (bin 2)
-constexpr int kChunk = 1020;            // bin-2 chunk: entries per warp item, chosen so the
-                                        // 16-byte-aligned window (1024 = 32 lanes x 8 int4)
-                                        // always covers the chunk
+constexpr int kTblBytes = 2048;         // per-warp tables: 4 x 512 (bin 1) | 2 x 1024 (bin 2)
+constexpr int kChunk = 1020;            // bin-2 chunk: entries per warp item; the 16-byte-
+                                        // aligned window (<= 1024 entries) covers it
+constexpr int kWin = 1024;              // window entries (32 lanes x 8 int4)
+
+template <class C>
+__host__ __device__ constexpr bool packed() { return sizeof(C) == 4 && C(-1) > C(0); }
+
+// dynamic shared memory per warp: [2 TMA stages (packed only)] [tables] [2 mbarriers]
+constexpr int kStage = kWin * 4;        // bytes per TMA stage: one bin-2 window
+// blocks per SM the round kernels are compiled for: packed mode is shared-memory bound to 2
+// (82 KB per block), plain mode can afford 3 (<= 85 registers)
+template <class C>
+constexpr int kMinBlocks = packed<C>() ? 2 : 3;
+template <class C> struct WarpSmem {
+  static constexpr int kBuf = packed<C>() ? 2 * kStage : 0;
+  static constexpr int kBytes = kBuf + kTblBytes + 16;  // + 2 mbarriers
+};
 
 // Device-resident loop state (in the workspace).
 struct Ctrl {
@@ -56,17 +76,19 @@ struct Ctrl {
   int32_t max_rounds;
   int32_t cnt[2][kBins];     // work items per parity (k & 1) and bin
   int32_t vcnt2[2];          // bin-2 worklist VERTICES per parity (items are chunks)
-  int32_t overflow;          // a first fit exceeded the color type (u16 -> rerun in i32)
+  int32_t overflow;          // a packed color or round number exceeded 16 bits
   int32_t round_cap;
   uint32_t bar_count;        // grid barrier (persistent kernel)
   uint32_t bar_gen;
-  int32_t big_count;         // slots handed to multi-chunk vertices by F_1
+  int32_t big_count;         // slots handed to bin-2 vertices by F_1
   int32_t max_color;
   int32_t violations;
   int32_t pad[3];
-  unsigned long long edges_acc[kBins];
+  unsigned long long edges_acc[kBins];    // sum of deg(v) over the pass's vertices (algorithmic)
+  unsigned long long entries_acc[kBins];  // CSR / list entries actually read by the pass
   unsigned long long verts_total[kBins + 1];   // [kBins] = F_1
   unsigned long long edges_total[kBins + 1];
+  unsigned long long entries_total[kBins + 1];
   unsigned long long pushes_total[kBins + 1];
   unsigned long long items_total;
   int32_t* round_sizes;
@@ -81,9 +103,12 @@ struct RoundArgs {
   int32_t* wl_t[2];           // bin 0 vertex lists, W_k in [k & 1]
   int32_t* wl_m[2];           // bin 1 vertex lists
   int64_t* wl_c[2];           // bin 2 chunk items: (v << 32) | chunk
-  int32_t* big_id;            // slot of each multi-chunk vertex (F_1)
-  uint32_t* acc_bits;         // [slot][32] partial forbidden sets
+  int32_t* big_id;            // slot of each bin-2 vertex (F_1)
+  uint32_t* acc_bits;         // [slot][32] partial forbidden sets of the running pass
   unsigned long long* acc_cnt;  // [slot] chunks finished | conflicts << 32
+  int32_t* adj[2];            // trimmed adjacency lists (packed mode), offsets = row_ptr
+  int32_t* len[2];            // [v] list length for the pass of parity p
+  uint32_t* fixed;            // [slot][32] colors of dropped (finalized) neighbours
   Ctrl* ctrl;
   int64_t nnz;
   int32_t n;
@@ -99,42 +124,89 @@ __device__ __forceinline__ T sel(int par, T a0, T a1) { return par ? a1 : a0; }
 __device__ __forceinline__ int32_t ld_cg(const int32_t* p) { return __ldcg(p); }
 __device__ __forceinline__ uint32_t ld_cg(const uint32_t* p) { return __ldcg(p); }
 
+// ---- color words: int32_t = plain color; uint32_t = (last round << 16) | color ----------
 template <bool Persist, class C>
-__device__ __forceinline__ int32_t ldc(const C* p) {
-  if constexpr (Persist) return (int32_t)__ldcg(p);
-  else return (int32_t)__ldg(p);
+__device__ __forceinline__ uint32_t ldraw(const C* p) {
+  if constexpr (Persist) return (uint32_t)__ldcg(p);
+  else return (uint32_t)__ldg(p);
 }
+template <class C>
+__device__ __forceinline__ int32_t cval(uint32_t raw) {
+  if constexpr (packed<C>()) return (int32_t)(raw & 0xffffu);
+  else return (int32_t)raw;
+}
+template <bool Persist, class C>
+__device__ __forceinline__ int32_t ldc(const C* p) { return cval<C>(ldraw<Persist>(p)); }
 
 template <class C>
-__device__ __forceinline__ C store_color(int32_t c, Ctrl* ctrl) {
-  if constexpr (sizeof(C) == 2) {
-    if (c > 65535) {
+__device__ __forceinline__ C cpack(int32_t color, int32_t last, Ctrl* ctrl) {
+  if constexpr (packed<C>()) {
+    if (color > 0xffff || last > 0xffff) {
       ctrl->overflow = 1;
-      return (C)65535;
+      return (C)0xffffffffu;
     }
+    return (C)(((uint32_t)last << 16) | (uint32_t)color);
+  } else {
+    (void)last;
+    (void)ctrl;
+    return (C)color;
   }
-  return (C)c;
 }
 
 __device__ __forceinline__ int bin_of(int64_t d, int small_max, int med_max) {
   return d <= small_max ? 0 : (d <= med_max ? 1 : 2);
 }
 
-// Chunks of a bin-2 row [s, e): [s + c * kChunk, s + (c + 1) * kChunk), c < ceil(deg / kChunk).
-__device__ __forceinline__ int32_t num_chunks(int64_t s, int64_t e) {
-  return (int32_t)((e - s + kChunk - 1) / kChunk);
+__device__ __forceinline__ int32_t num_chunks(int64_t len) {
+  return (int32_t)((len + kChunk - 1) / kChunk);
 }
 
 __device__ __forceinline__ void prefetch_l2(const void* p) {
   asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
 }
 
-// Release / acquire fences at GPU scope (lighter than the sequentially consistent
-// fence.sc.gpu that __threadfence() emits).
+// Release / acquire fence at GPU scope (lighter than the fence.sc.gpu of __threadfence()).
 __device__ __forceinline__ void fence_acq_rel_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
 
 __device__ __forceinline__ int64_t make_item(int32_t v, int32_t c) {
   return (int64_t)(((uint64_t)(uint32_t)v << 32) | (uint32_t)c);
+}
+
+// ---- TMA bulk copies + mbarriers (Blackwell async proxy) -------------------------------
+__device__ __forceinline__ uint32_t smem_addr(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_init_fence() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+// One elected thread: announce `bytes` of transaction and start the bulk copy global->smem.
+__device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t bytes,
+                                            uint64_t* bar) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)),
+               "r"(bytes)
+               : "memory");
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::
+          "r"(smem_addr(dst)),
+      "l"(src), "r"(bytes), "r"(smem_addr(bar))
+      : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
+  uint32_t done;
+  do {
+    asm volatile(
+        "{\n .reg .pred P;\n mbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2;\n"
+        " selp.u32 %0, 1, 0, P;\n}"
+        : "=r"(done)
+        : "r"(smem_addr(b)), "r"(parity)
+        : "memory");
+  } while (!done);
 }
 
 // ---------------------------------------------------------------------------------------
@@ -142,7 +214,8 @@ __device__ __forceinline__ int64_t make_item(int32_t v, int32_t c) {
 // color is 1 (first fit against an all-zero snapshot), so with rows sorted ascending
 //   LOWID: conflict(v) <=> first entry < v ;  PAPER: conflict(v) <=> last entry > v
 // (a self-loop can never satisfy the strict inequality); tent(v) = mex({1}) = 2.
-// Writes col[0] = C_1 (all 1), col[1] = C_2, and W_2 into the bins' lists [0].
+// Writes col[0] = C_1 (all 1), col[1] = C_2, and W_2 into the bins' lists [0]; bin-2
+// vertices of W_2 get a slot and (packed mode) their list length len[0][v] = deg(v).
 template <int TB, class C>
 __global__ void __launch_bounds__(256) k_first(RoundArgs<C> a, int sorted) {
   Ctrl* ctrl = a.ctrl;
@@ -167,23 +240,23 @@ __global__ void __launch_bounds__(256) k_first(RoundArgs<C> a, int sorted) {
           for (int64_t j = s; j < e && !conflict; ++j) conflict = lose<TB>(v, ldg_i32(a.col_idx + j));
         }
       }
-      X[v] = (C)1;
-      Y[v] = (C)(conflict ? 2 : 1);
+      X[v] = cpack<C>(1, 1, ctrl);
+      Y[v] = cpack<C>(conflict ? 2 : 1, conflict ? 2 : 1, ctrl);
     }
     const int b = bin_of(e - s, a.small_max, a.med_max);
     warp_push(conflict && b == 0, v, a.wl_t[0], &ctrl->cnt[0][0]);
     warp_push(conflict && b == 1, v, a.wl_m[0], &ctrl->cnt[0][1]);
-    // bin 2: one item per aligned chunk; multi-chunk vertices get an accumulator slot
+    // bin 2: ceil(deg / kChunk) items per vertex and an accumulator slot
     const bool big = conflict && b == 2;
-    const int32_t nch = big ? num_chunks(s, e) : 0;
+    const int32_t nch = big ? num_chunks(e - s) : 0;
     const unsigned mb = __ballot_sync(0xffffffffu, big);
     if (mb) {
-      const unsigned mm = __ballot_sync(0xffffffffu, nch > 1);
-      if (mm) {
-        int sb = 0;
-        if (lane == __ffs(mm) - 1) sb = atomicAdd(&ctrl->big_count, __popc(mm));
-        sb = __shfl_sync(0xffffffffu, sb, __ffs(mm) - 1);
-        if (nch > 1) a.big_id[v] = sb + __popc(mm & ((1u << lane) - 1u));
+      int sb = 0;
+      if (lane == __ffs(mb) - 1) sb = atomicAdd(&ctrl->big_count, __popc(mb));
+      sb = __shfl_sync(0xffffffffu, sb, __ffs(mb) - 1);
+      if (big) {
+        a.big_id[v] = sb + __popc(mb & ((1u << lane) - 1u));
+        if constexpr (packed<C>()) a.len[0][v] = (int32_t)(e - s);
       }
       int incl = nch;
 #pragma unroll
@@ -240,7 +313,20 @@ __device__ __forceinline__ uint32_t tbl_bits32(const uint8_t* tbl, int lane) {
   return bits;
 }
 
-// Exact warp first fit from `base` (all colors in [1, base) forbidden) — rare fallback.
+// First free color of a 1024-bit set spread over the warp (lane l holds colors
+// [32 l, 32 l + 32); bit 0 of lane 0 must already be set); -1 if all are taken.
+__device__ __forceinline__ int32_t bits_first_free(uint32_t word) {
+  const unsigned fb = __ballot_sync(0xffffffffu, word != 0xffffffffu);
+  if (!fb) return -1;
+  const int fl = __ffs(fb) - 1;
+  const uint32_t w2 = __shfl_sync(0xffffffffu, word, fl);
+  return fl * 32 + __ffs(~w2) - 1;
+}
+
+// Exact warp first fit over the FULL original row from `base` (all colors in [1, base)
+// forbidden): the rare fallback when a first fit exceeds the 1024-color table. Reads the
+// snapshot X, which holds the final colors of dropped neighbours, so it is exact in the
+// trimmed mode as well.
 template <bool Persist, class C>
 __device__ __noinline__ int32_t warp_first_fit_rescan(const int32_t* __restrict__ col_idx,
                                                       const C* X, int64_t s, int64_t e,
@@ -271,19 +357,26 @@ __device__ __noinline__ int32_t warp_first_fit_rescan(const int32_t* __restrict_
   }
 }
 
+__device__ __forceinline__ void clear_bytes(uint8_t* p, int bytes_per_lane, int lane) {
+  uint4* t = reinterpret_cast<uint4*>(p) + lane * (bytes_per_lane / 16);
+#pragma unroll
+  for (int q = 0; q < bytes_per_lane / 16; ++q) t[q] = make_uint4(0, 0, 0, 0);
+}
+
 // ---------------------------------------------------------------------------------------
-// Bin 2: one warp processes one chunk item [cs, ce) of row [s, e). Entries are read as int4
-// from the 16-byte-aligned window starting at cs rounded down to a multiple of 4 (1024
-// entries >= kChunk + 3); positions outside [cs, ce) are masked.
+// Bin 2, plain 32-bit colors (no trimming): one warp processes one chunk [cs, ce) of the
+// full row [s, e), read as int4 from the 16-byte-aligned window; outside [cs, ce) masked.
 template <int TB, bool Persist, class C>
-__device__ __forceinline__ void process_chunk(const RoundArgs<C>& a, int32_t v, int32_t c,
-                                              int64_t s, int64_t e, const C* X, C* Y,
-                                              int64_t* out, int32_t* out_cnt,
-                                              int32_t* out_vcnt, uint8_t* tbl, int lane,
-                                              unsigned long long& edges) {
+__device__ __forceinline__ void process_chunk_plain(const RoundArgs<C>& a, int k, int32_t v,
+                                                    int32_t c, int64_t s, int64_t e,
+                                                    const C* X, C* Y, int64_t* out,
+                                                    int32_t* out_cnt, int32_t* out_vcnt,
+                                                    uint8_t* tbl, int lane,
+                                                    unsigned long long& edges,
+                                                    unsigned long long& entries) {
   const int64_t cs = s + (int64_t)c * kChunk, ce = min(e, cs + kChunk);
   const int64_t wbase = cs & ~(int64_t)3;  // 16-byte aligned window start
-  const int32_t nch = num_chunks(s, e);
+  const int32_t nch = num_chunks(e - s);
   const int4* col4 = reinterpret_cast<const int4*>(a.col_idx + wbase);
   int32_t w[32];
 #pragma unroll
@@ -316,7 +409,10 @@ __device__ __forceinline__ void process_chunk(const RoundArgs<C>& a, int32_t v, 
     if ((uint32_t)w[u] < (uint32_t)kBigTbl) tbl[w[u]] = 1;
     conf |= (w[u] == xv) & ((lb >> u) & 1u);
   }
-  if (lane == 0) edges += (unsigned long long)(ce - cs);
+  if (lane == 0) {
+    entries += (unsigned long long)(ce - cs);
+    if (c == 0) edges += (unsigned long long)(e - s);
+  }
   __syncwarp();
   const bool any = __any_sync(0xffffffffu, conf);
   if (nch == 1) {
@@ -326,7 +422,7 @@ __device__ __forceinline__ void process_chunk(const RoundArgs<C>& a, int32_t v, 
       if (tent < 0) tent = warp_first_fit_rescan<Persist>(a.col_idx, X, s, e, kBigTbl, lane);
     }
     if (lane == 0) {
-      Y[v] = any ? store_color<C>(tent, a.ctrl) : (C)xv;
+      Y[v] = any ? cpack<C>(tent, k + 1, a.ctrl) : cpack<C>(xv, k, a.ctrl);
       if (any) {
         out[atomicAdd(out_cnt, 1)] = make_item(v, 0);
         atomicAdd(out_vcnt, 1);
@@ -353,18 +449,12 @@ __device__ __forceinline__ void process_chunk(const RoundArgs<C>& a, int32_t v, 
       int32_t tent = 0;
       if (conf_all) {
         if (lane == 0) word |= 1u;  // color 0
-        const unsigned fb = __ballot_sync(0xffffffffu, word != 0xffffffffu);
-        if (fb) {
-          const int fl = __ffs(fb) - 1;
-          const uint32_t w2 = __shfl_sync(0xffffffffu, word, fl);
-          tent = fl * 32 + __ffs(~w2) - 1;
-        } else {
-          tent = warp_first_fit_rescan<Persist>(a.col_idx, X, s, e, kBigTbl, lane);
-        }
+        tent = bits_first_free(word);
+        if (tent < 0) tent = warp_first_fit_rescan<Persist>(a.col_idx, X, s, e, kBigTbl, lane);
       }
       int32_t ob = 0;
       if (lane == 0) {
-        Y[v] = conf_all ? store_color<C>(tent, a.ctrl) : (C)xv;
+        Y[v] = conf_all ? cpack<C>(tent, k + 1, a.ctrl) : cpack<C>(xv, k, a.ctrl);
         if (conf_all) {
           ob = atomicAdd(out_cnt, nch);
           atomicAdd(out_vcnt, 1);
@@ -376,21 +466,255 @@ __device__ __forceinline__ void process_chunk(const RoundArgs<C>& a, int32_t v, 
       }
     }
   }
-  // clear the table for the next item (32 bytes per lane)
-  uint4* t4 = reinterpret_cast<uint4*>(tbl) + lane * 2;
-  t4[0] = make_uint4(0, 0, 0, 0);
-  t4[1] = make_uint4(0, 0, 0, 0);
+  clear_bytes(tbl, kBigTbl / 32, lane);
   __syncwarp();
+}
+
+// ---------------------------------------------------------------------------------------
+// Bin 2, packed colors, trimmed lists (see the header comment). Per warp: a 2-stage TMA
+// pipeline over the warp's chunk items i, i + NW, i + 2 NW, ...
+struct ChunkHdr {
+  int32_t v, c, len;
+  int64_t s;   // row offset (list start in adj[*] and col_idx)
+};
+
+template <int TB, bool Persist>
+__device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k, int p,
+                                             const uint32_t* X, uint32_t* Y, uint8_t* wsm,
+                                             int gw, int NW, int lane,
+                                             unsigned long long& edges,
+                                             unsigned long long& entries, uint32_t& ph) {
+  using C = uint32_t;
+  Ctrl* ctrl = a.ctrl;
+  const int nC = ld_cg(&ctrl->cnt[p][2]);
+  if (gw >= nC) return;
+  const int64_t* items = sel(p, (const int64_t*)a.wl_c[0], (const int64_t*)a.wl_c[1]);
+  int64_t* out = sel(p ^ 1, a.wl_c[0], a.wl_c[1]);
+  int32_t* out_cnt = &ctrl->cnt[p ^ 1][2];
+  int32_t* out_vcnt = &ctrl->vcnt2[p ^ 1];
+  const int32_t* src = sel(p, (const int32_t*)a.adj[0], (const int32_t*)a.adj[1]);
+  int32_t* dst = sel(p ^ 1, a.adj[0], a.adj[1]);
+  int32_t* len_cur = sel(p, a.len[0], a.len[1]);
+  int32_t* len_nxt = sel(p ^ 1, a.len[0], a.len[1]);
+  int32_t* bufs = reinterpret_cast<int32_t*>(wsm);
+  uint8_t* tbl_all = wsm + WarpSmem<C>::kBuf;
+  uint8_t* tbl_drop = tbl_all + kBigTbl;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(wsm + WarpSmem<C>::kBuf + kTblBytes);
+
+  auto issue = [&](const ChunkHdr& h, int st) {  // lane 0 only
+    const int64_t cs = h.s + (int64_t)h.c * kChunk;
+    const int64_t ce = min(h.s + (int64_t)h.len, cs + kChunk);
+    const int64_t w0 = cs & ~(int64_t)3;
+    const uint32_t bytes = (uint32_t)(((ce - w0 + 3) >> 2) << 4);
+    fence_proxy_async();  // generic-proxy reads of this stage happen-before the async write
+    tma_load_1d(bufs + st * (kStage / 4), src + w0, bytes, bars + st);
+  };
+  auto load_hdr = [&](int i, ChunkHdr& h) {
+    const int64_t it = __ldcg(items + i);
+    h.v = (int32_t)((uint64_t)it >> 32);
+    h.c = (int32_t)(uint32_t)it;
+    h.s = ldg_i64(a.row_ptr + h.v);
+    h.len = ld_cg(len_cur + h.v);
+  };
+
+  int i = gw;
+  ChunkHdr cur, nxt;
+  load_hdr(i, cur);
+  if (lane == 0) issue(cur, 0);
+  int in = i + NW;
+  nxt.v = nxt.c = nxt.len = 0;
+  nxt.s = 0;
+  if (in < nC) load_hdr(in, nxt);
+  int st = 0;
+  while (i < nC) {
+    if (in < nC && lane == 0) issue(nxt, st ^ 1);
+    const int inn = in + NW;
+    const int64_t it_nn = inn < nC ? __ldcg(items + inn) : 0;
+
+    // ---- chunk `cur` in stage st
+    const int32_t v = cur.v;
+    const int64_t cs = cur.s + (int64_t)cur.c * kChunk;
+    const int64_t ce = min(cur.s + (int64_t)cur.len, cs + kChunk);
+    const int64_t w0 = cs & ~(int64_t)3;
+    const int32_t nch = num_chunks(cur.len);
+    const int32_t xv = cval<C>(ldraw<Persist>(X + v));
+    mbar_wait(bars + st, (ph >> st) & 1u);
+    ph ^= 1u << st;
+    const int4* b4 = reinterpret_cast<const int4*>(bufs + st * (kStage / 4));
+    uint32_t cc[32];
+    uint32_t valid = 0, lb = 0;
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      const int4 t4 = b4[lane + 32 * q];
+      const int32_t wq[4] = {t4.x, t4.y, t4.z, t4.w};
+#pragma unroll
+      for (int t = 0; t < 4; ++t) {
+        const int64_t pos = w0 + 4 * (lane + 32 * q) + t;
+        const bool ok = pos >= cs && pos < ce;
+        valid |= ok ? (1u << (4 * q + t)) : 0u;
+        lb |= (ok && lose<TB>(v, wq[t])) ? (1u << (4 * q + t)) : 0u;
+        cc[4 * q + t] = ok ? ldraw<Persist>(X + wq[t]) : 0u;
+      }
+    }
+    bool conf = false;
+    uint32_t lv = 0;  // live bits
+#pragma unroll
+    for (int u = 0; u < 32; ++u) {
+      const int32_t col = cval<C>(cc[u]);
+      const bool live = (int32_t)(cc[u] >> 16) >= k;
+      const bool ok = (valid >> u) & 1u;
+      if ((uint32_t)col < (uint32_t)kBigTbl) {
+        tbl_all[col] = 1;
+        if (ok && !live) tbl_drop[col] = 1;
+      }
+      conf |= ok && col == xv && ((lb >> u) & 1u);
+      lv |= (ok && live) ? (1u << u) : 0u;
+    }
+    // next-next header: the item id has arrived by now
+    ChunkHdr nn;
+    nn.v = (int32_t)((uint64_t)it_nn >> 32);
+    nn.c = (int32_t)(uint32_t)it_nn;
+    nn.s = 0;
+    nn.len = 0;
+    if (inn < nC) {
+      nn.s = ldg_i64(a.row_ptr + nn.v);
+      nn.len = ld_cg(len_cur + nn.v);
+    }
+    if (lane == 0) {
+      entries += (unsigned long long)(ce - cs);
+      if (cur.c == 0) edges += (unsigned long long)(ldg_i64(a.row_ptr + v + 1) - cur.s);
+    }
+    __syncwarp();
+    const bool any = __any_sync(0xffffffffu, conf);
+
+    // live-entry compaction offsets: per int4 slot q, lane counts packed 8 bits per slot
+    uint32_t pk0 = 0, pk1 = 0;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) pk0 |= (uint32_t)__popc((lv >> (4 * q)) & 0xfu) << (8 * q);
+#pragma unroll
+    for (int q = 0; q < 4; ++q) pk1 |= (uint32_t)__popc((lv >> (4 * (q + 4))) & 0xfu) << (8 * q);
+    uint32_t in0 = pk0, in1 = pk1;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t t0 = __shfl_up_sync(0xffffffffu, in0, o);
+      const uint32_t t1 = __shfl_up_sync(0xffffffffu, in1, o);
+      if (lane >= o) {
+        in0 += t0;
+        in1 += t1;
+      }
+    }
+    const uint32_t tot0 = __shfl_sync(0xffffffffu, in0, 31);
+    const uint32_t tot1 = __shfl_sync(0xffffffffu, in1, 31);
+    const uint32_t ex0 = in0 - pk0, ex1 = in1 - pk1;
+    uint32_t live_total = 0;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) live_total += ((tot0 >> (8 * q)) & 0xffu) + ((tot1 >> (8 * q)) & 0xffu);
+    const int32_t* sbuf = bufs + st * (kStage / 4);
+    auto write_live = [&](int32_t* base) {
+      uint32_t qb = 0;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        const uint32_t sh = 8 * (q & 3);
+        const uint32_t tq = ((q < 4 ? tot0 : tot1) >> sh) & 0xffu;
+        uint32_t off = qb + (((q < 4 ? ex0 : ex1) >> sh) & 0xffu);
+        const int32_t* sq = sbuf + 4 * (lane + 32 * q);
+#pragma unroll
+        for (int t = 0; t < 4; ++t)
+          if ((lv >> (4 * q + t)) & 1u) base[off++] = sq[t];
+        qb += tq;
+      }
+    };
+
+    const int32_t slot = __ldg(a.big_id + v);
+    uint32_t* fx = a.fixed + (int64_t)slot * 32;
+    if (nch == 1) {
+      if (any) {
+        const uint32_t fo = ld_cg(fx + lane);
+        const uint32_t word = tbl_bits32(tbl_all, lane) | fo | (lane == 0 ? 1u : 0u);
+        int32_t tent = bits_first_free(word);
+        if (tent < 0) {
+          tent = warp_first_fit_rescan<Persist>(a.col_idx, X, cur.s,
+                                                ldg_i64(a.row_ptr + v + 1), kBigTbl, lane);
+        }
+        const uint32_t drop = tbl_bits32(tbl_drop, lane);
+        if (drop & ~fo) fx[lane] = fo | drop;
+        write_live(dst + cur.s);
+        if (lane == 0) {
+          len_nxt[v] = (int32_t)live_total;
+          Y[v] = cpack<C>(tent, k + 1, ctrl);
+          out[atomicAdd(out_cnt, 1)] = make_item(v, 0);  // live_total <= kChunk: one chunk
+          atomicAdd(out_vcnt, 1);
+        }
+      } else if (lane == 0) {
+        Y[v] = cpack<C>(xv, k, ctrl);
+      }
+    } else {
+      uint32_t* accb = a.acc_bits + (int64_t)slot * 32;
+      const uint32_t bits = tbl_bits32(tbl_all, lane);
+      const uint32_t drop = tbl_bits32(tbl_drop, lane);
+      if (bits) atomicOr(accb + lane, bits);
+      if (drop) atomicOr(fx + lane, drop);
+      int32_t lbase = 0;
+      if (lane == 0 && live_total) lbase = atomicAdd(len_nxt + v, (int32_t)live_total);
+      lbase = __shfl_sync(0xffffffffu, lbase, 0);
+      write_live(dst + cur.s + lbase);
+      __syncwarp();  // orders every lane's writes before lane 0's release below
+      unsigned long long old = 0;
+      if (lane == 0) {
+        fence_acq_rel_gpu();
+        old = atomicAdd(a.acc_cnt + slot, 1ull | ((unsigned long long)any << 32));
+      }
+      old = __shfl_sync(0xffffffffu, old, 0);
+      if ((uint32_t)old == (uint32_t)(nch - 1)) {  // last chunk of v in this pass
+        fence_acq_rel_gpu();
+        const uint32_t word = ld_cg(accb + lane) | ld_cg(fx + lane) | (lane == 0 ? 1u : 0u);
+        accb[lane] = 0u;
+        const bool conf_all = ((old >> 32) + (any ? 1ull : 0ull)) != 0ull;
+        int32_t tent = 0;
+        if (conf_all) {
+          tent = bits_first_free(word);
+          if (tent < 0) {
+            tent = warp_first_fit_rescan<Persist>(a.col_idx, X, cur.s,
+                                                  ldg_i64(a.row_ptr + v + 1), kBigTbl, lane);
+          }
+        }
+        int32_t ob = 0, nch2 = 0;
+        if (lane == 0) {
+          a.acc_cnt[slot] = 0ull;
+          len_cur[v] = 0;  // consumed; the pass after next accumulates into it
+          Y[v] = conf_all ? cpack<C>(tent, k + 1, ctrl) : cpack<C>(xv, k, ctrl);
+          if (conf_all) {
+            nch2 = num_chunks(ld_cg(len_nxt + v));
+            ob = atomicAdd(out_cnt, nch2);
+            atomicAdd(out_vcnt, 1);
+          }
+        }
+        if (conf_all) {
+          ob = __shfl_sync(0xffffffffu, ob, 0);
+          nch2 = __shfl_sync(0xffffffffu, nch2, 0);
+          for (int32_t t = lane; t < nch2; t += 32) out[ob + t] = make_item(v, t);
+        }
+      }
+    }
+    clear_bytes(tbl_all, kTblBytes / 32, lane);  // both tables
+    __syncwarp();
+    st ^= 1;
+    i = in;
+    in = inn;
+    cur = nxt;
+    nxt = nn;
+  }
 }
 
 // Bins 0 and 1: each 8-lane group of the warp processes one vertex (v < 0: idle group).
 // All loads of the row are issued up front (K per lane, group lanes interleaved so a
-// group's reads of a row are contiguous), then all color gathers.
+// group's reads of a row are contiguous), then all color gathers. (Staging these short
+// rows through TMA was measured slower: the per-copy cost exceeds the latency it hides.)
 template <int TB, bool Persist, class C, int K, bool Table>
-__device__ __forceinline__ void process_group(const RoundArgs<C>& a, int32_t v, int64_t s,
-                                              int64_t e, const C* X, C* Y, uint8_t* gtbl,
-                                              int gl, unsigned gmask, bool& push,
-                                              unsigned long long& edges) {
+__device__ __forceinline__ void process_group(const RoundArgs<C>& a, int k, int32_t v,
+                                              int64_t s, int64_t e, const C* X, C* Y,
+                                              uint8_t* gtbl, int gl, unsigned gmask,
+                                              bool& push, unsigned long long& edges) {
   int32_t w[K];
 #pragma unroll
   for (int u = 0; u < K; ++u) {
@@ -435,26 +759,56 @@ __device__ __forceinline__ void process_group(const RoundArgs<C>& a, int32_t v, 
       }
       // deg <= 256 => first fit <= 257 < kMedTbl: the table always has a free slot
     }
-    // clear the group's table (64 bytes per lane)
-    uint4* t4 = reinterpret_cast<uint4*>(gtbl) + gl * 4;
-#pragma unroll
-    for (int q = 0; q < 4; ++q) t4[q] = make_uint4(0, 0, 0, 0);
+    clear_bytes(gtbl, kMedTbl / kGroup, gl);
     __syncwarp();
   } else {
 #pragma unroll
     for (int o = 4; o > 0; o >>= 1) mask |= __shfl_xor_sync(0xffffffffu, mask, o);
     tent = __ffsll((long long)~mask) - 1;  // deg <= 62 => first fit <= 63
   }
-  if (v >= 0 && gl == 0) Y[v] = any ? store_color<C>(tent, a.ctrl) : (C)xv;
+  if (v >= 0 && gl == 0) Y[v] = any ? cpack<C>(tent, k + 1, a.ctrl) : cpack<C>(xv, k, a.ctrl);
   push = (v >= 0) && any && gl == 0;
+}
+
+// Bins 0/1 driver: warp w takes list positions 4w + g, 4(w + NW) + g, ... (g = group); the
+// next position's list entry and row offsets are prefetched, its row warmed into L2.
+template <int TB, bool Persist, class C, int K, bool Table>
+__device__ __forceinline__ void bin01(const RoundArgs<C>& a, int k, const int32_t* list, int nX,
+                                      int32_t* out, int32_t* out_cnt, const C* X, C* Y,
+                                      uint8_t* wsm, int gw, int NW, int lane,
+                                      unsigned long long& edges, unsigned long long& entries) {
+  const int g = lane >> 3, gl = lane & 7;
+  const unsigned gmask = 0xffu << (g * 8);
+  uint8_t* gtbl = wsm + WarpSmem<C>::kBuf + g * kMedTbl;
+  const int step = NW * 4;
+  int i = gw * 4 + g;
+  int32_t v = i < nX ? ld_cg(list + i) : -1;
+  int64_t s = v >= 0 ? ldg_i64(a.row_ptr + v) : 0, e = v >= 0 ? ldg_i64(a.row_ptr + v + 1) : 0;
+  for (int base = gw * 4; base < nX; base += step) {
+    const int in = i + step;
+    const int32_t vn = in < nX ? ld_cg(list + in) : -1;
+    const int64_t sn = vn >= 0 ? ldg_i64(a.row_ptr + vn) : 0;
+    const int64_t en = vn >= 0 ? ldg_i64(a.row_ptr + vn + 1) : 0;
+    if (Table && sn + 32 * gl < en) prefetch_l2(a.col_idx + sn + 32 * gl);  // 1 line / lane
+    bool push = false;
+    if (v >= 0 && gl == 0) entries += (unsigned long long)(e - s);
+    process_group<TB, Persist, C, K, Table>(a, k, v, s, e, X, Y, gtbl, gl, gmask, push, edges);
+    warp_push(push, v, out, out_cnt);
+    i = in;
+    v = vn;
+    s = sn;
+    e = en;
+  }
 }
 
 // One fused pass F_k over all three bins; every warp of the grid calls it. Static
 // round-robin assignment (warp w takes items w, w + NW, ...), with the next item's list
 // entry and row offsets prefetched while the current one is processed.
 template <int TB, bool Persist, class C>
-__device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, uint8_t* wtbl,
-                                           unsigned long long (&edges)[kBins]) {
+__device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, uint8_t* wsm,
+                                           unsigned long long (&edges)[kBins],
+                                           unsigned long long (&entries)[kBins],
+                                           uint32_t& ph) {
   Ctrl* ctrl = a.ctrl;
   const int p = k & 1;
   const int lane = threadIdx.x & 31;
@@ -462,8 +816,12 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, uint8_t
   const int NW = (int)((gridDim.x * blockDim.x) >> 5);
   const C* X = sel((k - 1) & 1, (const C*)a.col[0], (const C*)a.col[1]);
   C* Y = sel(k & 1, a.col[0], a.col[1]);
-  // ---- bin 2: chunk items, one per warp
-  {
+  uint8_t* wtbl = wsm + WarpSmem<C>::kBuf;
+  (void)wtbl;
+  // ---- bin 2
+  if constexpr (packed<C>()) {
+    bin2_trimmed<TB, Persist>(a, k, p, X, Y, wsm, gw, NW, lane, edges[2], entries[2], ph);
+  } else {
     const int nC = ld_cg(&ctrl->cnt[p][2]);
     const int64_t* items = sel(p, (const int64_t*)a.wl_c[0], (const int64_t*)a.wl_c[1]);
     int64_t* out = sel(p ^ 1, a.wl_c[0], a.wl_c[1]);
@@ -482,9 +840,9 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, uint8_t
         const int64_t ln = (csn & ~(int64_t)3) + 32 * lane;
         if (ln < en) prefetch_l2(a.col_idx + ln);
       }
-      process_chunk<TB, Persist, C>(a, v, (int32_t)(uint32_t)it, s, e, X, Y, out,
-                                    &ctrl->cnt[p ^ 1][2], &ctrl->vcnt2[p ^ 1], wtbl, lane,
-                                    edges[2]);
+      process_chunk_plain<TB, Persist, C>(a, k, v, (int32_t)(uint32_t)it, s, e, X, Y, out,
+                                          &ctrl->cnt[p ^ 1][2], &ctrl->vcnt2[p ^ 1], wtbl,
+                                          lane, edges[2], entries[2]);
       i = in;
       it = itn;
       v = vn;
@@ -492,76 +850,41 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, uint8_t
       e = en;
     }
   }
-  const int g = lane >> 3, gl = lane & 7;
-  const unsigned gmask = 0xffu << (g * 8);
   // ---- bin 1: four vertices per warp (one per 8-lane group), 512-byte tables
-  {
-    const int nM = ld_cg(&ctrl->cnt[p][1]);
-    const int32_t* list = sel(p, (const int32_t*)a.wl_m[0], (const int32_t*)a.wl_m[1]);
-    int32_t* out = sel(p ^ 1, a.wl_m[0], a.wl_m[1]);
-    int i = gw * 4 + g;
-    int32_t v = i < nM ? ld_cg(list + i) : -1;
-    int64_t s = v >= 0 ? ldg_i64(a.row_ptr + v) : 0, e = v >= 0 ? ldg_i64(a.row_ptr + v + 1) : 0;
-    for (int base = gw * 4; base < nM; base += NW * 4) {
-      const int in = i + NW * 4;
-      const int32_t vn = in < nM ? ld_cg(list + in) : -1;
-      const int64_t sn = vn >= 0 ? ldg_i64(a.row_ptr + vn) : 0;
-      const int64_t en = vn >= 0 ? ldg_i64(a.row_ptr + vn + 1) : 0;
-      if (sn + 32 * gl < en) prefetch_l2(a.col_idx + sn + 32 * gl);  // next row, 1 line / lane
-      bool push = false;
-      process_group<TB, Persist, C, kK1, true>(a, v, s, e, X, Y, wtbl + g * kMedTbl, gl, gmask,
-                                               push, edges[1]);
-      warp_push(push, v, out, &ctrl->cnt[p ^ 1][1]);
-      i = in;
-      v = vn;
-      s = sn;
-      e = en;
-    }
-  }
+  bin01<TB, Persist, C, kK1, true>(
+      a, k, sel(p, (const int32_t*)a.wl_m[0], (const int32_t*)a.wl_m[1]),
+      ld_cg(&ctrl->cnt[p][1]), sel(p ^ 1, a.wl_m[0], a.wl_m[1]), &ctrl->cnt[p ^ 1][1], X, Y,
+      wsm, gw, NW, lane, edges[1], entries[1]);
   // ---- bin 0: four vertices per warp, register masks
-  {
-    const int nT = ld_cg(&ctrl->cnt[p][0]);
-    const int32_t* list = sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]);
-    int32_t* out = sel(p ^ 1, a.wl_t[0], a.wl_t[1]);
-    int i = gw * 4 + g;
-    int32_t v = i < nT ? ld_cg(list + i) : -1;
-    int64_t s = v >= 0 ? ldg_i64(a.row_ptr + v) : 0, e = v >= 0 ? ldg_i64(a.row_ptr + v + 1) : 0;
-    for (int base = gw * 4; base < nT; base += NW * 4) {
-      const int in = i + NW * 4;
-      const int32_t vn = in < nT ? ld_cg(list + in) : -1;
-      const int64_t sn = vn >= 0 ? ldg_i64(a.row_ptr + vn) : 0;
-      const int64_t en = vn >= 0 ? ldg_i64(a.row_ptr + vn + 1) : 0;
-      bool push = false;
-      process_group<TB, Persist, C, kK0, false>(a, v, s, e, X, Y, nullptr, gl, gmask, push,
-                                                edges[0]);
-      warp_push(push, v, out, &ctrl->cnt[p ^ 1][0]);
-      i = in;
-      v = vn;
-      s = sn;
-      e = en;
-    }
-  }
+  bin01<TB, Persist, C, kK0, false>(
+      a, k, sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]),
+      ld_cg(&ctrl->cnt[p][0]), sel(p ^ 1, a.wl_t[0], a.wl_t[1]), &ctrl->cnt[p ^ 1][0], X, Y,
+      wsm, gw, NW, lane, edges[0], entries[0]);
 }
 
-// Block reduction of the three per-thread edge counters, one atomicAdd each per block.
-__device__ __forceinline__ void block_add3(unsigned long long (&x)[kBins], Ctrl* ctrl) {
-  __shared__ unsigned long long red[kBins][kBlock / 32];
+// Block reduction of the per-thread counters, one atomicAdd each per block.
+__device__ __forceinline__ void block_add6(unsigned long long (&x)[kBins],
+                                           unsigned long long (&y)[kBins], Ctrl* ctrl) {
+  __shared__ unsigned long long red[2 * kBins][kWarps];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
 #pragma unroll
-  for (int q = 0; q < kBins; ++q) {
-    unsigned long long y = x[q];
+  for (int q = 0; q < 2 * kBins; ++q) {
+    unsigned long long z = q < kBins ? x[q] : y[q - kBins];
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) y += __shfl_xor_sync(0xffffffffu, y, o);
-    if (lane == 0) red[q][wid] = y;
+    for (int o = 16; o > 0; o >>= 1) z += __shfl_xor_sync(0xffffffffu, z, o);
+    if (lane == 0) red[q][wid] = z;
   }
   __syncthreads();
   if (wid == 0) {
 #pragma unroll
-    for (int q = 0; q < kBins; ++q) {
-      unsigned long long y = lane < (kBlock / 32) ? red[q][lane] : 0ull;
+    for (int q = 0; q < 2 * kBins; ++q) {
+      unsigned long long z = lane < kWarps ? red[q][lane] : 0ull;
 #pragma unroll
-      for (int o = 16; o > 0; o >>= 1) y += __shfl_xor_sync(0xffffffffu, y, o);
-      if (lane == 0 && y) atomicAdd(&ctrl->edges_acc[q], y);
+      for (int o = 16; o > 0; o >>= 1) z += __shfl_xor_sync(0xffffffffu, z, o);
+      if (lane == 0 && z) {
+        if (q < kBins) atomicAdd(&ctrl->edges_acc[q], z);
+        else atomicAdd(&ctrl->entries_acc[q - kBins], z);
+      }
     }
   }
 }
@@ -599,9 +922,11 @@ __device__ __forceinline__ void advance_body(Ctrl* ctrl, bool first) {
   for (int q = 0; q < kBins; ++q) {
     c->verts_total[q] += (unsigned long long)vin[q];
     c->edges_total[q] += c->edges_acc[q];
+    c->entries_total[q] += c->entries_acc[q];
     c->pushes_total[q] += (unsigned long long)vout[q];
     e_all += c->edges_acc[q];
     c->edges_acc[q] = 0;
+    c->entries_acc[q] = 0;
     tot_in += vin[q];
   }
   c->items_total += (unsigned long long)c->cnt[p][2];
@@ -626,22 +951,35 @@ __global__ void k_advance(Ctrl* ctrl, int first) {
   if (threadIdx.x == 0 && blockIdx.x == 0) advance_body(ctrl, first != 0);
 }
 
-__device__ __forceinline__ void zero_smem(uint8_t* p, int bytes) {
-  uint4* q = reinterpret_cast<uint4*>(p);
-  for (int i = threadIdx.x; i < bytes / 16; i += blockDim.x) q[i] = make_uint4(0, 0, 0, 0);
+// Kernel prologue: zero the warp tables, initialise the warp's two TMA mbarriers.
+template <class C>
+__device__ __forceinline__ uint8_t* warp_smem_init(uint8_t* smem) {
+  const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  uint8_t* wsm = smem + wid * WarpSmem<C>::kBytes;
+  clear_bytes(wsm + WarpSmem<C>::kBuf, kTblBytes / 32, lane);
+  if constexpr (packed<C>()) {
+    if (lane == 0) {
+      uint64_t* bars = reinterpret_cast<uint64_t*>(wsm + WarpSmem<C>::kBuf + kTblBytes);
+      mbar_init(bars + 0, 1);  // bin-2 stages: one elected arrival per phase
+      mbar_init(bars + 1, 1);
+      mbar_init_fence();
+    }
+  }
+  __syncthreads();
+  return wsm;
 }
 
 // One pass per launch (host / graph loop modes); k_advance follows it on the stream.
 template <int TB, class C>
-__global__ void __launch_bounds__(kBlock, 3) k_round(RoundArgs<C> a) {
-  __shared__ __align__(16) uint8_t tbl[kBlock / 32][kWarpTbl];
+__global__ void __launch_bounds__(kBlock, kMinBlocks<C>) k_round(RoundArgs<C> a) {
+  extern __shared__ __align__(16) uint8_t dsmem[];
   Ctrl* ctrl = a.ctrl;
   if (!ctrl->active) return;  // uniform across the grid
-  zero_smem(&tbl[0][0], sizeof(tbl));
-  __syncthreads();
-  unsigned long long edges[kBins] = {0, 0, 0};
-  round_body<TB, false, C>(a, ctrl->k, tbl[threadIdx.x >> 5], edges);
-  block_add3(edges, ctrl);
+  uint8_t* wsm = warp_smem_init<C>(dsmem);
+  unsigned long long edges[kBins] = {0, 0, 0}, entries[kBins] = {0, 0, 0};
+  uint32_t ph = 0;
+  round_body<TB, false, C>(a, ctrl->k, wsm, edges, entries, ph);
+  block_add6(edges, entries, ctrl);
 }
 
 // Grid-wide barrier whose last arriving block runs advance_body (persistent kernel).
@@ -668,27 +1006,27 @@ __device__ __forceinline__ void grid_sync_advance(Ctrl* ctrl) {
 
 // All rounds in one cooperative launch (every block resident): pass, barrier+advance, ...
 template <int TB, class C>
-__global__ void __launch_bounds__(kBlock, 3) k_persistent(RoundArgs<C> a) {
-  __shared__ __align__(16) uint8_t tbl[kBlock / 32][kWarpTbl];
+__global__ void __launch_bounds__(kBlock, kMinBlocks<C>) k_persistent(RoundArgs<C> a) {
+  extern __shared__ __align__(16) uint8_t dsmem[];
   Ctrl* ctrl = a.ctrl;
-  zero_smem(&tbl[0][0], sizeof(tbl));
-  __syncthreads();
+  uint8_t* wsm = warp_smem_init<C>(dsmem);
+  uint32_t ph = 0;  // mbarrier phase bits of the warp's two TMA stages
   for (;;) {
     const int active = ld_cg(&ctrl->active);
     const int k = ld_cg(&ctrl->k);
     if (!active) break;  // uniform: read after the barrier by every thread
-    unsigned long long edges[kBins] = {0, 0, 0};
-    round_body<TB, true, C>(a, k, tbl[threadIdx.x >> 5], edges);
-    block_add3(edges, ctrl);
+    unsigned long long edges[kBins] = {0, 0, 0}, entries[kBins] = {0, 0, 0};
+    round_body<TB, true, C>(a, k, wsm, edges, entries, ph);
+    block_add6(edges, entries, ctrl);
     grid_sync_advance(ctrl);
   }
 }
 
-// Widen the final u16 colors into the caller's int32 output.
-__global__ void k_widen(const uint16_t* __restrict__ src, int32_t* __restrict__ dst, int64_t n) {
+// Final colors (packed words) into the caller's int32 output.
+__global__ void k_unpack(const uint32_t* __restrict__ src, int32_t* __restrict__ dst, int64_t n) {
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
        i += (int64_t)gridDim.x * blockDim.x)
-    dst[i] = (int32_t)src[i];
+    dst[i] = (int32_t)(src[i] & 0xffffu);
 }
 
 }  // namespace sgr
