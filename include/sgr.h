@@ -120,6 +120,7 @@ typedef struct {
   int64_t bin_vertices[3];           /* rounds >= 2, per degree bin (thread/group/chunk) */
   int64_t bin_edges[3];
   int64_t chunk_items;               /* warp work items processed in the chunk bin       */
+  int64_t bin_warp_cycles[3];        /* SM cycles warps spent in each bin (all rounds)   */
   int32_t grid_blocks;               /* blocks of the round kernel                        */
   int32_t color_bits;                /* width the coloring finished with (16 or 32)       */
 } sgr_stats;

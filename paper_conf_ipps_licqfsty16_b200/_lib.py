@@ -38,7 +38,8 @@ class Stats(ctypes.Structure):
                 ("kernel_launches", ctypes.c_int64 * SGR_K_COUNT),
                 ("kernel_bytes", ctypes.c_int64 * SGR_K_COUNT),
                 ("bin_vertices", ctypes.c_int64 * 3), ("bin_edges", ctypes.c_int64 * 3),
-                ("chunk_items", ctypes.c_int64), ("grid_blocks", ctypes.c_int32),
+                ("chunk_items", ctypes.c_int64), ("bin_warp_cycles", ctypes.c_int64 * 3),
+                ("grid_blocks", ctypes.c_int32),
                 ("color_bits", ctypes.c_int32)]
 
     def as_dict(self) -> dict:
@@ -51,6 +52,7 @@ class Stats(ctypes.Structure):
         d["bin_vertices"] = dict(zip(BINS, list(self.bin_vertices)))
         d["bin_edges"] = dict(zip(BINS, list(self.bin_edges)))
         d["chunk_items"] = self.chunk_items
+        d["bin_warp_cycles"] = dict(zip(BINS, list(self.bin_warp_cycles)))
         d["grid_blocks"] = self.grid_blocks
         d["color_bits"] = self.color_bits
         return d

@@ -54,7 +54,7 @@ Resolved resolve_opts(const sgr_opts* o, int64_t n) {
   r.loop_mode = (o->loop_mode == SGR_LOOP_HOST || o->loop_mode == SGR_LOOP_GRAPH)
                     ? o->loop_mode : SGR_LOOP_PERSISTENT;
   r.color_bits = o->color_bits == 32 ? 32 : 16;
-  r.small_max = o->bin_small_max > 0 ? std::min(o->bin_small_max, 62) : 32;
+  r.small_max = o->bin_small_max > 0 ? std::min(o->bin_small_max, kMaxSmall) : kMaxSmall;
   r.med_max = o->bin_med_max > 0 ? std::min(o->bin_med_max, kMaxMed) : kMaxMed;
   r.med_max = std::max(r.med_max, r.small_max);
   r.stream = (cudaStream_t)o->stream;
@@ -303,6 +303,7 @@ void fill_stats(const Ctrl& c, int64_t n, int64_t nnz, sgr_stats* st) {
     st->entries_read += (int64_t)c.entries_total[q];
   }
   st->chunk_items = (int64_t)c.items_total;
+  for (int q = 0; q < kBins; ++q) st->bin_warp_cycles[q] = (int64_t)c.bin_cycles[q];
   st->rounds = c.k - 1;
   st->num_colors = c.max_color;
   st->vertices_processed = n + vpass;

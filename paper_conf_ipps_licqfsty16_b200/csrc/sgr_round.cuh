@@ -11,8 +11,9 @@
 //
 // The pass is bound by the rate of scattered color gathers (~1 distinct 128-byte line per
 // SM-cycle, tools/gather_bench.cu) and by load latency. Work binning is static:
-//   bin 0  deg <= small_max (<= 62): 8 lanes per vertex (coalesced row reads), <= 8 entries
-//          per lane, all loads issued first, u64 register mask per lane, OR-reduced in-group
+//   bin 0  deg <= small_max (<= 32): 4 lanes per vertex (coalesced row reads), <= 8 entries
+//          per lane, the next vertex's row loaded while the current one's gathers are in
+//          flight, u64 register mask per lane, OR-reduced in-group
 //   bin 1  deg <= med_max (<= 256): 8 lanes per vertex, <= 32 entries per lane, 512-byte
 //          forbidden table (one byte per color) in shared memory
 //   bin 2  larger rows, one warp per chunk of <= kChunk entries. A vertex with several
@@ -44,7 +45,10 @@ constexpr int kBins = 3;
 constexpr int kBlock = 256;             // threads per block (8 warps)
 constexpr int kWarps = kBlock / 32;
 constexpr int kGroup = 8;               // lanes per vertex in bins 0 and 1
-constexpr int kK0 = 8;                  // entries per lane, bin 0 (8 x 8 = 64 >= 62)
+constexpr int kG0 = 4;                  // lanes per vertex in bin 0
+constexpr int kK0 = 8;                  // entries per lane, bin 0 (4 x 8 = 32 = max small)
+constexpr int kMaxSmall = kG0 * kK0;    // 32
+constexpr int kPushBuf = 64;            // per-warp push buffer (bins 0/1), flushed at >= 32
 constexpr int kK1 = 32;                 // entries per lane, bin 1 (8 x 32 = 256)
 constexpr int kMaxMed = kGroup * kK1;   // 256
 constexpr int kMedTbl = 512;            // bin-1 table bytes (colors < 512 > 257)
@@ -65,7 +69,9 @@ template <class C>
 constexpr int kMinBlocks = packed<C>() ? 2 : 3;
 template <class C> struct WarpSmem {
   static constexpr int kBuf = packed<C>() ? 2 * kStage : 0;
-  static constexpr int kBytes = kBuf + kTblBytes + 16;  // + 2 mbarriers
+  static constexpr int kPush = kBuf + kTblBytes;         // push buffer (kPushBuf int32)
+  static constexpr int kBars = kPush + kPushBuf * 4;     // 2 mbarriers
+  static constexpr int kBytes = kBars + 16;
 };
 
 // Device-resident loop state (in the workspace).
@@ -91,6 +97,7 @@ struct Ctrl {
   unsigned long long entries_total[kBins + 1];
   unsigned long long pushes_total[kBins + 1];
   unsigned long long items_total;
+  unsigned long long bin_cycles[kBins];   // warp-cycles spent in each bin (SM clock)
   int32_t* round_sizes;
   int64_t* round_edges;
 };
@@ -499,7 +506,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
   int32_t* bufs = reinterpret_cast<int32_t*>(wsm);
   uint8_t* tbl_all = wsm + WarpSmem<C>::kBuf;
   uint8_t* tbl_drop = tbl_all + kBigTbl;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(wsm + WarpSmem<C>::kBuf + kTblBytes);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(wsm + WarpSmem<C>::kBars);
 
   auto issue = [&](const ChunkHdr& h, int st) {  // lane 0 only
     const int64_t cs = h.s + (int64_t)h.c * kChunk;
@@ -531,44 +538,54 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
     const int inn = in + NW;
     const int64_t it_nn = inn < nC ? __ldcg(items + inn) : 0;
 
-    // ---- chunk `cur` in stage st
+    // ---- chunk `cur` in stage st: slots [off0, off0 + cnt) of the 16-byte-aligned window
     const int32_t v = cur.v;
     const int64_t cs = cur.s + (int64_t)cur.c * kChunk;
-    const int64_t ce = min(cur.s + (int64_t)cur.len, cs + kChunk);
-    const int64_t w0 = cs & ~(int64_t)3;
+    const int32_t cnt = (int32_t)(min(cur.s + (int64_t)cur.len, cs + kChunk) - cs);
+    const int32_t off0 = (int32_t)(cs & 3);
+    const int32_t nslots = off0 + cnt;
+    const int32_t nb = (nslots + 255) >> 8;  // batches of 256 slots = 2 int4 per lane
     const int32_t nch = num_chunks(cur.len);
     const int32_t xv = cval<C>(ldraw<Persist>(X + v));
+    const uint32_t klive = (uint32_t)k << 16;  // raw >= klive <=> neighbour still in W_k
     mbar_wait(bars + st, (ph >> st) & 1u);
     ph ^= 1u << st;
     const int4* b4 = reinterpret_cast<const int4*>(bufs + st * (kStage / 4));
-    uint32_t cc[32];
-    uint32_t valid = 0, lb = 0;
-#pragma unroll
-    for (int q = 0; q < 8; ++q) {
-      const int4 t4 = b4[lane + 32 * q];
-      const int32_t wq[4] = {t4.x, t4.y, t4.z, t4.w};
-#pragma unroll
-      for (int t = 0; t < 4; ++t) {
-        const int64_t pos = w0 + 4 * (lane + 32 * q) + t;
-        const bool ok = pos >= cs && pos < ce;
-        valid |= ok ? (1u << (4 * q + t)) : 0u;
-        lb |= (ok && lose<TB>(v, wq[t])) ? (1u << (4 * q + t)) : 0u;
-        cc[4 * q + t] = ok ? ldraw<Persist>(X + wq[t]) : 0u;
-      }
-    }
     bool conf = false;
-    uint32_t lv = 0;  // live bits
+    uint32_t lv = 0;  // live bits: bit 8 b + 4 qq + t
+    for (int bb = 0; bb < nb; ++bb) {
+      int32_t id[8];
+      uint32_t raw[8];
+      uint32_t okm = 0;
 #pragma unroll
-    for (int u = 0; u < 32; ++u) {
-      const int32_t col = cval<C>(cc[u]);
-      const bool live = (int32_t)(cc[u] >> 16) >= k;
-      const bool ok = (valid >> u) & 1u;
-      if ((uint32_t)col < (uint32_t)kBigTbl) {
-        tbl_all[col] = 1;
-        if (ok && !live) tbl_drop[col] = 1;
+      for (int qq = 0; qq < 2; ++qq) {
+        const int q = 2 * bb + qq;
+        const int4 t4 = b4[lane + 32 * q];
+        id[4 * qq + 0] = t4.x;
+        id[4 * qq + 1] = t4.y;
+        id[4 * qq + 2] = t4.z;
+        id[4 * qq + 3] = t4.w;
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+          const int32_t r = 4 * (lane + 32 * q) + t;
+          okm |= ((uint32_t)(r - off0) < (uint32_t)cnt) ? (1u << (4 * qq + t)) : 0u;
+        }
       }
-      conf |= ok && col == xv && ((lb >> u) & 1u);
-      lv |= (ok && live) ? (1u << u) : 0u;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) raw[j] = ((okm >> j) & 1u) ? ldraw<Persist>(X + id[j]) : 0u;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        if ((okm >> j) & 1u) {
+          // colors >= 1023 are clamped onto byte 1023; a first fit of 1023 or more is
+          // recomputed exactly from the full row (warp_first_fit_rescan)
+          const uint32_t ci = min(raw[j] & 0xffffu, (uint32_t)(kBigTbl - 1));
+          const bool live = raw[j] >= klive;
+          tbl_all[ci] = 1;
+          if (!live) tbl_drop[ci] = 1;
+          conf |= (int32_t)(raw[j] & 0xffffu) == xv && lose<TB>(v, id[j]);
+          lv |= live ? (1u << (8 * bb + j)) : 0u;
+        }
+      }
     }
     // next-next header: the item id has arrived by now
     ChunkHdr nn;
@@ -581,47 +598,36 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
       nn.len = ld_cg(len_cur + nn.v);
     }
     if (lane == 0) {
-      entries += (unsigned long long)(ce - cs);
+      entries += (unsigned long long)cnt;
       if (cur.c == 0) edges += (unsigned long long)(ldg_i64(a.row_ptr + v + 1) - cur.s);
     }
     __syncwarp();
     const bool any = __any_sync(0xffffffffu, conf);
-
-    // live-entry compaction offsets: per int4 slot q, lane counts packed 8 bits per slot
-    uint32_t pk0 = 0, pk1 = 0;
-#pragma unroll
-    for (int q = 0; q < 4; ++q) pk0 |= (uint32_t)__popc((lv >> (4 * q)) & 0xfu) << (8 * q);
-#pragma unroll
-    for (int q = 0; q < 4; ++q) pk1 |= (uint32_t)__popc((lv >> (4 * (q + 4))) & 0xfu) << (8 * q);
-    uint32_t in0 = pk0, in1 = pk1;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t t0 = __shfl_up_sync(0xffffffffu, in0, o);
-      const uint32_t t1 = __shfl_up_sync(0xffffffffu, in1, o);
-      if (lane >= o) {
-        in0 += t0;
-        in1 += t1;
-      }
-    }
-    const uint32_t tot0 = __shfl_sync(0xffffffffu, in0, 31);
-    const uint32_t tot1 = __shfl_sync(0xffffffffu, in1, 31);
-    const uint32_t ex0 = in0 - pk0, ex1 = in1 - pk1;
-    uint32_t live_total = 0;
-#pragma unroll
-    for (int q = 0; q < 4; ++q) live_total += ((tot0 >> (8 * q)) & 0xffu) + ((tot1 >> (8 * q)) & 0xffu);
+    const uint32_t live_total = (uint32_t)__reduce_add_sync(0xffffffffu, (uint32_t)__popc(lv));
     const int32_t* sbuf = bufs + st * (kStage / 4);
+    // compacted live list in window order: per batch, per int4 slot q, lanes in order
     auto write_live = [&](int32_t* base) {
       uint32_t qb = 0;
+      for (int bb = 0; bb < nb; ++bb) {
+        const uint32_t pk = (uint32_t)__popc((lv >> (8 * bb)) & 0xfu) |
+                            ((uint32_t)__popc((lv >> (8 * bb + 4)) & 0xfu) << 16);
+        uint32_t inc = pk;
 #pragma unroll
-      for (int q = 0; q < 8; ++q) {
-        const uint32_t sh = 8 * (q & 3);
-        const uint32_t tq = ((q < 4 ? tot0 : tot1) >> sh) & 0xffu;
-        uint32_t off = qb + (((q < 4 ? ex0 : ex1) >> sh) & 0xffu);
-        const int32_t* sq = sbuf + 4 * (lane + 32 * q);
+        for (int o = 1; o < 32; o <<= 1) {
+          const uint32_t tt = __shfl_up_sync(0xffffffffu, inc, o);
+          if (lane >= o) inc += tt;
+        }
+        const uint32_t tot = __shfl_sync(0xffffffffu, inc, 31);
+        const uint32_t ex = inc - pk;
 #pragma unroll
-        for (int t = 0; t < 4; ++t)
-          if ((lv >> (4 * q + t)) & 1u) base[off++] = sq[t];
-        qb += tq;
+        for (int qq = 0; qq < 2; ++qq) {
+          uint32_t off = qb + ((ex >> (16 * qq)) & 0xffffu);
+          const int32_t* sq = sbuf + 4 * (lane + 32 * (2 * bb + qq));
+#pragma unroll
+          for (int t = 0; t < 4; ++t)
+            if ((lv >> (8 * bb + 4 * qq + t)) & 1u) base[off++] = sq[t];
+          qb += (tot >> (16 * qq)) & 0xffffu;
+        }
       }
     };
 
@@ -632,9 +638,9 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
         const uint32_t fo = ld_cg(fx + lane);
         const uint32_t word = tbl_bits32(tbl_all, lane) | fo | (lane == 0 ? 1u : 0u);
         int32_t tent = bits_first_free(word);
-        if (tent < 0) {
+        if (tent < 0 || tent >= kBigTbl - 1) {  // beyond the exact range of the table
           tent = warp_first_fit_rescan<Persist>(a.col_idx, X, cur.s,
-                                                ldg_i64(a.row_ptr + v + 1), kBigTbl, lane);
+                                                ldg_i64(a.row_ptr + v + 1), kBigTbl - 1, lane);
         }
         const uint32_t drop = tbl_bits32(tbl_drop, lane);
         if (drop & ~fo) fx[lane] = fo | drop;
@@ -673,9 +679,9 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
         int32_t tent = 0;
         if (conf_all) {
           tent = bits_first_free(word);
-          if (tent < 0) {
+          if (tent < 0 || tent >= kBigTbl - 1) {  // beyond the exact range of the table
             tent = warp_first_fit_rescan<Persist>(a.col_idx, X, cur.s,
-                                                  ldg_i64(a.row_ptr + v + 1), kBigTbl, lane);
+                                                  ldg_i64(a.row_ptr + v + 1), kBigTbl - 1, lane);
           }
         }
         int32_t ob = 0, nch2 = 0;
@@ -770,6 +776,108 @@ __device__ __forceinline__ void process_group(const RoundArgs<C>& a, int k, int3
   push = (v >= 0) && any && gl == 0;
 }
 
+// Per-warp buffered worklist push (bins 0/1): lanes with `pred` append `v` to a shared-
+// memory buffer; when 32 or more are pending the warp flushes them with ONE atomicAdd on the
+// global counter and a contiguous store. All 32 lanes must call; `pending` is warp-uniform.
+__device__ __forceinline__ void push_buffered(bool pred, int32_t v, int32_t* pbuf, int& pending,
+                                              int32_t* list, int32_t* count, int lane) {
+  const unsigned m = __ballot_sync(0xffffffffu, pred);
+  if (pred) pbuf[pending + __popc(m & ((1u << lane) - 1u))] = v;
+  pending += __popc(m);
+  if (pending >= 32) {
+    __syncwarp();
+    int base = 0;
+    if (lane == 0) base = atomicAdd(count, pending);
+    base = __shfl_sync(0xffffffffu, base, 0);
+    for (int t = lane; t < pending; t += 32) list[base + t] = pbuf[t];
+    __syncwarp();
+    pending = 0;
+  }
+}
+__device__ __forceinline__ void push_flush(int32_t* pbuf, int& pending, int32_t* list,
+                                           int32_t* count, int lane) {
+  if (pending == 0) return;
+  __syncwarp();
+  int base = 0;
+  if (lane == 0) base = atomicAdd(count, pending);
+  base = __shfl_sync(0xffffffffu, base, 0);
+  for (int t = lane; t < pending; t += 32) list[base + t] = pbuf[t];
+  __syncwarp();
+  pending = 0;
+}
+
+// Bin 0 driver: 4-lane groups, 8 vertices per warp per step; list entries and row offsets
+// prefetched two steps ahead, the row entries one step ahead (so they are in flight while
+// the current vertices' color gathers are), pushes buffered per warp.
+template <int TB, bool Persist, class C>
+__device__ __forceinline__ void bin0(const RoundArgs<C>& a, int k, const int32_t* list, int nX,
+                                     int32_t* out, int32_t* out_cnt, const C* X, C* Y,
+                                     uint8_t* wsm, int gw, int NW, int lane,
+                                     unsigned long long& edges, unsigned long long& entries) {
+  constexpr int G = kG0, VPW = 32 / kG0;
+  if (gw * VPW >= nX) return;
+  const int g = lane / G, gl = lane % G;
+  const unsigned gmask = ((1u << G) - 1u) << (g * G);
+  int32_t* pbuf = reinterpret_cast<int32_t*>(wsm + WarpSmem<C>::kPush);
+  int pending = 0;
+  const int step = NW * VPW;
+  auto load_row = [&](int32_t vv, int64_t ss, int64_t ee, int32_t (&w)[kK0]) {
+#pragma unroll
+    for (int u = 0; u < kK0; ++u) {
+      const int64_t j = ss + gl + G * u;
+      w[u] = (vv >= 0 && j < ee) ? __ldg(a.col_idx + j) : -1;
+    }
+  };
+  int i = gw * VPW + g;
+  int32_t v = i < nX ? ld_cg(list + i) : -1;
+  int64_t s = v >= 0 ? ldg_i64(a.row_ptr + v) : 0, e = v >= 0 ? ldg_i64(a.row_ptr + v + 1) : 0;
+  int32_t w[kK0];
+  load_row(v, s, e, w);
+  int32_t v1 = i + step < nX ? ld_cg(list + i + step) : -1;
+  int64_t s1 = v1 >= 0 ? ldg_i64(a.row_ptr + v1) : 0, e1 = v1 >= 0 ? ldg_i64(a.row_ptr + v1 + 1) : 0;
+  for (int base = gw * VPW; base < nX; base += step) {
+    const int32_t v2 = i + 2 * step < nX ? ld_cg(list + i + 2 * step) : -1;
+    const int32_t xv = v >= 0 ? ldc<Persist>(X + v) : 0;
+    uint32_t lb = 0;
+#pragma unroll
+    for (int u = 0; u < kK0; ++u) lb |= (w[u] >= 0 && lose<TB>(v, w[u])) ? (1u << u) : 0u;
+    int32_t c[kK0];
+#pragma unroll
+    for (int u = 0; u < kK0; ++u) c[u] = (w[u] >= 0) ? ldc<Persist>(X + w[u]) : 0;
+    int32_t wn[kK0];
+    load_row(v1, s1, e1, wn);  // next vertex's row, in flight with the gathers above
+    bool conf = false;
+    uint64_t mask = 1ull;  // bit 0 = color 0, never a candidate
+#pragma unroll
+    for (int u = 0; u < kK0; ++u) {
+      mask |= ((uint32_t)c[u] < 64u) ? (1ull << c[u]) : 0ull;
+      conf |= (c[u] == xv) & ((lb >> u) & 1u);
+    }
+#pragma unroll
+    for (int o = G / 2; o > 0; o >>= 1) mask |= __shfl_xor_sync(0xffffffffu, mask, o);
+    const bool any = (__ballot_sync(0xffffffffu, conf) & gmask) != 0u;
+    if (v >= 0 && gl == 0) {
+      const int32_t tent = __ffsll((long long)~mask) - 1;  // deg <= 32 => first fit <= 33
+      Y[v] = any ? cpack<C>(tent, k + 1, a.ctrl) : cpack<C>(xv, k, a.ctrl);
+      edges += (unsigned long long)(e - s);
+      entries += (unsigned long long)(e - s);
+    }
+    push_buffered(v >= 0 && any && gl == 0, v, pbuf, pending, out, out_cnt, lane);
+    const int64_t s2 = v2 >= 0 ? ldg_i64(a.row_ptr + v2) : 0;
+    const int64_t e2 = v2 >= 0 ? ldg_i64(a.row_ptr + v2 + 1) : 0;
+    i += step;
+    v = v1;
+    s = s1;
+    e = e1;
+#pragma unroll
+    for (int u = 0; u < kK0; ++u) w[u] = wn[u];
+    v1 = v2;
+    s1 = s2;
+    e1 = e2;
+  }
+  push_flush(pbuf, pending, out, out_cnt, lane);
+}
+
 // Bins 0/1 driver: warp w takes list positions 4w + g, 4(w + NW) + g, ... (g = group); the
 // next position's list entry and row offsets are prefetched, its row warmed into L2.
 template <int TB, bool Persist, class C, int K, bool Table>
@@ -780,6 +888,8 @@ __device__ __forceinline__ void bin01(const RoundArgs<C>& a, int k, const int32_
   const int g = lane >> 3, gl = lane & 7;
   const unsigned gmask = 0xffu << (g * 8);
   uint8_t* gtbl = wsm + WarpSmem<C>::kBuf + g * kMedTbl;
+  int32_t* pbuf = reinterpret_cast<int32_t*>(wsm + WarpSmem<C>::kPush);
+  int pending = 0;
   const int step = NW * 4;
   int i = gw * 4 + g;
   int32_t v = i < nX ? ld_cg(list + i) : -1;
@@ -793,12 +903,13 @@ __device__ __forceinline__ void bin01(const RoundArgs<C>& a, int k, const int32_
     bool push = false;
     if (v >= 0 && gl == 0) entries += (unsigned long long)(e - s);
     process_group<TB, Persist, C, K, Table>(a, k, v, s, e, X, Y, gtbl, gl, gmask, push, edges);
-    warp_push(push, v, out, out_cnt);
+    push_buffered(push, v, pbuf, pending, out, out_cnt, lane);
     i = in;
     v = vn;
     s = sn;
     e = en;
   }
+  push_flush(pbuf, pending, out, out_cnt, lane);
 }
 
 // One fused pass F_k over all three bins; every warp of the grid calls it. Static
@@ -808,7 +919,7 @@ template <int TB, bool Persist, class C>
 __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, uint8_t* wsm,
                                            unsigned long long (&edges)[kBins],
                                            unsigned long long (&entries)[kBins],
-                                           uint32_t& ph) {
+                                           uint32_t& ph, unsigned long long (&cyc)[kBins]) {
   Ctrl* ctrl = a.ctrl;
   const int p = k & 1;
   const int lane = threadIdx.x & 31;
@@ -818,6 +929,7 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, uint8_t
   C* Y = sel(k & 1, a.col[0], a.col[1]);
   uint8_t* wtbl = wsm + WarpSmem<C>::kBuf;
   (void)wtbl;
+  long long t0 = clock64();
   // ---- bin 2
   if constexpr (packed<C>()) {
     bin2_trimmed<TB, Persist>(a, k, p, X, Y, wsm, gw, NW, lane, edges[2], entries[2], ph);
@@ -850,16 +962,21 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, uint8_t
       e = en;
     }
   }
+  long long t1 = clock64();
+  cyc[2] += (unsigned long long)(t1 - t0);
   // ---- bin 1: four vertices per warp (one per 8-lane group), 512-byte tables
   bin01<TB, Persist, C, kK1, true>(
       a, k, sel(p, (const int32_t*)a.wl_m[0], (const int32_t*)a.wl_m[1]),
       ld_cg(&ctrl->cnt[p][1]), sel(p ^ 1, a.wl_m[0], a.wl_m[1]), &ctrl->cnt[p ^ 1][1], X, Y,
       wsm, gw, NW, lane, edges[1], entries[1]);
-  // ---- bin 0: four vertices per warp, register masks
-  bin01<TB, Persist, C, kK0, false>(
+  long long t2 = clock64();
+  cyc[1] += (unsigned long long)(t2 - t1);
+  // ---- bin 0: eight vertices per warp, register masks
+  bin0<TB, Persist, C>(
       a, k, sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]),
       ld_cg(&ctrl->cnt[p][0]), sel(p ^ 1, a.wl_t[0], a.wl_t[1]), &ctrl->cnt[p ^ 1][0], X, Y,
       wsm, gw, NW, lane, edges[0], entries[0]);
+  cyc[0] += (unsigned long long)(clock64() - t2);
 }
 
 // Block reduction of the per-thread counters, one atomicAdd each per block.
@@ -959,7 +1076,7 @@ __device__ __forceinline__ uint8_t* warp_smem_init(uint8_t* smem) {
   clear_bytes(wsm + WarpSmem<C>::kBuf, kTblBytes / 32, lane);
   if constexpr (packed<C>()) {
     if (lane == 0) {
-      uint64_t* bars = reinterpret_cast<uint64_t*>(wsm + WarpSmem<C>::kBuf + kTblBytes);
+      uint64_t* bars = reinterpret_cast<uint64_t*>(wsm + WarpSmem<C>::kBars);
       mbar_init(bars + 0, 1);  // bin-2 stages: one elected arrival per phase
       mbar_init(bars + 1, 1);
       mbar_init_fence();
@@ -977,9 +1094,12 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks<C>) k_round(RoundArgs<C> a)
   if (!ctrl->active) return;  // uniform across the grid
   uint8_t* wsm = warp_smem_init<C>(dsmem);
   unsigned long long edges[kBins] = {0, 0, 0}, entries[kBins] = {0, 0, 0};
+  unsigned long long cyc[kBins] = {0, 0, 0};
   uint32_t ph = 0;
-  round_body<TB, false, C>(a, ctrl->k, wsm, edges, entries, ph);
+  round_body<TB, false, C>(a, ctrl->k, wsm, edges, entries, ph, cyc);
   block_add6(edges, entries, ctrl);
+  if ((threadIdx.x & 31) == 0)
+    for (int q = 0; q < kBins; ++q) atomicAdd(&ctrl->bin_cycles[q], cyc[q]);
 }
 
 // Grid-wide barrier whose last arriving block runs advance_body (persistent kernel).
@@ -1011,15 +1131,18 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks<C>) k_persistent(RoundArgs<
   Ctrl* ctrl = a.ctrl;
   uint8_t* wsm = warp_smem_init<C>(dsmem);
   uint32_t ph = 0;  // mbarrier phase bits of the warp's two TMA stages
+  unsigned long long cyc[kBins] = {0, 0, 0};
   for (;;) {
     const int active = ld_cg(&ctrl->active);
     const int k = ld_cg(&ctrl->k);
     if (!active) break;  // uniform: read after the barrier by every thread
     unsigned long long edges[kBins] = {0, 0, 0}, entries[kBins] = {0, 0, 0};
-    round_body<TB, true, C>(a, k, wsm, edges, entries, ph);
+    round_body<TB, true, C>(a, k, wsm, edges, entries, ph, cyc);
     block_add6(edges, entries, ctrl);
     grid_sync_advance(ctrl);
   }
+  if ((threadIdx.x & 31) == 0)
+    for (int q = 0; q < kBins; ++q) atomicAdd(&ctrl->bin_cycles[q], cyc[q]);
 }
 
 // Final colors (packed words) into the caller's int32 output.

@@ -107,7 +107,7 @@ def test_degree_bins_and_windows(tb, bins, mode, bits):
                loop_mode=mode, color_bits=bits)
 
 
-@pytest.mark.parametrize("k", [64, 257, 520])
+@pytest.mark.parametrize("k", [64, 257, 520, 1100])
 def test_complete_graphs_large_mex(k):
     g = gen.from_edges(k, [(i, j) for i in range(k) for j in range(i + 1, k)])
     for bins in [(0, 0), (1, 1), (62, 256), (1, 2)]:
