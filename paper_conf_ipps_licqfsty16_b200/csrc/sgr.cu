@@ -4,6 +4,7 @@
 
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <vector>
@@ -194,6 +195,10 @@ static int round_grid(bool persistent) {
       : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_round<TB, C>, kBlock,
                                                       round_smem<C>());
   if (e != cudaSuccess || per_sm <= 0) per_sm = 1;
+  if (const char* env = getenv("SGR_BLOCKS_PER_SM")) {  // experiments: shrink the grid
+    const int lim = atoi(env);
+    if (lim > 0 && lim < per_sm) per_sm = lim;
+  }
   return per_sm * num_sms();
 }
 

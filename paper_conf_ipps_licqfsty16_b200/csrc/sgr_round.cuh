@@ -39,6 +39,15 @@
 
 #include "sgr_common.cuh"
 
+#ifndef SGR_QB
+#define SGR_QB 2  // int4 slots per lane per batch (batch = 128 * SGR_QB window slots)
+#endif
+constexpr int kQB = SGR_QB;
+constexpr int kJB = 4 * kQB;  // entries per lane per batch
+#ifndef SGR_NO_TMA
+#define SGR_NO_TMA 0
+#endif
+
 namespace sgr {
 
 constexpr int kBins = 3;
@@ -70,7 +79,8 @@ constexpr int kMinBlocks = packed<C>() ? 2 : 3;
 template <class C> struct WarpSmem {
   static constexpr int kBuf = packed<C>() ? 2 * kStage : 0;
   static constexpr int kPush = kBuf + kTblBytes;         // push buffer (kPushBuf int32)
-  static constexpr int kBars = kPush + kPushBuf * 4;     // 2 mbarriers
+  static constexpr int kItems = kPush + kPushBuf * 4;    // bin-2 item buffer (32 int64)
+  static constexpr int kBars = kItems + 32 * 8;          // 2 mbarriers
   static constexpr int kBytes = kBars + 16;
 };
 
@@ -177,6 +187,23 @@ __device__ __forceinline__ void fence_acq_rel_gpu() { asm volatile("fence.acq_re
 
 __device__ __forceinline__ int64_t make_item(int32_t v, int32_t c) {
   return (int64_t)(((uint64_t)(uint32_t)v << 32) | (uint32_t)c);
+}
+// Bin-2 items of the trimmed mode carry the adjacency buffer holding the vertex's list in
+// bit 31 of the chunk field.
+constexpr uint32_t kBufBit = 0x80000000u;
+
+// Ticket increment with release+acquire semantics at GPU scope: every write this thread
+// (and, through the preceding __syncwarp, its warp) made is visible to whoever observes
+// the new count, and this thread observes the others'.
+__device__ __forceinline__ unsigned long long atom_add_acq_rel(unsigned long long* p,
+                                                               unsigned long long v) {
+  unsigned long long r;
+  asm volatile("atom.acq_rel.gpu.global.add.u64 %0, [%1], %2;" : "=l"(r) : "l"(p), "l"(v) : "memory");
+  return r;
+}
+// Generic-proxy global writes before later async-proxy (TMA) reads of the same locations.
+__device__ __forceinline__ void fence_proxy_async_global() {
+  asm volatile("fence.proxy.async.global;" ::: "memory");
 }
 
 // ---- TMA bulk copies + mbarriers (Blackwell async proxy) -------------------------------
@@ -305,18 +332,15 @@ __device__ __forceinline__ int32_t tbl_first_free_warp(const uint8_t* tbl, int l
   return -1;
 }
 
-// 32 bits = nonzero-ness of bytes [32 * lane, 32 * lane + 32) of a 1024-byte table.
+// 32 bits = the bytes [32 * lane, 32 * lane + 32) of a 1024-byte table whose bytes are 0 or
+// 1: multiplying a word of four 0/1 bytes by 0x01020408 gathers the bytes into bits 24-27.
 __device__ __forceinline__ uint32_t tbl_bits32(const uint8_t* tbl, int lane) {
   const uint4* t = reinterpret_cast<const uint4*>(tbl) + lane * 2;
   const uint4 a = t[0], b = t[1];
   const uint32_t w[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
   uint32_t bits = 0;
 #pragma unroll
-  for (int q = 0; q < 8; ++q) {
-    const uint32_t z = __vcmpne4(w[q], 0u);  // 0xff per nonzero byte
-    const uint32_t nib = ((z >> 7) & 1u) | ((z >> 14) & 2u) | ((z >> 21) & 4u) | ((z >> 28) & 8u);
-    bits |= nib << (4 * q);
-  }
+  for (int q = 0; q < 8; ++q) bits |= ((w[q] * 0x01020408u) >> 24) << (4 * q);
   return bits;
 }
 
@@ -481,8 +505,8 @@ __device__ __forceinline__ void process_chunk_plain(const RoundArgs<C>& a, int k
 // Bin 2, packed colors, trimmed lists (see the header comment). Per warp: a 2-stage TMA
 // pipeline over the warp's chunk items i, i + NW, i + 2 NW, ...
 struct ChunkHdr {
-  int32_t v, c, len;
-  int64_t s;   // row offset (list start in adj[*] and col_idx)
+  int32_t v, c, len, slot, buf;
+  int64_t s, e;   // original row [s, e): list start in adj[*] and col_idx
 };
 
 template <int TB, bool Persist>
@@ -499,14 +523,26 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
   int64_t* out = sel(p ^ 1, a.wl_c[0], a.wl_c[1]);
   int32_t* out_cnt = &ctrl->cnt[p ^ 1][2];
   int32_t* out_vcnt = &ctrl->vcnt2[p ^ 1];
-  const int32_t* src = sel(p, (const int32_t*)a.adj[0], (const int32_t*)a.adj[1]);
-  int32_t* dst = sel(p ^ 1, a.adj[0], a.adj[1]);
   int32_t* len_cur = sel(p, a.len[0], a.len[1]);
   int32_t* len_nxt = sel(p ^ 1, a.len[0], a.len[1]);
   int32_t* bufs = reinterpret_cast<int32_t*>(wsm);
   uint8_t* tbl_all = wsm + WarpSmem<C>::kBuf;
   uint8_t* tbl_drop = tbl_all + kBigTbl;
   uint64_t* bars = reinterpret_cast<uint64_t*>(wsm + WarpSmem<C>::kBars);
+  // Next-round items are buffered per warp and flushed with one atomicAdd per <= 32 items
+  // (the bin's item and vertex counters are single hot addresses).
+  int64_t* ibuf = reinterpret_cast<int64_t*>(wsm + WarpSmem<C>::kItems);
+  int ipend = 0, vpend = 0;  // warp-uniform
+  auto iflush = [&]() {
+    if (ipend == 0) return;
+    __syncwarp();
+    int ob = 0;
+    if (lane == 0) ob = atomicAdd(out_cnt, ipend);
+    ob = __shfl_sync(0xffffffffu, ob, 0);
+    if (lane < ipend) out[ob + lane] = ibuf[lane];
+    __syncwarp();
+    ipend = 0;
+  };
 
   auto issue = [&](const ChunkHdr& h, int st) {  // lane 0 only
     const int64_t cs = h.s + (int64_t)h.c * kChunk;
@@ -514,27 +550,36 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
     const int64_t w0 = cs & ~(int64_t)3;
     const uint32_t bytes = (uint32_t)(((ce - w0 + 3) >> 2) << 4);
     fence_proxy_async();  // generic-proxy reads of this stage happen-before the async write
-    tma_load_1d(bufs + st * (kStage / 4), src + w0, bytes, bars + st);
+    tma_load_1d(bufs + st * (kStage / 4), sel(h.buf, (const int32_t*)a.adj[0],
+                                              (const int32_t*)a.adj[1]) + w0,
+                bytes, bars + st);
   };
-  auto load_hdr = [&](int i, ChunkHdr& h) {
-    const int64_t it = __ldcg(items + i);
+  auto finish_hdr = [&](int64_t it, ChunkHdr& h) {  // everything but the item itself
     h.v = (int32_t)((uint64_t)it >> 32);
-    h.c = (int32_t)(uint32_t)it;
+    h.c = (int32_t)((uint32_t)it & ~kBufBit);
+    h.buf = ((uint32_t)it & kBufBit) ? 1 : 0;
     h.s = ldg_i64(a.row_ptr + h.v);
+    h.e = ldg_i64(a.row_ptr + h.v + 1);
     h.len = ld_cg(len_cur + h.v);
+    h.slot = __ldg(a.big_id + h.v);
   };
+  auto load_hdr = [&](int i, ChunkHdr& h) { finish_hdr(__ldcg(items + i), h); };
 
   int i = gw;
   ChunkHdr cur, nxt;
   load_hdr(i, cur);
+#if !SGR_NO_TMA
   if (lane == 0) issue(cur, 0);
+#endif
   int in = i + NW;
-  nxt.v = nxt.c = nxt.len = 0;
-  nxt.s = 0;
+  nxt.v = nxt.c = nxt.len = nxt.slot = nxt.buf = 0;
+  nxt.s = nxt.e = 0;
   if (in < nC) load_hdr(in, nxt);
   int st = 0;
   while (i < nC) {
+#if !SGR_NO_TMA
     if (in < nC && lane == 0) issue(nxt, st ^ 1);
+#endif
     const int inn = in + NW;
     const int64_t it_nn = inn < nC ? __ldcg(items + inn) : 0;
 
@@ -544,37 +589,48 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
     const int32_t cnt = (int32_t)(min(cur.s + (int64_t)cur.len, cs + kChunk) - cs);
     const int32_t off0 = (int32_t)(cs & 3);
     const int32_t nslots = off0 + cnt;
-    const int32_t nb = (nslots + 255) >> 8;  // batches of 256 slots = 2 int4 per lane
+    const int32_t nb = (nslots + 128 * kQB - 1) / (128 * kQB);  // batches of kQB int4 per lane
     const int32_t nch = num_chunks(cur.len);
     const int32_t xv = cval<C>(ldraw<Persist>(X + v));
     const uint32_t klive = (uint32_t)k << 16;  // raw >= klive <=> neighbour still in W_k
+#if SGR_NO_TMA
+    {  // A/B: the warp stages its own window (16-byte loads + shared stores), no TMA
+      const int4* g4 = reinterpret_cast<const int4*>(
+          sel(cur.buf, (const int32_t*)a.adj[0], (const int32_t*)a.adj[1]) + (cs & ~(int64_t)3));
+      int4* s4 = reinterpret_cast<int4*>(bufs + st * (kStage / 4));
+      for (int q = 0; 4 * 32 * q < nslots; ++q)
+        if (4 * (lane + 32 * q) < nslots) s4[lane + 32 * q] = __ldcg(g4 + lane + 32 * q);
+      __syncwarp();
+    }
+#else
     mbar_wait(bars + st, (ph >> st) & 1u);
     ph ^= 1u << st;
+#endif
     const int4* b4 = reinterpret_cast<const int4*>(bufs + st * (kStage / 4));
     bool conf = false;
-    uint32_t lv = 0;  // live bits: bit 8 b + 4 qq + t
+    uint32_t lv = 0;  // live bits: bit kJB b + 4 qq + t
     for (int bb = 0; bb < nb; ++bb) {
-      int32_t id[8];
-      uint32_t raw[8];
+      int32_t id[kJB];
+      uint32_t raw[kJB];
       uint32_t okm = 0;
 #pragma unroll
-      for (int qq = 0; qq < 2; ++qq) {
-        const int q = 2 * bb + qq;
+      for (int qq = 0; qq < kQB; ++qq) {
+        const int q = kQB * bb + qq;
         const int4 t4 = b4[lane + 32 * q];
         id[4 * qq + 0] = t4.x;
         id[4 * qq + 1] = t4.y;
         id[4 * qq + 2] = t4.z;
         id[4 * qq + 3] = t4.w;
-#pragma unroll
-        for (int t = 0; t < 4; ++t) {
-          const int32_t r = 4 * (lane + 32 * q) + t;
-          okm |= ((uint32_t)(r - off0) < (uint32_t)cnt) ? (1u << (4 * qq + t)) : 0u;
+        {  // slots [r0, r0 + 4) of this int4 against the valid range [off0, nslots)
+          const int32_t r0 = 4 * (lane + 32 * q);
+          const int32_t lo = max(off0 - r0, 0), hi = min(nslots - r0, 4);
+          okm |= lo < hi ? (((1u << hi) - 1u) & ~((1u << lo) - 1u)) << (4 * qq) : 0u;
         }
       }
 #pragma unroll
-      for (int j = 0; j < 8; ++j) raw[j] = ((okm >> j) & 1u) ? ldraw<Persist>(X + id[j]) : 0u;
+      for (int j = 0; j < kJB; ++j) raw[j] = ((okm >> j) & 1u) ? ldraw<Persist>(X + id[j]) : 0u;
 #pragma unroll
-      for (int j = 0; j < 8; ++j) {
+      for (int j = 0; j < kJB; ++j) {
         if ((okm >> j) & 1u) {
           // colors >= 1023 are clamped onto byte 1023; a first fit of 1023 or more is
           // recomputed exactly from the full row (warp_first_fit_rescan)
@@ -583,74 +639,76 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
           tbl_all[ci] = 1;
           if (!live) tbl_drop[ci] = 1;
           conf |= (int32_t)(raw[j] & 0xffffu) == xv && lose<TB>(v, id[j]);
-          lv |= live ? (1u << (8 * bb + j)) : 0u;
+          lv |= live ? (1u << (kJB * bb + j)) : 0u;
         }
       }
     }
     // next-next header: the item id has arrived by now
     ChunkHdr nn;
-    nn.v = (int32_t)((uint64_t)it_nn >> 32);
-    nn.c = (int32_t)(uint32_t)it_nn;
-    nn.s = 0;
-    nn.len = 0;
-    if (inn < nC) {
-      nn.s = ldg_i64(a.row_ptr + nn.v);
-      nn.len = ld_cg(len_cur + nn.v);
-    }
+    nn.v = nn.c = nn.len = nn.slot = nn.buf = 0;
+    nn.s = nn.e = 0;
+    if (inn < nC) finish_hdr(it_nn, nn);
     if (lane == 0) {
       entries += (unsigned long long)cnt;
-      if (cur.c == 0) edges += (unsigned long long)(ldg_i64(a.row_ptr + v + 1) - cur.s);
+      if (cur.c == 0) edges += (unsigned long long)(cur.e - cur.s);
     }
     __syncwarp();
     const bool any = __any_sync(0xffffffffu, conf);
     const uint32_t live_total = (uint32_t)__reduce_add_sync(0xffffffffu, (uint32_t)__popc(lv));
     const int32_t* sbuf = bufs + st * (kStage / 4);
-    // compacted live list in window order: per batch, per int4 slot q, lanes in order
+    // compacted live list in window order (batch, int4 slot q, lane, t): positions from
+    // ballots — lane offset = live entries of lower lanes in the same q
+    const unsigned lt_mask = (1u << lane) - 1u;
     auto write_live = [&](int32_t* base) {
       uint32_t qb = 0;
       for (int bb = 0; bb < nb; ++bb) {
-        const uint32_t pk = (uint32_t)__popc((lv >> (8 * bb)) & 0xfu) |
-                            ((uint32_t)__popc((lv >> (8 * bb + 4)) & 0xfu) << 16);
-        uint32_t inc = pk;
 #pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-          const uint32_t tt = __shfl_up_sync(0xffffffffu, inc, o);
-          if (lane >= o) inc += tt;
-        }
-        const uint32_t tot = __shfl_sync(0xffffffffu, inc, 31);
-        const uint32_t ex = inc - pk;
+        for (int qq = 0; qq < kQB; ++qq) {
+          const int sh = kJB * bb + 4 * qq;
+          uint32_t pre = 0, tot = 0;
 #pragma unroll
-        for (int qq = 0; qq < 2; ++qq) {
-          uint32_t off = qb + ((ex >> (16 * qq)) & 0xffffu);
-          const int32_t* sq = sbuf + 4 * (lane + 32 * (2 * bb + qq));
+          for (int t = 0; t < 4; ++t) {
+            const unsigned bal = __ballot_sync(0xffffffffu, (lv >> (sh + t)) & 1u);
+            pre += __popc(bal & lt_mask);
+            tot += __popc(bal);
+          }
+          uint32_t off = qb + pre;
+          const int32_t* sq = sbuf + 4 * (lane + 32 * (kQB * bb + qq));
 #pragma unroll
           for (int t = 0; t < 4; ++t)
-            if ((lv >> (8 * bb + 4 * qq + t)) & 1u) base[off++] = sq[t];
-          qb += (tot >> (16 * qq)) & 0xffffu;
+            if ((lv >> (sh + t)) & 1u) base[off++] = sq[t];
+          qb += tot;
         }
       }
+      fence_proxy_async_global();  // the next pass reads these lists with TMA
     };
 
-    const int32_t slot = __ldg(a.big_id + v);
+    const int32_t slot = cur.slot;
     uint32_t* fx = a.fixed + (int64_t)slot * 32;
+    int32_t* lst_same = sel(cur.buf, a.adj[0], a.adj[1]);
+    int32_t* lst_other = sel(cur.buf, a.adj[1], a.adj[0]);
     if (nch == 1) {
       if (any) {
         const uint32_t fo = ld_cg(fx + lane);
         const uint32_t word = tbl_bits32(tbl_all, lane) | fo | (lane == 0 ? 1u : 0u);
         int32_t tent = bits_first_free(word);
         if (tent < 0 || tent >= kBigTbl - 1) {  // beyond the exact range of the table
-          tent = warp_first_fit_rescan<Persist>(a.col_idx, X, cur.s,
-                                                ldg_i64(a.row_ptr + v + 1), kBigTbl - 1, lane);
+          tent = warp_first_fit_rescan<Persist>(a.col_idx, X, cur.s, cur.e, kBigTbl - 1, lane);
         }
         const uint32_t drop = tbl_bits32(tbl_drop, lane);
         if (drop & ~fo) fx[lane] = fo | drop;
-        write_live(dst + cur.s);
+        // single chunk: the warp owns the whole list, so it is compacted in place, and not
+        // rewritten at all when nothing was dropped
+        if (live_total < (uint32_t)cnt) write_live(lst_same + cur.s);
         if (lane == 0) {
           len_nxt[v] = (int32_t)live_total;
           Y[v] = cpack<C>(tent, k + 1, ctrl);
-          out[atomicAdd(out_cnt, 1)] = make_item(v, 0);  // live_total <= kChunk: one chunk
-          atomicAdd(out_vcnt, 1);
+          // live <= kChunk: one chunk, the list stays in its buffer
+          ibuf[ipend] = make_item(v, (int32_t)(cur.buf ? kBufBit : 0u));
         }
+        ++ipend;
+        ++vpend;
+        if (ipend == 32) iflush();
       } else if (lane == 0) {
         Y[v] = cpack<C>(xv, k, ctrl);
       }
@@ -663,13 +721,10 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
       int32_t lbase = 0;
       if (lane == 0 && live_total) lbase = atomicAdd(len_nxt + v, (int32_t)live_total);
       lbase = __shfl_sync(0xffffffffu, lbase, 0);
-      write_live(dst + cur.s + lbase);
+      write_live(lst_other + cur.s + lbase);
       __syncwarp();  // orders every lane's writes before lane 0's release below
       unsigned long long old = 0;
-      if (lane == 0) {
-        fence_acq_rel_gpu();
-        old = atomicAdd(a.acc_cnt + slot, 1ull | ((unsigned long long)any << 32));
-      }
+      if (lane == 0) old = atom_add_acq_rel(a.acc_cnt + slot, 1ull | ((unsigned long long)any << 32));
       old = __shfl_sync(0xffffffffu, old, 0);
       if ((uint32_t)old == (uint32_t)(nch - 1)) {  // last chunk of v in this pass
         fence_acq_rel_gpu();
@@ -680,25 +735,31 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
         if (conf_all) {
           tent = bits_first_free(word);
           if (tent < 0 || tent >= kBigTbl - 1) {  // beyond the exact range of the table
-            tent = warp_first_fit_rescan<Persist>(a.col_idx, X, cur.s,
-                                                  ldg_i64(a.row_ptr + v + 1), kBigTbl - 1, lane);
+            tent = warp_first_fit_rescan<Persist>(a.col_idx, X, cur.s, cur.e, kBigTbl - 1, lane);
           }
         }
-        int32_t ob = 0, nch2 = 0;
+        int32_t nch2 = 0;
         if (lane == 0) {
           a.acc_cnt[slot] = 0ull;
           len_cur[v] = 0;  // consumed; the pass after next accumulates into it
           Y[v] = conf_all ? cpack<C>(tent, k + 1, ctrl) : cpack<C>(xv, k, ctrl);
-          if (conf_all) {
-            nch2 = num_chunks(ld_cg(len_nxt + v));
-            ob = atomicAdd(out_cnt, nch2);
-            atomicAdd(out_vcnt, 1);
-          }
+          if (conf_all) nch2 = num_chunks(ld_cg(len_nxt + v));
         }
         if (conf_all) {
-          ob = __shfl_sync(0xffffffffu, ob, 0);
           nch2 = __shfl_sync(0xffffffffu, nch2, 0);
-          for (int32_t t = lane; t < nch2; t += 32) out[ob + t] = make_item(v, t);
+          const uint32_t nbuf = cur.buf ? 0u : kBufBit;  // the list moved to the other buffer
+          ++vpend;
+          if (ipend + nch2 > 32) iflush();
+          if (nch2 > 32) {  // a hub with many chunks: direct
+            int ob = 0;
+            if (lane == 0) ob = atomicAdd(out_cnt, nch2);
+            ob = __shfl_sync(0xffffffffu, ob, 0);
+            for (int32_t t = lane; t < nch2; t += 32) out[ob + t] = make_item(v, (int32_t)(t | nbuf));
+          } else {
+            if (lane < nch2) ibuf[ipend + lane] = make_item(v, (int32_t)(lane | nbuf));
+            ipend += nch2;
+            if (ipend == 32) iflush();
+          }
         }
       }
     }
@@ -710,68 +771,65 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
     cur = nxt;
     nxt = nn;
   }
+  iflush();
+  if (lane == 0 && vpend) atomicAdd(out_vcnt, vpend);
 }
 
-// Bins 0 and 1: each 8-lane group of the warp processes one vertex (v < 0: idle group).
-// All loads of the row are issued up front (K per lane, group lanes interleaved so a
-// group's reads of a row are contiguous), then all color gathers. (Staging these short
-// rows through TMA was measured slower: the per-copy cost exceeds the latency it hides.)
-template <int TB, bool Persist, class C, int K, bool Table>
+// Bin 1: each 8-lane group of the warp processes one vertex (v < 0: idle group) in batches
+// of 64 row entries (8 per lane: all eight loads, then all eight gathers); only as many
+// batches as the row needs are issued. 32-bit relative indices throughout.
+template <int TB, bool Persist, class C>
 __device__ __forceinline__ void process_group(const RoundArgs<C>& a, int k, int32_t v,
                                               int64_t s, int64_t e, const C* X, C* Y,
                                               uint8_t* gtbl, int gl, unsigned gmask,
                                               bool& push, unsigned long long& edges) {
-  int32_t w[K];
-#pragma unroll
-  for (int u = 0; u < K; ++u) {
-    const int64_t j = s + gl + kGroup * u;
-    w[u] = (v >= 0 && j < e) ? __ldg(a.col_idx + j) : -1;
-  }
+  const int32_t cnt = v >= 0 ? (int32_t)(e - s) : 0;  // <= 256
+  const int32_t* row = a.col_idx + s;
   const int32_t xv = v >= 0 ? ldc<Persist>(X + v) : 0;
-  uint32_t lb = 0;
-#pragma unroll
-  for (int u = 0; u < K; ++u) lb |= (w[u] >= 0 && lose<TB>(v, w[u])) ? (1u << u) : 0u;
-#pragma unroll
-  for (int u = 0; u < K; ++u) w[u] = (w[u] >= 0) ? ldc<Persist>(X + w[u]) : 0;  // colors
   bool conf = false;
-  uint64_t mask = 1ull;  // bit 0 = color 0, never a candidate
+  const int32_t nb = (cnt + 63) >> 6;
+  for (int32_t bb = 0; bb < nb; ++bb) {
+    int32_t w[8];
 #pragma unroll
-  for (int u = 0; u < K; ++u) {
-    if constexpr (Table) {
-      if ((uint32_t)w[u] < (uint32_t)kMedTbl) gtbl[w[u]] = 1;
-    } else {
-      mask |= ((uint32_t)w[u] < 64u) ? (1ull << w[u]) : 0ull;
+    for (int u = 0; u < 8; ++u) {
+      const int32_t r = 64 * bb + gl + kGroup * u;
+      w[u] = r < cnt ? __ldg(row + r) : -1;
     }
-    conf |= (w[u] == xv) & ((lb >> u) & 1u);
+    uint32_t lb = 0;
+#pragma unroll
+    for (int u = 0; u < 8; ++u) lb |= (w[u] >= 0 && lose<TB>(v, w[u])) ? (1u << u) : 0u;
+#pragma unroll
+    for (int u = 0; u < 8; ++u) w[u] = w[u] >= 0 ? ldc<Persist>(X + w[u]) : -1;  // colors
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      if (w[u] >= 0) {
+        // deg <= 256 => first fit <= 257: colors >= 511 are clamped onto an unused byte
+        gtbl[min(w[u], kMedTbl - 1)] = 1;
+        conf |= w[u] == xv && ((lb >> u) & 1u);
+      }
+    }
   }
-  if (v >= 0 && gl == 0) edges += (unsigned long long)(e - s);
+  if (v >= 0 && gl == 0) edges += (unsigned long long)cnt;
+  __syncwarp();
   const bool any = (__ballot_sync(0xffffffffu, conf) & gmask) != 0u;
   int32_t tent = 0;
-  if constexpr (Table) {
-    __syncwarp();
-    if (v >= 0 && any) {  // the group scans its table 32 bytes (8 words) per step
-      const uint32_t* t32 = reinterpret_cast<const uint32_t*>(gtbl);
-      for (int it = 0; it < kMedTbl / 32; ++it) {
-        uint32_t word = t32[it * 8 + gl];
-        if (it == 0 && gl == 0) word |= 0xffu;
-        const uint32_t z = __vcmpeq4(word, 0u);
-        const unsigned b = __ballot_sync(gmask, z != 0u) & gmask;
-        if (b) {
-          const int fl = __ffs(b) - 1;  // absolute lane
-          const uint32_t zz = __shfl_sync(gmask, z, fl);
-          tent = (it * 8 + (fl & 7)) * 4 + (__ffs(zz) - 1) / 8;
-          break;
-        }
+  if (v >= 0 && any) {  // the group scans its table 32 bytes (8 words) per step
+    const uint32_t* t32 = reinterpret_cast<const uint32_t*>(gtbl);
+    for (int it = 0; it < kMedTbl / 32; ++it) {
+      uint32_t word = t32[it * 8 + gl];
+      if (it == 0 && gl == 0) word |= 0xffu;
+      const uint32_t z = __vcmpeq4(word, 0u);
+      const unsigned b = __ballot_sync(gmask, z != 0u) & gmask;
+      if (b) {
+        const int fl = __ffs(b) - 1;  // absolute lane
+        const uint32_t zz = __shfl_sync(gmask, z, fl);
+        tent = (it * 8 + (fl & 7)) * 4 + (__ffs(zz) - 1) / 8;
+        break;
       }
-      // deg <= 256 => first fit <= 257 < kMedTbl: the table always has a free slot
     }
-    clear_bytes(gtbl, kMedTbl / kGroup, gl);
-    __syncwarp();
-  } else {
-#pragma unroll
-    for (int o = 4; o > 0; o >>= 1) mask |= __shfl_xor_sync(0xffffffffu, mask, o);
-    tent = __ffsll((long long)~mask) - 1;  // deg <= 62 => first fit <= 63
   }
+  clear_bytes(gtbl, kMedTbl / kGroup, gl);
+  __syncwarp();
   if (v >= 0 && gl == 0) Y[v] = any ? cpack<C>(tent, k + 1, a.ctrl) : cpack<C>(xv, k, a.ctrl);
   push = (v >= 0) && any && gl == 0;
 }
@@ -822,11 +880,10 @@ __device__ __forceinline__ void bin0(const RoundArgs<C>& a, int k, const int32_t
   int pending = 0;
   const int step = NW * VPW;
   auto load_row = [&](int32_t vv, int64_t ss, int64_t ee, int32_t (&w)[kK0]) {
+    const int32_t cnt = vv >= 0 ? (int32_t)(ee - ss) : 0;
+    const int32_t* row = a.col_idx + ss;
 #pragma unroll
-    for (int u = 0; u < kK0; ++u) {
-      const int64_t j = ss + gl + G * u;
-      w[u] = (vv >= 0 && j < ee) ? __ldg(a.col_idx + j) : -1;
-    }
+    for (int u = 0; u < kK0; ++u) w[u] = (gl + G * u < cnt) ? __ldg(row + gl + G * u) : -1;
   };
   int i = gw * VPW + g;
   int32_t v = i < nX ? ld_cg(list + i) : -1;
@@ -847,17 +904,17 @@ __device__ __forceinline__ void bin0(const RoundArgs<C>& a, int k, const int32_t
     int32_t wn[kK0];
     load_row(v1, s1, e1, wn);  // next vertex's row, in flight with the gathers above
     bool conf = false;
-    uint64_t mask = 1ull;  // bit 0 = color 0, never a candidate
+    uint32_t mask = 0;  // bit i = color i + 1 present (deg <= 32 => first fit <= 33)
 #pragma unroll
     for (int u = 0; u < kK0; ++u) {
-      mask |= ((uint32_t)c[u] < 64u) ? (1ull << c[u]) : 0ull;
+      mask |= ((uint32_t)(c[u] - 1) < 32u) ? (1u << (c[u] - 1)) : 0u;
       conf |= (c[u] == xv) & ((lb >> u) & 1u);
     }
 #pragma unroll
     for (int o = G / 2; o > 0; o >>= 1) mask |= __shfl_xor_sync(0xffffffffu, mask, o);
     const bool any = (__ballot_sync(0xffffffffu, conf) & gmask) != 0u;
     if (v >= 0 && gl == 0) {
-      const int32_t tent = __ffsll((long long)~mask) - 1;  // deg <= 32 => first fit <= 33
+      const int32_t tent = ~mask ? __ffs(~mask) : 33;
       Y[v] = any ? cpack<C>(tent, k + 1, a.ctrl) : cpack<C>(xv, k, a.ctrl);
       edges += (unsigned long long)(e - s);
       entries += (unsigned long long)(e - s);
@@ -880,8 +937,8 @@ __device__ __forceinline__ void bin0(const RoundArgs<C>& a, int k, const int32_t
 
 // Bins 0/1 driver: warp w takes list positions 4w + g, 4(w + NW) + g, ... (g = group); the
 // next position's list entry and row offsets are prefetched, its row warmed into L2.
-template <int TB, bool Persist, class C, int K, bool Table>
-__device__ __forceinline__ void bin01(const RoundArgs<C>& a, int k, const int32_t* list, int nX,
+template <int TB, bool Persist, class C>
+__device__ __forceinline__ void bin1(const RoundArgs<C>& a, int k, const int32_t* list, int nX,
                                       int32_t* out, int32_t* out_cnt, const C* X, C* Y,
                                       uint8_t* wsm, int gw, int NW, int lane,
                                       unsigned long long& edges, unsigned long long& entries) {
@@ -899,10 +956,10 @@ __device__ __forceinline__ void bin01(const RoundArgs<C>& a, int k, const int32_
     const int32_t vn = in < nX ? ld_cg(list + in) : -1;
     const int64_t sn = vn >= 0 ? ldg_i64(a.row_ptr + vn) : 0;
     const int64_t en = vn >= 0 ? ldg_i64(a.row_ptr + vn + 1) : 0;
-    if (Table && sn + 32 * gl < en) prefetch_l2(a.col_idx + sn + 32 * gl);  // 1 line / lane
+    if (sn + 32 * gl < en) prefetch_l2(a.col_idx + sn + 32 * gl);  // 1 line / lane
     bool push = false;
     if (v >= 0 && gl == 0) entries += (unsigned long long)(e - s);
-    process_group<TB, Persist, C, K, Table>(a, k, v, s, e, X, Y, gtbl, gl, gmask, push, edges);
+    process_group<TB, Persist, C>(a, k, v, s, e, X, Y, gtbl, gl, gmask, push, edges);
     push_buffered(push, v, pbuf, pending, out, out_cnt, lane);
     i = in;
     v = vn;
@@ -965,7 +1022,7 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, uint8_t
   long long t1 = clock64();
   cyc[2] += (unsigned long long)(t1 - t0);
   // ---- bin 1: four vertices per warp (one per 8-lane group), 512-byte tables
-  bin01<TB, Persist, C, kK1, true>(
+  bin1<TB, Persist, C>(
       a, k, sel(p, (const int32_t*)a.wl_m[0], (const int32_t*)a.wl_m[1]),
       ld_cg(&ctrl->cnt[p][1]), sel(p ^ 1, a.wl_m[0], a.wl_m[1]), &ctrl->cnt[p ^ 1][1], X, Y,
       wsm, gw, NW, lane, edges[1], entries[1]);
