@@ -41,6 +41,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--loop-mode", default="auto")
+    ap.add_argument("--dist", action="store_true",
+                    help="use the multi-GPU (NCCL) path even for one rank")
     return ap.parse_args()
 
 
@@ -302,7 +304,7 @@ def main():
     if args.impl == "reference":
         return run_reference(args)
     world = int(os.environ.get("WORLD_SIZE", "1"))
-    if world > 1 or args.gpus > 1:
+    if world > 1 or args.gpus > 1 or args.dist:
         from paper_conf_ipps_licqfsty16_b200 import benchdist
         return benchdist.run(args)
     return run_single(args)

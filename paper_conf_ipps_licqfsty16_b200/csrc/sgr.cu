@@ -11,6 +11,7 @@
 
 #include "sgr.h"
 #include "sgr_internal.h"
+#include "sgr_host.cuh"
 #include "sgr_round.cuh"
 #include "sgr_step.cuh"
 
@@ -43,8 +44,6 @@ int num_sms() {
   return sms[dev];
 }
 
-static size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
-
 Resolved resolve_opts(const sgr_opts* o, int64_t n) {
   Resolved r;
   sgr_opts d;
@@ -69,100 +68,6 @@ Resolved resolve_opts(const sgr_opts* o, int64_t n) {
   return r;
 }
 
-// Workspace layout (bytes, each piece 256-aligned):
-//   Ctrl | colors: 2 x n words | wl_t: 2 x n i32 | wl_m: 2 x cap_m i32 | wl_c: 2 x cap_c i64 |
-//   big_id: n i32 | acc_bits: cap_big x 32 u32 | acc_cnt: cap_big u64 |
-//   (packed mode) fixed: cap_big x 32 u32 | len: 2 x n i32 | adj: 2 x (nnz + 16) i32
-// 32-bit mode: the caller's colors_out is one of the two ping-pong buffers. Packed mode
-// (16-bit color + 16-bit round, trimming) uses two workspace buffers and unpacks at the end.
-struct Layout {
-  bool packed;
-  int64_t cap_m, cap_c, cap_big;
-  size_t off_col, off_t, off_m, off_c, off_big, off_accb, off_accc, off_fixed, off_len, off_adj;
-  size_t zero_begin, zero_end, total;
-};
-
-static Layout layout(int64_t n, int64_t nnz, const Resolved& r) {
-  Layout L;
-  L.packed = r.color_bits == 16;
-  L.cap_m = std::min<int64_t>(n, nnz / (r.small_max + 1) + 1);
-  // each bin-2 vertex (deg > med_max) has <= deg / kChunk + 1 chunks
-  L.cap_c = nnz / kChunk + nnz / (r.med_max + 1) + 2;
-  L.cap_big = nnz / (r.med_max + 1) + 1;
-  const size_t nb = align_up((size_t)n * 4, 256);
-  size_t o = align_up(sizeof(Ctrl), 256);
-  L.off_col = o;
-  o += 2 * nb;
-  L.off_t = o;
-  o += 2 * nb;
-  L.off_m = o;
-  o += 2 * align_up((size_t)L.cap_m * 4, 256);
-  L.off_c = o;
-  o += 2 * align_up((size_t)L.cap_c * 8, 256);
-  L.off_big = o;
-  o += nb;
-  L.off_accb = o;
-  L.zero_begin = o;
-  o += align_up((size_t)L.cap_big * 128, 256);
-  L.off_accc = o;
-  o += align_up((size_t)L.cap_big * 8, 256);
-  L.off_fixed = L.off_len = L.off_adj = o;
-  if (L.packed) {
-    L.off_fixed = o;
-    o += align_up((size_t)L.cap_big * 128, 256);
-    L.off_len = o;
-    o += 2 * nb;
-  }
-  L.zero_end = o;  // accumulators, fixed sets and list lengths start at zero
-  if (L.packed) {
-    L.off_adj = o;
-    o += 2 * align_up((size_t)(nnz + 16) * 4, 256);
-  }
-  L.total = o;
-  return L;
-}
-
-size_t ws_bytes(int64_t n, int64_t nnz, const Resolved& r) { return layout(n, nnz, r).total; }
-
-template <class C>
-static void build_args(RoundArgs<C>& a, const sgr_csr* csr, int64_t n, int64_t nnz,
-                       int32_t* colors, void* ws, const Layout& L, const Resolved& r) {
-  memset(&a, 0, sizeof(a));
-  char* b = (char*)ws;
-  const size_t nb = align_up((size_t)n * 4, 256);
-  a.row_ptr = csr->row_ptr;
-  a.col_idx = csr->col_idx;
-  if constexpr (packed<C>()) {
-    a.col[0] = (C*)(b + L.off_col);
-    a.col[1] = (C*)(b + L.off_col + nb);
-    a.fixed = (uint32_t*)(b + L.off_fixed);
-    a.len[0] = (int32_t*)(b + L.off_len);
-    a.len[1] = (int32_t*)(b + L.off_len + nb);
-    const size_t ab = align_up((size_t)(nnz + 16) * 4, 256);
-    a.adj[0] = (int32_t*)(b + L.off_adj);
-    a.adj[1] = (int32_t*)(b + L.off_adj + ab);
-  } else {
-    a.col[0] = (C*)colors;
-    a.col[1] = (C*)(b + L.off_col);
-  }
-  a.wl_t[0] = (int32_t*)(b + L.off_t);
-  a.wl_t[1] = (int32_t*)(b + L.off_t + nb);
-  const size_t sm = align_up((size_t)L.cap_m * 4, 256);
-  a.wl_m[0] = (int32_t*)(b + L.off_m);
-  a.wl_m[1] = (int32_t*)(b + L.off_m + sm);
-  const size_t sc = align_up((size_t)L.cap_c * 8, 256);
-  a.wl_c[0] = (int64_t*)(b + L.off_c);
-  a.wl_c[1] = (int64_t*)(b + L.off_c + sc);
-  a.big_id = (int32_t*)(b + L.off_big);
-  a.acc_bits = (uint32_t*)(b + L.off_accb);
-  a.acc_cnt = (unsigned long long*)(b + L.off_accc);
-  a.ctrl = (Ctrl*)b;
-  a.n = (int32_t)n;
-  a.nnz = nnz;
-  a.small_max = r.small_max;
-  a.med_max = r.med_max;
-}
-
 // Pinned host slots for termination flags (reused across calls on this thread).
 static int32_t* pinned_flags() {
   static thread_local int32_t* p = nullptr;
@@ -170,37 +75,7 @@ static int32_t* pinned_flags() {
   return p;
 }
 
-int first_grid(int64_t n) {
-  return (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, (int64_t)num_sms() * 8));
-}
-
-template <class C>
-static constexpr size_t round_smem() { return (size_t)kWarps * WarpSmem<C>::kBytes; }
-
-// Blocks of the round kernels: as many as are co-resident (persistent: required).
-template <int TB, class C>
-static int round_grid(bool persistent) {
-  static bool attr_set = false;
-  if (!attr_set) {  // opt in to > 48 KB of dynamic shared memory
-    cudaFuncSetAttribute(k_persistent<TB, C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)round_smem<C>());
-    cudaFuncSetAttribute(k_round<TB, C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)round_smem<C>());
-    attr_set = true;
-  }
-  int per_sm = 0;
-  cudaError_t e = persistent
-      ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_persistent<TB, C>, kBlock,
-                                                      round_smem<C>())
-      : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_round<TB, C>, kBlock,
-                                                      round_smem<C>());
-  if (e != cudaSuccess || per_sm <= 0) per_sm = 1;
-  if (const char* env = getenv("SGR_BLOCKS_PER_SM")) {  // experiments: shrink the grid
-    const int lim = atoi(env);
-    if (lim > 0 && lim < per_sm) per_sm = lim;
-  }
-  return per_sm * num_sms();
-}
+size_t ws_bytes(int64_t n, int64_t nnz, const Resolved& r) { return layout(n, nnz, r).total; }
 
 // ----- CUDA-graph cache: one graph = `batch` round passes -----------------------------------
 struct GraphKey {

@@ -1,10 +1,250 @@
-// sgr_dist.cu — multi-GPU layer: nnz-balanced contiguous vertex ranges.
+// sgr_dist.cu — multi-GPU layer.
+//
+// The graph is split into contiguous vertex ranges balanced by nnz (sgr_partition). Every
+// partition owns the rows of its range (local row offsets, GLOBAL column ids) and keeps a
+// full replica of the color array. A round is:
+//   1. the fused pass F_k over the partition's owned worklists (the same kernels as one GPU;
+//      row_ptr is shifted by -v_begin so global ids index the local offsets),
+//   2. k_pack: the partition's part of W_{k+1} as (v, new color word) records,
+//   3. an all-gather of the records (NCCL over NVLink between ranks, or device copies
+//      between partitions that share one GPU),
+//   4. k_apply: every replica writes the other partitions' records into both ping-pong
+//      buffers (a remote vertex is never written by the local pass).
+// Round k's records are a subset of W_k, so the largest count of the previous exchange is
+// a valid capacity for the padded all-gather: one collective per round (plus one counts
+// gather before the first). The result is bit-identical to one GPU: the passes read the
+// same snapshot values, only the owner computes each vertex.
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cstring>
+#include <functional>
+#include <vector>
 
 #include "sgr.h"
+#include "sgr_host.cuh"
 #include "sgr_internal.h"
+#include "sgr_round.cuh"
+#include "sgr_step.cuh"
+
+#if SGR_HAVE_NCCL
+#include <nccl.h>
+#endif
+
+namespace sgr {
+
+struct DistComm {
+#if SGR_HAVE_NCCL
+  ncclComm_t comm = nullptr;
+#endif
+  int rank = 0, world = 1, device = 0;
+};
+
+struct Part {
+  int64_t lo = 0, hi = 0, nnz = 0;
+  sgr_csr csr{};        // owned rows: row_ptr (hi - lo + 1 local offsets), col_idx (global ids)
+  void* ws = nullptr;   // workspace (layout(n_global, nnz_local))
+  int32_t* colors = nullptr;  // plain mode ping-pong partner / final output
+  uint2* send = nullptr;
+  bool own_colors = false;
+};
+
+using Gather = std::function<sgr_status(std::vector<Part>& parts, uint2* recv, int32_t cap,
+                                        cudaStream_t s)>;
+
+#define DCK(call)                                                            \
+  do {                                                                       \
+    cudaError_t e_ = (call);                                                 \
+    if (e_ != cudaSuccess) return cuda_fail(e_, #call, __LINE__);           \
+  } while (0)
+
+// Runs the rounds for every partition in `parts` (all on the current device, one stream).
+// `me0` is the index of parts[0] among all `world` partitions (NCCL: the rank).
+template <int TB, class C>
+static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_t n,
+                            int32_t* colors_out, sgr_stats* stats, const Gather& gather,
+                            int64_t cap_hint, const Resolved& r) {
+  cudaStream_t s = r.stream;
+  const int P = (int)parts.size();
+  std::vector<Layout> Ls;
+  std::vector<RoundArgs<C>> args(P);
+  // a record count never exceeds its owner's range: size by the largest range anywhere
+  int64_t cap_max = std::max<int64_t>(1, cap_hint);
+  for (int i = 0; i < P; ++i) cap_max = std::max(cap_max, parts[i].hi - parts[i].lo);
+  for (int i = 0; i < P; ++i) {
+    Part& pt = parts[i];
+    Ls.push_back(layout(n, pt.nnz, r));
+    DCK(cudaMallocAsync(&pt.ws, Ls[i].total, s));
+    DCK(cudaMallocAsync((void**)&pt.send, (size_t)(cap_max + 1) * sizeof(uint2), s));
+    if (!packed<C>() && (i > 0 || !colors_out)) {
+      DCK(cudaMallocAsync((void**)&pt.colors, (size_t)n * 4, s));
+      pt.own_colors = true;
+    } else {
+      pt.colors = colors_out;
+    }
+    sgr_csr shifted{pt.csr.row_ptr - pt.lo, pt.csr.col_idx};
+    build_args<C>(args[i], &shifted, n, pt.nnz, pt.colors, pt.ws, Ls[i], r);
+    args[i].v_begin = (int32_t)pt.lo;
+    args[i].v_end = (int32_t)pt.hi;
+    Ctrl hc;
+    memset(&hc, 0, sizeof(hc));
+    hc.k = 1;
+    hc.max_rounds = INT32_MAX;
+    DCK(cudaMemcpyAsync(args[i].ctrl, &hc, sizeof(Ctrl), cudaMemcpyHostToDevice, s));
+    DCK(cudaMemsetAsync((char*)pt.ws + Ls[i].zero_begin, 0, Ls[i].zero_end - Ls[i].zero_begin, s));
+    if constexpr (packed<C>()) {
+      if (pt.nnz > 0)
+        DCK(cudaMemcpyAsync(args[i].adj[0], pt.csr.col_idx, (size_t)pt.nnz * 4,
+                            cudaMemcpyDeviceToDevice, s));
+    }
+    k_fill_c1<C><<<first_grid(n), 256, 0, s>>>(args[i]);
+    k_first<TB, C><<<first_grid(pt.hi - pt.lo), 256, 0, s>>>(args[i], 1);
+    k_advance<<<1, 32, 0, s>>>(args[i].ctrl, 1, 0);
+  }
+  DCK(cudaGetLastError());
+  const int grid = round_grid<TB, C>(false);
+  uint2* recv = nullptr;
+  DCK(cudaMallocAsync((void**)&recv, (size_t)world * (cap_max + 1) * sizeof(uint2), s));
+  std::vector<uint2> hdr(world);
+  int32_t* counts_host = nullptr;
+  DCK(cudaMallocHost(&counts_host, sizeof(int32_t) * world));
+
+  // one exchange: pack -> all-gather with capacity cap -> apply; returns per-part counts
+  auto exchange = [&](int32_t cap, std::vector<int32_t>& cnt) -> sgr_status {
+    for (int i = 0; i < P; ++i) {
+      DCK(cudaMemsetAsync(parts[i].send, 0, sizeof(uint2), s));
+      k_pack<C><<<first_grid(parts[i].hi - parts[i].lo + 1), 256, 0, s>>>(args[i], parts[i].send, cap);
+    }
+    DCK(cudaGetLastError());
+    sgr_status st = gather(parts, recv, cap, s);
+    if (st != SGR_OK) return st;
+    for (int i = 0; i < P; ++i)
+      k_apply<C><<<first_grid(cap), 256, 0, s>>>(args[i], recv, world, cap + 1, me0 + i);
+    DCK(cudaGetLastError());
+    DCK(cudaMemcpy2DAsync(counts_host, sizeof(int32_t), recv, (size_t)(cap + 1) * sizeof(uint2),
+                          sizeof(int32_t), world, cudaMemcpyDeviceToHost, s));
+    DCK(cudaStreamSynchronize(s));
+    cnt.assign(counts_host, counts_host + world);
+    return SGR_OK;
+  };
+
+  sgr_status status = SGR_OK;
+  cudaEvent_t ev0, ev1;
+  cudaEventCreate(&ev0);
+  cudaEventCreate(&ev1);
+  std::vector<int32_t> cnt;
+  // W_2: a counts-only round first, so the data gather is sized by the real maximum
+  {
+    for (int i = 0; i < P; ++i) DCK(cudaMemsetAsync(parts[i].send, 0, sizeof(uint2), s));
+    for (int i = 0; i < P; ++i)
+      k_pack<C><<<first_grid(parts[i].hi - parts[i].lo + 1), 256, 0, s>>>(args[i], parts[i].send, 0);
+    status = gather(parts, recv, 0, s);
+    if (status == SGR_OK) {
+      DCK(cudaMemcpy2DAsync(counts_host, sizeof(int32_t), recv, sizeof(uint2), sizeof(int32_t),
+                            world, cudaMemcpyDeviceToHost, s));
+      DCK(cudaStreamSynchronize(s));
+    }
+  }
+  cudaEventRecord(ev0, s);
+  int32_t cap = 0;
+  for (int q = 0; q < world && status == SGR_OK; ++q) cap = std::max(cap, counts_host[q]);
+  int64_t vertices = n, rounds = 1;
+  if (status == SGR_OK) status = exchange(cap, cnt);  // W_2 records
+  int64_t total = 0;
+  for (int32_t c : cnt) total += c;
+  if (total > 0) rounds = 2;
+  vertices += total;
+  while (status == SGR_OK && total > 0) {
+    if (rounds > r.max_rounds) {
+      set_error("sgr_color_dist: max_rounds (%d) reached", r.max_rounds);
+      status = SGR_ENOCONV;
+      break;
+    }
+    cap = *std::max_element(cnt.begin(), cnt.end());
+    for (int i = 0; i < P; ++i) {
+      k_round<TB, C><<<grid, kBlock, round_smem<C>(), s>>>(args[i]);
+      k_advance<<<1, 32, 0, s>>>(args[i].ctrl, 0, 1);
+    }
+    DCK(cudaGetLastError());
+    status = exchange(cap, cnt);
+    total = 0;
+    for (int32_t c : cnt) total += c;
+    vertices += total;
+    if (total > 0) ++rounds;
+  }
+  cudaEventRecord(ev1, s);
+  if (status == SGR_OK) {
+    RoundArgs<C>& a0 = args[0];
+    if constexpr (packed<C>()) {
+      k_unpack<<<first_grid(n), 256, 0, s>>>(a0.col[0], colors_out, n);
+    } else if (a0.col[0] != (C*)colors_out) {
+      DCK(cudaMemcpyAsync(colors_out, a0.col[0], (size_t)n * 4, cudaMemcpyDeviceToDevice, s));
+    }
+    k_max_color<<<first_grid(n), 256, 0, s>>>(colors_out, n, &a0.ctrl->max_color);
+    DCK(cudaGetLastError());
+    std::vector<Ctrl> fin(P);
+    for (int i = 0; i < P; ++i)
+      DCK(cudaMemcpyAsync(&fin[i], args[i].ctrl, sizeof(Ctrl), cudaMemcpyDeviceToHost, s));
+    DCK(cudaStreamSynchronize(s));
+    int overflow = 0;
+    for (int i = 0; i < P; ++i) overflow |= fin[i].overflow;
+    if (overflow) {
+      set_error("sgr_color_dist: a color or round number exceeded 16 bits; use color_bits=32");
+      status = SGR_EUNSUPPORTED;
+    }
+    if (stats) {
+      memset(stats, 0, sizeof(*stats));
+      for (int i = 0; i < P; ++i) {
+        sgr_stats t;
+        memset(&t, 0, sizeof(t));
+        fill_stats(fin[i], 0, 0, &t);
+        stats->edges_scanned += t.edges_scanned;
+        stats->entries_read += t.entries_read;
+        stats->bytes_algorithmic += t.bytes_algorithmic;
+        stats->chunk_items += t.chunk_items;
+        for (int q = 0; q < 3; ++q) {
+          stats->bin_vertices[q] += t.bin_vertices[q];
+          stats->bin_edges[q] += t.bin_edges[q];
+          stats->bin_warp_cycles[q] += t.bin_warp_cycles[q];
+        }
+      }
+      int64_t nnz_parts = 0;
+      for (auto& pt : parts) nnz_parts += pt.nnz;
+      stats->edges_scanned += nnz_parts;  // round 1 (local rows)
+      stats->rounds = (int32_t)rounds;
+      stats->num_colors = fin[0].max_color;
+      // F_1 + advance + fill per part, 5 launches per part per exchange round, final
+      stats->launches = (int32_t)(P * 3 + (rounds + 1) * P * 5 + 2);
+      stats->vertices_processed = vertices;
+      stats->grid_blocks = grid;
+      stats->color_bits = packed<C>() ? 16 : 32;
+      cudaEventElapsedTime(&stats->elapsed_ms, ev0, ev1);
+    }
+  }
+  cudaEventDestroy(ev0);
+  cudaEventDestroy(ev1);
+  cudaFreeHost(counts_host);
+  cudaFreeAsync(recv, s);
+  for (auto& pt : parts) {
+    cudaFreeAsync(pt.ws, s);
+    cudaFreeAsync(pt.send, s);
+    if (pt.own_colors) cudaFreeAsync(pt.colors, s);
+  }
+  cudaStreamSynchronize(s);
+  return status;
+}
+
+template <class... A>
+static sgr_status dispatch(const Resolved& r, A&&... args) {
+  if (r.color_bits == 16) {
+    return r.tiebreak ? run_parts<1, uint32_t>(std::forward<A>(args)..., r)
+                      : run_parts<0, uint32_t>(std::forward<A>(args)..., r);
+  }
+  return r.tiebreak ? run_parts<1, int32_t>(std::forward<A>(args)..., r)
+                    : run_parts<0, int32_t>(std::forward<A>(args)..., r);
+}
+
+}  // namespace sgr
 
 using namespace sgr;
 
@@ -25,38 +265,171 @@ sgr_status sgr_partition(const int64_t* row_ptr, int64_t n, int32_t P, int64_t* 
   return SGR_OK;
 }
 
+sgr_status sgr_color_partitioned(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t P,
+                                 const int64_t* ranges, int32_t* colors_out, sgr_stats* stats,
+                                 const sgr_opts* opts) {
+  if (!csr || n < 0 || nnz < 0 || P < 1 || !ranges || n >= ((int64_t)1 << 31)) return SGR_EINVAL;
+  if (stats) memset(stats, 0, sizeof(*stats));
+  if (n == 0) return SGR_OK;
+  if (!csr->row_ptr || !colors_out || (nnz > 0 && !csr->col_idx)) return SGR_EINVAL;
+  if (((uintptr_t)csr->col_idx & 15u) != 0) {
+    set_error("sgr_color_partitioned: col_idx must be 16-byte aligned");
+    return SGR_EINVAL;
+  }
+  if (ranges[0] != 0 || ranges[P] != n) return SGR_EINVAL;
+  for (int p = 0; p < P; ++p)
+    if (ranges[p + 1] < ranges[p]) return SGR_EINVAL;
+  const Resolved r = resolve_opts(opts, n);
+  // local CSRs: offsets relative to the range's first row (host copy of row_ptr needed)
+  std::vector<int64_t> rp(n + 1);
+  if (cudaMemcpy(rp.data(), csr->row_ptr, (size_t)(n + 1) * 8, cudaMemcpyDeviceToHost) != cudaSuccess)
+    return cuda_fail(cudaGetLastError(), "row_ptr D2H", __LINE__);
+  std::vector<Part> parts(P);
+  std::vector<int64_t*> local_rp(P, nullptr);
+  std::vector<int32_t*> local_ci(P, nullptr);
+  cudaStream_t s = r.stream;
+  for (int p = 0; p < P; ++p) {
+    Part& pt = parts[p];
+    pt.lo = ranges[p];
+    pt.hi = ranges[p + 1];
+    const int64_t b = rp[pt.lo], e = rp[pt.hi];
+    pt.nnz = e - b;
+    std::vector<int64_t> lrp(pt.hi - pt.lo + 1);
+    for (int64_t v = pt.lo; v <= pt.hi; ++v) lrp[v - pt.lo] = rp[v] - b;
+    DCK(cudaMallocAsync((void**)&local_rp[p], lrp.size() * 8, s));
+    DCK(cudaMallocAsync((void**)&local_ci[p], (size_t)std::max<int64_t>(pt.nnz, 4) * 4, s));
+    DCK(cudaMemcpyAsync(local_rp[p], lrp.data(), lrp.size() * 8, cudaMemcpyHostToDevice, s));
+    if (pt.nnz > 0)
+      DCK(cudaMemcpyAsync(local_ci[p], csr->col_idx + b, (size_t)pt.nnz * 4, cudaMemcpyDeviceToDevice, s));
+    DCK(cudaStreamSynchronize(s));  // lrp is a host temporary
+    pt.csr = sgr_csr{local_rp[p], local_ci[p]};
+  }
+  // the all-gather between partitions that share this device: device copies
+  Gather gather = [](std::vector<Part>& ps, uint2* recv, int32_t cap, cudaStream_t st) -> sgr_status {
+    for (size_t q = 0; q < ps.size(); ++q)
+      DCK(cudaMemcpyAsync(recv + q * (size_t)(cap + 1), ps[q].send, (size_t)(cap + 1) * sizeof(uint2),
+                          cudaMemcpyDeviceToDevice, st));
+    return SGR_OK;
+  };
+  const sgr_status st = dispatch(r, parts, P, 0, n, colors_out, stats, gather, (int64_t)0);
+  for (int p = 0; p < P; ++p) {
+    cudaFreeAsync(local_rp[p], s);
+    cudaFreeAsync(local_ci[p], s);
+  }
+  cudaStreamSynchronize(s);
+  return st;
+}
+
 sgr_status sgr_nccl_unique_id(void* id_out) {
+#if SGR_HAVE_NCCL
+  if (!id_out) return SGR_EINVAL;
+  ncclUniqueId id;
+  const ncclResult_t rc = ncclGetUniqueId(&id);
+  if (rc != ncclSuccess) {
+    set_error("ncclGetUniqueId: %s", ncclGetErrorString(rc));
+    return SGR_ENCCL;
+  }
+  static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId size");
+  memcpy(id_out, &id, sizeof(id));
+  return SGR_OK;
+#else
   (void)id_out;
-  set_error("sgr_nccl_unique_id: not built yet");
+  set_error("built without NCCL");
   return SGR_EUNSUPPORTED;
+#endif
 }
 
 sgr_status sgr_comm_init(void** comm, int32_t rank, int32_t world, const void* id, int32_t device) {
-  (void)comm; (void)rank; (void)world; (void)id; (void)device;
-  set_error("sgr_comm_init: not built yet");
+  if (!comm || !id || world < 1 || rank < 0 || rank >= world) return SGR_EINVAL;
+#if SGR_HAVE_NCCL
+  if (cudaSetDevice(device) != cudaSuccess) return cuda_fail(cudaGetLastError(), "cudaSetDevice", __LINE__);
+  DistComm* c = new DistComm();
+  c->rank = rank;
+  c->world = world;
+  c->device = device;
+  ncclUniqueId uid;
+  memcpy(&uid, id, sizeof(uid));
+  const ncclResult_t rc = ncclCommInitRank(&c->comm, world, uid, rank);
+  if (rc != ncclSuccess) {
+    delete c;
+    set_error("ncclCommInitRank: %s", ncclGetErrorString(rc));
+    return SGR_ENCCL;
+  }
+  *comm = c;
+  return SGR_OK;
+#else
+  (void)device;
+  set_error("built without NCCL");
   return SGR_EUNSUPPORTED;
+#endif
 }
 
 sgr_status sgr_comm_destroy(void* comm) {
-  (void)comm;
+  if (!comm) return SGR_OK;
+  DistComm* c = (DistComm*)comm;
+#if SGR_HAVE_NCCL
+  if (c->comm) ncclCommDestroy(c->comm);
+#endif
+  delete c;
   return SGR_OK;
 }
 
 sgr_status sgr_color_dist(void* comm, const sgr_csr* local, int64_t n_global, int64_t v_begin,
                           int64_t v_end, int64_t nnz_local, int32_t* colors_out, sgr_stats* stats,
                           const sgr_opts* opts) {
+  if (!comm || !local || n_global < 0 || v_begin < 0 || v_end < v_begin || v_end > n_global ||
+      nnz_local < 0 || n_global >= ((int64_t)1 << 31))
+    return SGR_EINVAL;
+  if (stats) memset(stats, 0, sizeof(*stats));
+  if (n_global == 0) return SGR_OK;
+  if (!local->row_ptr || !colors_out || (nnz_local > 0 && !local->col_idx)) return SGR_EINVAL;
+  if (((uintptr_t)local->col_idx & 15u) != 0) {
+    set_error("sgr_color_dist: col_idx must be 16-byte aligned");
+    return SGR_EINVAL;
+  }
+#if SGR_HAVE_NCCL
+  DistComm* c = (DistComm*)comm;
+  const Resolved r = resolve_opts(opts, n_global);
+  std::vector<Part> parts(1);
+  parts[0].lo = v_begin;
+  parts[0].hi = v_end;
+  parts[0].nnz = nnz_local;
+  parts[0].csr = *local;
+  // every rank must size its buffers by the LARGEST range: agree on it first
+  int64_t* d_sz = nullptr;
+  cudaStream_t s = r.stream;
+  DCK(cudaMallocAsync((void**)&d_sz, 8 * (size_t)(c->world + 1), s));
+  const int64_t mine = v_end - v_begin;
+  DCK(cudaMemcpyAsync(d_sz + c->world, &mine, 8, cudaMemcpyHostToDevice, s));
+  ncclResult_t rc = ncclAllGather(d_sz + c->world, d_sz, 1, ncclInt64, c->comm, s);
+  if (rc != ncclSuccess) {
+    set_error("ncclAllGather: %s", ncclGetErrorString(rc));
+    return SGR_ENCCL;
+  }
+  std::vector<int64_t> sizes(c->world);
+  DCK(cudaMemcpyAsync(sizes.data(), d_sz, 8 * (size_t)c->world, cudaMemcpyDeviceToHost, s));
+  DCK(cudaStreamSynchronize(s));
+  cudaFreeAsync(d_sz, s);
+  Gather gather = [c](std::vector<Part>& ps, uint2* recv, int32_t cap, cudaStream_t st) -> sgr_status {
+    const ncclResult_t e = ncclAllGather(ps[0].send, recv, (size_t)(cap + 1) * 2, ncclUint32,
+                                         c->comm, st);
+    if (e != ncclSuccess) {
+      set_error("ncclAllGather: %s", ncclGetErrorString(e));
+      return SGR_ENCCL;
+    }
+    return SGR_OK;
+  };
+  // partitions on other ranks may be larger than ours: every buffer is sized by the
+  // largest range, so all ranks use the same padded record counts
+  int64_t cap_all = 0;
+  for (int64_t z : sizes) cap_all = std::max(cap_all, z);
+  return dispatch(r, parts, c->world, c->rank, n_global, colors_out, stats, gather, cap_all);
+#else
   (void)comm; (void)local; (void)n_global; (void)v_begin; (void)v_end; (void)nnz_local;
   (void)colors_out; (void)stats; (void)opts;
-  set_error("sgr_color_dist: not built yet");
+  set_error("built without NCCL");
   return SGR_EUNSUPPORTED;
-}
-
-sgr_status sgr_color_partitioned(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t P,
-                                 const int64_t* ranges, int32_t* colors_out, sgr_stats* stats,
-                                 const sgr_opts* opts) {
-  (void)csr; (void)n; (void)nnz; (void)P; (void)ranges; (void)colors_out; (void)stats; (void)opts;
-  set_error("sgr_color_partitioned: not built yet");
-  return SGR_EUNSUPPORTED;
+#endif
 }
 
 }  // extern "C"

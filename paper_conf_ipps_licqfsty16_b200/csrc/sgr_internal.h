@@ -33,7 +33,6 @@ sgr_status cuda_fail(cudaError_t e, const char* what, int line);
 int num_sms();
 Resolved resolve_opts(const sgr_opts* o, int64_t n);
 size_t ws_bytes(int64_t n, int64_t nnz, const Resolved& r);
-int first_grid(int64_t n);
 void fill_stats(const Ctrl& c, int64_t n, int64_t nnz, sgr_stats* st);
 
 }  // namespace sgr

@@ -131,6 +131,8 @@ struct RoundArgs {
   int32_t n;
   int32_t small_max;
   int32_t med_max;
+  int32_t v_begin;            // owned vertex range [v_begin, v_end) (multi-GPU: a partition)
+  int32_t v_end;
   int32_t pad;
 };
 
@@ -256,8 +258,8 @@ __global__ void __launch_bounds__(256) k_first(RoundArgs<C> a, int sorted) {
   C* __restrict__ X = a.col[0];
   C* __restrict__ Y = a.col[1];
   const int lane = threadIdx.x & 31;
-  const int64_t n = a.n;
-  for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < n;
+  const int64_t n = a.v_end;
+  for (int64_t base = (int64_t)a.v_begin + (int64_t)blockIdx.x * blockDim.x; base < n;
        base += (int64_t)gridDim.x * blockDim.x) {
     const int64_t vi = base + threadIdx.x;
     bool conflict = false;
@@ -1067,7 +1069,7 @@ __device__ __forceinline__ void block_add6(unsigned long long (&x)[kBins],
 // counters into totals and the trace, consume W_k, advance k and decide whether W_{k+1}
 // is non-empty. A pass over an empty W_k changes nothing, so any surplus pass a host loop
 // issues before it sees `active == 0` is a no-op.
-__device__ __forceinline__ void advance_body(Ctrl* ctrl, bool first) {
+__device__ __forceinline__ void advance_body(Ctrl* ctrl, bool first, bool force = false) {
   volatile Ctrl* c = ctrl;
   if (first) {  // after F_1: W_2 is in parity 0
     int tot = 0;
@@ -1085,7 +1087,7 @@ __device__ __forceinline__ void advance_body(Ctrl* ctrl, bool first) {
   const int k = c->k;
   const int p = k & 1;
   const int items_in = c->cnt[p][0] + c->cnt[p][1] + c->cnt[p][2];
-  if (items_in == 0) {
+  if (items_in == 0 && !force) {  // (multi-GPU ranks advance in lockstep: force)
     c->active = 0;
     return;
   }
@@ -1121,8 +1123,76 @@ __device__ __forceinline__ void advance_body(Ctrl* ctrl, bool first) {
   }
 }
 
-__global__ void k_advance(Ctrl* ctrl, int first) {
-  if (threadIdx.x == 0 && blockIdx.x == 0) advance_body(ctrl, first != 0);
+static __global__ void k_advance(Ctrl* ctrl, int first, int force = 0) {
+  if (threadIdx.x == 0 && blockIdx.x == 0) advance_body(ctrl, first != 0, force != 0);
+}
+
+// ---------------------------------------------------------------------------------------
+// Multi-GPU exchange. After pass F_k the rank's next worklists hold its
+// owned part of W_{k+1}; every other replica needs those vertices' new color words.
+// Record = (v, word); slot 0 of a send buffer carries (count, 0).
+template <class C>
+__global__ void k_pack(RoundArgs<C> a, uint2* send, int32_t cap) {
+  Ctrl* ctrl = a.ctrl;
+  const int k = ctrl->k;  // already advanced: W_k's lists are the new ones
+  const int p = k & 1;
+  const C* Y = sel((k - 1) & 1, (const C*)a.col[0], (const C*)a.col[1]);
+  const int nT = ctrl->cnt[p][0], nM = ctrl->cnt[p][1], nC = ctrl->cnt[p][2];
+  const int32_t* lt = sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]);
+  const int32_t* lm = sel(p, (const int32_t*)a.wl_m[0], (const int32_t*)a.wl_m[1]);
+  const int64_t* lc = sel(p, (const int64_t*)a.wl_c[0], (const int64_t*)a.wl_c[1]);
+  int32_t* count = reinterpret_cast<int32_t*>(&send[0].x);
+  const int64_t total = (int64_t)nT + nM + nC;
+  for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < total;
+       base += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t i = base + threadIdx.x;
+    int32_t v = -1;
+    if (i < nT) v = lt[i];
+    else if (i < nT + nM) v = lm[i - nT];
+    else if (i < total) {
+      const int64_t it = lc[i - nT - nM];
+      if (((uint32_t)it & ~kBufBit) == 0u) v = (int32_t)((uint64_t)it >> 32);  // chunk 0
+    }
+    const unsigned m = __ballot_sync(0xffffffffu, v >= 0);
+    if (m) {
+      const int lane = threadIdx.x & 31;
+      int b = 0;
+      if (lane == __ffs(m) - 1) b = atomicAdd(count, __popc(m));
+      b = __shfl_sync(0xffffffffu, b, __ffs(m) - 1);
+      if (v >= 0) {
+        const int slot = b + __popc(m & ((1u << lane) - 1u));
+        if (slot < cap) send[1 + slot] = make_uint2((uint32_t)v, (uint32_t)Y[v]);
+      }
+    }
+  }
+}
+
+// Apply every other part's records to this replica: both ping-pong buffers, because a
+// remote vertex is only ever written by these updates.
+template <class C>
+__global__ void k_apply(RoundArgs<C> a, const uint2* recv, int32_t parts, int32_t stride,
+                        int32_t me) {
+  for (int q = 0; q < parts; ++q) {
+    if (q == me) continue;
+    const uint2* r = recv + (int64_t)q * stride;
+    const int32_t cnt = (int32_t)r[0].x;
+    for (int32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += gridDim.x * blockDim.x) {
+      const uint2 rec = r[1 + i];
+      a.col[0][rec.x] = (C)rec.y;
+      a.col[1][rec.x] = (C)rec.y;
+    }
+  }
+}
+
+// Initialise both color buffers of a replica to C_1 (every vertex colored 1 in round 1).
+template <class C>
+__global__ void k_fill_c1(RoundArgs<C> a) {
+  const C one = packed<C>() ? (C)((1u << 16) | 1u) : (C)1;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < a.n;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    a.col[0][i] = one;
+    a.col[1][i] = one;
+  }
 }
 
 // Kernel prologue: zero the warp tables, initialise the warp's two TMA mbarriers.
@@ -1203,7 +1273,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks<C>) k_persistent(RoundArgs<
 }
 
 // Final colors (packed words) into the caller's int32 output.
-__global__ void k_unpack(const uint32_t* __restrict__ src, int32_t* __restrict__ dst, int64_t n) {
+static __global__ void k_unpack(const uint32_t* __restrict__ src, int32_t* __restrict__ dst, int64_t n) {
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
        i += (int64_t)gridDim.x * blockDim.x)
     dst[i] = (int32_t)(src[i] & 0xffffu);

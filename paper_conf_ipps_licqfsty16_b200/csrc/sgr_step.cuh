@@ -8,7 +8,7 @@
 
 namespace sgr {
 
-__global__ void k_max_color(const int32_t* __restrict__ c, int64_t n, int32_t* out) {
+static __global__ void k_max_color(const int32_t* __restrict__ c, int64_t n, int32_t* out) {
   int32_t m = 0;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
        i += (int64_t)gridDim.x * blockDim.x)
@@ -21,7 +21,7 @@ __global__ void k_max_color(const int32_t* __restrict__ c, int64_t n, int32_t* o
 // Step entry points (Algorithm 5 split line by line; not on the fused hot path).
 
 // Alg. 5 l.4-10: warp per listed vertex, exact for any degree.
-__global__ void __launch_bounds__(256) k_assign_step(const int64_t* __restrict__ row_ptr,
+static __global__ void __launch_bounds__(256) k_assign_step(const int64_t* __restrict__ row_ptr,
                                                      const int32_t* __restrict__ col_idx,
                                                      const int32_t* __restrict__ wl, int64_t len,
                                                      const int32_t* __restrict__ X,
@@ -38,7 +38,7 @@ __global__ void __launch_bounds__(256) k_assign_step(const int64_t* __restrict__
 }
 
 // Alg. 5 l.9: colors[wl[i]] = tent[i].
-__global__ void k_commit_step(const int32_t* __restrict__ wl, const int32_t* __restrict__ tent,
+static __global__ void k_commit_step(const int32_t* __restrict__ wl, const int32_t* __restrict__ tent,
                               int64_t len, int32_t* __restrict__ colors) {
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < len;
        i += (int64_t)gridDim.x * blockDim.x)
@@ -71,7 +71,7 @@ __global__ void __launch_bounds__(256) k_detect_step(const int64_t* __restrict__
 // Order-preserving compaction (Fig. 5): tile counts -> scan -> scatter.
 constexpr int kCompactTile = 1024;  // elements per tile (256 threads x 4)
 
-__global__ void __launch_bounds__(256) k_compact_count(const uint8_t* __restrict__ flags,
+static __global__ void __launch_bounds__(256) k_compact_count(const uint8_t* __restrict__ flags,
                                                        int64_t len, int32_t* __restrict__ tile_cnt) {
   const int64_t t0 = (int64_t)blockIdx.x * kCompactTile;
   int c = 0;
@@ -91,7 +91,7 @@ __global__ void __launch_bounds__(256) k_compact_count(const uint8_t* __restrict
 }
 
 // Exclusive scan of tile counts by one block (tiles <= a few million: sequential chunks).
-__global__ void __launch_bounds__(1024) k_compact_scan(int32_t* __restrict__ tile_cnt, int64_t tiles,
+static __global__ void __launch_bounds__(1024) k_compact_scan(int32_t* __restrict__ tile_cnt, int64_t tiles,
                                                        int64_t* __restrict__ total) {
   __shared__ int64_t carry_s;
   __shared__ int64_t warp_s[32];
@@ -129,7 +129,7 @@ __global__ void __launch_bounds__(1024) k_compact_scan(int32_t* __restrict__ til
   if (threadIdx.x == 0) *total = carry_s;
 }
 
-__global__ void __launch_bounds__(256) k_compact_scatter(const int32_t* __restrict__ wl,
+static __global__ void __launch_bounds__(256) k_compact_scatter(const int32_t* __restrict__ wl,
                                                          const uint8_t* __restrict__ flags,
                                                          int64_t len,
                                                          const int32_t* __restrict__ tile_off,
@@ -166,7 +166,7 @@ __global__ void __launch_bounds__(256) k_compact_scatter(const int32_t* __restri
 }
 
 // Device CSR validation: 1 offsets, 2 range, 4 unsorted.
-__global__ void k_validate(const int64_t* __restrict__ row_ptr, const int32_t* __restrict__ col_idx,
+static __global__ void k_validate(const int64_t* __restrict__ row_ptr, const int32_t* __restrict__ col_idx,
                            int64_t n, int64_t nnz, int32_t* violations) {
   int viol = 0;
   for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n;

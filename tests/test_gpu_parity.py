@@ -268,3 +268,57 @@ def test_full_size_configs_bit_exact(cfg):
     per-vertex loops; identical to the single-threaded oracle by construction)."""
     g = gen.config(cfg)
     check_full(g, LOW)
+
+
+# ----------------------------------------------------------------------------- multi-GPU path
+@pytest.mark.parametrize("P", [1, 2, 3, 5, 8])
+@pytest.mark.parametrize("tb", [LOW, PAP])
+def test_partitioned_equals_single_gpu(P, tb):
+    """The distributed exchange protocol (sgr_dist.cu: pack -> padded all-gather -> apply into
+    both replica buffers, lockstep advance) on P partitions of one device is bit-exact."""
+    for g in (gen.config(1), degree_boundary_graph(), random_graph(7, n=300)):
+        rp, ci = dev(g)
+        ref = oracle.jacobi(g, tb)
+        res = sgr.color_partitioned(rp, ci, P, tiebreak=RULE[tb])
+        assert np.array_equal(res.colors.cpu().numpy(), ref.colors), (g.name, P)
+        assert res.stats["rounds"] == ref.rounds
+        assert res.stats["vertices_processed"] == ref.vertices_processed
+        assert res.stats["num_colors"] == ref.num_colors
+
+
+@pytest.mark.parametrize("bits", [16, 32])
+def test_partitioned_random_ranges_and_widths(bits):
+    g = gen.rmat(14, 8, 0.57, 0.19, 0.19, seed=3)
+    rp, ci = dev(g)
+    ref = sgr.color(rp, ci).colors
+    rng = np.random.default_rng(0)
+    for P in (2, 4, 7):
+        cuts = np.sort(rng.integers(0, g.n + 1, P - 1))
+        ranges = np.concatenate([[0], cuts, [g.n]]).astype(np.int64)
+        res = sgr.color_partitioned(rp, ci, P, ranges=ranges, color_bits=bits)
+        assert torch.equal(res.colors, ref), (P, ranges)
+
+
+def test_nccl_world1_color_dist():
+    """sgr_comm_init + sgr_color_dist over a one-rank NCCL communicator (the box has one
+    GPU; multi-rank NCCL is exercised by bench.py under torchrun on a multi-GPU node)."""
+    import socket
+
+    import torch.distributed as dist
+    from paper_conf_ipps_licqfsty16_b200.dist import Comm, color_dist
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    dist.init_process_group("nccl", init_method=f"tcp://127.0.0.1:{port}", rank=0,
+                            world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        comm = Comm(0, 1, 0)
+        for g in (gen.config(1), degree_boundary_graph()):
+            rp, ci = dev(g)
+            res = color_dist(comm, rp, ci, g.n, 0, g.n)
+            ref = oracle.jacobi(g, LOW)
+            assert np.array_equal(res.colors.cpu().numpy(), ref.colors)
+            assert res.stats["rounds"] == ref.rounds
+        comm.close()
+    finally:
+        dist.destroy_process_group()
