@@ -31,6 +31,21 @@ sgr_status cuda_fail(cudaError_t e, const char* what, int line) {
   return SGR_ECUDA;
 }
 
+// Keep freed stream-ordered allocations in the device's default pool (the default release
+// threshold of 0 hands GB-sized workspaces back to the driver at every synchronize, and
+// the next call pays for fresh allocations).
+void keep_pool_memory() {
+  static bool done[64] = {false};
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64 || done[dev]) return;
+  cudaMemPool_t pool;
+  if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+    uint64_t thr = UINT64_MAX;
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+  }
+  done[dev] = true;
+}
+
 int num_sms() {
   static int sms[64] = {0};
   int dev = 0;
@@ -452,6 +467,7 @@ sgr_status sgr_color_ex(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* col
   }
   const Resolved r = resolve_opts(opts, n);
   cudaStream_t s = r.stream;
+  keep_pool_memory();
   const Layout L = layout(n, nnz, r);
   void* ws = workspace;
   bool own = false;
@@ -492,6 +508,7 @@ sgr_status sgr_color_host(const int64_t* row_ptr, const int32_t* col_idx, int64_
   if (n == 0) return SGR_OK;
   const Resolved r = resolve_opts(opts, n);
   cudaStream_t s = r.stream;
+  keep_pool_memory();
   int64_t* d_rp = nullptr;
   int32_t* d_ci = nullptr;
   int32_t* d_col = nullptr;

@@ -65,6 +65,7 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
                             int32_t* colors_out, sgr_stats* stats, const Gather& gather,
                             int64_t cap_hint, const Resolved& r) {
   cudaStream_t s = r.stream;
+  keep_pool_memory();
   const int P = (int)parts.size();
   std::vector<Layout> Ls;
   std::vector<RoundArgs<C>> args(P);

@@ -31,6 +31,7 @@ struct Resolved {
 void set_error(const char* fmt, ...);
 sgr_status cuda_fail(cudaError_t e, const char* what, int line);
 int num_sms();
+void keep_pool_memory();
 Resolved resolve_opts(const sgr_opts* o, int64_t n);
 size_t ws_bytes(int64_t n, int64_t nnz, const Resolved& r);
 void fill_stats(const Ctrl& c, int64_t n, int64_t nnz, sgr_stats* st);
