@@ -129,6 +129,7 @@ static sgr_status get_graph(const RoundArgs<C>& a, int grid, int batch, cudaGrap
   }
   for (int b = 0; b < batch; ++b) {
     k_round<TB, C><<<grid, kBlock, round_smem<C>(), cs>>>(a);
+    if constexpr (packed<C>()) k_finalize<TB, C><<<grid, kBlock, 0, cs>>>(a);
     k_advance<<<1, 32, 0, cs>>>(a.ctrl, 0);
   }
   cudaGraph_t graph;
@@ -199,6 +200,11 @@ void fill_stats(const Ctrl& c, int64_t n, int64_t nnz, sgr_stats* st) {
   }
   st->chunk_items = (int64_t)c.items_total;
   for (int q = 0; q < kBins; ++q) st->bin_warp_cycles[q] = (int64_t)c.bin_cycles[q];
+  if (const char* env = getenv("SGR_PHASES")) {  // experiments: bin-2 phase breakdown
+    (void)env;
+    fprintf(stderr, "sgr phases (warp-cycles): issue %llu wait %llu gather %llu post %llu\n",
+            c.phase_cycles[0], c.phase_cycles[1], c.phase_cycles[2], c.phase_cycles[3]);
+  }
   st->rounds = c.k - 1;
   st->num_colors = c.max_color;
   st->vertices_processed = n + vpass;
@@ -299,7 +305,10 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
           le = cudaGraphLaunch(gexec, s);
         } else {
           for (int b = 0; b < r.batch; ++b) {
-            prof.timed(SGR_K_ROUND, s, [&] { k_round<TB, C><<<grid, kBlock, round_smem<C>(), s>>>(a); });
+            prof.timed(SGR_K_ROUND, s, [&] {
+              k_round<TB, C><<<grid, kBlock, round_smem<C>(), s>>>(a);
+              if constexpr (packed<C>()) k_finalize<TB, C><<<grid, kBlock, 0, s>>>(a);
+            });
             prof.timed(SGR_K_CTRL, s, [&] { k_advance<<<1, 32, 0, s>>>(a.ctrl, 0); });
           }
           le = cudaGetLastError();

@@ -164,6 +164,7 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
     cap = *std::max_element(cnt.begin(), cnt.end());
     for (int i = 0; i < P; ++i) {
       k_round<TB, C><<<grid, kBlock, round_smem<C>(), s>>>(args[i]);
+      if constexpr (packed<C>()) k_finalize<TB, C><<<grid, kBlock, 0, s>>>(args[i]);
       k_advance<<<1, 32, 0, s>>>(args[i].ctrl, 0, 1);
     }
     DCK(cudaGetLastError());

@@ -22,7 +22,8 @@ inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 struct Layout {
   bool packed;
   int64_t cap_m, cap_c, cap_big;
-  size_t off_col, off_t, off_m, off_c, off_big, off_accb, off_accc, off_fixed, off_len, off_adj;
+  size_t off_col, off_t, off_m, off_c, off_big, off_accb, off_accc, off_fixed, off_len, off_adj,
+      off_fin;
   size_t zero_begin, zero_end, total;
 };
 
@@ -58,6 +59,8 @@ inline Layout layout(int64_t n, int64_t nnz, const Resolved& r) {
     o += 2 * nb;
   }
   L.zero_end = o;  // accumulators, fixed sets and list lengths start at zero
+  L.off_fin = o;
+  o += align_up((size_t)L.cap_big * 4, 256);
   if (L.packed) {
     L.off_adj = o;
     o += 2 * align_up((size_t)(nnz + 16) * 4, 256);
@@ -79,6 +82,7 @@ inline void build_args(RoundArgs<C>& a, const sgr_csr* csr, int64_t n, int64_t n
     a.col[0] = (C*)(b + L.off_col);
     a.col[1] = (C*)(b + L.off_col + nb);
     a.fixed = (uint32_t*)(b + L.off_fixed);
+    a.fin = (int32_t*)(b + L.off_fin);
     a.len[0] = (int32_t*)(b + L.off_len);
     a.len[1] = (int32_t*)(b + L.off_len + nb);
     const size_t ab = align_up((size_t)(nnz + 16) * 4, 256);

@@ -99,7 +99,8 @@ struct Ctrl {
   int32_t big_count;         // slots handed to bin-2 vertices by F_1
   int32_t max_color;
   int32_t violations;
-  int32_t pad[3];
+  int32_t fin_cnt;           // multi-chunk bin-2 vertices awaiting the finalize phase
+  int32_t pad[2];
   unsigned long long edges_acc[kBins];    // sum of deg(v) over the pass's vertices (algorithmic)
   unsigned long long entries_acc[kBins];  // CSR / list entries actually read by the pass
   unsigned long long verts_total[kBins + 1];   // [kBins] = F_1
@@ -108,6 +109,7 @@ struct Ctrl {
   unsigned long long pushes_total[kBins + 1];
   unsigned long long items_total;
   unsigned long long bin_cycles[kBins];   // warp-cycles spent in each bin (SM clock)
+  unsigned long long phase_cycles[4];     // bin 2 (trimmed) phases: issue, wait, gather, post
   int32_t* round_sizes;
   int64_t* round_edges;
 };
@@ -126,6 +128,7 @@ struct RoundArgs {
   int32_t* adj[2];            // trimmed adjacency lists (packed mode), offsets = row_ptr
   int32_t* len[2];            // [v] list length for the pass of parity p
   uint32_t* fixed;            // [slot][32] colors of dropped (finalized) neighbours
+  int32_t* fin;               // finalize list: multi-chunk vertices of the pass (v | buf << 31)
   Ctrl* ctrl;
   int64_t nnz;
   int32_t n;
@@ -567,6 +570,8 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
   };
   auto load_hdr = [&](int i, ChunkHdr& h) { finish_hdr(__ldcg(items + i), h); };
 
+  unsigned long long pc0 = 0, pc1 = 0, pc2 = 0, pc3 = 0;  // phase cycles (lane 0 adds)
+  long long tq = clock64();
   int i = gw;
   ChunkHdr cur, nxt;
   load_hdr(i, cur);
@@ -605,8 +610,12 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
       __syncwarp();
     }
 #else
+    const long long ta = clock64();
+    pc0 += (unsigned long long)(ta - tq);
     mbar_wait(bars + st, (ph >> st) & 1u);
     ph ^= 1u << st;
+    const long long tb = clock64();
+    pc1 += (unsigned long long)(tb - ta);
 #endif
     const int4* b4 = reinterpret_cast<const int4*>(bufs + st * (kStage / 4));
     bool conf = false;
@@ -645,6 +654,10 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
         }
       }
     }
+#if !SGR_NO_TMA
+    const long long tc = clock64();
+    pc2 += (unsigned long long)(tc - tb);
+#endif
     // next-next header: the item id has arrived by now
     ChunkHdr nn;
     nn.v = nn.c = nn.len = nn.slot = nn.buf = 0;
@@ -715,6 +728,9 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
         Y[v] = cpack<C>(xv, k, ctrl);
       }
     } else {
+      // several chunks: publish this chunk's partial forbidden set, dropped colors and
+      // compacted live entries; the finalize phase after the pass decides conflict and
+      // first fit once every chunk is in (no per-chunk fences or tickets)
       uint32_t* accb = a.acc_bits + (int64_t)slot * 32;
       const uint32_t bits = tbl_bits32(tbl_all, lane);
       const uint32_t drop = tbl_bits32(tbl_drop, lane);
@@ -724,49 +740,17 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
       if (lane == 0 && live_total) lbase = atomicAdd(len_nxt + v, (int32_t)live_total);
       lbase = __shfl_sync(0xffffffffu, lbase, 0);
       write_live(lst_other + cur.s + lbase);
-      __syncwarp();  // orders every lane's writes before lane 0's release below
-      unsigned long long old = 0;
-      if (lane == 0) old = atom_add_acq_rel(a.acc_cnt + slot, 1ull | ((unsigned long long)any << 32));
-      old = __shfl_sync(0xffffffffu, old, 0);
-      if ((uint32_t)old == (uint32_t)(nch - 1)) {  // last chunk of v in this pass
-        fence_acq_rel_gpu();
-        const uint32_t word = ld_cg(accb + lane) | ld_cg(fx + lane) | (lane == 0 ? 1u : 0u);
-        accb[lane] = 0u;
-        const bool conf_all = ((old >> 32) + (any ? 1ull : 0ull)) != 0ull;
-        int32_t tent = 0;
-        if (conf_all) {
-          tent = bits_first_free(word);
-          if (tent < 0 || tent >= kBigTbl - 1) {  // beyond the exact range of the table
-            tent = warp_first_fit_rescan<Persist>(a.col_idx, X, cur.s, cur.e, kBigTbl - 1, lane);
-          }
-        }
-        int32_t nch2 = 0;
-        if (lane == 0) {
-          a.acc_cnt[slot] = 0ull;
-          len_cur[v] = 0;  // consumed; the pass after next accumulates into it
-          Y[v] = conf_all ? cpack<C>(tent, k + 1, ctrl) : cpack<C>(xv, k, ctrl);
-          if (conf_all) nch2 = num_chunks(ld_cg(len_nxt + v));
-        }
-        if (conf_all) {
-          nch2 = __shfl_sync(0xffffffffu, nch2, 0);
-          const uint32_t nbuf = cur.buf ? 0u : kBufBit;  // the list moved to the other buffer
-          ++vpend;
-          if (ipend + nch2 > 32) iflush();
-          if (nch2 > 32) {  // a hub with many chunks: direct
-            int ob = 0;
-            if (lane == 0) ob = atomicAdd(out_cnt, nch2);
-            ob = __shfl_sync(0xffffffffu, ob, 0);
-            for (int32_t t = lane; t < nch2; t += 32) out[ob + t] = make_item(v, (int32_t)(t | nbuf));
-          } else {
-            if (lane < nch2) ibuf[ipend + lane] = make_item(v, (int32_t)(lane | nbuf));
-            ipend += nch2;
-            if (ipend == 32) iflush();
-          }
-        }
+      if (lane == 0) {
+        if (any) atomicOr(a.acc_cnt + slot, 1ull);  // conflict flag
+        if (cur.c == 0) a.fin[atomicAdd(&ctrl->fin_cnt, 1)] = (int32_t)((uint32_t)v | (cur.buf ? kBufBit : 0u));
       }
     }
     clear_bytes(tbl_all, kTblBytes / 32, lane);  // both tables
     __syncwarp();
+#if !SGR_NO_TMA
+    tq = clock64();
+    pc3 += (unsigned long long)(tq - tc);
+#endif
     st ^= 1;
     i = in;
     in = inn;
@@ -775,6 +759,67 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
   }
   iflush();
   if (lane == 0 && vpend) atomicAdd(out_vcnt, vpend);
+  if (lane == 0) {
+    atomicAdd(&ctrl->phase_cycles[0], pc0);
+    atomicAdd(&ctrl->phase_cycles[1], pc1);
+    atomicAdd(&ctrl->phase_cycles[2], pc2);
+    atomicAdd(&ctrl->phase_cycles[3], pc3);
+  }
+}
+
+// Finalize phase of a trimmed pass (after every chunk of the pass is done): for each
+// multi-chunk bin-2 vertex, the merged forbidden set is the OR of its chunks' partial sets
+// and its fixed set; conflict is the OR of the chunks' flags (Alg. 5 l.12-15), the first
+// fit the lowest free color (l.8). Writes Y[v], pushes the vertex's next-round chunk items
+// (its compacted list now lives in the other buffer), and resets the accumulators.
+template <int TB, bool Persist>
+__device__ __forceinline__ void finalize_body(const RoundArgs<uint32_t>& a, int k) {
+  using C = uint32_t;
+  Ctrl* ctrl = a.ctrl;
+  const int p = k & 1;
+  const int lane = threadIdx.x & 31;
+  const int gw = (int)((blockIdx.x * blockDim.x + threadIdx.x) >> 5);
+  const int NW = (int)((gridDim.x * blockDim.x) >> 5);
+  const int nF = ld_cg(&ctrl->fin_cnt);
+  const C* X = sel((k - 1) & 1, (const C*)a.col[0], (const C*)a.col[1]);
+  C* Y = sel(k & 1, a.col[0], a.col[1]);
+  int64_t* out = sel(p ^ 1, a.wl_c[0], a.wl_c[1]);
+  int32_t* len_cur = sel(p, a.len[0], a.len[1]);
+  int32_t* len_nxt = sel(p ^ 1, a.len[0], a.len[1]);
+  for (int i = gw; i < nF; i += NW) {
+    const uint32_t f = (uint32_t)ld_cg(a.fin + i);
+    const int32_t v = (int32_t)(f & ~kBufBit);
+    const int32_t slot = __ldg(a.big_id + v);
+    uint32_t* accb = a.acc_bits + (int64_t)slot * 32;
+    const uint32_t word = ld_cg(accb + lane) | ld_cg(a.fixed + (int64_t)slot * 32 + lane) |
+                          (lane == 0 ? 1u : 0u);
+    const bool conf = (__ldcg(a.acc_cnt + slot) & 1ull) != 0ull;
+    accb[lane] = 0u;
+    int32_t tent = 0;
+    if (conf) {
+      tent = bits_first_free(word);
+      if (tent < 0 || tent >= kBigTbl - 1)  // beyond the exact range of the table
+        tent = warp_first_fit_rescan<Persist>(a.col_idx, X, ldg_i64(a.row_ptr + v),
+                                              ldg_i64(a.row_ptr + v + 1), kBigTbl - 1, lane);
+    }
+    int32_t ob = 0, nch2 = 0;
+    if (lane == 0) {
+      a.acc_cnt[slot] = 0ull;
+      len_cur[v] = 0;  // consumed; the pass after next accumulates into it
+      Y[v] = conf ? cpack<C>(tent, k + 1, ctrl) : cpack<C>(cval<C>(ldraw<Persist>(X + v)), k, ctrl);
+      if (conf) {
+        nch2 = num_chunks(ld_cg(len_nxt + v));
+        ob = atomicAdd(&ctrl->cnt[p ^ 1][2], nch2);
+        atomicAdd(&ctrl->vcnt2[p ^ 1], 1);
+      }
+    }
+    if (conf) {
+      ob = __shfl_sync(0xffffffffu, ob, 0);
+      nch2 = __shfl_sync(0xffffffffu, nch2, 0);
+      const uint32_t nbuf = (f & kBufBit) ? 0u : kBufBit;  // the list moved to the other buffer
+      for (int32_t t = lane; t < nch2; t += 32) out[ob + t] = make_item(v, (int32_t)(t | nbuf));
+    }
+  }
 }
 
 // Bin 1: each 8-lane group of the warp processes one vertex (v < 0: idle group) in batches
@@ -1106,6 +1151,7 @@ __device__ __forceinline__ void advance_body(Ctrl* ctrl, bool first, bool force 
     tot_in += vin[q];
   }
   c->items_total += (unsigned long long)c->cnt[p][2];
+  c->fin_cnt = 0;
   for (int q = 0; q < kBins; ++q) c->cnt[p][q] = 0;
   c->vcnt2[p] = 0;
   if (k - 1 < c->round_cap) {
@@ -1229,8 +1275,17 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks<C>) k_round(RoundArgs<C> a)
     for (int q = 0; q < kBins; ++q) atomicAdd(&ctrl->bin_cycles[q], cyc[q]);
 }
 
+// Finalize phase as its own launch (host / graph loop modes), between k_round and k_advance.
+template <int TB, class C>
+__global__ void __launch_bounds__(kBlock) k_finalize(RoundArgs<C> a) {
+  if constexpr (packed<C>()) {
+    if (!a.ctrl->active) return;
+    finalize_body<TB, false>(a, a.ctrl->k);
+  }
+}
+
 // Grid-wide barrier whose last arriving block runs advance_body (persistent kernel).
-__device__ __forceinline__ void grid_sync_advance(Ctrl* ctrl) {
+__device__ __forceinline__ void grid_sync_advance(Ctrl* ctrl, bool advance = true) {
   __syncthreads();
   if (threadIdx.x == 0) {
     volatile uint32_t* gen_p = &ctrl->bar_gen;
@@ -1239,7 +1294,7 @@ __device__ __forceinline__ void grid_sync_advance(Ctrl* ctrl) {
     const uint32_t arrived = atomicAdd(&ctrl->bar_count, 1u);
     if (arrived == gridDim.x - 1) {
       __threadfence();
-      advance_body(ctrl, false);
+      if (advance) advance_body(ctrl, false);
       *(volatile uint32_t*)&ctrl->bar_count = 0u;
       __threadfence();
       atomicAdd(&ctrl->bar_gen, 1u);
@@ -1266,6 +1321,10 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks<C>) k_persistent(RoundArgs<
     unsigned long long edges[kBins] = {0, 0, 0}, entries[kBins] = {0, 0, 0};
     round_body<TB, true, C>(a, k, wsm, edges, entries, ph, cyc);
     block_add6(edges, entries, ctrl);
+    if constexpr (packed<C>()) {  // multi-chunk vertices are decided once all chunks are in
+      grid_sync_advance(ctrl, false);
+      finalize_body<TB, true>(a, k);
+    }
     grid_sync_advance(ctrl);
   }
   if ((threadIdx.x & 31) == 0)

@@ -139,8 +139,9 @@ int main(int argc, char** argv) {
     printf("%-34s %8.3f ms  %7.1f G gathers/s  (%.2f per SM-cycle @1.9GHz)\n", name, ms,
            m / ms / 1e6, m / (ms * 1e-3) / sms / 1.9e9);
   };
-  const int grid = sms * 8, blk = 256;
-  printf("n=%lld m=%lld locality=%d sms=%d\n", n, m, locality, sms);
+  const int bps = argc > 4 ? atoi(argv[4]) : 8;  // blocks of 256 threads per SM
+  const int grid = sms * bps, blk = 256;
+  printf("n=%lld m=%lld locality=%d sms=%d blocks/SM=%d\n", n, m, locality, sms, bps);
   timeit("stream idx only", [&] { k_stream<<<grid, blk>>>(d_idx, m, d_out); });
   timeit("default ld (U=8)", [&] { k_gather<0, 8><<<grid, blk>>>(d_idx, m, d_x, d_out); });
   timeit("ld.cg (U=8)", [&] { k_gather<1, 8><<<grid, blk>>>(d_idx, m, d_x, d_out); });
@@ -148,6 +149,8 @@ int main(int argc, char** argv) {
   timeit("ld.nc.L1::no_allocate (U=8)", [&] { k_gather<3, 8><<<grid, blk>>>(d_idx, m, d_x, d_out); });
   timeit("ldg (U=2)", [&] { k_gather<2, 2><<<grid, blk>>>(d_idx, m, d_x, d_out); });
   timeit("ldg (U=16)", [&] { k_gather<2, 16><<<grid, blk>>>(d_idx, m, d_x, d_out); });
+  timeit("ldg (U=32)", [&] { k_gather<2, 32><<<grid, blk>>>(d_idx, m, d_x, d_out); });
+  timeit("ld.cg (U=16)", [&] { k_gather<1, 16><<<grid, blk>>>(d_idx, m, d_x, d_out); });
   if (tex) timeit("tex1Dfetch (U=8)", [&] { k_gather_tex<8><<<grid, blk>>>(d_idx, m, tex, d_out); });
   timeit("u16 ldg (U=8)", [&] { k_gather16<8><<<grid, blk>>>(d_idx, m, d_x16, d_out); });
   return 0;
