@@ -82,10 +82,10 @@ typedef struct {
   int32_t tiebreak;      /* sgr_tiebreak; default LOWID_KEEPS */
   int32_t max_rounds;    /* 0 = n+1 (never reached) */
   int32_t loop_mode;     /* sgr_loop_mode */
-  int32_t color_bits;    /* 16 (default): packed 16-bit color + 16-bit round words, with
-                            live-neighbour trimming of high-degree rows; a color or round
-                            above 65535 triggers an automatic 32-bit rerun. 32: plain int32
-                            colors, full rows every round */
+  int32_t color_bits;    /* 16 (default): 16-bit words (12-bit color + round mod 16), with
+                            live-neighbour trimming of high-degree rows; a color above 4095
+                            triggers an automatic 32-bit rerun. 32: plain int32 colors,
+                            full rows every round */
   int32_t bin_small_max; /* degree bins: d <= small -> 8 lanes/vertex, register mask (<= 62);
                             0 = 32 */
   int32_t bin_med_max;   /* small < d <= med -> 8 lanes/vertex, smem table (<= 256); 0 = 256;
@@ -99,6 +99,9 @@ typedef struct {
   int32_t profile;       /* != 0: time every kernel launch with CUDA events */
   float* round_ms;       /* optional HOST buffer (round_cap): with profile != 0 and the host
                             loop, device time of each round pass k = 2, 3, ... */
+  int32_t color_cap;     /* test hook: 0 = 4095, the largest color a 16-bit word holds; a
+                            smaller cap sends colorings whose colors exceed it down the
+                            automatic 32-bit rerun path (results are unchanged) */
 } sgr_opts;
 
 /* Kernel classes (stats->kernel_*): F_1, the fused round pass(es), loop control, final. */

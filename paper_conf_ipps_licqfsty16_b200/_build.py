@@ -70,9 +70,10 @@ def build_oracle(force=False):
     return out
 
 
-def build_cuda(force=False):
+def build_cuda(force=False, out=None, extra=(), tag="obj"):
+    """libsgr.so; `out`/`extra` build an alternative (tools/variants.py experiments)."""
     LIB.mkdir(exist_ok=True)
-    out = LIB / "libsgr.so"
+    out = Path(out) if out else LIB / "libsgr.so"
     cu = sorted(CSRC.glob("*.cu"))
     if not cu:
         return None
@@ -81,13 +82,13 @@ def build_cuda(force=False):
         return out
     nccl_inc, nccl_lib = _nccl_dirs()
     flags = ["-O3", "-std=c++17", "-lineinfo", *ARCH, "-Xcompiler", "-fPIC,-Wall",
-             "-Xptxas", "-v", "--expt-relaxed-constexpr", "-I", INCLUDE, "-I", CSRC]
+             "-Xptxas", "-v", "--expt-relaxed-constexpr", "-I", INCLUDE, "-I", CSRC, *extra]
     link = ["-shared", "-lcudart"]
     if nccl_inc is not None:
         flags += ["-DSGR_HAVE_NCCL=1", "-I", nccl_inc]
         link += ["-L", nccl_lib, "-l:libnccl.so.2", f"-Xlinker=-rpath,{nccl_lib}"]
     objs = []
-    bdir = LIB / "obj"
+    bdir = LIB / tag
     bdir.mkdir(exist_ok=True)
     for src in cu:
         obj = bdir / (src.stem + ".o")

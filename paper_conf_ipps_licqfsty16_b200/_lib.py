@@ -5,9 +5,13 @@ There is no fallback: if the CUDA library is missing or fails to load, every cal
 from __future__ import annotations
 
 import ctypes
+import os
 from pathlib import Path
 
 LIBPATH = Path(__file__).resolve().parent / "lib" / "libsgr.so"
+# experiments only (tools/variants.py): load an alternative build of the same library
+if os.environ.get("SGR_LIBPATH"):
+    LIBPATH = Path(os.environ["SGR_LIBPATH"])
 
 SGR_K_COUNT = 4
 KERNEL_CLASSES = ("first", "round", "control", "final")
@@ -25,7 +29,8 @@ class Opts(ctypes.Structure):
                 ("stream", ctypes.c_void_p), ("round_sizes", ctypes.c_void_p),
                 ("round_edges", ctypes.c_void_p), ("round_cap", ctypes.c_int32),
                 ("validate", ctypes.c_int32), ("rounds_per_batch", ctypes.c_int32),
-                ("profile", ctypes.c_int32), ("round_ms", ctypes.c_void_p)]
+                ("profile", ctypes.c_int32), ("round_ms", ctypes.c_void_p),
+                ("color_cap", ctypes.c_int32)]
 
 
 class Stats(ctypes.Structure):

@@ -80,6 +80,8 @@ Resolved resolve_opts(const sgr_opts* o, int64_t n) {
   r.batch = o->rounds_per_batch > 0 ? o->rounds_per_batch : 8;
   r.profile = o->profile;
   r.round_ms = o->round_ms;
+  r.color_cap = (o->color_cap > 0 && o->color_cap < (int32_t)kColorMask) ? o->color_cap
+                                                                         : (int32_t)kColorMask;
   return r;
 }
 
@@ -361,7 +363,7 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
         if (m.first == SGR_K_ROUND && r.round_ms && ri < r.round_cap) r.round_ms[ri++] = ms;
       }
     }
-    if (fin.status == 1) {
+    if (fin.status == 1 && !fin.overflow) {
       set_error("sgr_color: max_rounds (%d) reached", r.max_rounds);
       status = SGR_ENOCONV;
     }
@@ -376,9 +378,9 @@ static sgr_status run_any(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* c
                           sgr_stats* stats, const Resolved& r, void* ws, const Layout& L) {
   int overflow = 0;
   if (r.color_bits == 16) {
-    const sgr_status st = run_color<TB, uint32_t>(csr, n, nnz, colors_out, stats, r, ws, L, &overflow);
+    const sgr_status st = run_color<TB, Packed>(csr, n, nnz, colors_out, stats, r, ws, L, &overflow);
     if (st != SGR_OK || !overflow) return st;
-    // a color or round number exceeded 16 bits: the packed run is discarded and redone
+    // a color exceeded 12 bits (4095): the packed run is discarded and redone
     // with plain 32-bit colors (no trimming)
   }
   Resolved r32 = r;

@@ -63,7 +63,7 @@ using Gather = std::function<sgr_status(std::vector<Part>& parts, uint2* recv, i
 template <int TB, class C>
 static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_t n,
                             int32_t* colors_out, sgr_stats* stats, const Gather& gather,
-                            int64_t cap_hint, const Resolved& r) {
+                            int64_t cap_hint, const Resolved& r, int* overflow_out) {
   cudaStream_t s = r.stream;
   keep_pool_memory();
   const int P = (int)parts.size();
@@ -107,8 +107,9 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
   uint2* recv = nullptr;
   DCK(cudaMallocAsync((void**)&recv, (size_t)world * (cap_max + 1) * sizeof(uint2), s));
   std::vector<uint2> hdr(world);
-  int32_t* counts_host = nullptr;
-  DCK(cudaMallocHost(&counts_host, sizeof(int32_t) * world));
+  int32_t* counts_host = nullptr;  // per part: (record count, overflow flag)
+  DCK(cudaMallocHost(&counts_host, 2 * sizeof(int32_t) * world));
+  bool overflow_seen = false;
 
   // one exchange: pack -> all-gather with capacity cap -> apply; returns per-part counts
   auto exchange = [&](int32_t cap, std::vector<int32_t>& cnt) -> sgr_status {
@@ -122,10 +123,15 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
     for (int i = 0; i < P; ++i)
       k_apply<C><<<first_grid(cap), 256, 0, s>>>(args[i], recv, world, cap + 1, me0 + i);
     DCK(cudaGetLastError());
-    DCK(cudaMemcpy2DAsync(counts_host, sizeof(int32_t), recv, (size_t)(cap + 1) * sizeof(uint2),
-                          sizeof(int32_t), world, cudaMemcpyDeviceToHost, s));
+    DCK(cudaMemcpy2DAsync(counts_host, sizeof(uint2), recv, (size_t)(cap + 1) * sizeof(uint2),
+                          sizeof(uint2), world, cudaMemcpyDeviceToHost, s));
     DCK(cudaStreamSynchronize(s));
-    cnt.assign(counts_host, counts_host + world);
+    cnt.resize(world);
+    for (int q = 0; q < world; ++q) {
+      cnt[q] = counts_host[2 * q];
+      if (counts_host[2 * q + 1]) overflow_seen = true;
+    }
+    if (overflow_seen) std::fill(cnt.begin(), cnt.end(), 0);  // stop; rerun with int32 words
     return SGR_OK;
   };
 
@@ -141,14 +147,18 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
       k_pack<C><<<first_grid(parts[i].hi - parts[i].lo + 1), 256, 0, s>>>(args[i], parts[i].send, 0);
     status = gather(parts, recv, 0, s);
     if (status == SGR_OK) {
-      DCK(cudaMemcpy2DAsync(counts_host, sizeof(int32_t), recv, sizeof(uint2), sizeof(int32_t),
+      DCK(cudaMemcpy2DAsync(counts_host, sizeof(uint2), recv, sizeof(uint2), sizeof(uint2),
                             world, cudaMemcpyDeviceToHost, s));
       DCK(cudaStreamSynchronize(s));
     }
   }
   cudaEventRecord(ev0, s);
   int32_t cap = 0;
-  for (int q = 0; q < world && status == SGR_OK; ++q) cap = std::max(cap, counts_host[q]);
+  for (int q = 0; q < world && status == SGR_OK; ++q) {
+    cap = std::max(cap, counts_host[2 * q]);
+    if (counts_host[2 * q + 1]) overflow_seen = true;
+  }
+  if (overflow_seen) cap = 0;
   int64_t vertices = n, rounds = 1;
   if (status == SGR_OK) status = exchange(cap, cnt);  // W_2 records
   int64_t total = 0;
@@ -188,12 +198,13 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
     for (int i = 0; i < P; ++i)
       DCK(cudaMemcpyAsync(&fin[i], args[i].ctrl, sizeof(Ctrl), cudaMemcpyDeviceToHost, s));
     DCK(cudaStreamSynchronize(s));
-    int overflow = 0;
+    int overflow = overflow_seen ? 1 : 0;
     for (int i = 0; i < P; ++i) overflow |= fin[i].overflow;
-    if (overflow) {
-      set_error("sgr_color_dist: a color or round number exceeded 16 bits; use color_bits=32");
+    if (overflow && !packed<C>()) {
+      set_error("sgr_color_dist: 32-bit color overflow");
       status = SGR_EUNSUPPORTED;
     }
+    if (overflow && packed<C>()) *overflow_out = 1;  // every rank saw the same flags
     if (stats) {
       memset(stats, 0, sizeof(*stats));
       for (int i = 0; i < P; ++i) {
@@ -236,14 +247,20 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
   return status;
 }
 
+// Packed (16-bit) words first; if any partition's first fit exceeded the color cap, every
+// rank saw the flag in the same exchange and the whole coloring is redone with int32 words.
 template <class... A>
 static sgr_status dispatch(const Resolved& r, A&&... args) {
+  int overflow = 0;
   if (r.color_bits == 16) {
-    return r.tiebreak ? run_parts<1, uint32_t>(std::forward<A>(args)..., r)
-                      : run_parts<0, uint32_t>(std::forward<A>(args)..., r);
+    const sgr_status st = r.tiebreak ? run_parts<1, Packed>(args..., r, &overflow)
+                                     : run_parts<0, Packed>(args..., r, &overflow);
+    if (st != SGR_OK || !overflow) return st;
   }
-  return r.tiebreak ? run_parts<1, int32_t>(std::forward<A>(args)..., r)
-                    : run_parts<0, int32_t>(std::forward<A>(args)..., r);
+  Resolved r32 = r;
+  r32.color_bits = 32;
+  return r.tiebreak ? run_parts<1, int32_t>(args..., r32, &overflow)
+                    : run_parts<0, int32_t>(args..., r32, &overflow);
 }
 
 }  // namespace sgr

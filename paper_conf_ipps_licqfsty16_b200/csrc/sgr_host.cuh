@@ -14,11 +14,11 @@ namespace sgr {
 inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
 // Workspace layout (bytes, each piece 256-aligned):
-//   Ctrl | colors: 2 x n words | wl_t: 2 x n i32 | wl_m: 2 x cap_m i32 | wl_c: 2 x cap_c i64 |
+//   Ctrl | colors: 2 x n words (u16 packed / i32) | wl_t: 2 x n i32 | wl_m: 2 x cap_m i32 | wl_c: 2 x cap_c i64 |
 //   big_id: n i32 | acc_bits: cap_big x 32 u32 | acc_cnt: cap_big u64 |
 //   (packed mode) fixed: cap_big x 32 u32 | len: 2 x n i32 | adj: 2 x (nnz + 16) i32
 // 32-bit mode: the caller's colors_out is one of the two ping-pong buffers. Packed mode
-// (16-bit color + 16-bit round, trimming) uses two workspace buffers and unpacks at the end.
+// (12-bit color + round mod 16, trimming) uses two workspace buffers and unpacks at the end.
 struct Layout {
   bool packed;
   int64_t cap_m, cap_c, cap_big;
@@ -37,7 +37,7 @@ inline Layout layout(int64_t n, int64_t nnz, const Resolved& r) {
   const size_t nb = align_up((size_t)n * 4, 256);
   size_t o = align_up(sizeof(Ctrl), 256);
   L.off_col = o;
-  o += 2 * nb;
+  o += 2 * align_up((size_t)n * (L.packed ? sizeof(Packed) : 4), 256);
   L.off_t = o;
   o += 2 * nb;
   L.off_m = o;
@@ -80,7 +80,7 @@ inline void build_args(RoundArgs<C>& a, const sgr_csr* csr, int64_t n, int64_t n
   a.col_idx = csr->col_idx;
   if constexpr (packed<C>()) {
     a.col[0] = (C*)(b + L.off_col);
-    a.col[1] = (C*)(b + L.off_col + nb);
+    a.col[1] = (C*)(b + L.off_col + align_up((size_t)n * sizeof(C), 256));
     a.fixed = (uint32_t*)(b + L.off_fixed);
     a.fin = (int32_t*)(b + L.off_fin);
     a.len[0] = (int32_t*)(b + L.off_len);
@@ -110,6 +110,7 @@ inline void build_args(RoundArgs<C>& a, const sgr_csr* csr, int64_t n, int64_t n
   a.v_end = (int32_t)n;
   a.small_max = r.small_max;
   a.med_max = r.med_max;
+  a.color_cap = r.color_cap;
 }
 
 inline int first_grid(int64_t n) {

@@ -26,6 +26,7 @@ struct Resolved {
   int batch;
   int profile;
   float* round_ms;
+  int32_t color_cap;
 };
 
 void set_error(const char* fmt, ...);

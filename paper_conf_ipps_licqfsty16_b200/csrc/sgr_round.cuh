@@ -21,9 +21,11 @@
 //          to finish (atomic ticket) decides conflict and first fit.
 //
 // Live-neighbour trimming (bin 2, packed colors; DESIGN.md §3 proof (vii)): a neighbour
-// that has left the worklist never changes color again. Colors are stored packed as
-// (last round the vertex was in W) << 16 | color, so one gather also says whether the
-// neighbour is still live (last >= k). Each bin-2 vertex keeps its adjacency list in a
+// that has left the worklist never changes color again. Colors are stored as 16-bit words
+// (last round the vertex was in W, mod 16) << 12 | color, so one gather also says whether
+// the neighbour is still live (last == k mod 16; a neighbour that left exactly 16 r rounds
+// ago looks live and is kept one more round, which is harmless: only live neighbours must
+// never be dropped). Each bin-2 vertex keeps its adjacency list in a
 // double-buffered copy adj[2] (same offsets as col_idx) and a 1024-bit set F of the colors
 // of the neighbours it has dropped; every pass reads the current list, drops the neighbours
 // that are no longer live (their colors go to F), and writes the compacted list for the
@@ -60,22 +62,44 @@ constexpr int kMaxSmall = kG0 * kK0;    // 32
 constexpr int kPushBuf = 64;            // per-warp push buffer (bins 0/1), flushed at >= 32
 constexpr int kK1 = 32;                 // entries per lane, bin 1 (8 x 32 = 256)
 constexpr int kMaxMed = kGroup * kK1;   // 256
-constexpr int kMedTbl = 512;            // bin-1 table bytes (colors < 512 > 257)
-constexpr int kBigTbl = 1024;           // bin-2 table bytes (colors < 1024)
-constexpr int kTblBytes = 2048;         // per-warp tables: 4 x 512 (bin 1) | 2 x 1024 (bin 2)
-constexpr int kChunk = 1020;            // bin-2 chunk: entries per warp item; the 16-byte-
-                                        // aligned window (<= 1024 entries) covers it
-constexpr int kWin = 1024;              // window entries (32 lanes x 8 int4)
+// Forbidden-color sets in shared memory: SGR_BITTBL = 1 one bit per color (shared atomicOr),
+// 0 one byte per color (plain byte stores). Bit sets leave more of the SM's unified
+// L1/shared storage to the L1 cache that serves the color gathers.
+#ifndef SGR_BITTBL
+#define SGR_BITTBL 0
+#endif
+constexpr int kMedTbl = 512;            // bin-1 set: colors < 512 (first fit <= 257)
+constexpr int kBigTbl = 1024;           // bin-2 set: colors < 1024
+constexpr int kTblDiv = SGR_BITTBL ? 8 : 1;
+constexpr int kMedTblB = kMedTbl / kTblDiv;  // bytes
+constexpr int kBigTblB = kBigTbl / kTblDiv;
+constexpr int kTblBytes = 2 * kBigTblB;      // per-warp tables: 4 x bin-1 | 2 x bin-2
+#ifndef SGR_WIN
+#define SGR_WIN 1024
+#endif
+constexpr int kWin = SGR_WIN;           // window entries (32 lanes x kWin / 128 int4)
+constexpr int kChunk = kWin - 4;        // bin-2 chunk: entries per warp item; the 16-byte-
+                                        // aligned window (<= kWin entries) covers it
+static_assert(kWin == 512 || kWin == 1024, "window: 512 or 1024 entries");
 
+// Working color word. Packed (default): uint16_t = (last round mod 16) << 12 | color, color
+// <= 4095 (a larger first fit sets the overflow flag and the coloring is redone with plain
+// int32 words, which have no round field and no trimming).
+using Packed = uint16_t;
+constexpr uint32_t kColorMask = 0xfffu;
+constexpr int kRoundShift = 12;
 template <class C>
-__host__ __device__ constexpr bool packed() { return sizeof(C) == 4 && C(-1) > C(0); }
+__host__ __device__ constexpr bool packed() { return sizeof(C) == 2; }
 
 // dynamic shared memory per warp: [2 TMA stages (packed only)] [tables] [2 mbarriers]
 constexpr int kStage = kWin * 4;        // bytes per TMA stage: one bin-2 window
 // blocks per SM the round kernels are compiled for: packed mode is shared-memory bound to 2
 // (82 KB per block), plain mode can afford 3 (<= 85 registers)
+#ifndef SGR_MINB
+#define SGR_MINB 2
+#endif
 template <class C>
-constexpr int kMinBlocks = packed<C>() ? 2 : 3;
+constexpr int kMinBlocks = packed<C>() ? SGR_MINB : 3;
 template <class C> struct WarpSmem {
   static constexpr int kBuf = packed<C>() ? 2 * kStage : 0;
   static constexpr int kPush = kBuf + kTblBytes;         // push buffer (kPushBuf int32)
@@ -92,7 +116,7 @@ struct Ctrl {
   int32_t max_rounds;
   int32_t cnt[2][kBins];     // work items per parity (k & 1) and bin
   int32_t vcnt2[2];          // bin-2 worklist VERTICES per parity (items are chunks)
-  int32_t overflow;          // a packed color or round number exceeded 16 bits
+  int32_t overflow;          // a packed color exceeded 12 bits (4095)
   int32_t round_cap;
   uint32_t bar_count;        // grid barrier (persistent kernel)
   uint32_t bar_gen;
@@ -136,7 +160,7 @@ struct RoundArgs {
   int32_t med_max;
   int32_t v_begin;            // owned vertex range [v_begin, v_end) (multi-GPU: a partition)
   int32_t v_end;
-  int32_t pad;
+  int32_t color_cap;          // packed mode: largest color a 16-bit word holds (<= 4095)
 };
 
 // Parameter-struct selects without dynamic indexing (which would spill it to the stack).
@@ -146,7 +170,7 @@ __device__ __forceinline__ T sel(int par, T a0, T a1) { return par ? a1 : a0; }
 __device__ __forceinline__ int32_t ld_cg(const int32_t* p) { return __ldcg(p); }
 __device__ __forceinline__ uint32_t ld_cg(const uint32_t* p) { return __ldcg(p); }
 
-// ---- color words: int32_t = plain color; uint32_t = (last round << 16) | color ----------
+// ---- color words: int32_t = plain color; Packed = (last round mod 16) << 12 | color ------
 template <bool Persist, class C>
 __device__ __forceinline__ uint32_t ldraw(const C* p) {
   if constexpr (Persist) return (uint32_t)__ldcg(p);
@@ -154,23 +178,23 @@ __device__ __forceinline__ uint32_t ldraw(const C* p) {
 }
 template <class C>
 __device__ __forceinline__ int32_t cval(uint32_t raw) {
-  if constexpr (packed<C>()) return (int32_t)(raw & 0xffffu);
+  if constexpr (packed<C>()) return (int32_t)(raw & kColorMask);
   else return (int32_t)raw;
 }
 template <bool Persist, class C>
 __device__ __forceinline__ int32_t ldc(const C* p) { return cval<C>(ldraw<Persist>(p)); }
 
 template <class C>
-__device__ __forceinline__ C cpack(int32_t color, int32_t last, Ctrl* ctrl) {
+__device__ __forceinline__ C cpack(int32_t color, int32_t last, const RoundArgs<C>& a) {
   if constexpr (packed<C>()) {
-    if (color > 0xffff || last > 0xffff) {
-      ctrl->overflow = 1;
-      return (C)0xffffffffu;
+    if (color > a.color_cap) {  // color_cap = 4095 unless a test lowers it
+      a.ctrl->overflow = 1;
+      return (C)kColorMask;
     }
-    return (C)(((uint32_t)last << 16) | (uint32_t)color);
+    return (C)((((uint32_t)last & 15u) << kRoundShift) | (uint32_t)color);
   } else {
     (void)last;
-    (void)ctrl;
+    (void)a;
     return (C)color;
   }
 }
@@ -279,8 +303,8 @@ __global__ void __launch_bounds__(256) k_first(RoundArgs<C> a, int sorted) {
           for (int64_t j = s; j < e && !conflict; ++j) conflict = lose<TB>(v, ldg_i32(a.col_idx + j));
         }
       }
-      X[v] = cpack<C>(1, 1, ctrl);
-      Y[v] = cpack<C>(conflict ? 2 : 1, conflict ? 2 : 1, ctrl);
+      X[v] = cpack<C>(1, 1, a);
+      Y[v] = cpack<C>(conflict ? 2 : 1, conflict ? 2 : 1, a);
     }
     const int b = bin_of(e - s, a.small_max, a.med_max);
     warp_push(conflict && b == 0, v, a.wl_t[0], &ctrl->cnt[0][0]);
@@ -316,7 +340,26 @@ __global__ void __launch_bounds__(256) k_first(RoundArgs<C> a, int sorted) {
 }
 
 // ---------------------------------------------------------------------------------------
-// Forbidden-table helpers (bytes in shared memory, one per color).
+// Forbidden-set helpers (shared memory; bits or bytes per color, see SGR_BITTBL).
+
+__device__ __forceinline__ void set_add(uint8_t* tbl, uint32_t c) {
+#if SGR_BITTBL
+  atomicOr(reinterpret_cast<uint32_t*>(tbl) + (c >> 5), 1u << (c & 31u));
+#else
+  tbl[c] = 1;
+#endif
+}
+
+// Zero `bytes` of a set, the `nl` lanes of a group sharing the work (lane index l < nl).
+__device__ __forceinline__ void set_clear(uint8_t* p, int bytes, int l, int nl) {
+  if ((bytes / 16) % nl == 0) {
+    uint4* t = reinterpret_cast<uint4*>(p);
+    for (int q = l; q < bytes / 16; q += nl) t[q] = make_uint4(0u, 0u, 0u, 0u);
+  } else {
+    uint32_t* t = reinterpret_cast<uint32_t*>(p);
+    for (int q = l; q < bytes / 4; q += nl) t[q] = 0u;
+  }
+}
 
 // First free color >= 1 of a warp-owned table of N bytes (N multiple of 128); -1 if full.
 template <int N>
@@ -337,9 +380,12 @@ __device__ __forceinline__ int32_t tbl_first_free_warp(const uint8_t* tbl, int l
   return -1;
 }
 
-// 32 bits = the bytes [32 * lane, 32 * lane + 32) of a 1024-byte table whose bytes are 0 or
-// 1: multiplying a word of four 0/1 bytes by 0x01020408 gathers the bytes into bits 24-27.
+// 32 bits = colors [32 * lane, 32 * lane + 32) of a 1024-color set. Byte sets: multiplying a
+// word of four 0/1 bytes by 0x01020408 gathers the bytes into bits 24-27.
 __device__ __forceinline__ uint32_t tbl_bits32(const uint8_t* tbl, int lane) {
+#if SGR_BITTBL
+  return reinterpret_cast<const uint32_t*>(tbl)[lane];
+#else
   const uint4* t = reinterpret_cast<const uint4*>(tbl) + lane * 2;
   const uint4 a = t[0], b = t[1];
   const uint32_t w[8] = {a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w};
@@ -347,6 +393,7 @@ __device__ __forceinline__ uint32_t tbl_bits32(const uint8_t* tbl, int lane) {
 #pragma unroll
   for (int q = 0; q < 8; ++q) bits |= ((w[q] * 0x01020408u) >> 24) << (4 * q);
   return bits;
+#endif
 }
 
 // First free color of a 1024-bit set spread over the warp (lane l holds colors
@@ -393,12 +440,6 @@ __device__ __noinline__ int32_t warp_first_fit_rescan(const int32_t* __restrict_
   }
 }
 
-__device__ __forceinline__ void clear_bytes(uint8_t* p, int bytes_per_lane, int lane) {
-  uint4* t = reinterpret_cast<uint4*>(p) + lane * (bytes_per_lane / 16);
-#pragma unroll
-  for (int q = 0; q < bytes_per_lane / 16; ++q) t[q] = make_uint4(0, 0, 0, 0);
-}
-
 // ---------------------------------------------------------------------------------------
 // Bin 2, plain 32-bit colors (no trimming): one warp processes one chunk [cs, ce) of the
 // full row [s, e), read as int4 from the 16-byte-aligned window; outside [cs, ce) masked.
@@ -414,9 +455,9 @@ __device__ __forceinline__ void process_chunk_plain(const RoundArgs<C>& a, int k
   const int64_t wbase = cs & ~(int64_t)3;  // 16-byte aligned window start
   const int32_t nch = num_chunks(e - s);
   const int4* col4 = reinterpret_cast<const int4*>(a.col_idx + wbase);
-  int32_t w[32];
+  int32_t w[kWin / 32];
 #pragma unroll
-  for (int q = 0; q < 8; ++q) {
+  for (int q = 0; q < kWin / 128; ++q) {
     const int64_t p0 = wbase + 4 * (lane + 32 * q);
     int4 t = make_int4(-1, -1, -1, -1);
     if (p0 + 3 >= cs && p0 < ce) {
@@ -436,13 +477,13 @@ __device__ __forceinline__ void process_chunk_plain(const RoundArgs<C>& a, int k
   const int32_t xv = ldc<Persist>(X + v);
   uint32_t lb = 0;  // lose(v, w) bits
 #pragma unroll
-  for (int u = 0; u < 32; ++u) lb |= (w[u] >= 0 && lose<TB>(v, w[u])) ? (1u << u) : 0u;
+  for (int u = 0; u < kWin / 32; ++u) lb |= (w[u] >= 0 && lose<TB>(v, w[u])) ? (1u << u) : 0u;
 #pragma unroll
-  for (int u = 0; u < 32; ++u) w[u] = (w[u] >= 0) ? ldc<Persist>(X + w[u]) : 0;  // now colors
+  for (int u = 0; u < kWin / 32; ++u) w[u] = (w[u] >= 0) ? ldc<Persist>(X + w[u]) : 0;  // now colors
   bool conf = false;
 #pragma unroll
-  for (int u = 0; u < 32; ++u) {
-    if ((uint32_t)w[u] < (uint32_t)kBigTbl) tbl[w[u]] = 1;
+  for (int u = 0; u < kWin / 32; ++u) {
+    if ((uint32_t)w[u] < (uint32_t)kBigTbl) set_add(tbl, (uint32_t)w[u]);
     conf |= (w[u] == xv) & ((lb >> u) & 1u);
   }
   if (lane == 0) {
@@ -454,11 +495,15 @@ __device__ __forceinline__ void process_chunk_plain(const RoundArgs<C>& a, int k
   if (nch == 1) {
     int32_t tent = 0;
     if (any) {
+#if SGR_BITTBL
+      tent = bits_first_free(tbl_bits32(tbl, lane) | (lane == 0 ? 1u : 0u));
+#else
       tent = tbl_first_free_warp<kBigTbl>(tbl, lane);
+#endif
       if (tent < 0) tent = warp_first_fit_rescan<Persist>(a.col_idx, X, s, e, kBigTbl, lane);
     }
     if (lane == 0) {
-      Y[v] = any ? cpack<C>(tent, k + 1, a.ctrl) : cpack<C>(xv, k, a.ctrl);
+      Y[v] = any ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a);
       if (any) {
         out[atomicAdd(out_cnt, 1)] = make_item(v, 0);
         atomicAdd(out_vcnt, 1);
@@ -490,7 +535,7 @@ __device__ __forceinline__ void process_chunk_plain(const RoundArgs<C>& a, int k
       }
       int32_t ob = 0;
       if (lane == 0) {
-        Y[v] = conf_all ? cpack<C>(tent, k + 1, a.ctrl) : cpack<C>(xv, k, a.ctrl);
+        Y[v] = conf_all ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a);
         if (conf_all) {
           ob = atomicAdd(out_cnt, nch);
           atomicAdd(out_vcnt, 1);
@@ -502,7 +547,7 @@ __device__ __forceinline__ void process_chunk_plain(const RoundArgs<C>& a, int k
       }
     }
   }
-  clear_bytes(tbl, kBigTbl / 32, lane);
+  set_clear(tbl, kBigTblB, lane, 32);
   __syncwarp();
 }
 
@@ -515,12 +560,12 @@ struct ChunkHdr {
 };
 
 template <int TB, bool Persist>
-__device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k, int p,
-                                             const uint32_t* X, uint32_t* Y, uint8_t* wsm,
+__device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, int p,
+                                             const Packed* X, Packed* Y, uint8_t* wsm,
                                              int gw, int NW, int lane,
                                              unsigned long long& edges,
                                              unsigned long long& entries, uint32_t& ph) {
-  using C = uint32_t;
+  using C = Packed;
   Ctrl* ctrl = a.ctrl;
   const int nC = ld_cg(&ctrl->cnt[p][2]);
   if (gw >= nC) return;
@@ -532,7 +577,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
   int32_t* len_nxt = sel(p ^ 1, a.len[0], a.len[1]);
   int32_t* bufs = reinterpret_cast<int32_t*>(wsm);
   uint8_t* tbl_all = wsm + WarpSmem<C>::kBuf;
-  uint8_t* tbl_drop = tbl_all + kBigTbl;
+  uint8_t* tbl_drop = tbl_all + kBigTblB;
   uint64_t* bars = reinterpret_cast<uint64_t*>(wsm + WarpSmem<C>::kBars);
   // Next-round items are buffered per warp and flushed with one atomicAdd per <= 32 items
   // (the bin's item and vertex counters are single hot addresses).
@@ -599,7 +644,10 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
     const int32_t nb = (nslots + 128 * kQB - 1) / (128 * kQB);  // batches of kQB int4 per lane
     const int32_t nch = num_chunks(cur.len);
     const int32_t xv = cval<C>(ldraw<Persist>(X + v));
-    const uint32_t klive = (uint32_t)k << 16;  // raw >= klive <=> neighbour still in W_k
+    // a neighbour still in W_k was written by pass k-1 with last = k; one that has left W
+    // has last < k and is recognised unless last = k mod 16, in which case it simply stays
+    // in the list one more round (never the reverse: live neighbours are never dropped)
+    const uint32_t klive = (uint32_t)k & 15u;
 #if SGR_NO_TMA
     {  // A/B: the warp stages its own window (16-byte loads + shared stores), no TMA
       const int4* g4 = reinterpret_cast<const int4*>(
@@ -645,11 +693,11 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
         if ((okm >> j) & 1u) {
           // colors >= 1023 are clamped onto byte 1023; a first fit of 1023 or more is
           // recomputed exactly from the full row (warp_first_fit_rescan)
-          const uint32_t ci = min(raw[j] & 0xffffu, (uint32_t)(kBigTbl - 1));
-          const bool live = raw[j] >= klive;
-          tbl_all[ci] = 1;
-          if (!live) tbl_drop[ci] = 1;
-          conf |= (int32_t)(raw[j] & 0xffffu) == xv && lose<TB>(v, id[j]);
+          const uint32_t ci = min(raw[j] & kColorMask, (uint32_t)(kBigTbl - 1));
+          const bool live = (raw[j] >> kRoundShift) == klive;
+          set_add(tbl_all, ci);
+          if (!live) set_add(tbl_drop, ci);
+          conf |= (int32_t)(raw[j] & kColorMask) == xv && lose<TB>(v, id[j]);
           lv |= live ? (1u << (kJB * bb + j)) : 0u;
         }
       }
@@ -717,7 +765,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
         if (live_total < (uint32_t)cnt) write_live(lst_same + cur.s);
         if (lane == 0) {
           len_nxt[v] = (int32_t)live_total;
-          Y[v] = cpack<C>(tent, k + 1, ctrl);
+          Y[v] = cpack<C>(tent, k + 1, a);
           // live <= kChunk: one chunk, the list stays in its buffer
           ibuf[ipend] = make_item(v, (int32_t)(cur.buf ? kBufBit : 0u));
         }
@@ -725,7 +773,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
         ++vpend;
         if (ipend == 32) iflush();
       } else if (lane == 0) {
-        Y[v] = cpack<C>(xv, k, ctrl);
+        Y[v] = cpack<C>(xv, k, a);
       }
     } else {
       // several chunks: publish this chunk's partial forbidden set, dropped colors and
@@ -745,7 +793,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
         if (cur.c == 0) a.fin[atomicAdd(&ctrl->fin_cnt, 1)] = (int32_t)((uint32_t)v | (cur.buf ? kBufBit : 0u));
       }
     }
-    clear_bytes(tbl_all, kTblBytes / 32, lane);  // both tables
+    set_clear(tbl_all, kTblBytes, lane, 32);  // both sets
     __syncwarp();
 #if !SGR_NO_TMA
     tq = clock64();
@@ -773,8 +821,8 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<uint32_t>& a, int k
 // fit the lowest free color (l.8). Writes Y[v], pushes the vertex's next-round chunk items
 // (its compacted list now lives in the other buffer), and resets the accumulators.
 template <int TB, bool Persist>
-__device__ __forceinline__ void finalize_body(const RoundArgs<uint32_t>& a, int k) {
-  using C = uint32_t;
+__device__ __forceinline__ void finalize_body(const RoundArgs<Packed>& a, int k) {
+  using C = Packed;
   Ctrl* ctrl = a.ctrl;
   const int p = k & 1;
   const int lane = threadIdx.x & 31;
@@ -806,7 +854,7 @@ __device__ __forceinline__ void finalize_body(const RoundArgs<uint32_t>& a, int 
     if (lane == 0) {
       a.acc_cnt[slot] = 0ull;
       len_cur[v] = 0;  // consumed; the pass after next accumulates into it
-      Y[v] = conf ? cpack<C>(tent, k + 1, ctrl) : cpack<C>(cval<C>(ldraw<Persist>(X + v)), k, ctrl);
+      Y[v] = conf ? cpack<C>(tent, k + 1, a) : cpack<C>(cval<C>(ldraw<Persist>(X + v)), k, a);
       if (conf) {
         nch2 = num_chunks(ld_cg(len_nxt + v));
         ob = atomicAdd(&ctrl->cnt[p ^ 1][2], nch2);
@@ -851,7 +899,7 @@ __device__ __forceinline__ void process_group(const RoundArgs<C>& a, int k, int3
     for (int u = 0; u < 8; ++u) {
       if (w[u] >= 0) {
         // deg <= 256 => first fit <= 257: colors >= 511 are clamped onto an unused byte
-        gtbl[min(w[u], kMedTbl - 1)] = 1;
+        set_add(gtbl, (uint32_t)min(w[u], kMedTbl - 1));
         conf |= w[u] == xv && ((lb >> u) & 1u);
       }
     }
@@ -862,6 +910,16 @@ __device__ __forceinline__ void process_group(const RoundArgs<C>& a, int k, int3
   int32_t tent = 0;
   if (v >= 0 && any) {  // the group scans its table 32 bytes (8 words) per step
     const uint32_t* t32 = reinterpret_cast<const uint32_t*>(gtbl);
+#if SGR_BITTBL
+    {  // 512 bits = 16 words, two per lane of the group
+      uint32_t w0 = t32[2 * gl], w1 = t32[2 * gl + 1];
+      if (gl == 0) w0 |= 1u;  // color 0
+      const int f = (~w0) ? (__ffs(~w0) - 1) : ((~w1) ? 32 + __ffs(~w1) - 1 : 64);
+      const unsigned b = __ballot_sync(gmask, f < 64) & gmask;
+      const int fl = __ffs(b) - 1;  // the group's lane 0 always has a free color (deg <= 256)
+      tent = (fl & 7) * 64 + __shfl_sync(gmask, f, fl);
+    }
+#else
     for (int it = 0; it < kMedTbl / 32; ++it) {
       uint32_t word = t32[it * 8 + gl];
       if (it == 0 && gl == 0) word |= 0xffu;
@@ -874,10 +932,11 @@ __device__ __forceinline__ void process_group(const RoundArgs<C>& a, int k, int3
         break;
       }
     }
+#endif
   }
-  clear_bytes(gtbl, kMedTbl / kGroup, gl);
+  set_clear(gtbl, kMedTblB, gl, kGroup);
   __syncwarp();
-  if (v >= 0 && gl == 0) Y[v] = any ? cpack<C>(tent, k + 1, a.ctrl) : cpack<C>(xv, k, a.ctrl);
+  if (v >= 0 && gl == 0) Y[v] = any ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a);
   push = (v >= 0) && any && gl == 0;
 }
 
@@ -962,7 +1021,7 @@ __device__ __forceinline__ void bin0(const RoundArgs<C>& a, int k, const int32_t
     const bool any = (__ballot_sync(0xffffffffu, conf) & gmask) != 0u;
     if (v >= 0 && gl == 0) {
       const int32_t tent = ~mask ? __ffs(~mask) : 33;
-      Y[v] = any ? cpack<C>(tent, k + 1, a.ctrl) : cpack<C>(xv, k, a.ctrl);
+      Y[v] = any ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a);
       edges += (unsigned long long)(e - s);
       entries += (unsigned long long)(e - s);
     }
@@ -991,7 +1050,7 @@ __device__ __forceinline__ void bin1(const RoundArgs<C>& a, int k, const int32_t
                                       unsigned long long& edges, unsigned long long& entries) {
   const int g = lane >> 3, gl = lane & 7;
   const unsigned gmask = 0xffu << (g * 8);
-  uint8_t* gtbl = wsm + WarpSmem<C>::kBuf + g * kMedTbl;
+  uint8_t* gtbl = wsm + WarpSmem<C>::kBuf + g * kMedTblB;
   int32_t* pbuf = reinterpret_cast<int32_t*>(wsm + WarpSmem<C>::kPush);
   int pending = 0;
   const int step = NW * 4;
@@ -1121,7 +1180,7 @@ __device__ __forceinline__ void advance_body(Ctrl* ctrl, bool first, bool force 
     for (int q = 0; q < kBins; ++q) tot += c->cnt[0][q];
     c->pushes_total[kBins] = (unsigned long long)(c->cnt[0][0] + c->cnt[0][1] + c->vcnt2[0]);
     c->k = 2;
-    c->active = tot > 0;
+    c->active = tot > 0 && !c->overflow;
     if (c->active && c->max_rounds < 2) {
       c->status = 1;
       c->active = 0;
@@ -1160,7 +1219,8 @@ __device__ __forceinline__ void advance_body(Ctrl* ctrl, bool first, bool force 
   }
   c->k = k + 1;
   const int items_out = c->cnt[p ^ 1][0] + c->cnt[p ^ 1][1] + c->cnt[p ^ 1][2];
-  c->active = items_out > 0;
+  // a packed color overflowed: stop here, the host reruns with 32-bit colors
+  c->active = items_out > 0 && !c->overflow;
   if (c->active && k + 1 > c->max_rounds) {  // W_{k+1} non-empty beyond the cap
     c->status = 1;
     c->active = 0;
@@ -1188,6 +1248,7 @@ __global__ void k_pack(RoundArgs<C> a, uint2* send, int32_t cap) {
   const int32_t* lm = sel(p, (const int32_t*)a.wl_m[0], (const int32_t*)a.wl_m[1]);
   const int64_t* lc = sel(p, (const int64_t*)a.wl_c[0], (const int64_t*)a.wl_c[1]);
   int32_t* count = reinterpret_cast<int32_t*>(&send[0].x);
+  if (blockIdx.x == 0 && threadIdx.x == 0) send[0].y = (uint32_t)ctrl->overflow;
   const int64_t total = (int64_t)nT + nM + nC;
   for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < total;
        base += (int64_t)gridDim.x * blockDim.x) {
@@ -1233,7 +1294,7 @@ __global__ void k_apply(RoundArgs<C> a, const uint2* recv, int32_t parts, int32_
 // Initialise both color buffers of a replica to C_1 (every vertex colored 1 in round 1).
 template <class C>
 __global__ void k_fill_c1(RoundArgs<C> a) {
-  const C one = packed<C>() ? (C)((1u << 16) | 1u) : (C)1;
+  const C one = packed<C>() ? (C)((1u << kRoundShift) | 1u) : (C)1;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < a.n;
        i += (int64_t)gridDim.x * blockDim.x) {
     a.col[0][i] = one;
@@ -1246,7 +1307,7 @@ template <class C>
 __device__ __forceinline__ uint8_t* warp_smem_init(uint8_t* smem) {
   const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
   uint8_t* wsm = smem + wid * WarpSmem<C>::kBytes;
-  clear_bytes(wsm + WarpSmem<C>::kBuf, kTblBytes / 32, lane);
+  set_clear(wsm + WarpSmem<C>::kBuf, kTblBytes, lane, 32);
   if constexpr (packed<C>()) {
     if (lane == 0) {
       uint64_t* bars = reinterpret_cast<uint64_t*>(wsm + WarpSmem<C>::kBars);
@@ -1332,10 +1393,10 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks<C>) k_persistent(RoundArgs<
 }
 
 // Final colors (packed words) into the caller's int32 output.
-static __global__ void k_unpack(const uint32_t* __restrict__ src, int32_t* __restrict__ dst, int64_t n) {
+static __global__ void k_unpack(const Packed* __restrict__ src, int32_t* __restrict__ dst, int64_t n) {
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
        i += (int64_t)gridDim.x * blockDim.x)
-    dst[i] = (int32_t)(src[i] & 0xffffu);
+    dst[i] = (int32_t)(src[i] & kColorMask);
 }
 
 }  // namespace sgr

@@ -84,7 +84,8 @@ def degree_boundary_graph():
     (first fits above 64 and 256; K_300 rows straddle 1024-aligned chunk boundaries)."""
     edges = []
     n = 0
-    for d in [0, 1, 2, 31, 32, 33, 61, 62, 63, 64, 65, 255, 256, 257, 1019, 1020, 1021, 2040,
+    for d in [0, 1, 2, 31, 32, 33, 61, 62, 63, 64, 65, 255, 256, 257, 507, 508, 509, 1015, 1016,
+              1017, 1019, 1020, 1021, 2040,
               2041, 2047, 2048, 2049, 4095, 4096, 4097, 9000]:
         c = n
         edges += [(c, c + 1 + i) for i in range(d)]
@@ -105,6 +106,16 @@ def degree_boundary_graph():
 def test_degree_bins_and_windows(tb, bins, mode, bits):
     check_full(degree_boundary_graph(), tb, bin_small_max=bins[0], bin_med_max=bins[1],
                loop_mode=mode, color_bits=bits)
+
+
+@pytest.mark.parametrize("cap,bits", [(40, 32), (299, 32), (300, 16), (0, 16)])
+def test_color_overflow_rerun(cap, bits):
+    """A first fit above the 16-bit word's color range (lowered by the color_cap test hook)
+    discards the packed run and redoes the coloring with plain int32 words: same result."""
+    g = degree_boundary_graph()  # contains K_300: colors up to 300
+    for tb in (LOW, PAP):
+        res, _ = check_full(g, tb, color_cap=cap)
+        assert res.stats["color_bits"] == bits, (cap, res.stats["color_bits"])
 
 
 @pytest.mark.parametrize("k", [64, 257, 520, 1100])
@@ -284,6 +295,20 @@ def test_partitioned_equals_single_gpu(P, tb):
         assert res.stats["rounds"] == ref.rounds
         assert res.stats["vertices_processed"] == ref.vertices_processed
         assert res.stats["num_colors"] == ref.num_colors
+
+
+@pytest.mark.parametrize("P", [1, 3])
+def test_partitioned_color_overflow_rerun(P):
+    """Partitions see a packed overflow in the same exchange and all redo the coloring
+    with int32 words (color_cap lowered below K_300's colors by the test hook)."""
+    g = degree_boundary_graph()
+    rp, ci = dev(g)
+    for tb in (LOW, PAP):
+        ref = oracle.jacobi(g, tb)
+        res = sgr.color_partitioned(rp, ci, P, tiebreak=RULE[tb], color_cap=40)
+        assert np.array_equal(res.colors.cpu().numpy(), ref.colors), (P, tb)
+        assert res.stats["color_bits"] == 32
+        assert res.stats["rounds"] == ref.rounds
 
 
 @pytest.mark.parametrize("bits", [16, 32])
