@@ -235,6 +235,7 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
   int32_t launches = 0;
   const bool persistent = r.loop_mode == SGR_LOOP_PERSISTENT;
   const int grid = round_grid<TB, C>(persistent);
+  const int grid_flat = persistent ? round_grid<TB, C, false>(true) : grid;
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
   sgr_status status = SGR_OK;
   do {
@@ -276,12 +277,16 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
     }
 
     if (persistent) {
+      // both builds are enqueued; the one that does not match F_1's bins returns at once
       prof.timed(SGR_K_ROUND, s, [&] {
         void* args[] = {(void*)&a};
-        le = cudaLaunchCooperativeKernel((const void*)k_persistent<TB, C>, grid, kBlock, args,
-                                         round_smem<C>(), s);
+        le = cudaLaunchCooperativeKernel((const void*)k_persistent<TB, C, true>, grid, kBlock,
+                                         args, round_smem<C, true>(), s);
+        if (le == cudaSuccess)
+          le = cudaLaunchCooperativeKernel((const void*)k_persistent<TB, C, false>, grid_flat,
+                                           kBlock, args, round_smem<C, false>(), s);
       });
-      launches += 1;
+      launches += 2;
       if (le != cudaSuccess) {
         status = cuda_fail(le, "cooperative launch of k_persistent", __LINE__);
         break;
@@ -352,7 +357,7 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
       fill_stats(fin, n, nnz, stats);
       cudaEventElapsedTime(&stats->elapsed_ms, ev0, ev1);
       stats->launches = launches;
-      stats->grid_blocks = grid;
+      stats->grid_blocks = fin.big_count ? grid : grid_flat;
       stats->color_bits = packed<C>() ? 16 : 32;
       int32_t ri = 0;
       for (auto& m : prof.marks) {

@@ -117,24 +117,24 @@ inline int first_grid(int64_t n) {
   return (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, (int64_t)num_sms() * 8));
 }
 
-template <class C>
-constexpr size_t round_smem() { return (size_t)kWarps * WarpSmem<C>::kBytes; }
+template <class C, bool Hub = true>
+constexpr size_t round_smem() { return (size_t)kWarps * WarpSmem<C, Hub>::kBytes; }
 
 // Blocks of the round kernels: as many as are co-resident (persistent: required).
-template <int TB, class C>
+template <int TB, class C, bool Hub = true>
 inline int round_grid(bool persistent) {
   static bool attr_set = false;
   if (!attr_set) {  // opt in to > 48 KB of dynamic shared memory
-    cudaFuncSetAttribute(k_persistent<TB, C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)round_smem<C>());
+    cudaFuncSetAttribute(k_persistent<TB, C, Hub>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)round_smem<C, Hub>());
     cudaFuncSetAttribute(k_round<TB, C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)round_smem<C>());
     attr_set = true;
   }
   int per_sm = 0;
   cudaError_t e = persistent
-      ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_persistent<TB, C>, kBlock,
-                                                      round_smem<C>())
+      ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_persistent<TB, C, Hub>, kBlock,
+                                                      round_smem<C, Hub>())
       : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_round<TB, C>, kBlock,
                                                       round_smem<C>());
   if (e != cudaSuccess || per_sm <= 0) per_sm = 1;

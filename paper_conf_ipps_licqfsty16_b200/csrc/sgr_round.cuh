@@ -91,21 +91,30 @@ constexpr int kRoundShift = 12;
 template <class C>
 __host__ __device__ constexpr bool packed() { return sizeof(C) == 2; }
 
-// dynamic shared memory per warp: [2 TMA stages (packed only)] [tables] [2 mbarriers]
+// Two builds of the round kernels: Hub (bins 0-2) and flat (bins 0-1 only), chosen per
+// coloring by whether F_1 put any vertex into bin 2 (bins are static, so then bin 2 stays
+// empty). The flat build needs no TMA stages, so it leaves most of the SM's unified
+// L1/shared storage to the L1 cache that serves the color gathers, and runs 3 blocks/SM.
+//
+// dynamic shared memory per warp: [2 TMA stages (Hub, packed)] [tables] [push buffer]
+// [bin-2 item buffer, 2 mbarriers (Hub)]
 constexpr int kStage = kWin * 4;        // bytes per TMA stage: one bin-2 window
-// blocks per SM the round kernels are compiled for: packed mode is shared-memory bound to 2
-// (82 KB per block), plain mode can afford 3 (<= 85 registers)
+// blocks per SM the round kernels are compiled for: the packed Hub build is shared-memory
+// bound to 2 (86 KB per block); the others can afford 3 (<= 85 registers)
 #ifndef SGR_MINB
 #define SGR_MINB 2
 #endif
-template <class C>
-constexpr int kMinBlocks = packed<C>() ? SGR_MINB : 3;
-template <class C> struct WarpSmem {
-  static constexpr int kBuf = packed<C>() ? 2 * kStage : 0;
+#ifndef SGR_FLATB
+#define SGR_FLATB 3
+#endif
+template <class C, bool Hub = true>
+constexpr int kMinBlocks = (packed<C>() && Hub) ? SGR_MINB : (Hub ? 3 : SGR_FLATB);
+template <class C, bool Hub = true> struct WarpSmem {
+  static constexpr int kBuf = (packed<C>() && Hub) ? 2 * kStage : 0;
   static constexpr int kPush = kBuf + kTblBytes;         // push buffer (kPushBuf int32)
   static constexpr int kItems = kPush + kPushBuf * 4;    // bin-2 item buffer (32 int64)
-  static constexpr int kBars = kItems + 32 * 8;          // 2 mbarriers
-  static constexpr int kBytes = kBars + 16;
+  static constexpr int kBars = kItems + (Hub ? 32 * 8 : 0);  // 2 mbarriers
+  static constexpr int kBytes = kBars + (Hub ? 16 : 0);
 };
 
 // Device-resident loop state (in the workspace).
@@ -973,7 +982,7 @@ __device__ __forceinline__ void push_flush(int32_t* pbuf, int& pending, int32_t*
 // Bin 0 driver: 4-lane groups, 8 vertices per warp per step; list entries and row offsets
 // prefetched two steps ahead, the row entries one step ahead (so they are in flight while
 // the current vertices' color gathers are), pushes buffered per warp.
-template <int TB, bool Persist, class C>
+template <int TB, bool Persist, class C, bool Hub>
 __device__ __forceinline__ void bin0(const RoundArgs<C>& a, int k, const int32_t* list, int nX,
                                      int32_t* out, int32_t* out_cnt, const C* X, C* Y,
                                      uint8_t* wsm, int gw, int NW, int lane,
@@ -982,7 +991,7 @@ __device__ __forceinline__ void bin0(const RoundArgs<C>& a, int k, const int32_t
   if (gw * VPW >= nX) return;
   const int g = lane / G, gl = lane % G;
   const unsigned gmask = ((1u << G) - 1u) << (g * G);
-  int32_t* pbuf = reinterpret_cast<int32_t*>(wsm + WarpSmem<C>::kPush);
+  int32_t* pbuf = reinterpret_cast<int32_t*>(wsm + WarpSmem<C, Hub>::kPush);
   int pending = 0;
   const int step = NW * VPW;
   auto load_row = [&](int32_t vv, int64_t ss, int64_t ee, int32_t (&w)[kK0]) {
@@ -1043,15 +1052,15 @@ __device__ __forceinline__ void bin0(const RoundArgs<C>& a, int k, const int32_t
 
 // Bins 0/1 driver: warp w takes list positions 4w + g, 4(w + NW) + g, ... (g = group); the
 // next position's list entry and row offsets are prefetched, its row warmed into L2.
-template <int TB, bool Persist, class C>
+template <int TB, bool Persist, class C, bool Hub>
 __device__ __forceinline__ void bin1(const RoundArgs<C>& a, int k, const int32_t* list, int nX,
                                       int32_t* out, int32_t* out_cnt, const C* X, C* Y,
                                       uint8_t* wsm, int gw, int NW, int lane,
                                       unsigned long long& edges, unsigned long long& entries) {
   const int g = lane >> 3, gl = lane & 7;
   const unsigned gmask = 0xffu << (g * 8);
-  uint8_t* gtbl = wsm + WarpSmem<C>::kBuf + g * kMedTblB;
-  int32_t* pbuf = reinterpret_cast<int32_t*>(wsm + WarpSmem<C>::kPush);
+  uint8_t* gtbl = wsm + WarpSmem<C, Hub>::kBuf + g * kMedTblB;
+  int32_t* pbuf = reinterpret_cast<int32_t*>(wsm + WarpSmem<C, Hub>::kPush);
   int pending = 0;
   const int step = NW * 4;
   int i = gw * 4 + g;
@@ -1078,7 +1087,7 @@ __device__ __forceinline__ void bin1(const RoundArgs<C>& a, int k, const int32_t
 // One fused pass F_k over all three bins; every warp of the grid calls it. Static
 // round-robin assignment (warp w takes items w, w + NW, ...), with the next item's list
 // entry and row offsets prefetched while the current one is processed.
-template <int TB, bool Persist, class C>
+template <int TB, bool Persist, class C, bool Hub>
 __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, uint8_t* wsm,
                                            unsigned long long (&edges)[kBins],
                                            unsigned long long (&entries)[kBins],
@@ -1090,11 +1099,12 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, uint8_t
   const int NW = (int)((gridDim.x * blockDim.x) >> 5);
   const C* X = sel((k - 1) & 1, (const C*)a.col[0], (const C*)a.col[1]);
   C* Y = sel(k & 1, a.col[0], a.col[1]);
-  uint8_t* wtbl = wsm + WarpSmem<C>::kBuf;
+  uint8_t* wtbl = wsm + WarpSmem<C, Hub>::kBuf;
   (void)wtbl;
   long long t0 = clock64();
-  // ---- bin 2
-  if constexpr (packed<C>()) {
+  // ---- bin 2 (Hub build only; the flat build runs when bin 2 is empty)
+  if constexpr (!Hub) {
+  } else if constexpr (packed<C>()) {
     bin2_trimmed<TB, Persist>(a, k, p, X, Y, wsm, gw, NW, lane, edges[2], entries[2], ph);
   } else {
     const int nC = ld_cg(&ctrl->cnt[p][2]);
@@ -1128,14 +1138,14 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, uint8_t
   long long t1 = clock64();
   cyc[2] += (unsigned long long)(t1 - t0);
   // ---- bin 1: four vertices per warp (one per 8-lane group), 512-byte tables
-  bin1<TB, Persist, C>(
+  bin1<TB, Persist, C, Hub>(
       a, k, sel(p, (const int32_t*)a.wl_m[0], (const int32_t*)a.wl_m[1]),
       ld_cg(&ctrl->cnt[p][1]), sel(p ^ 1, a.wl_m[0], a.wl_m[1]), &ctrl->cnt[p ^ 1][1], X, Y,
       wsm, gw, NW, lane, edges[1], entries[1]);
   long long t2 = clock64();
   cyc[1] += (unsigned long long)(t2 - t1);
   // ---- bin 0: eight vertices per warp, register masks
-  bin0<TB, Persist, C>(
+  bin0<TB, Persist, C, Hub>(
       a, k, sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]),
       ld_cg(&ctrl->cnt[p][0]), sel(p ^ 1, a.wl_t[0], a.wl_t[1]), &ctrl->cnt[p ^ 1][0], X, Y,
       wsm, gw, NW, lane, edges[0], entries[0]);
@@ -1303,14 +1313,14 @@ __global__ void k_fill_c1(RoundArgs<C> a) {
 }
 
 // Kernel prologue: zero the warp tables, initialise the warp's two TMA mbarriers.
-template <class C>
+template <class C, bool Hub = true>
 __device__ __forceinline__ uint8_t* warp_smem_init(uint8_t* smem) {
   const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  uint8_t* wsm = smem + wid * WarpSmem<C>::kBytes;
-  set_clear(wsm + WarpSmem<C>::kBuf, kTblBytes, lane, 32);
-  if constexpr (packed<C>()) {
+  uint8_t* wsm = smem + wid * WarpSmem<C, Hub>::kBytes;
+  set_clear(wsm + WarpSmem<C, Hub>::kBuf, kTblBytes, lane, 32);
+  if constexpr (packed<C>() && Hub) {
     if (lane == 0) {
-      uint64_t* bars = reinterpret_cast<uint64_t*>(wsm + WarpSmem<C>::kBars);
+      uint64_t* bars = reinterpret_cast<uint64_t*>(wsm + WarpSmem<C, Hub>::kBars);
       mbar_init(bars + 0, 1);  // bin-2 stages: one elected arrival per phase
       mbar_init(bars + 1, 1);
       mbar_init_fence();
@@ -1330,7 +1340,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks<C>) k_round(RoundArgs<C> a)
   unsigned long long edges[kBins] = {0, 0, 0}, entries[kBins] = {0, 0, 0};
   unsigned long long cyc[kBins] = {0, 0, 0};
   uint32_t ph = 0;
-  round_body<TB, false, C>(a, ctrl->k, wsm, edges, entries, ph, cyc);
+  round_body<TB, false, C, true>(a, ctrl->k, wsm, edges, entries, ph, cyc);
   block_add6(edges, entries, ctrl);
   if ((threadIdx.x & 31) == 0)
     for (int q = 0; q < kBins; ++q) atomicAdd(&ctrl->bin_cycles[q], cyc[q]);
@@ -1368,11 +1378,14 @@ __device__ __forceinline__ void grid_sync_advance(Ctrl* ctrl, bool advance = tru
 }
 
 // All rounds in one cooperative launch (every block resident): pass, barrier+advance, ...
-template <int TB, class C>
-__global__ void __launch_bounds__(kBlock, kMinBlocks<C>) k_persistent(RoundArgs<C> a) {
+// The host enqueues both builds; each returns at once unless it is the right one for this
+// coloring (Hub iff F_1 put a vertex into bin 2), so the choice needs no host round trip.
+template <int TB, class C, bool Hub>
+__global__ void __launch_bounds__(kBlock, kMinBlocks<C, Hub>) k_persistent(RoundArgs<C> a) {
   extern __shared__ __align__(16) uint8_t dsmem[];
   Ctrl* ctrl = a.ctrl;
-  uint8_t* wsm = warp_smem_init<C>(dsmem);
+  if ((ld_cg(&ctrl->big_count) != 0) != Hub) return;  // uniform across the grid
+  uint8_t* wsm = warp_smem_init<C, Hub>(dsmem);
   uint32_t ph = 0;  // mbarrier phase bits of the warp's two TMA stages
   unsigned long long cyc[kBins] = {0, 0, 0};
   for (;;) {
@@ -1380,9 +1393,9 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks<C>) k_persistent(RoundArgs<
     const int k = ld_cg(&ctrl->k);
     if (!active) break;  // uniform: read after the barrier by every thread
     unsigned long long edges[kBins] = {0, 0, 0}, entries[kBins] = {0, 0, 0};
-    round_body<TB, true, C>(a, k, wsm, edges, entries, ph, cyc);
+    round_body<TB, true, C, Hub>(a, k, wsm, edges, entries, ph, cyc);
     block_add6(edges, entries, ctrl);
-    if constexpr (packed<C>()) {  // multi-chunk vertices are decided once all chunks are in
+    if constexpr (packed<C>() && Hub) {  // multi-chunk vertices: decided once all chunks are in
       grid_sync_advance(ctrl, false);
       finalize_body<TB, true>(a, k);
     }
