@@ -99,6 +99,8 @@ typedef struct {
   int32_t profile;       /* != 0: time every kernel launch with CUDA events */
   float* round_ms;       /* optional HOST buffer (round_cap): with profile != 0 and the host
                             loop, device time of each round pass k = 2, 3, ... */
+  int64_t* round_ns;     /* optional DEVICE buffer (round_cap): %globaltimer (ns) when pass
+                            k = 2, 3, ... ended, written by the loop control (profiling) */
   int32_t color_cap;     /* test hook: 0 = 4095, the largest color a 16-bit word holds; a
                             smaller cap sends colorings whose colors exceed it down the
                             automatic 32-bit rerun path (results are unchanged) */

@@ -68,7 +68,7 @@ def _check_csr(row_ptr, col_idx):
 def make_opts(tiebreak="lowid", stream=None, max_rounds=0, loop_mode="auto", color_bits=0,
               bin_small_max=0, bin_med_max=0, validate=False, rounds_per_batch=0,
               profile=False, round_sizes=None, round_edges=None, round_cap=0,
-              round_ms=None, color_cap=0) -> Opts:
+              round_ms=None, color_cap=0, round_ns=None) -> Opts:
     o = Opts()
     load().sgr_opts_default(ctypes.byref(o))
     o.tiebreak = _tb(tiebreak)
@@ -86,6 +86,7 @@ def make_opts(tiebreak="lowid", stream=None, max_rounds=0, loop_mode="auto", col
     o.round_cap = int(round_cap)
     o.round_ms = round_ms.ctypes.data if round_ms is not None else None
     o.color_cap = int(color_cap)
+    o.round_ns = round_ns.data_ptr() if round_ns is not None else None
     return o
 
 

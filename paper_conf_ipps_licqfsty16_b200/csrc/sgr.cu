@@ -75,7 +75,8 @@ Resolved resolve_opts(const sgr_opts* o, int64_t n) {
   r.stream = (cudaStream_t)o->stream;
   r.round_sizes = o->round_sizes;
   r.round_edges = o->round_edges;
-  r.round_cap = (o->round_sizes || o->round_edges) ? o->round_cap : 0;
+  r.round_ns = o->round_ns;
+  r.round_cap = (o->round_sizes || o->round_edges || o->round_ns) ? o->round_cap : 0;
   r.validate = o->validate;
   r.batch = o->rounds_per_batch > 0 ? o->rounds_per_batch : 8;
   r.profile = o->profile;
@@ -246,6 +247,7 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
     hc.round_cap = r.round_cap;
     hc.round_sizes = r.round_sizes;
     hc.round_edges = r.round_edges;
+    hc.round_ns = r.round_ns;
     cudaError_t le = cudaMemcpyAsync(a.ctrl, &hc, sizeof(Ctrl), cudaMemcpyHostToDevice, s);
     if (le == cudaSuccess)
       le = cudaMemsetAsync((char*)ws + L.zero_begin, 0, L.zero_end - L.zero_begin, s);

@@ -27,6 +27,7 @@ struct Resolved {
   int profile;
   float* round_ms;
   int32_t color_cap;
+  int64_t* round_ns;
 };
 
 void set_error(const char* fmt, ...);

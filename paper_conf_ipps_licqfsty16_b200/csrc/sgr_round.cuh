@@ -117,14 +117,27 @@ template <class C, bool Hub = true> struct WarpSmem {
   static constexpr int kBytes = kBars + (Hub ? 16 : 0);
 };
 
+// Work counts of one worklist W_k (32 bytes: one pair of vector loads).
+struct alignas(32) Counts {
+  int32_t t;                 // bin 0 vertices
+  int32_t m;                 // bin 1 vertices
+  int32_t c;                 // bin 2 chunk items
+  int32_t cv;                // bin 2 vertices
+  int32_t fin;               // pass k: multi-chunk bin-2 vertices awaiting the finalize phase
+  int32_t pad[3];
+};
+// W_k's counts live in ring slot k % 3: pass k reads slot k % 3 and pushes W_{k+1} into
+// slot (k+1) % 3, while slot (k+2) % 3 (W_{k-1}, read by the finished pass k-1) is folded
+// into the totals and zeroed. So no single thread has to advance anything between passes:
+// after the barrier every block reads the next counts itself.
+__host__ __device__ __forceinline__ int rs(int k) { return k % 3; }
+
 // Device-resident loop state (in the workspace).
 struct Ctrl {
   int32_t k;                 // index of the next fused pass F_k (k = 2 after F_1)
-  int32_t active;            // 1 while W_k is non-empty
+  int32_t active;            // 1 while W_k is non-empty (host / graph loop modes)
   int32_t status;            // 0 ok, 1 = max_rounds reached with W non-empty
   int32_t max_rounds;
-  int32_t cnt[2][kBins];     // work items per parity (k & 1) and bin
-  int32_t vcnt2[2];          // bin-2 worklist VERTICES per parity (items are chunks)
   int32_t overflow;          // a packed color exceeded 12 bits (4095)
   int32_t round_cap;
   uint32_t bar_count;        // grid barrier (persistent kernel)
@@ -132,10 +145,10 @@ struct Ctrl {
   int32_t big_count;         // slots handed to bin-2 vertices by F_1
   int32_t max_color;
   int32_t violations;
-  int32_t fin_cnt;           // multi-chunk bin-2 vertices awaiting the finalize phase
-  int32_t pad[2];
-  unsigned long long edges_acc[kBins];    // sum of deg(v) over the pass's vertices (algorithmic)
-  unsigned long long entries_acc[kBins];  // CSR / list entries actually read by the pass
+  int32_t pad[5];
+  Counts ring[3];
+  unsigned long long edges_acc[3][kBins];    // per ring slot: sum of deg(v) over the pass's
+  unsigned long long entries_acc[3][kBins];  // vertices / list entries actually read
   unsigned long long verts_total[kBins + 1];   // [kBins] = F_1
   unsigned long long edges_total[kBins + 1];
   unsigned long long entries_total[kBins + 1];
@@ -145,6 +158,7 @@ struct Ctrl {
   unsigned long long phase_cycles[4];     // bin 2 (trimmed) phases: issue, wait, gather, post
   int32_t* round_sizes;
   int64_t* round_edges;
+  int64_t* round_ns;          // %globaltimer at the end of each pass (profiling)
 };
 
 template <class C>
@@ -316,8 +330,9 @@ __global__ void __launch_bounds__(256) k_first(RoundArgs<C> a, int sorted) {
       Y[v] = cpack<C>(conflict ? 2 : 1, conflict ? 2 : 1, a);
     }
     const int b = bin_of(e - s, a.small_max, a.med_max);
-    warp_push(conflict && b == 0, v, a.wl_t[0], &ctrl->cnt[0][0]);
-    warp_push(conflict && b == 1, v, a.wl_m[0], &ctrl->cnt[0][1]);
+    Counts* w2 = &ctrl->ring[rs(2)];
+    warp_push(conflict && b == 0, v, a.wl_t[0], &w2->t);
+    warp_push(conflict && b == 1, v, a.wl_m[0], &w2->m);
     // bin 2: ceil(deg / kChunk) items per vertex and an accumulator slot
     const bool big = conflict && b == 2;
     const int32_t nch = big ? num_chunks(e - s) : 0;
@@ -339,8 +354,8 @@ __global__ void __launch_bounds__(256) k_first(RoundArgs<C> a, int sorted) {
       const int total = __shfl_sync(0xffffffffu, incl, 31);
       int ib = 0;
       if (lane == 0) {
-        ib = atomicAdd(&ctrl->cnt[0][2], total);
-        atomicAdd(&ctrl->vcnt2[0], __popc(mb));
+        ib = atomicAdd(&w2->c, total);
+        atomicAdd(&w2->cv, __popc(mb));
       }
       ib = __shfl_sync(0xffffffffu, ib, 0) + incl - nch;
       for (int32_t t = 0; t < nch; ++t) a.wl_c[0][ib + t] = make_item(v, t);
@@ -571,17 +586,16 @@ struct ChunkHdr {
 template <int TB, bool Persist>
 __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, int p,
                                              const Packed* X, Packed* Y, uint8_t* wsm,
-                                             int gw, int NW, int lane,
+                                             int gw, int NW, int lane, int nC,
                                              unsigned long long& edges,
                                              unsigned long long& entries, uint32_t& ph) {
   using C = Packed;
   Ctrl* ctrl = a.ctrl;
-  const int nC = ld_cg(&ctrl->cnt[p][2]);
   if (gw >= nC) return;
   const int64_t* items = sel(p, (const int64_t*)a.wl_c[0], (const int64_t*)a.wl_c[1]);
   int64_t* out = sel(p ^ 1, a.wl_c[0], a.wl_c[1]);
-  int32_t* out_cnt = &ctrl->cnt[p ^ 1][2];
-  int32_t* out_vcnt = &ctrl->vcnt2[p ^ 1];
+  int32_t* out_cnt = &ctrl->ring[rs(k + 1)].c;
+  int32_t* out_vcnt = &ctrl->ring[rs(k + 1)].cv;
   int32_t* len_cur = sel(p, a.len[0], a.len[1]);
   int32_t* len_nxt = sel(p ^ 1, a.len[0], a.len[1]);
   int32_t* bufs = reinterpret_cast<int32_t*>(wsm);
@@ -799,7 +813,8 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
       write_live(lst_other + cur.s + lbase);
       if (lane == 0) {
         if (any) atomicOr(a.acc_cnt + slot, 1ull);  // conflict flag
-        if (cur.c == 0) a.fin[atomicAdd(&ctrl->fin_cnt, 1)] = (int32_t)((uint32_t)v | (cur.buf ? kBufBit : 0u));
+        if (cur.c == 0)
+          a.fin[atomicAdd(&ctrl->ring[rs(k)].fin, 1)] = (int32_t)((uint32_t)v | (cur.buf ? kBufBit : 0u));
       }
     }
     set_clear(tbl_all, kTblBytes, lane, 32);  // both sets
@@ -837,7 +852,7 @@ __device__ __forceinline__ void finalize_body(const RoundArgs<Packed>& a, int k)
   const int lane = threadIdx.x & 31;
   const int gw = (int)((blockIdx.x * blockDim.x + threadIdx.x) >> 5);
   const int NW = (int)((gridDim.x * blockDim.x) >> 5);
-  const int nF = ld_cg(&ctrl->fin_cnt);
+  const int nF = ld_cg(&ctrl->ring[rs(k)].fin);
   const C* X = sel((k - 1) & 1, (const C*)a.col[0], (const C*)a.col[1]);
   C* Y = sel(k & 1, a.col[0], a.col[1]);
   int64_t* out = sel(p ^ 1, a.wl_c[0], a.wl_c[1]);
@@ -866,8 +881,8 @@ __device__ __forceinline__ void finalize_body(const RoundArgs<Packed>& a, int k)
       Y[v] = conf ? cpack<C>(tent, k + 1, a) : cpack<C>(cval<C>(ldraw<Persist>(X + v)), k, a);
       if (conf) {
         nch2 = num_chunks(ld_cg(len_nxt + v));
-        ob = atomicAdd(&ctrl->cnt[p ^ 1][2], nch2);
-        atomicAdd(&ctrl->vcnt2[p ^ 1], 1);
+        ob = atomicAdd(&ctrl->ring[rs(k + 1)].c, nch2);
+        atomicAdd(&ctrl->ring[rs(k + 1)].cv, 1);
       }
     }
     if (conf) {
@@ -1088,7 +1103,8 @@ __device__ __forceinline__ void bin1(const RoundArgs<C>& a, int k, const int32_t
 // round-robin assignment (warp w takes items w, w + NW, ...), with the next item's list
 // entry and row offsets prefetched while the current one is processed.
 template <int TB, bool Persist, class C, bool Hub>
-__device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, uint8_t* wsm,
+__device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, const Counts& w,
+                                           uint8_t* wsm,
                                            unsigned long long (&edges)[kBins],
                                            unsigned long long (&entries)[kBins],
                                            uint32_t& ph, unsigned long long (&cyc)[kBins]) {
@@ -1105,9 +1121,9 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, uint8_t
   // ---- bin 2 (Hub build only; the flat build runs when bin 2 is empty)
   if constexpr (!Hub) {
   } else if constexpr (packed<C>()) {
-    bin2_trimmed<TB, Persist>(a, k, p, X, Y, wsm, gw, NW, lane, edges[2], entries[2], ph);
+    bin2_trimmed<TB, Persist>(a, k, p, X, Y, wsm, gw, NW, lane, w.c, edges[2], entries[2], ph);
   } else {
-    const int nC = ld_cg(&ctrl->cnt[p][2]);
+    const int nC = w.c;
     const int64_t* items = sel(p, (const int64_t*)a.wl_c[0], (const int64_t*)a.wl_c[1]);
     int64_t* out = sel(p ^ 1, a.wl_c[0], a.wl_c[1]);
     int i = gw;
@@ -1126,7 +1142,7 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, uint8_t
         if (ln < en) prefetch_l2(a.col_idx + ln);
       }
       process_chunk_plain<TB, Persist, C>(a, k, v, (int32_t)(uint32_t)it, s, e, X, Y, out,
-                                          &ctrl->cnt[p ^ 1][2], &ctrl->vcnt2[p ^ 1], wtbl,
+                                          &ctrl->ring[rs(k + 1)].c, &ctrl->ring[rs(k + 1)].cv, wtbl,
                                           lane, edges[2], entries[2]);
       i = in;
       it = itn;
@@ -1140,21 +1156,21 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, uint8_t
   // ---- bin 1: four vertices per warp (one per 8-lane group), 512-byte tables
   bin1<TB, Persist, C, Hub>(
       a, k, sel(p, (const int32_t*)a.wl_m[0], (const int32_t*)a.wl_m[1]),
-      ld_cg(&ctrl->cnt[p][1]), sel(p ^ 1, a.wl_m[0], a.wl_m[1]), &ctrl->cnt[p ^ 1][1], X, Y,
+      w.m, sel(p ^ 1, a.wl_m[0], a.wl_m[1]), &ctrl->ring[rs(k + 1)].m, X, Y,
       wsm, gw, NW, lane, edges[1], entries[1]);
   long long t2 = clock64();
   cyc[1] += (unsigned long long)(t2 - t1);
   // ---- bin 0: eight vertices per warp, register masks
   bin0<TB, Persist, C, Hub>(
       a, k, sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]),
-      ld_cg(&ctrl->cnt[p][0]), sel(p ^ 1, a.wl_t[0], a.wl_t[1]), &ctrl->cnt[p ^ 1][0], X, Y,
+      w.t, sel(p ^ 1, a.wl_t[0], a.wl_t[1]), &ctrl->ring[rs(k + 1)].t, X, Y,
       wsm, gw, NW, lane, edges[0], entries[0]);
   cyc[0] += (unsigned long long)(clock64() - t2);
 }
 
 // Block reduction of the per-thread counters, one atomicAdd each per block.
 __device__ __forceinline__ void block_add6(unsigned long long (&x)[kBins],
-                                           unsigned long long (&y)[kBins], Ctrl* ctrl) {
+                                           unsigned long long (&y)[kBins], Ctrl* ctrl, int k) {
   __shared__ unsigned long long red[2 * kBins][kWarps];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
 #pragma unroll
@@ -1172,70 +1188,95 @@ __device__ __forceinline__ void block_add6(unsigned long long (&x)[kBins],
 #pragma unroll
       for (int o = 16; o > 0; o >>= 1) z += __shfl_xor_sync(0xffffffffu, z, o);
       if (lane == 0 && z) {
-        if (q < kBins) atomicAdd(&ctrl->edges_acc[q], z);
-        else atomicAdd(&ctrl->entries_acc[q - kBins], z);
+        if (q < kBins) atomicAdd(&ctrl->edges_acc[rs(k)][q], z);
+        else atomicAdd(&ctrl->entries_acc[rs(k)][q - kBins], z);
       }
     }
   }
 }
 
-// End of pass F_k (one thread, after every block of the pass is done): fold the pass's
-// counters into totals and the trace, consume W_k, advance k and decide whether W_{k+1}
-// is non-empty. A pass over an empty W_k changes nothing, so any surplus pass a host loop
-// issues before it sees `active == 0` is a no-op.
-__device__ __forceinline__ void advance_body(Ctrl* ctrl, bool first, bool force = false) {
-  volatile Ctrl* c = ctrl;
-  if (first) {  // after F_1: W_2 is in parity 0
-    int tot = 0;
-    for (int q = 0; q < kBins; ++q) tot += c->cnt[0][q];
-    c->pushes_total[kBins] = (unsigned long long)(c->cnt[0][0] + c->cnt[0][1] + c->vcnt2[0]);
-    c->k = 2;
-    c->active = tot > 0 && !c->overflow;
-    if (c->active && c->max_rounds < 2) {
-      c->status = 1;
-      c->active = 0;
-      for (int q = 0; q < kBins; ++q) c->cnt[0][q] = 0;
-    }
-    return;
+// Counts written by other blocks' atomics: read at L2 (ld.global.cg), never a stale L1 line.
+__device__ __forceinline__ Counts ld_counts(const Counts* p) {
+  const int4* q = reinterpret_cast<const int4*>(p);
+  const int4 x = __ldcg(q), y = __ldcg(q + 1);
+  Counts w;
+  w.t = x.x; w.m = x.y; w.c = x.z; w.cv = x.w;
+  w.fin = y.x; w.pad[0] = y.y; w.pad[1] = y.z; w.pad[2] = y.w;
+  return w;
+}
+
+__device__ __forceinline__ void stamp_round(Ctrl* c, int idx) {
+  if (c->round_ns && idx < c->round_cap) {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    c->round_ns[idx] = (int64_t)t;
   }
-  const int k = c->k;
-  const int p = k & 1;
-  const int items_in = c->cnt[p][0] + c->cnt[p][1] + c->cnt[p][2];
-  if (items_in == 0 && !force) {  // (multi-GPU ranks advance in lockstep: force)
+}
+
+// After F_1 (one thread): W_2's counts are in ring slot 2.
+__device__ __forceinline__ void first_body(Ctrl* c) {
+  const Counts w = ld_counts(&c->ring[rs(2)]);
+  c->pushes_total[kBins] = (unsigned long long)(w.t + w.m + w.cv);
+  c->k = 2;
+  c->active = (w.t + w.m + w.c) > 0 && !__ldcg(&c->overflow);
+  if (c->active && c->max_rounds < 2) {
+    c->status = 1;
     c->active = 0;
-    return;
   }
-  const int vin[kBins] = {c->cnt[p][0], c->cnt[p][1], c->vcnt2[p]};
-  const int vout[kBins] = {c->cnt[p ^ 1][0], c->cnt[p ^ 1][1], c->vcnt2[p ^ 1]};
+  stamp_round(c, 0);
+}
+
+// Fold finished pass F_k into the totals and the trace (one thread, any time after every
+// block of pass k is done and before pass k+2 pushes into slot k % 3), then zero slot k % 3.
+// A pass over an empty W_k changes nothing, so surplus passes are no-ops.
+__device__ __forceinline__ void fold_pass(Ctrl* c, int k) {
+  const Counts win = ld_counts(&c->ring[rs(k)]), wout = ld_counts(&c->ring[rs(k + 1)]);
+  const int vin[kBins] = {win.t, win.m, win.cv};
+  const int vout[kBins] = {wout.t, wout.m, wout.cv};
   unsigned long long e_all = 0;
   int tot_in = 0;
   for (int q = 0; q < kBins; ++q) {
+    const unsigned long long e = __ldcg(&c->edges_acc[rs(k)][q]);
+    const unsigned long long x = __ldcg(&c->entries_acc[rs(k)][q]);
     c->verts_total[q] += (unsigned long long)vin[q];
-    c->edges_total[q] += c->edges_acc[q];
-    c->entries_total[q] += c->entries_acc[q];
+    c->edges_total[q] += e;
+    c->entries_total[q] += x;
     c->pushes_total[q] += (unsigned long long)vout[q];
-    e_all += c->edges_acc[q];
-    c->edges_acc[q] = 0;
-    c->entries_acc[q] = 0;
+    c->edges_acc[rs(k)][q] = 0ull;
+    c->entries_acc[rs(k)][q] = 0ull;
+    e_all += e;
     tot_in += vin[q];
   }
-  c->items_total += (unsigned long long)c->cnt[p][2];
-  c->fin_cnt = 0;
-  for (int q = 0; q < kBins; ++q) c->cnt[p][q] = 0;
-  c->vcnt2[p] = 0;
+  c->items_total += (unsigned long long)win.c;
+  c->ring[rs(k)] = Counts{};
   if (k - 1 < c->round_cap) {
     if (c->round_sizes) c->round_sizes[k - 1] = tot_in;
     if (c->round_edges) c->round_edges[k - 1] = (int64_t)e_all;
   }
+  stamp_round(c, k - 1);
+}
+
+__device__ __forceinline__ int items_of(const Counts& w) { return w.t + w.m + w.c; }
+
+// Host / graph loop modes, after pass F_k (and its finalize): fold it, advance k and decide
+// whether W_{k+1} is non-empty. Multi-GPU ranks advance in lockstep (force).
+__device__ __forceinline__ void advance_body(Ctrl* ctrl, bool first, bool force = false) {
+  Ctrl* c = ctrl;
+  if (first) {
+    first_body(c);
+    return;
+  }
+  const int k = c->k;
+  if (items_of(ld_counts(&c->ring[rs(k)])) == 0 && !force) {
+    c->active = 0;
+    return;
+  }
+  fold_pass(c, k);
   c->k = k + 1;
-  const int items_out = c->cnt[p ^ 1][0] + c->cnt[p ^ 1][1] + c->cnt[p ^ 1][2];
-  // a packed color overflowed: stop here, the host reruns with 32-bit colors
-  c->active = items_out > 0 && !c->overflow;
+  c->active = items_of(ld_counts(&c->ring[rs(k + 1)])) > 0 && !__ldcg(&c->overflow);
   if (c->active && k + 1 > c->max_rounds) {  // W_{k+1} non-empty beyond the cap
     c->status = 1;
     c->active = 0;
-    for (int q = 0; q < kBins; ++q) c->cnt[p ^ 1][q] = 0;
-    c->vcnt2[p ^ 1] = 0;
   }
 }
 
@@ -1253,7 +1294,8 @@ __global__ void k_pack(RoundArgs<C> a, uint2* send, int32_t cap) {
   const int k = ctrl->k;  // already advanced: W_k's lists are the new ones
   const int p = k & 1;
   const C* Y = sel((k - 1) & 1, (const C*)a.col[0], (const C*)a.col[1]);
-  const int nT = ctrl->cnt[p][0], nM = ctrl->cnt[p][1], nC = ctrl->cnt[p][2];
+  const Counts w = ctrl->ring[rs(k)];
+  const int nT = w.t, nM = w.m, nC = w.c;
   const int32_t* lt = sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]);
   const int32_t* lm = sel(p, (const int32_t*)a.wl_m[0], (const int32_t*)a.wl_m[1]);
   const int64_t* lc = sel(p, (const int64_t*)a.wl_c[0], (const int64_t*)a.wl_c[1]);
@@ -1340,8 +1382,10 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks<C>) k_round(RoundArgs<C> a)
   unsigned long long edges[kBins] = {0, 0, 0}, entries[kBins] = {0, 0, 0};
   unsigned long long cyc[kBins] = {0, 0, 0};
   uint32_t ph = 0;
-  round_body<TB, false, C, true>(a, ctrl->k, wsm, edges, entries, ph, cyc);
-  block_add6(edges, entries, ctrl);
+  const int k = ctrl->k;
+  const Counts w = ctrl->ring[rs(k)];
+  round_body<TB, false, C, true>(a, k, w, wsm, edges, entries, ph, cyc);
+  block_add6(edges, entries, ctrl, k);
   if ((threadIdx.x & 31) == 0)
     for (int q = 0; q < kBins; ++q) atomicAdd(&ctrl->bin_cycles[q], cyc[q]);
 }
@@ -1355,51 +1399,77 @@ __global__ void __launch_bounds__(kBlock) k_finalize(RoundArgs<C> a) {
   }
 }
 
-// Grid-wide barrier whose last arriving block runs advance_body (persistent kernel).
-__device__ __forceinline__ void grid_sync_advance(Ctrl* ctrl, bool advance = true) {
+__device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_gpu(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ uint32_t atom_add_acq_rel_u32(uint32_t* p, uint32_t v) {
+  uint32_t r;
+  asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], %2;" : "=r"(r) : "l"(p), "r"(v) : "memory");
+  return r;
+}
+
+// Grid-wide barrier of the persistent kernel (every block resident). Thread 0 of each block
+// arrives with an acq_rel atomic (publishing, via the preceding bar.sync, every write of
+// its block); the last arrival resets the count and releases the new generation.
+__device__ __forceinline__ void grid_sync(Ctrl* ctrl) {
   __syncthreads();
   if (threadIdx.x == 0) {
-    volatile uint32_t* gen_p = &ctrl->bar_gen;
-    const uint32_t gen = *gen_p;
-    __threadfence();
-    const uint32_t arrived = atomicAdd(&ctrl->bar_count, 1u);
+    const uint32_t gen = ld_acquire_gpu(&ctrl->bar_gen);
+    const uint32_t arrived = atom_add_acq_rel_u32(&ctrl->bar_count, 1u);
     if (arrived == gridDim.x - 1) {
-      __threadfence();
-      if (advance) advance_body(ctrl, false);
-      *(volatile uint32_t*)&ctrl->bar_count = 0u;
-      __threadfence();
-      atomicAdd(&ctrl->bar_gen, 1u);
+      ctrl->bar_count = 0u;
+      st_release_gpu(&ctrl->bar_gen, gen + 1u);
     } else {
-      while (*gen_p == gen) __nanosleep(32);
+      while (ld_acquire_gpu(&ctrl->bar_gen) == gen) __nanosleep(20);
     }
-    __threadfence();
   }
   __syncthreads();
 }
 
-// All rounds in one cooperative launch (every block resident): pass, barrier+advance, ...
-// The host enqueues both builds; each returns at once unless it is the right one for this
-// coloring (Hub iff F_1 put a vertex into bin 2), so the choice needs no host round trip.
+
+// All rounds in one cooperative launch (every block resident). Each block tracks k itself
+// and reads W_k's counts after the barrier that ends pass k-1; block 0 folds pass k-1 into
+// the totals while pass k runs. The host enqueues both builds; each returns at once unless
+// it is the right one for this coloring (Hub iff F_1 put a vertex into bin 2), so the
+// choice needs no host round trip.
 template <int TB, class C, bool Hub>
 __global__ void __launch_bounds__(kBlock, kMinBlocks<C, Hub>) k_persistent(RoundArgs<C> a) {
   extern __shared__ __align__(16) uint8_t dsmem[];
   Ctrl* ctrl = a.ctrl;
   if ((ld_cg(&ctrl->big_count) != 0) != Hub) return;  // uniform across the grid
+  if (!ld_cg(&ctrl->active)) return;                   // F_1 left W_2 empty
   uint8_t* wsm = warp_smem_init<C, Hub>(dsmem);
   uint32_t ph = 0;  // mbarrier phase bits of the warp's two TMA stages
   unsigned long long cyc[kBins] = {0, 0, 0};
-  for (;;) {
-    const int active = ld_cg(&ctrl->active);
-    const int k = ld_cg(&ctrl->k);
-    if (!active) break;  // uniform: read after the barrier by every thread
+  const int max_rounds = ld_cg(&ctrl->max_rounds);
+  const bool leader = blockIdx.x == 0 && threadIdx.x == 0;
+  int k = 2;
+  for (;; ++k) {
+    const Counts w = ld_counts(&ctrl->ring[rs(k)]);
+    const int overflow = ld_cg(&ctrl->overflow);
+    if (leader && k > 2) fold_pass(ctrl, k - 1);
+    const bool active = items_of(w) > 0 && !overflow;
+    if (!active || k > max_rounds) {  // uniform: every block read the same values
+      if (leader) {
+        ctrl->k = k;
+        ctrl->active = 0;
+        if (active) ctrl->status = 1;  // W_k non-empty beyond the cap
+      }
+      break;
+    }
     unsigned long long edges[kBins] = {0, 0, 0}, entries[kBins] = {0, 0, 0};
-    round_body<TB, true, C, Hub>(a, k, wsm, edges, entries, ph, cyc);
-    block_add6(edges, entries, ctrl);
+    round_body<TB, true, C, Hub>(a, k, w, wsm, edges, entries, ph, cyc);
+    block_add6(edges, entries, ctrl, k);
     if constexpr (packed<C>() && Hub) {  // multi-chunk vertices: decided once all chunks are in
-      grid_sync_advance(ctrl, false);
+      grid_sync(ctrl);
       finalize_body<TB, true>(a, k);
     }
-    grid_sync_advance(ctrl);
+    grid_sync(ctrl);
   }
   if ((threadIdx.x & 31) == 0)
     for (int q = 0; q < kBins; ++q) atomicAdd(&ctrl->bin_cycles[q], cyc[q]);

@@ -22,7 +22,8 @@ import paper_conf_ipps_licqfsty16_b200 as sgr
 from paper_conf_ipps_licqfsty16_b200 import gen
 out = {}
 for cfg in %(configs)r:
-    g = gen.config(cfg)
+    # -1: path of 4000 vertices (4000 rounds of <= 4000 vertices: per-round loop overhead)
+    g = gen.stencil2d(4000, 1, 5) if cfg == -1 else gen.config(cfg)
     rp = torch.from_numpy(g.row_ptr).cuda(); ci = torch.from_numpy(g.col_idx).cuda()
     colors = torch.empty(g.n, dtype=torch.int32, device="cuda")
     ws = torch.empty(sgr.workspace_bytes(g.n, g.nnz), dtype=torch.uint8, device="cuda")
@@ -71,7 +72,7 @@ def main():
             continue
         res = json.loads(line[0][7:])
         txt = "  ".join(f"c{c}: {r['ms']:.2f} ms (min {r['min']:.2f}, grid {r['grid']}, "
-                        f"same={r['same']})" for c, r in res.items())
+                        f"R {r['rounds']}, same={r['same']})" for c, r in res.items())
         print(f"{os.path.basename(v):28s} {txt}", flush=True)
 
 
