@@ -124,7 +124,7 @@ struct alignas(32) Counts {
   int32_t c;                 // bin 2 chunk items
   int32_t cv;                // bin 2 vertices
   int32_t fin;               // pass k: multi-chunk bin-2 vertices awaiting the finalize phase
-  int32_t pad[3];
+  int32_t pad[3];            // pad[0]: pass k's bin-2 work cursor
 };
 // W_k's counts live in ring slot k % 3: pass k reads slot k % 3 and pushes W_{k+1} into
 // slot (k+1) % 3, while slot (k+2) % 3 (W_{k-1}, read by the finished pass k-1) is folded
@@ -581,6 +581,8 @@ __device__ __forceinline__ void process_chunk_plain(const RoundArgs<C>& a, int k
 struct ChunkHdr {
   int32_t v, c, len, slot, buf;
   int64_t s, e;   // original row [s, e): list start in adj[*] and col_idx
+  uint32_t fo;    // single-chunk vertex: this lane's word of its fixed set (prefetched)
+  uint32_t xraw;  // X[v] word (prefetched; decoded at use, so the load is not waited for)
 };
 
 template <int TB, bool Persist>
@@ -637,26 +639,51 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
     h.slot = __ldg(a.big_id + h.v);
   };
   auto load_hdr = [&](int i, ChunkHdr& h) { finish_hdr(__ldcg(items + i), h); };
+  // second-stage header loads, issued one chunk ahead (they need slot / v)
+  auto finish_hdr2 = [&](ChunkHdr& h) {
+    // unconditional loads (a select on the result would wait for it); fo is only used when
+    // the vertex has a single chunk, and fixed + slot * 32 is always a valid address
+    h.fo = ld_cg(a.fixed + (int64_t)h.slot * 32 + lane);
+    h.xraw = ldraw<Persist>(X + h.v);
+  };
+  auto zero_hdr = [](ChunkHdr& h) {
+    h.v = h.c = h.len = h.slot = h.buf = 0;
+    h.s = h.e = 0;
+    h.fo = 0u;
+    h.xraw = 0u;
+  };
 
+  // Work distribution: the warp's first four items are gw + j NW (j < 4); after that it
+  // takes the next unclaimed item from a per-pass cursor, so warps that drew short chunks
+  // take more of them. Software pipeline over the warp's items: while chunk i is processed,
+  // the next chunk's list window streams in (TMA) and its fixed set and own color load, the
+  // one after's header loads, the third one's item id and the fourth one's claim are in
+  // flight, so nothing the next iteration needs is waited for at the end of this one.
+  int* cursor = &ctrl->ring[rs(k)].pad[0];
   unsigned long long pc0 = 0, pc1 = 0, pc2 = 0, pc3 = 0;  // phase cycles (lane 0 adds)
   long long tq = clock64();
-  int i = gw;
+  int i = gw, in = gw + NW, inn = gw + 2 * NW, innn = gw + 3 * NW;
   ChunkHdr cur, nxt;
   load_hdr(i, cur);
+  finish_hdr2(cur);
 #if !SGR_NO_TMA
   if (lane == 0) issue(cur, 0);
 #endif
-  int in = i + NW;
-  nxt.v = nxt.c = nxt.len = nxt.slot = nxt.buf = 0;
-  nxt.s = nxt.e = 0;
+  zero_hdr(nxt);
   if (in < nC) load_hdr(in, nxt);
+  int64_t it_nn = inn < nC ? __ldcg(items + inn) : 0;
   int st = 0;
   while (i < nC) {
 #if !SGR_NO_TMA
     if (in < nC && lane == 0) issue(nxt, st ^ 1);
 #endif
-    const int inn = in + NW;
-    const int64_t it_nn = inn < nC ? __ldcg(items + inn) : 0;
+    if (in < nC) finish_hdr2(nxt);
+    ChunkHdr nn;
+    zero_hdr(nn);
+    if (inn < nC) finish_hdr(it_nn, nn);
+    const int64_t it_nnn = innn < nC ? __ldcg(items + innn) : 0;
+    int claim = nC;  // the item after innn (monotone: once past nC, stop claiming)
+    if (lane == 0 && innn < nC) claim = 4 * NW + atomicAdd(cursor, 1);
 
     // ---- chunk `cur` in stage st: slots [off0, off0 + cnt) of the 16-byte-aligned window
     const int32_t v = cur.v;
@@ -666,7 +693,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
     const int32_t nslots = off0 + cnt;
     const int32_t nb = (nslots + 128 * kQB - 1) / (128 * kQB);  // batches of kQB int4 per lane
     const int32_t nch = num_chunks(cur.len);
-    const int32_t xv = cval<C>(ldraw<Persist>(X + v));
+    const int32_t xv = cval<C>(cur.xraw);
     // a neighbour still in W_k was written by pass k-1 with last = k; one that has left W
     // has last < k and is recognised unless last = k mod 16, in which case it simply stays
     // in the list one more round (never the reverse: live neighbours are never dropped)
@@ -729,11 +756,6 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
     const long long tc = clock64();
     pc2 += (unsigned long long)(tc - tb);
 #endif
-    // next-next header: the item id has arrived by now
-    ChunkHdr nn;
-    nn.v = nn.c = nn.len = nn.slot = nn.buf = 0;
-    nn.s = nn.e = 0;
-    if (inn < nC) finish_hdr(it_nn, nn);
     if (lane == 0) {
       entries += (unsigned long long)cnt;
       if (cur.c == 0) edges += (unsigned long long)(cur.e - cur.s);
@@ -766,7 +788,6 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
           qb += tot;
         }
       }
-      fence_proxy_async_global();  // the next pass reads these lists with TMA
     };
 
     const int32_t slot = cur.slot;
@@ -775,7 +796,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
     int32_t* lst_other = sel(cur.buf, a.adj[1], a.adj[0]);
     if (nch == 1) {
       if (any) {
-        const uint32_t fo = ld_cg(fx + lane);
+        const uint32_t fo = cur.fo;
         const uint32_t word = tbl_bits32(tbl_all, lane) | fo | (lane == 0 ? 1u : 0u);
         int32_t tent = bits_first_free(word);
         if (tent < 0 || tent >= kBigTbl - 1) {  // beyond the exact range of the table
@@ -802,20 +823,21 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
       // several chunks: publish this chunk's partial forbidden set, dropped colors and
       // compacted live entries; the finalize phase after the pass decides conflict and
       // first fit once every chunk is in (no per-chunk fences or tickets)
+      // (the atomics whose results are needed are issued first, consumed last)
+      int32_t lbase = 0, fpos = 0;
+      if (lane == 0) {
+        if (live_total) lbase = atomicAdd(len_nxt + v, (int32_t)live_total);
+        if (cur.c == 0) fpos = atomicAdd(&ctrl->ring[rs(k)].fin, 1);
+        if (any) atomicOr(a.acc_cnt + slot, 1ull);  // conflict flag
+      }
       uint32_t* accb = a.acc_bits + (int64_t)slot * 32;
       const uint32_t bits = tbl_bits32(tbl_all, lane);
       const uint32_t drop = tbl_bits32(tbl_drop, lane);
       if (bits) atomicOr(accb + lane, bits);
       if (drop) atomicOr(fx + lane, drop);
-      int32_t lbase = 0;
-      if (lane == 0 && live_total) lbase = atomicAdd(len_nxt + v, (int32_t)live_total);
       lbase = __shfl_sync(0xffffffffu, lbase, 0);
       write_live(lst_other + cur.s + lbase);
-      if (lane == 0) {
-        if (any) atomicOr(a.acc_cnt + slot, 1ull);  // conflict flag
-        if (cur.c == 0)
-          a.fin[atomicAdd(&ctrl->ring[rs(k)].fin, 1)] = (int32_t)((uint32_t)v | (cur.buf ? kBufBit : 0u));
-      }
+      if (lane == 0 && cur.c == 0) a.fin[fpos] = (int32_t)((uint32_t)v | (cur.buf ? kBufBit : 0u));
     }
     set_clear(tbl_all, kTblBytes, lane, 32);  // both sets
     __syncwarp();
@@ -826,11 +848,16 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
     st ^= 1;
     i = in;
     in = inn;
+    inn = innn;
+    innn = __shfl_sync(0xffffffffu, claim, 0);
     cur = nxt;
     nxt = nn;
+    it_nn = it_nnn;
   }
   iflush();
   if (lane == 0 && vpend) atomicAdd(out_vcnt, vpend);
+  // once per pass: this thread's list writes before the next pass's TMA (async-proxy) reads
+  fence_proxy_async_global();
   if (lane == 0) {
     atomicAdd(&ctrl->phase_cycles[0], pc0);
     atomicAdd(&ctrl->phase_cycles[1], pc1);
