@@ -251,10 +251,6 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
     cudaError_t le = cudaMemcpyAsync(a.ctrl, &hc, sizeof(Ctrl), cudaMemcpyHostToDevice, s);
     if (le == cudaSuccess)
       le = cudaMemsetAsync((char*)ws + L.zero_begin, 0, L.zero_end - L.zero_begin, s);
-    if constexpr (packed<C>()) {  // the bin-2 lists start as the full rows
-      if (le == cudaSuccess && nnz > 0)
-        le = cudaMemcpyAsync(a.adj[0], csr->col_idx, (size_t)nnz * 4, cudaMemcpyDeviceToDevice, s);
-    }
     if (le != cudaSuccess) {
       status = cuda_fail(le, "workspace init", __LINE__);
       break;

@@ -93,11 +93,6 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
     hc.max_rounds = INT32_MAX;
     DCK(cudaMemcpyAsync(args[i].ctrl, &hc, sizeof(Ctrl), cudaMemcpyHostToDevice, s));
     DCK(cudaMemsetAsync((char*)pt.ws + Ls[i].zero_begin, 0, Ls[i].zero_end - Ls[i].zero_begin, s));
-    if constexpr (packed<C>()) {
-      if (pt.nnz > 0)
-        DCK(cudaMemcpyAsync(args[i].adj[0], pt.csr.col_idx, (size_t)pt.nnz * 4,
-                            cudaMemcpyDeviceToDevice, s));
-    }
     k_fill_c1<C><<<first_grid(n), 256, 0, s>>>(args[i]);
     k_first<TB, C><<<first_grid(pt.hi - pt.lo), 256, 0, s>>>(args[i], 1);
     k_advance<<<1, 32, 0, s>>>(args[i].ctrl, 1, 0);

@@ -113,8 +113,10 @@ inline void build_args(RoundArgs<C>& a, const sgr_csr* csr, int64_t n, int64_t n
   a.color_cap = r.color_cap;
 }
 
+// Streaming per-vertex kernels (F_1, unpack, max): one thread per vertex up to 64 blocks
+// per SM, so the dependent row_ptr -> col_idx loads of many vertices are in flight.
 inline int first_grid(int64_t n) {
-  return (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, (int64_t)num_sms() * 8));
+  return (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, (int64_t)num_sms() * 64));
 }
 
 template <class C, bool Hub = true>

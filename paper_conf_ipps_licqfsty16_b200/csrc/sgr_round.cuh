@@ -619,15 +619,18 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
     ipend = 0;
   };
 
+  // Pass 2 reads the rows straight from col_idx (every list is still the full row); later
+  // passes read the compacted lists in adj[buf].
+  auto list_src = [&](int buf) -> const int32_t* {
+    return k == 2 ? a.col_idx : sel(buf, (const int32_t*)a.adj[0], (const int32_t*)a.adj[1]);
+  };
   auto issue = [&](const ChunkHdr& h, int st) {  // lane 0 only
     const int64_t cs = h.s + (int64_t)h.c * kChunk;
     const int64_t ce = min(h.s + (int64_t)h.len, cs + kChunk);
     const int64_t w0 = cs & ~(int64_t)3;
     const uint32_t bytes = (uint32_t)(((ce - w0 + 3) >> 2) << 4);
     fence_proxy_async();  // generic-proxy reads of this stage happen-before the async write
-    tma_load_1d(bufs + st * (kStage / 4), sel(h.buf, (const int32_t*)a.adj[0],
-                                              (const int32_t*)a.adj[1]) + w0,
-                bytes, bars + st);
+    tma_load_1d(bufs + st * (kStage / 4), list_src(h.buf) + w0, bytes, bars + st);
   };
   auto finish_hdr = [&](int64_t it, ChunkHdr& h) {  // everything but the item itself
     h.v = (int32_t)((uint64_t)it >> 32);
@@ -700,8 +703,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
     const uint32_t klive = (uint32_t)k & 15u;
 #if SGR_NO_TMA
     {  // A/B: the warp stages its own window (16-byte loads + shared stores), no TMA
-      const int4* g4 = reinterpret_cast<const int4*>(
-          sel(cur.buf, (const int32_t*)a.adj[0], (const int32_t*)a.adj[1]) + (cs & ~(int64_t)3));
+      const int4* g4 = reinterpret_cast<const int4*>(list_src(cur.buf) + (cs & ~(int64_t)3));
       int4* s4 = reinterpret_cast<int4*>(bufs + st * (kStage / 4));
       for (int q = 0; 4 * 32 * q < nslots; ++q)
         if (4 * (lane + 32 * q) < nslots) s4[lane + 32 * q] = __ldcg(g4 + lane + 32 * q);
@@ -805,8 +807,8 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
         const uint32_t drop = tbl_bits32(tbl_drop, lane);
         if (drop & ~fo) fx[lane] = fo | drop;
         // single chunk: the warp owns the whole list, so it is compacted in place, and not
-        // rewritten at all when nothing was dropped
-        if (live_total < (uint32_t)cnt) write_live(lst_same + cur.s);
+        // rewritten at all when nothing was dropped (pass 2 read col_idx: always written)
+        if (k == 2 || live_total < (uint32_t)cnt) write_live(lst_same + cur.s);
         if (lane == 0) {
           len_nxt[v] = (int32_t)live_total;
           Y[v] = cpack<C>(tent, k + 1, a);
