@@ -46,6 +46,24 @@ def parse():
     return ap.parse_args()
 
 
+# Scattered color-gather ceiling of one B200 (tools/gather_bench.cu: random 4-byte gathers
+# into a 64 MB L2-resident array, ~1 distinct 128-byte line per SM-cycle; see
+# profiles/r01_ncu_summary.md). The round kernel's binding resource besides HBM.
+GATHER_PEAK_G = 271.0
+
+
+def ncu_traffic(workload: str, kernel: str):
+    """DRAM bytes per launch of `kernel` from the committed ncu --set full capture
+    (profiles/ncu_traffic.json, written from `ncu -i ... --page raw`), or None."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if not os.path.exists(p):
+        return None
+    with open(p) as f:
+        d = json.load(f)
+    e = d.get(workload, {}).get(kernel)
+    return None if e is None else int(e["dram_read_bytes"] + e["dram_write_bytes"])
+
+
 def peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -238,7 +256,8 @@ def run_single(args):
     achieved = kb[dom] / (kms[dom] * 1e-3) / 1e9 if kms[dom] > 0 else 0.0
     total_kernel_ms = sum(kms.values())
     roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak,
-                "unit": "GB/s", "frac": achieved / peak, "traffic": None,
+                "unit": "GB/s", "frac": achieved / peak,
+                "traffic": ncu_traffic(workload_name(args.config), dom),
                 "peak_source": peak_src,
                 "launches_per_step": kl[dom] / args.steps,
                 "algorithmic_bytes_per_launch": kb[dom] / max(kl[dom], 1),
@@ -248,7 +267,15 @@ def run_single(args):
                 "whole_step": {"algorithmic_GBps": st["bytes_algorithmic"] / (ms * 1e-3) / 1e9,
                                "frac": st["bytes_algorithmic"] / (ms * 1e-3) / 1e9 / peak},
                 "bin_edges": st["bin_edges"], "bin_vertices": st["bin_vertices"],
-                "chunk_items": st["chunk_items"], "grid_blocks": st["grid_blocks"]}
+                "chunk_items": st["chunk_items"], "grid_blocks": st["grid_blocks"],
+                "entries_read_per_nnz": st["entries_read"] / g.nnz,
+                "entries_written_per_nnz": st["entries_written"] / g.nnz,
+                "color_bits": st["color_bits"]}
+    # the same kernel against the scattered-gather ceiling (one color gather per entry read)
+    g_rate = st["entries_read"] / (kms["round"] / args.steps * 1e-3) / 1e9 if kms.get("round") else 0.0
+    roofline["gather"] = {"achieved": g_rate, "peak": GATHER_PEAK_G, "unit": "G gathers/s",
+                          "frac": g_rate / GATHER_PEAK_G,
+                          "peak_source": "measured, tools/gather_bench.cu (profiles/r01_ncu_summary.md)"}
 
     # e2e: the same coloring through sgr_color_host from pinned host buffers
     e2e = None

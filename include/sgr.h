@@ -128,6 +128,7 @@ typedef struct {
   int64_t bin_warp_cycles[3];        /* SM cycles warps spent in each bin (all rounds)   */
   int32_t grid_blocks;               /* blocks of the round kernel                        */
   int32_t color_bits;                /* width the coloring finished with (16 or 32)       */
+  int64_t entries_written;           /* compacted neighbour-list entries written (bin 2)  */
 } sgr_stats;
 
 void sgr_opts_default(sgr_opts* opts);

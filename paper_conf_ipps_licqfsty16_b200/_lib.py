@@ -45,7 +45,7 @@ class Stats(ctypes.Structure):
                 ("bin_vertices", ctypes.c_int64 * 3), ("bin_edges", ctypes.c_int64 * 3),
                 ("chunk_items", ctypes.c_int64), ("bin_warp_cycles", ctypes.c_int64 * 3),
                 ("grid_blocks", ctypes.c_int32),
-                ("color_bits", ctypes.c_int32)]
+                ("color_bits", ctypes.c_int32), ("entries_written", ctypes.c_int64)]
 
     def as_dict(self) -> dict:
         d = {k: getattr(self, k) for k in ("rounds", "num_colors", "vertices_processed",
@@ -59,6 +59,7 @@ class Stats(ctypes.Structure):
         d["chunk_items"] = self.chunk_items
         d["bin_warp_cycles"] = dict(zip(BINS, list(self.bin_warp_cycles)))
         d["grid_blocks"] = self.grid_blocks
+        d["entries_written"] = self.entries_written
         d["color_bits"] = self.color_bits
         return d
 

@@ -188,20 +188,23 @@ struct Prof {
 };
 
 // Byte model and counters from the final Ctrl.
-void fill_stats(const Ctrl& c, int64_t n, int64_t nnz, sgr_stats* st) {
+void fill_stats(const Ctrl& c, int64_t n, int64_t nnz, sgr_stats* st, int cb) {
   int64_t vpass = 0, epass = 0, b_round = 0;
   for (int q = 0; q < kBins; ++q) {
     vpass += (int64_t)c.verts_total[q];
     epass += (int64_t)c.edges_total[q];
     st->bin_vertices[q] = (int64_t)c.verts_total[q];
     st->bin_edges[q] = (int64_t)c.edges_total[q];
-    // per worklist vertex: 4 B id + 16 B row pair + 4 B X[v] + 4 B Y[v]; 8 B per scanned
-    // entry actually read (4 B list entry + 4 B X[w]); 4 B per vertex pushed to W_{k+1}
-    b_round += 28 * (int64_t)c.verts_total[q] + 8 * (int64_t)c.entries_total[q] +
+    // per worklist vertex: 4 B id + 16 B row pair + X[v] + Y[v] words; per adjacency entry
+    // actually read: 4 B list entry + an X[w] word (cb = 2 packed, 4 plain); 4 B per vertex
+    // pushed to W_{k+1}; 4 B per compacted list entry written (below)
+    b_round += (20 + 2 * cb) * (int64_t)c.verts_total[q] + (4 + cb) * (int64_t)c.entries_total[q] +
                4 * (int64_t)c.pushes_total[q];
     st->entries_read += (int64_t)c.entries_total[q];
   }
   st->chunk_items = (int64_t)c.items_total;
+  st->entries_written = (int64_t)c.list_writes_total;
+  b_round += 4 * (int64_t)c.list_writes_total;
   for (int q = 0; q < kBins; ++q) st->bin_warp_cycles[q] = (int64_t)c.bin_cycles[q];
   if (const char* env = getenv("SGR_PHASES")) {  // experiments: bin-2 phase breakdown
     (void)env;
@@ -212,9 +215,10 @@ void fill_stats(const Ctrl& c, int64_t n, int64_t nnz, sgr_stats* st) {
   st->num_colors = c.max_color;
   st->vertices_processed = n + vpass;
   st->edges_scanned = nnz + epass;
-  // F_1 per vertex: 8 B row offset + 4 B first/last entry + 4 B + 4 B color writes; 4 B/push
-  const int64_t b_first = 20 * n + 4 * (int64_t)c.pushes_total[kBins];
-  const int64_t b_final = 4 * n;
+  // F_1 per vertex: 8 B row offset + 4 B first/last entry + two color-word writes; 4 B/push.
+  // Final: packed, read a word + write int32 (max fused); plain, the max-color read.
+  const int64_t b_first = (12 + 2 * cb) * n + 4 * (int64_t)c.pushes_total[kBins];
+  const int64_t b_final = (cb == 2 ? 6 : 4) * n;
   st->bytes_algorithmic = b_first + b_round + b_final;
   st->kernel_bytes[SGR_K_FIRST] = b_first;
   st->kernel_bytes[SGR_K_ROUND] = b_round;
@@ -338,10 +342,12 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
     }
 
     prof.timed(SGR_K_FINAL, s, [&] {
-      if constexpr (packed<C>()) k_unpack<<<first_grid(n), 256, 0, s>>>(a.col[0], colors_out, n);
-      k_max_color<<<first_grid(n), 256, 0, s>>>(colors_out, n, &a.ctrl->max_color);
+      if constexpr (packed<C>())
+        k_unpack<<<reduce_grid(n), 256, 0, s>>>(a.col[0], colors_out, n, &a.ctrl->max_color);
+      else
+        k_max_color<<<reduce_grid(n), 256, 0, s>>>(colors_out, n, &a.ctrl->max_color);
     });
-    launches += packed<C>() ? 2 : 1;
+    launches += 1;
     cudaEventRecord(ev1, s);
     Ctrl fin;
     cudaMemcpyAsync(&fin, a.ctrl, sizeof(Ctrl), cudaMemcpyDeviceToHost, s);
@@ -352,7 +358,7 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
     }
     *overflow_out = fin.overflow;
     if (stats) {
-      fill_stats(fin, n, nnz, stats);
+      fill_stats(fin, n, nnz, stats, (int)sizeof(C));
       cudaEventElapsedTime(&stats->elapsed_ms, ev0, ev1);
       stats->launches = launches;
       stats->grid_blocks = fin.big_count ? grid : grid_flat;

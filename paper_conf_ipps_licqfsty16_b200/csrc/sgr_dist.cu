@@ -183,11 +183,12 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
   if (status == SGR_OK) {
     RoundArgs<C>& a0 = args[0];
     if constexpr (packed<C>()) {
-      k_unpack<<<first_grid(n), 256, 0, s>>>(a0.col[0], colors_out, n);
-    } else if (a0.col[0] != (C*)colors_out) {
-      DCK(cudaMemcpyAsync(colors_out, a0.col[0], (size_t)n * 4, cudaMemcpyDeviceToDevice, s));
+      k_unpack<<<reduce_grid(n), 256, 0, s>>>(a0.col[0], colors_out, n, &a0.ctrl->max_color);
+    } else {
+      if (a0.col[0] != (C*)colors_out)
+        DCK(cudaMemcpyAsync(colors_out, a0.col[0], (size_t)n * 4, cudaMemcpyDeviceToDevice, s));
+      k_max_color<<<reduce_grid(n), 256, 0, s>>>(colors_out, n, &a0.ctrl->max_color);
     }
-    k_max_color<<<first_grid(n), 256, 0, s>>>(colors_out, n, &a0.ctrl->max_color);
     DCK(cudaGetLastError());
     std::vector<Ctrl> fin(P);
     for (int i = 0; i < P; ++i)
@@ -205,9 +206,10 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
       for (int i = 0; i < P; ++i) {
         sgr_stats t;
         memset(&t, 0, sizeof(t));
-        fill_stats(fin[i], 0, 0, &t);
+        fill_stats(fin[i], 0, 0, &t, (int)sizeof(C));
         stats->edges_scanned += t.edges_scanned;
         stats->entries_read += t.entries_read;
+        stats->entries_written += t.entries_written;
         stats->bytes_algorithmic += t.bytes_algorithmic;
         stats->chunk_items += t.chunk_items;
         for (int q = 0; q < 3; ++q) {

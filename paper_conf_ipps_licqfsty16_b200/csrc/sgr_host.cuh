@@ -118,6 +118,10 @@ inline void build_args(RoundArgs<C>& a, const sgr_csr* csr, int64_t n, int64_t n
 inline int first_grid(int64_t n) {
   return (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, (int64_t)num_sms() * 64));
 }
+// Per-vertex kernels that end in one atomic per warp (unpack + max): 8 blocks per SM.
+inline int reduce_grid(int64_t n) {
+  return (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, (int64_t)num_sms() * 8));
+}
 
 template <class C, bool Hub = true>
 constexpr size_t round_smem() { return (size_t)kWarps * WarpSmem<C, Hub>::kBytes; }

@@ -36,6 +36,6 @@ int num_sms();
 void keep_pool_memory();
 Resolved resolve_opts(const sgr_opts* o, int64_t n);
 size_t ws_bytes(int64_t n, int64_t nnz, const Resolved& r);
-void fill_stats(const Ctrl& c, int64_t n, int64_t nnz, sgr_stats* st);
+void fill_stats(const Ctrl& c, int64_t n, int64_t nnz, sgr_stats* st, int cb);
 
 }  // namespace sgr

@@ -154,6 +154,7 @@ struct Ctrl {
   unsigned long long entries_total[kBins + 1];
   unsigned long long pushes_total[kBins + 1];
   unsigned long long items_total;
+  unsigned long long list_writes_total;   // compacted list entries written (bin 2, packed)
   unsigned long long bin_cycles[kBins];   // warp-cycles spent in each bin (SM clock)
   unsigned long long phase_cycles[4];     // bin 2 (trimmed) phases: issue, wait, gather, post
   int32_t* round_sizes;
@@ -663,6 +664,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
   // one after's header loads, the third one's item id and the fourth one's claim are in
   // flight, so nothing the next iteration needs is waited for at the end of this one.
   int* cursor = &ctrl->ring[rs(k)].pad[0];
+  unsigned long long lwrites = 0;  // warp-uniform
   unsigned long long pc0 = 0, pc1 = 0, pc2 = 0, pc3 = 0;  // phase cycles (lane 0 adds)
   long long tq = clock64();
   int i = gw, in = gw + NW, inn = gw + 2 * NW, innn = gw + 3 * NW;
@@ -808,7 +810,10 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
         if (drop & ~fo) fx[lane] = fo | drop;
         // single chunk: the warp owns the whole list, so it is compacted in place, and not
         // rewritten at all when nothing was dropped (pass 2 read col_idx: always written)
-        if (k == 2 || live_total < (uint32_t)cnt) write_live(lst_same + cur.s);
+        if (k == 2 || live_total < (uint32_t)cnt) {
+          write_live(lst_same + cur.s);
+          lwrites += live_total;
+        }
         if (lane == 0) {
           len_nxt[v] = (int32_t)live_total;
           Y[v] = cpack<C>(tent, k + 1, a);
@@ -839,6 +844,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
       if (drop) atomicOr(fx + lane, drop);
       lbase = __shfl_sync(0xffffffffu, lbase, 0);
       write_live(lst_other + cur.s + lbase);
+      lwrites += live_total;
       if (lane == 0 && cur.c == 0) a.fin[fpos] = (int32_t)((uint32_t)v | (cur.buf ? kBufBit : 0u));
     }
     set_clear(tbl_all, kTblBytes, lane, 32);  // both sets
@@ -858,6 +864,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
   }
   iflush();
   if (lane == 0 && vpend) atomicAdd(out_vcnt, vpend);
+  if (lane == 0 && lwrites) atomicAdd(&ctrl->list_writes_total, lwrites);
   // once per pass: this thread's list writes before the next pass's TMA (async-proxy) reads
   fence_proxy_async_global();
   if (lane == 0) {
@@ -1504,11 +1511,18 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks<C, Hub>) k_persistent(Round
     for (int q = 0; q < kBins; ++q) atomicAdd(&ctrl->bin_cycles[q], cyc[q]);
 }
 
-// Final colors (packed words) into the caller's int32 output.
-static __global__ void k_unpack(const Packed* __restrict__ src, int32_t* __restrict__ dst, int64_t n) {
+// Final colors (packed words) into the caller's int32 output, and their maximum.
+static __global__ void k_unpack(const Packed* __restrict__ src, int32_t* __restrict__ dst, int64_t n,
+                                int32_t* max_out) {
+  int32_t m = 0;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
-       i += (int64_t)gridDim.x * blockDim.x)
-    dst[i] = (int32_t)(src[i] & kColorMask);
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t c = (int32_t)(src[i] & kColorMask);
+    dst[i] = c;
+    m = max(m, c);
+  }
+  m = (int32_t)__reduce_max_sync(0xffffffffu, (unsigned)m);
+  if ((threadIdx.x & 31) == 0 && m) atomicMax(max_out, m);
 }
 
 }  // namespace sgr
