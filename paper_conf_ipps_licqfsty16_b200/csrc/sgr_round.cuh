@@ -80,7 +80,7 @@ constexpr int kTblBytes = 2 * kBigTblB;      // per-warp tables: 4 x bin-1 | 2 x
 constexpr int kWin = SGR_WIN;           // window entries (32 lanes x kWin / 128 int4)
 constexpr int kChunk = kWin - 4;        // bin-2 chunk: entries per warp item; the 16-byte-
                                         // aligned window (<= kWin entries) covers it
-static_assert(kWin == 512 || kWin == 1024, "window: 512 or 1024 entries");
+static_assert(kWin == 512 || kWin == 768 || kWin == 1024, "window: 512, 768 or 1024 entries");
 
 // Working color word. Packed (default): uint16_t = (last round mod 16) << 12 | color, color
 // <= 4095 (a larger first fit sets the overflow flag and the coloring is redone with plain
@@ -272,17 +272,47 @@ __device__ __forceinline__ void mbar_init_fence() {
 __device__ __forceinline__ void fence_proxy_async() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
+#ifndef SGR_L2HINT
+#define SGR_L2HINT 1
+#endif
+#ifndef SGR_ROWNA
+#define SGR_ROWNA 0
+#endif
 // One elected thread: announce `bytes` of transaction and start the bulk copy global->smem.
+// SGR_L2HINT: the lists stream through L2 with evict-first priority (they are read once
+// per pass), so the color arrays the gathers hit stay resident.
 __device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t bytes,
                                             uint64_t* bar) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)),
                "r"(bytes)
                : "memory");
+#if SGR_L2HINT
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+      " [%0], [%1], %2, [%3], %4;" ::"r"(smem_addr(dst)),
+      "l"(src), "r"(bytes), "r"(smem_addr(bar)), "l"(pol)
+      : "memory");
+#else
   asm volatile(
       "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::
           "r"(smem_addr(dst)),
       "l"(src), "r"(bytes), "r"(smem_addr(bar))
       : "memory");
+#endif
+}
+
+// Row entries of bins 0 and 1 (streamed once per pass). SGR_ROWNA: bypass L1 allocation,
+// leaving L1 to the color gathers.
+__device__ __forceinline__ int32_t ld_row(const int32_t* p) {
+#if SGR_ROWNA
+  int32_t r;
+  asm volatile("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(r) : "l"(p));
+  return r;
+#else
+  return __ldg(p);
+#endif
 }
 __device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
   uint32_t done;
@@ -948,7 +978,7 @@ __device__ __forceinline__ void process_group(const RoundArgs<C>& a, int k, int3
 #pragma unroll
     for (int u = 0; u < 8; ++u) {
       const int32_t r = 64 * bb + gl + kGroup * u;
-      w[u] = r < cnt ? __ldg(row + r) : -1;
+      w[u] = r < cnt ? ld_row(row + r) : -1;
     }
     uint32_t lb = 0;
 #pragma unroll
@@ -1049,7 +1079,7 @@ __device__ __forceinline__ void bin0(const RoundArgs<C>& a, int k, const int32_t
     const int32_t cnt = vv >= 0 ? (int32_t)(ee - ss) : 0;
     const int32_t* row = a.col_idx + ss;
 #pragma unroll
-    for (int u = 0; u < kK0; ++u) w[u] = (gl + G * u < cnt) ? __ldg(row + gl + G * u) : -1;
+    for (int u = 0; u < kK0; ++u) w[u] = (gl + G * u < cnt) ? ld_row(row + gl + G * u) : -1;
   };
   int i = gw * VPW + g;
   int32_t v = i < nX ? ld_cg(list + i) : -1;

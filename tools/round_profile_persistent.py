@@ -32,5 +32,10 @@ for k in range(2, R + 1):
     u = us[k - 2]
     if k < 12 or k % args.every == 0 or k > R - 3:
         print(f"{k:3d} {sizes[k-1]:9d} {edges[k-1]:11d} {u:8.1f} {edges[k-1]/max(u,1e-3)/1e3:7.1f}")
+cum = np.cumsum(us)
+for lo, hi in [(2, 11), (12, 30), (31, 60), (61, 100), (101, 150), (151, 200), (201, R)]:
+    sel = slice(lo - 2, min(hi, R) - 1)
+    print(f"rounds {lo:3d}-{min(hi, R):3d}: {us[sel].sum()/1e3:7.2f} ms, entries {np.sum(edges[lo-1:min(hi, R)])/1e6:9.1f} M")
+np.save("/tmp/round_us.npy", us)
 small = us[np.asarray(sizes[1:R]) < 1000]
 print(f"passes with |W| < 1000: {len(small)}, {small.sum()/1e3:.2f} ms, median {np.median(small) if len(small) else 0:.1f} us")
