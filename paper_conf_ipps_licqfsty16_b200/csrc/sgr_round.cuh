@@ -195,10 +195,26 @@ __device__ __forceinline__ int32_t ld_cg(const int32_t* p) { return __ldcg(p); }
 __device__ __forceinline__ uint32_t ld_cg(const uint32_t* p) { return __ldcg(p); }
 
 // ---- color words: int32_t = plain color; Packed = (last round mod 16) << 12 | color ------
+// Snapshot reads. A per-pass launch may use the read-only path (the buffer is not written
+// while it runs). The persistent kernel writes each buffer in alternate passes, so its
+// reads must be coherent: SGR_GATHER_CA = 0 reads at L2 (ld.global.cg); 1 uses plain
+// L1-cached loads, relying on the PTX memory model: every pass starts after the grid
+// barrier's ld.acquire.gpu (thread 0) + bar.sync, which orders these weak loads after the
+// previous pass's writes (the acquire invalidates the SM's L1).
+#ifndef SGR_GATHER_CA
+#define SGR_GATHER_CA 1
+#endif
 template <bool Persist, class C>
 __device__ __forceinline__ uint32_t ldraw(const C* p) {
-  if constexpr (Persist) return (uint32_t)__ldcg(p);
-  else return (uint32_t)__ldg(p);
+  if constexpr (Persist) {
+#if SGR_GATHER_CA
+    return (uint32_t)*p;
+#else
+    return (uint32_t)__ldcg(p);
+#endif
+  } else {
+    return (uint32_t)__ldg(p);
+  }
 }
 template <class C>
 __device__ __forceinline__ int32_t cval(uint32_t raw) {
