@@ -7,6 +7,8 @@ the fused path's worklists through their sizes and the final colors.
 """
 from __future__ import annotations
 
+import os
+
 import numpy as np
 import pytest
 
@@ -279,6 +281,19 @@ def test_full_size_configs_bit_exact(cfg):
     per-vertex loops; identical to the single-threaded oracle by construction)."""
     g = gen.config(cfg)
     check_full(g, LOW)
+
+
+@pytest.mark.slow
+@pytest.mark.skipif(os.environ.get("SGR_TEST_CFG5") != "1",
+                    reason="cfg5 (R-MAT s27, 2.1 G entries): ~10 min; set SGR_TEST_CFG5=1")
+def test_cfg5_full_size():
+    """BASELINE config 5 (R-MAT scale 27, nnz 2.13e9, int64 offsets) on one GPU against the
+    full oracle (OpenMP), plus the partitioned protocol on 2 partitions of the same device."""
+    g = gen.config(5)
+    res, ref = check_full(g, LOW)
+    rp, ci = dev(g)
+    part = sgr.color_partitioned(rp, ci, 2)
+    assert np.array_equal(part.colors.cpu().numpy(), ref.colors)
 
 
 # ----------------------------------------------------------------------------- multi-GPU path
