@@ -139,7 +139,8 @@ def oracle_run(g, tiebreak: int, edges_total: int | None, budget_s: float = 30.0
         return {"seconds": t_probe, "cores": cores, "sample": "full run", "result": probe}
     total = edges_total
     est = None if not total else t_probe * total / max(probe.edges_scanned, 1)
-    if est is not None and est <= budget_s:
+    # total unknown (reference arm, first step): run it in full once to learn it
+    if est is None or est <= budget_s:
         t0 = time.perf_counter()
         full = oracle.jacobi(g, tiebreak, nthreads=cores)
         return {"seconds": time.perf_counter() - t0, "cores": cores, "sample": "full run",
@@ -182,7 +183,7 @@ def run_reference(args):
     value = g.nnz / t / 1e9
     sample = "full oracle run per step" if res is not None else r["sample"]
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "GTEPS",
-            "n_gpus": 0, "steps": len(times), "warmup": args.warmup, "ms_per_step": t * 1e3,
+            "n_gpus": args.gpus, "device": "host cpu", "steps": len(times), "warmup": args.warmup, "ms_per_step": t * 1e3,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
             "dtype": "int32", "data": "synthetic",
             "config": {"workload": workload_name(args.config), "n": g.n, "nnz": g.nnz,
