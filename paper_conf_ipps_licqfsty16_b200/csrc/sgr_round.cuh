@@ -49,6 +49,12 @@ constexpr int kJB = 4 * kQB;  // entries per lane per batch
 #ifndef SGR_NO_TMA
 #define SGR_NO_TMA 0
 #endif
+#ifndef SGR_SLAYOUT
+#define SGR_SLAYOUT 1  // bin 2: lane-consecutive window slots (see bin2_trimmed)
+#endif
+#ifndef SGR_XPIPE
+#define SGR_XPIPE 0  // bin 2: next batch's gathers in flight while this batch is consumed
+#endif
 
 namespace sgr {
 
@@ -766,12 +772,52 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
     pc1 += (unsigned long long)(tb - ta);
 #endif
     const int4* b4 = reinterpret_cast<const int4*>(bufs + st * (kStage / 4));
+    (void)b4;
+    // live entries are compacted into the front of this stage as the batches go (a batch's
+    // outputs land below its own slots, whose ids every lane already holds in registers)
+    int32_t* sbuf = bufs + st * (kStage / 4);
     bool conf = false;
-    uint32_t lv = 0;  // live bits: bit kJB b + 4 qq + t
-    for (int bb = 0; bb < nb; ++bb) {
-      int32_t id[kJB];
-      uint32_t raw[kJB];
-      uint32_t okm = 0;
+    uint32_t lpos = 0;  // warp-uniform: live entries of the finished batches
+    const unsigned lt_mask = (1u << lane) - 1u;
+#if SGR_SLAYOUT
+    // batch bb: window slots 32 (kJB bb + j) + lane, j < kJB: consecutive lanes read
+    // consecutive (sorted) list entries, so neighbours close in id share a cache line
+    // within one gather instruction
+    auto fetch = [&](int bb, int32_t (&id)[kJB], uint32_t (&raw)[kJB], uint32_t& okm) {
+      okm = 0;
+#pragma unroll
+      for (int j = 0; j < kJB; ++j) {
+        const int32_t r = 32 * (kJB * bb + j) + lane;
+        id[j] = sbuf[r];
+        okm |= (r >= off0 && r < nslots) ? (1u << j) : 0u;
+      }
+#pragma unroll
+      for (int j = 0; j < kJB; ++j) raw[j] = ((okm >> j) & 1u) ? ldraw<Persist>(X + id[j]) : 0u;
+    };
+    auto consume = [&](const int32_t (&id)[kJB], const uint32_t (&raw)[kJB], uint32_t okm) {
+#pragma unroll
+      for (int j = 0; j < kJB; ++j) {
+        bool live = false;
+        if ((okm >> j) & 1u) {
+          // colors >= 1023 are clamped onto byte 1023; a first fit of 1023 or more is
+          // recomputed exactly from the full row (warp_first_fit_rescan)
+          const uint32_t ci = min(raw[j] & kColorMask, (uint32_t)(kBigTbl - 1));
+          live = (raw[j] >> kRoundShift) == klive;
+          set_add(tbl_all, ci);
+          if (!live) set_add(tbl_drop, ci);
+          conf |= (int32_t)(raw[j] & kColorMask) == xv && lose<TB>(v, id[j]);
+        }
+        // compaction in window order (the list stays sorted): a live entry's position is
+        // at most its own slot, and every lane already holds this batch's ids
+        const unsigned bal = __ballot_sync(0xffffffffu, live);
+        if (live) sbuf[lpos + __popc(bal & lt_mask)] = id[j];
+        lpos += (uint32_t)__popc(bal);
+      }
+    };
+#else
+    // batch bb: this lane's kJB window slots (kQB int4 of the stage) and their gathers
+    auto fetch = [&](int bb, int32_t (&id)[kJB], uint32_t (&raw)[kJB], uint32_t& okm) {
+      okm = 0;
 #pragma unroll
       for (int qq = 0; qq < kQB; ++qq) {
         const int q = kQB * bb + qq;
@@ -788,6 +834,9 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
       }
 #pragma unroll
       for (int j = 0; j < kJB; ++j) raw[j] = ((okm >> j) & 1u) ? ldraw<Persist>(X + id[j]) : 0u;
+    };
+    auto consume = [&](const int32_t (&id)[kJB], const uint32_t (&raw)[kJB], uint32_t okm) {
+      uint32_t lb = 0;  // live bits of this batch
 #pragma unroll
       for (int j = 0; j < kJB; ++j) {
         if ((okm >> j) & 1u) {
@@ -798,10 +847,51 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
           set_add(tbl_all, ci);
           if (!live) set_add(tbl_drop, ci);
           conf |= (int32_t)(raw[j] & kColorMask) == xv && lose<TB>(v, id[j]);
-          lv |= live ? (1u << (kJB * bb + j)) : 0u;
+          lb |= live ? (1u << j) : 0u;
         }
       }
+      // positions: lane-major within the batch (the list is a set; order is free). They
+      // land below the batch's own slots, never on a later batch's.
+      const uint32_t c8 = (uint32_t)__popc(lb);
+      uint32_t incl = c8;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t t = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += t;
+      }
+      uint32_t pos = lpos + incl - c8;
+#pragma unroll
+      for (int j = 0; j < kJB; ++j)
+        if ((lb >> j) & 1u) sbuf[pos++] = id[j];
+      lpos += __shfl_sync(0xffffffffu, incl, 31);
+    };
+#endif
+#if SGR_XPIPE
+    {  // the next batch's slots are read and its gathers issued before this batch is consumed
+      int32_t id[kJB], idn[kJB];
+      uint32_t raw[kJB], rawn[kJB];
+      uint32_t okm, okmn = 0;
+      fetch(0, id, raw, okm);
+      for (int bb = 0; bb < nb; ++bb) {
+        if (bb + 1 < nb) fetch(bb + 1, idn, rawn, okmn);
+        consume(id, raw, okm);
+#pragma unroll
+        for (int j = 0; j < kJB; ++j) {
+          id[j] = idn[j];
+          raw[j] = rawn[j];
+        }
+        okm = okmn;
+      }
     }
+#else
+    for (int bb = 0; bb < nb; ++bb) {
+      int32_t id[kJB];
+      uint32_t raw[kJB];
+      uint32_t okm;
+      fetch(bb, id, raw, okm);
+      consume(id, raw, okm);
+    }
+#endif
 #if !SGR_NO_TMA
     const long long tc = clock64();
     pc2 += (unsigned long long)(tc - tb);
@@ -812,32 +902,10 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
     }
     __syncwarp();
     const bool any = __any_sync(0xffffffffu, conf);
-    const uint32_t live_total = (uint32_t)__reduce_add_sync(0xffffffffu, (uint32_t)__popc(lv));
-    const int32_t* sbuf = bufs + st * (kStage / 4);
-    // compacted live list in window order (batch, int4 slot q, lane, t): positions from
-    // ballots — lane offset = live entries of lower lanes in the same q
-    const unsigned lt_mask = (1u << lane) - 1u;
+    const uint32_t live_total = lpos;
+    // the compacted live list (front of the stage) to global memory, coalesced
     auto write_live = [&](int32_t* base) {
-      uint32_t qb = 0;
-      for (int bb = 0; bb < nb; ++bb) {
-#pragma unroll
-        for (int qq = 0; qq < kQB; ++qq) {
-          const int sh = kJB * bb + 4 * qq;
-          uint32_t pre = 0, tot = 0;
-#pragma unroll
-          for (int t = 0; t < 4; ++t) {
-            const unsigned bal = __ballot_sync(0xffffffffu, (lv >> (sh + t)) & 1u);
-            pre += __popc(bal & lt_mask);
-            tot += __popc(bal);
-          }
-          uint32_t off = qb + pre;
-          const int32_t* sq = sbuf + 4 * (lane + 32 * (kQB * bb + qq));
-#pragma unroll
-          for (int t = 0; t < 4; ++t)
-            if ((lv >> (sh + t)) & 1u) base[off++] = sq[t];
-          qb += tot;
-        }
-      }
+      for (uint32_t q = lane; q < live_total; q += 32) base[q] = sbuf[q];
     };
 
     const int32_t slot = cur.slot;
@@ -940,38 +1008,70 @@ __device__ __forceinline__ void finalize_body(const RoundArgs<Packed>& a, int k)
   int64_t* out = sel(p ^ 1, a.wl_c[0], a.wl_c[1]);
   int32_t* len_cur = sel(p, a.len[0], a.len[1]);
   int32_t* len_nxt = sel(p ^ 1, a.len[0], a.len[1]);
-  for (int i = gw; i < nF; i += NW) {
-    const uint32_t f = (uint32_t)ld_cg(a.fin + i);
+  // 32 vertices per warp step, one per lane for the scalar work (loads, item pushes: one
+  // aggregated atomicAdd per counter per warp); the 1024-bit first fits go vertex by vertex
+  // across the warp, the next vertex's set words loaded while the current one is decided
+  for (int base = gw * 32; base < nF; base += NW * 32) {
+    const int i = base + lane;
+    const bool valid = i < nF;
+    const uint32_t f = valid ? (uint32_t)ld_cg(a.fin + i) : 0u;
     const int32_t v = (int32_t)(f & ~kBufBit);
-    const int32_t slot = __ldg(a.big_id + v);
-    uint32_t* accb = a.acc_bits + (int64_t)slot * 32;
-    const uint32_t word = ld_cg(accb + lane) | ld_cg(a.fixed + (int64_t)slot * 32 + lane) |
-                          (lane == 0 ? 1u : 0u);
-    const bool conf = (__ldcg(a.acc_cnt + slot) & 1ull) != 0ull;
-    accb[lane] = 0u;
-    int32_t tent = 0;
-    if (conf) {
-      tent = bits_first_free(word);
-      if (tent < 0 || tent >= kBigTbl - 1)  // beyond the exact range of the table
-        tent = warp_first_fit_rescan<Persist>(a.col_idx, X, ldg_i64(a.row_ptr + v),
-                                              ldg_i64(a.row_ptr + v + 1), kBigTbl - 1, lane);
+    const int32_t slot = valid ? __ldg(a.big_id + v) : 0;
+    const bool conf = valid && (__ldcg(a.acc_cnt + slot) & 1ull) != 0ull;
+    const uint32_t xraw = valid ? ldraw<Persist>(X + v) : 0u;
+    const int32_t nch2 = conf ? num_chunks(ld_cg(len_nxt + v)) : 0;
+    int32_t incl = nch2;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int32_t t = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += t;
     }
-    int32_t ob = 0, nch2 = 0;
+    const int32_t total = __shfl_sync(0xffffffffu, incl, 31);
+    const unsigned cm = __ballot_sync(0xffffffffu, conf);
+    const unsigned vm = __ballot_sync(0xffffffffu, valid);
+    int32_t ob = 0;
     if (lane == 0) {
-      a.acc_cnt[slot] = 0ull;
-      len_cur[v] = 0;  // consumed; the pass after next accumulates into it
-      Y[v] = conf ? cpack<C>(tent, k + 1, a) : cpack<C>(cval<C>(ldraw<Persist>(X + v)), k, a);
-      if (conf) {
-        nch2 = num_chunks(ld_cg(len_nxt + v));
-        ob = atomicAdd(&ctrl->ring[rs(k + 1)].c, nch2);
-        atomicAdd(&ctrl->ring[rs(k + 1)].cv, 1);
+      if (total) ob = atomicAdd(&ctrl->ring[rs(k + 1)].c, total);
+      if (cm) atomicAdd(&ctrl->ring[rs(k + 1)].cv, __popc(cm));
+    }
+    // per vertex j: merged set = partial sets of its chunks | fixed set | color 0
+    int32_t tent = 0;
+    unsigned rem = vm;
+    uint32_t wn = 0u;
+    int jn = -1;
+    if (rem) {
+      jn = __ffs(rem) - 1;
+      const int32_t sj = __shfl_sync(0xffffffffu, slot, jn);
+      wn = ld_cg(a.acc_bits + (int64_t)sj * 32 + lane) | ld_cg(a.fixed + (int64_t)sj * 32 + lane);
+    }
+    while (rem) {
+      const int j = jn;
+      const uint32_t word = wn | (lane == 0 ? 1u : 0u);
+      const int32_t sj = __shfl_sync(0xffffffffu, slot, j);
+      rem &= rem - 1u;
+      if (rem) {
+        jn = __ffs(rem) - 1;
+        const int32_t sn = __shfl_sync(0xffffffffu, slot, jn);
+        wn = ld_cg(a.acc_bits + (int64_t)sn * 32 + lane) | ld_cg(a.fixed + (int64_t)sn * 32 + lane);
+      }
+      a.acc_bits[(int64_t)sj * 32 + lane] = 0u;
+      if ((cm >> j) & 1u) {
+        int32_t t = bits_first_free(word);
+        if (t < 0 || t >= kBigTbl - 1) {  // beyond the exact range of the table
+          const int32_t vj = __shfl_sync(0xffffffffu, v, j);
+          t = warp_first_fit_rescan<Persist>(a.col_idx, X, ldg_i64(a.row_ptr + vj),
+                                             ldg_i64(a.row_ptr + vj + 1), kBigTbl - 1, lane);
+        }
+        if (lane == j) tent = t;
       }
     }
-    if (conf) {
-      ob = __shfl_sync(0xffffffffu, ob, 0);
-      nch2 = __shfl_sync(0xffffffffu, nch2, 0);
+    ob = __shfl_sync(0xffffffffu, ob, 0) + incl - nch2;
+    if (valid) {
+      a.acc_cnt[slot] = 0ull;
+      len_cur[v] = 0;  // consumed; the pass after next accumulates into it
+      Y[v] = conf ? cpack<C>(tent, k + 1, a) : cpack<C>(cval<C>(xraw), k, a);
       const uint32_t nbuf = (f & kBufBit) ? 0u : kBufBit;  // the list moved to the other buffer
-      for (int32_t t = lane; t < nch2; t += 32) out[ob + t] = make_item(v, (int32_t)(t | nbuf));
+      for (int32_t t = 0; t < nch2; ++t) out[ob + t] = make_item(v, (int32_t)(t | nbuf));
     }
   }
 }
