@@ -208,8 +208,9 @@ void fill_stats(const Ctrl& c, int64_t n, int64_t nnz, sgr_stats* st, int cb) {
   for (int q = 0; q < kBins; ++q) st->bin_warp_cycles[q] = (int64_t)c.bin_cycles[q];
   if (const char* env = getenv("SGR_PHASES")) {  // experiments: bin-2 phase breakdown
     (void)env;
-    fprintf(stderr, "sgr phases (warp-cycles): issue %llu wait %llu gather %llu post %llu\n",
-            c.phase_cycles[0], c.phase_cycles[1], c.phase_cycles[2], c.phase_cycles[3]);
+    fprintf(stderr, "sgr phases (warp-cycles): issue %llu wait %llu gather %llu post %llu | barrier %llu finalize %llu counters %llu\n",
+            c.phase_cycles[0], c.phase_cycles[1], c.phase_cycles[2], c.phase_cycles[3],
+            c.phase_cycles[4], c.phase_cycles[5], c.phase_cycles[6]);
   }
   st->rounds = c.k - 1;
   st->num_colors = c.max_color;

@@ -60,7 +60,7 @@ inline Layout layout(int64_t n, int64_t nnz, const Resolved& r) {
   }
   L.zero_end = o;  // accumulators, fixed sets and list lengths start at zero
   L.off_fin = o;
-  o += align_up((size_t)L.cap_big * 4, 256);
+  o += align_up((size_t)L.cap_big * 8, 256);
   if (L.packed) {
     L.off_adj = o;
     o += 2 * align_up((size_t)(nnz + 16) * 4, 256);
@@ -82,7 +82,7 @@ inline void build_args(RoundArgs<C>& a, const sgr_csr* csr, int64_t n, int64_t n
     a.col[0] = (C*)(b + L.off_col);
     a.col[1] = (C*)(b + L.off_col + align_up((size_t)n * sizeof(C), 256));
     a.fixed = (uint32_t*)(b + L.off_fixed);
-    a.fin = (int32_t*)(b + L.off_fin);
+    a.fin = (int64_t*)(b + L.off_fin);
     a.len[0] = (int32_t*)(b + L.off_len);
     a.len[1] = (int32_t*)(b + L.off_len + nb);
     const size_t ab = align_up((size_t)(nnz + 16) * 4, 256);

@@ -52,6 +52,9 @@ constexpr int kJB = 4 * kQB;  // entries per lane per batch
 #ifndef SGR_SLAYOUT
 #define SGR_SLAYOUT 1  // bin 2: lane-consecutive window slots (see bin2_trimmed)
 #endif
+#ifndef SGR_BIN0_THREAD
+#define SGR_BIN0_THREAD 0  // bin 0: one thread per vertex (else 4-lane groups)
+#endif
 #ifndef SGR_XPIPE
 #define SGR_XPIPE 0  // bin 2: next batch's gathers in flight while this batch is consumed
 #endif
@@ -162,7 +165,8 @@ struct Ctrl {
   unsigned long long items_total;
   unsigned long long list_writes_total;   // compacted list entries written (bin 2, packed)
   unsigned long long bin_cycles[kBins];   // warp-cycles spent in each bin (SM clock)
-  unsigned long long phase_cycles[4];     // bin 2 (trimmed) phases: issue, wait, gather, post
+  unsigned long long phase_cycles[8];     // bin 2 (trimmed) phases: issue, wait, gather, post;
+                                          // [4] grid barriers, [5] finalize, [6] counters
   int32_t* round_sizes;
   int64_t* round_edges;
   int64_t* round_ns;          // %globaltimer at the end of each pass (profiling)
@@ -182,7 +186,8 @@ struct RoundArgs {
   int32_t* adj[2];            // trimmed adjacency lists (packed mode), offsets = row_ptr
   int32_t* len[2];            // [v] list length for the pass of parity p
   uint32_t* fixed;            // [slot][32] colors of dropped (finalized) neighbours
-  int32_t* fin;               // finalize list: multi-chunk vertices of the pass (v | buf << 31)
+  int64_t* fin;               // finalize list: multi-chunk vertices of the pass
+                              // (slot << 32 | buf << 31 | v)
   Ctrl* ctrl;
   int64_t nnz;
   int32_t n;
@@ -335,6 +340,10 @@ __device__ __forceinline__ int32_t ld_row(const int32_t* p) {
 #else
   return __ldg(p);
 #endif
+}
+__device__ __forceinline__ int4 ld_row4(const int4* p) { return __ldg(p); }
+__device__ __forceinline__ void prefetch_l1(const void* p) {
+  asm volatile("prefetch.global.L1 [%0];" ::"l"(p));
 }
 __device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
   uint32_t done;
@@ -959,7 +968,8 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
       lbase = __shfl_sync(0xffffffffu, lbase, 0);
       write_live(lst_other + cur.s + lbase);
       lwrites += live_total;
-      if (lane == 0 && cur.c == 0) a.fin[fpos] = (int32_t)((uint32_t)v | (cur.buf ? kBufBit : 0u));
+      if (lane == 0 && cur.c == 0)
+        a.fin[fpos] = (int64_t)(((uint64_t)(uint32_t)slot << 32) | (uint32_t)v | (cur.buf ? kBufBit : 0u));
     }
     set_clear(tbl_all, kTblBytes, lane, 32);  // both sets
     __syncwarp();
@@ -1008,18 +1018,44 @@ __device__ __forceinline__ void finalize_body(const RoundArgs<Packed>& a, int k)
   int64_t* out = sel(p ^ 1, a.wl_c[0], a.wl_c[1]);
   int32_t* len_cur = sel(p, a.len[0], a.len[1]);
   int32_t* len_nxt = sel(p ^ 1, a.len[0], a.len[1]);
-  // 32 vertices per warp step, one per lane for the scalar work (loads, item pushes: one
-  // aggregated atomicAdd per counter per warp); the 1024-bit first fits go vertex by vertex
-  // across the warp, the next vertex's set words loaded while the current one is decided
-  for (int base = gw * 32; base < nF; base += NW * 32) {
+  // B <= 32 vertices per warp (spread over every warp of the grid), one per lane: its
+  // conflict flag, its two 1024-bit sets (partial sets of its chunks, fixed set) as 16
+  // vector loads issued together, first fit by a scan of the merged words, item pushes with
+  // one aggregated atomicAdd per counter per warp
+  const int B = min(32, (nF + NW - 1) / NW);
+  for (int base = gw * B; base < nF; base += NW * B) {
     const int i = base + lane;
-    const bool valid = i < nF;
-    const uint32_t f = valid ? (uint32_t)ld_cg(a.fin + i) : 0u;
-    const int32_t v = (int32_t)(f & ~kBufBit);
-    const int32_t slot = valid ? __ldg(a.big_id + v) : 0;
-    const bool conf = valid && (__ldcg(a.acc_cnt + slot) & 1ull) != 0ull;
-    const uint32_t xraw = valid ? ldraw<Persist>(X + v) : 0u;
-    const int32_t nch2 = conf ? num_chunks(ld_cg(len_nxt + v)) : 0;
+    const bool valid = lane < B && i < nF;
+    const uint64_t f = valid ? (uint64_t)__ldcg(a.fin + i) : 0ull;
+    const int32_t v = (int32_t)((uint32_t)f & ~kBufBit);
+    const int32_t slot = (int32_t)(f >> 32);
+    bool conf = false;
+    int32_t nch2 = 0, tent = -1;
+    uint32_t xraw = 0u;
+    uint4* accb = reinterpret_cast<uint4*>(a.acc_bits + (int64_t)slot * 32);
+    if (valid) {
+      const uint4* fxb = reinterpret_cast<const uint4*>(a.fixed + (int64_t)slot * 32);
+      uint4 m[8];
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        const uint4 x = __ldcg(accb + q), y = __ldcg(fxb + q);
+        m[q] = make_uint4(x.x | y.x, x.y | y.y, x.z | y.z, x.w | y.w);
+      }
+      conf = (__ldcg(a.acc_cnt + slot) & 1ull) != 0ull;
+      xraw = ldraw<Persist>(X + v);
+      const int32_t ln = ld_cg(len_nxt + v);
+      nch2 = conf ? num_chunks(ln) : 0;
+      m[0].x |= 1u;  // color 0
+#pragma unroll
+      for (int q = 7; q >= 0; --q) {  // lowest word with a zero bit
+        const uint32_t w4[4] = {m[q].x, m[q].y, m[q].z, m[q].w};
+#pragma unroll
+        for (int t = 3; t >= 0; --t)
+          if (w4[t] != 0xffffffffu) tent = 32 * (4 * q + t) + __ffs(~w4[t]) - 1;
+      }
+#pragma unroll
+      for (int q = 0; q < 8; ++q) accb[q] = make_uint4(0u, 0u, 0u, 0u);
+    }
     int32_t incl = nch2;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
@@ -1028,49 +1064,27 @@ __device__ __forceinline__ void finalize_body(const RoundArgs<Packed>& a, int k)
     }
     const int32_t total = __shfl_sync(0xffffffffu, incl, 31);
     const unsigned cm = __ballot_sync(0xffffffffu, conf);
-    const unsigned vm = __ballot_sync(0xffffffffu, valid);
     int32_t ob = 0;
     if (lane == 0) {
       if (total) ob = atomicAdd(&ctrl->ring[rs(k + 1)].c, total);
       if (cm) atomicAdd(&ctrl->ring[rs(k + 1)].cv, __popc(cm));
     }
-    // per vertex j: merged set = partial sets of its chunks | fixed set | color 0
-    int32_t tent = 0;
-    unsigned rem = vm;
-    uint32_t wn = 0u;
-    int jn = -1;
-    if (rem) {
-      jn = __ffs(rem) - 1;
-      const int32_t sj = __shfl_sync(0xffffffffu, slot, jn);
-      wn = ld_cg(a.acc_bits + (int64_t)sj * 32 + lane) | ld_cg(a.fixed + (int64_t)sj * 32 + lane);
-    }
-    while (rem) {
-      const int j = jn;
-      const uint32_t word = wn | (lane == 0 ? 1u : 0u);
-      const int32_t sj = __shfl_sync(0xffffffffu, slot, j);
-      rem &= rem - 1u;
-      if (rem) {
-        jn = __ffs(rem) - 1;
-        const int32_t sn = __shfl_sync(0xffffffffu, slot, jn);
-        wn = ld_cg(a.acc_bits + (int64_t)sn * 32 + lane) | ld_cg(a.fixed + (int64_t)sn * 32 + lane);
-      }
-      a.acc_bits[(int64_t)sj * 32 + lane] = 0u;
-      if ((cm >> j) & 1u) {
-        int32_t t = bits_first_free(word);
-        if (t < 0 || t >= kBigTbl - 1) {  // beyond the exact range of the table
-          const int32_t vj = __shfl_sync(0xffffffffu, v, j);
-          t = warp_first_fit_rescan<Persist>(a.col_idx, X, ldg_i64(a.row_ptr + vj),
-                                             ldg_i64(a.row_ptr + vj + 1), kBigTbl - 1, lane);
-        }
-        if (lane == j) tent = t;
-      }
+    // first fits beyond the exact range of the table: warp rescans of the full rows (rare)
+    unsigned rm = __ballot_sync(0xffffffffu, conf && (tent < 0 || tent >= kBigTbl - 1));
+    while (rm) {
+      const int j = __ffs(rm) - 1;
+      rm &= rm - 1u;
+      const int32_t vj = __shfl_sync(0xffffffffu, v, j);
+      const int32_t t = warp_first_fit_rescan<Persist>(a.col_idx, X, ldg_i64(a.row_ptr + vj),
+                                                       ldg_i64(a.row_ptr + vj + 1), kBigTbl - 1, lane);
+      if (lane == j) tent = t;
     }
     ob = __shfl_sync(0xffffffffu, ob, 0) + incl - nch2;
     if (valid) {
       a.acc_cnt[slot] = 0ull;
       len_cur[v] = 0;  // consumed; the pass after next accumulates into it
       Y[v] = conf ? cpack<C>(tent, k + 1, a) : cpack<C>(cval<C>(xraw), k, a);
-      const uint32_t nbuf = (f & kBufBit) ? 0u : kBufBit;  // the list moved to the other buffer
+      const uint32_t nbuf = ((uint32_t)f & kBufBit) ? 0u : kBufBit;  // the list moved buffers
       for (int32_t t = 0; t < nch2; ++t) out[ob + t] = make_item(v, (int32_t)(t | nbuf));
     }
   }
@@ -1247,6 +1261,88 @@ __device__ __forceinline__ void bin0(const RoundArgs<C>& a, int k, const int32_t
   push_flush(pbuf, pending, out, out_cnt, lane);
 }
 
+// Bin 0, one thread per vertex (SGR_BIN0_THREAD): lane L of the warp takes list position
+// 32 step + L. Its row (<= 32 entries) is read as <= 9 int4 of the 16-byte-aligned window,
+// then every entry's color is gathered at once (<= 32 loads in flight per lane, 1024 per
+// warp), and mask / first fit / conflict are per-lane register work (no shuffles). When the
+// worklist is ordered (stencils), the 32 lanes' j-th neighbours are 32 consecutive ids: one
+// cache line per gather instruction. The next step's list entry and row offsets are
+// prefetched, its row warmed into L1.
+template <int TB, bool Persist, class C, bool Hub>
+__device__ __forceinline__ void bin0_thread(const RoundArgs<C>& a, int k, const int32_t* list,
+                                            int nX, int32_t* out, int32_t* out_cnt, const C* X,
+                                            C* Y, uint8_t* wsm, int gw, int NW, int lane,
+                                            unsigned long long& edges,
+                                            unsigned long long& entries) {
+  constexpr int kQ = 9;  // int4 per window: offset <= 3 + 32 entries
+  if (gw * 32 >= nX) return;
+  int32_t* pbuf = reinterpret_cast<int32_t*>(wsm + WarpSmem<C, Hub>::kPush);
+  int pending = 0;
+  const int step = NW * 32;
+  int i = gw * 32 + lane;
+  int32_t v = i < nX ? ld_cg(list + i) : -1;
+  int64_t s = v >= 0 ? ldg_i64(a.row_ptr + v) : 0, e = v >= 0 ? ldg_i64(a.row_ptr + v + 1) : 0;
+  for (int base = gw * 32; base < nX; base += step) {
+    const int in = i + step;
+    const int32_t vn = in < nX ? ld_cg(list + in) : -1;
+    const int32_t xv = v >= 0 ? ldc<Persist>(X + v) : 0;
+    const int64_t w0 = s & ~(int64_t)3;
+    const int32_t off = (int32_t)(s - w0), cnt = (int32_t)(e - s);
+    const int32_t nq = (off + cnt + 3) >> 2;
+    int32_t id[4 * kQ];
+    const int4* win = reinterpret_cast<const int4*>(a.col_idx + w0);
+#pragma unroll
+    for (int q = 0; q < kQ; ++q) {
+      int4 t = make_int4(0, 0, 0, 0);
+      if (q < nq) {
+        if (w0 + 4 * q + 4 <= a.nnz) {
+          t = ld_row4(win + q);
+        } else {  // the array's last, partial 16-byte group: never read past nnz
+          const int64_t p0 = w0 + 4 * q;
+          t.x = ld_row(a.col_idx + p0);
+          if (p0 + 1 < a.nnz) t.y = ld_row(a.col_idx + p0 + 1);
+          if (p0 + 2 < a.nnz) t.z = ld_row(a.col_idx + p0 + 2);
+        }
+      }
+      id[4 * q + 0] = t.x;
+      id[4 * q + 1] = t.y;
+      id[4 * q + 2] = t.z;
+      id[4 * q + 3] = t.w;
+    }
+    // valid slots [off, off + cnt) of the window
+    const uint64_t vm = cnt > 0 ? (((cnt >= 64 ? ~0ull : ((1ull << cnt) - 1ull))) << off) : 0ull;
+    uint64_t lb = 0;
+#pragma unroll
+    for (int r = 0; r < 4 * kQ; ++r)
+      lb |= (((vm >> r) & 1ull) && lose<TB>(v, id[r])) ? (1ull << r) : 0ull;
+    int32_t c[4 * kQ];
+#pragma unroll
+    for (int r = 0; r < 4 * kQ; ++r) c[r] = ((vm >> r) & 1ull) ? ldc<Persist>(X + id[r]) : 0;
+    const int64_t sn = vn >= 0 ? ldg_i64(a.row_ptr + vn) : 0;
+    const int64_t en = vn >= 0 ? ldg_i64(a.row_ptr + vn + 1) : 0;
+    bool conf = false;
+    uint32_t mask = 0;  // bit i = color i + 1 present (deg <= 32 => first fit <= 33)
+#pragma unroll
+    for (int r = 0; r < 4 * kQ; ++r) {
+      mask |= ((uint32_t)(c[r] - 1) < 32u) ? (1u << (c[r] - 1)) : 0u;
+      conf |= (c[r] == xv) & (((lb >> r) & 1ull) != 0ull);
+    }
+    if (v >= 0) {
+      const int32_t tent = ~mask ? __ffs(~mask) : 33;
+      Y[v] = conf ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a);
+      edges += (unsigned long long)cnt;
+      entries += (unsigned long long)cnt;
+    }
+    push_buffered(v >= 0 && conf, v, pbuf, pending, out, out_cnt, lane);
+    if (en > sn) prefetch_l1(a.col_idx + sn);
+    i = in;
+    v = vn;
+    s = sn;
+    e = en;
+  }
+  push_flush(pbuf, pending, out, out_cnt, lane);
+}
+
 // Bins 0/1 driver: warp w takes list positions 4w + g, 4(w + NW) + g, ... (g = group); the
 // next position's list entry and row offsets are prefetched, its row warmed into L2.
 template <int TB, bool Persist, class C, bool Hub>
@@ -1343,7 +1439,11 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, const C
   long long t2 = clock64();
   cyc[1] += (unsigned long long)(t2 - t1);
   // ---- bin 0: eight vertices per warp, register masks
+#if SGR_BIN0_THREAD
+  bin0_thread<TB, Persist, C, Hub>(
+#else
   bin0<TB, Persist, C, Hub>(
+#endif
       a, k, sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]),
       w.t, sel(p ^ 1, a.wl_t[0], a.wl_t[1]), &ctrl->ring[rs(k + 1)].t, X, Y,
       wsm, gw, NW, lane, edges[0], entries[0]);
@@ -1628,6 +1728,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks<C, Hub>) k_persistent(Round
   uint8_t* wsm = warp_smem_init<C, Hub>(dsmem);
   uint32_t ph = 0;  // mbarrier phase bits of the warp's two TMA stages
   unsigned long long cyc[kBins] = {0, 0, 0};
+  unsigned long long pcx[3] = {0, 0, 0};  // barrier waits, finalize, counter reduction
   const int max_rounds = ld_cg(&ctrl->max_rounds);
   const bool leader = blockIdx.x == 0 && threadIdx.x == 0;
   int k = 2;
@@ -1646,15 +1747,28 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks<C, Hub>) k_persistent(Round
     }
     unsigned long long edges[kBins] = {0, 0, 0}, entries[kBins] = {0, 0, 0};
     round_body<TB, true, C, Hub>(a, k, w, wsm, edges, entries, ph, cyc);
+    const long long t0 = clock64();
     block_add6(edges, entries, ctrl, k);
+    const long long t1 = clock64();
+    pcx[2] += (unsigned long long)(t1 - t0);
     if constexpr (packed<C>() && Hub) {  // multi-chunk vertices: decided once all chunks are in
       grid_sync(ctrl);
+      const long long t2 = clock64();
       finalize_body<TB, true>(a, k);
+      const long long t3 = clock64();
+      pcx[0] += (unsigned long long)(t2 - t1);
+      pcx[1] += (unsigned long long)(t3 - t2);
+      grid_sync(ctrl);
+      pcx[0] += (unsigned long long)(clock64() - t3);
+    } else {
+      grid_sync(ctrl);
+      pcx[0] += (unsigned long long)(clock64() - t1);
     }
-    grid_sync(ctrl);
   }
-  if ((threadIdx.x & 31) == 0)
+  if ((threadIdx.x & 31) == 0) {
     for (int q = 0; q < kBins; ++q) atomicAdd(&ctrl->bin_cycles[q], cyc[q]);
+    for (int q = 0; q < 3; ++q) atomicAdd(&ctrl->phase_cycles[4 + q], pcx[q]);
+  }
 }
 
 // Final colors (packed words) into the caller's int32 output, and their maximum.
