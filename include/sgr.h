@@ -151,6 +151,17 @@ sgr_status sgr_color_host(const int64_t* row_ptr, const int32_t* col_idx, int64_
                           int64_t nnz, int32_t* colors_out, sgr_stats* stats,
                           const sgr_opts* opts);
 
+/* Topology-driven mapping of the same method: the paper's Algorithm 4 (T-base,
+ * P:194-196) under the Jacobi reading. Every iteration visits all n vertices, one thread
+ * per vertex: the uncolored ones take a first fit against the iteration's snapshot, then
+ * every vertex is checked for a conflict (Alg. 4 l.15-21) and the host reads the `changed`
+ * count (l.22). Same contract, same result (colors, rounds, |W_r|) as sgr_color; slower by
+ * design (it rescans V every iteration) — the comparison the paper makes against Alg. 5.
+ * Uses opts->tiebreak, max_rounds, stream and round_sizes/round_cap (|W_r| per iteration);
+ * device scratch from the stream-ordered allocator; synchronizes the stream. */
+sgr_status sgr_color_topo(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* colors_out,
+                          sgr_stats* stats, const sgr_opts* opts);
+
 /* ---- one-round step entry points: Algorithm 5 split line by line (all device pointers,
  * asynchronous on opts->stream; opts may be NULL) ---------------------------------------- */
 

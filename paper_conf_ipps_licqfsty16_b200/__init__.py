@@ -26,7 +26,7 @@ from ._lib import Csr, Opts, Stats, check, load
 TIEBREAK = {"lowid": 0, "lowid_keeps": 0, "paper": 1}
 LOOP = {"auto": 0, "graph": 1, "persistent": 2, "host": 3}
 
-__all__ = ["color", "color_host", "color_partitioned", "color_dist", "assign", "commit",
+__all__ = ["color", "color_host", "color_topo", "color_partitioned", "color_dist", "assign", "commit",
            "detect", "compact", "validate_csr", "partition", "workspace_bytes", "gen",
            "ColorResult", "TIEBREAK"]
 
@@ -136,6 +136,29 @@ def color(row_ptr, col_idx, tiebreak="lowid", *, out=None, stream=None, trace=Fa
         res.round_sizes = rs[:R].cpu().numpy()
         res.round_edges = re[:R].cpu().numpy()
         res.extra["round_ms"] = rms[:R]
+    return res
+
+
+def color_topo(row_ptr, col_idx, tiebreak="lowid", *, out=None, stream=None, trace=False,
+               **opt_kw) -> ColorResult:
+    """Topology-driven mapping (the paper's Algorithm 4, T-base): every iteration visits all
+    vertices, one thread each, and the host reads the `changed` count. Same result as
+    color() (colors, rounds, |W_r|); the comparison mapping, not the fast path."""
+    torch = _torch()
+    _check_csr(row_ptr, col_idx)
+    n = row_ptr.numel() - 1
+    nnz = col_idx.numel()
+    colors = out if out is not None else torch.empty(n, dtype=torch.int32, device=row_ptr.device)
+    _require_cuda(colors)
+    rs = torch.zeros(n + 2, dtype=torch.int32, device=row_ptr.device) if trace else None
+    opts = make_opts(tiebreak, stream, round_sizes=rs, round_cap=(n + 2) if trace else 0, **opt_kw)
+    csr = Csr(row_ptr.data_ptr(), col_idx.data_ptr() if nnz else None)
+    st = Stats()
+    check(load().sgr_color_topo(ctypes.byref(csr), n, nnz, colors.data_ptr() if n else None,
+                                ctypes.byref(st), ctypes.byref(opts)), "sgr_color_topo")
+    res = ColorResult(colors, st.as_dict())
+    if trace:
+        res.round_sizes = rs[:res.stats["rounds"]].cpu().numpy()
     return res
 
 

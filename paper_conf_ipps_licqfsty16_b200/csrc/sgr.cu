@@ -14,6 +14,7 @@
 #include "sgr_host.cuh"
 #include "sgr_round.cuh"
 #include "sgr_step.cuh"
+#include "sgr_topo.cuh"
 
 namespace sgr {
 
@@ -546,6 +547,113 @@ sgr_status sgr_color_host(const int64_t* row_ptr, const int32_t* col_idx, int64_
   cudaFreeAsync(d_col, s);
   CK(cudaStreamSynchronize(s));
   return st;
+}
+
+// ----- topology-driven mapping (Algorithm 4; sgr_topo.cuh) -------------------
+sgr_status sgr_color_topo(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* colors_out,
+                          sgr_stats* stats, const sgr_opts* opts) {
+  if (!csr || n < 0 || nnz < 0 || n >= ((int64_t)1 << 31)) {
+    set_error("sgr_color_topo: invalid sizes or csr");
+    return SGR_EINVAL;
+  }
+  if (stats) memset(stats, 0, sizeof(*stats));
+  if (n == 0) return SGR_OK;
+  if (!csr->row_ptr || !colors_out || (nnz > 0 && !csr->col_idx)) {
+    set_error("sgr_color_topo: null pointer");
+    return SGR_EINVAL;
+  }
+  const Resolved r = resolve_opts(opts, n);
+  cudaStream_t s = r.stream;
+  keep_pool_memory();
+  // workspace: flag[n] | T[n] | changed | edges
+  const size_t nb = align_up((size_t)n * 4, 256);
+  char* ws = nullptr;
+  CK(cudaMallocAsync((void**)&ws, 2 * nb + 256, s));
+  int32_t* flag = (int32_t*)ws;
+  int32_t* buf[2] = {colors_out, (int32_t*)(ws + nb)};
+  int32_t* changed = (int32_t*)(ws + 2 * nb);
+  unsigned long long* edges = (unsigned long long*)(ws + 2 * nb + 64);
+  int32_t* hcnt = nullptr;
+  CK(cudaMallocHost((void**)&hcnt, sizeof(int32_t)));
+  cudaEvent_t e0, e1;
+  CK(cudaEventCreate(&e0));
+  CK(cudaEventCreate(&e1));
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, (int64_t)num_sms() * 16));
+  std::vector<int32_t> sizes;
+  sgr_status status = SGR_OK;
+  int launches = 0;
+  CK(cudaMemsetAsync(edges, 0, 8, s));
+  CK(cudaEventRecord(e0, s));
+  k_topo_init<<<grid, 256, 0, s>>>(n, flag, buf[0]);
+  ++launches;
+  int32_t cnt = (int32_t)n;  // |W_1| = n
+  int32_t rr = 1;
+  int cur = 0;
+  while (cnt > 0) {
+    if (rr > r.max_rounds) {
+      status = SGR_ENOCONV;
+      set_error("sgr_color_topo: max_rounds reached");
+      break;
+    }
+    sizes.push_back(cnt);
+    k_topo_assign<<<grid, 256, 0, s>>>(csr->row_ptr, csr->col_idx, n, rr, flag, buf[cur],
+                                       buf[cur ^ 1], edges);
+    CK(cudaMemsetAsync(changed, 0, 4, s));
+    if (r.tiebreak)
+      k_topo_detect<1><<<grid, 256, 0, s>>>(csr->row_ptr, csr->col_idx, n, rr, buf[cur ^ 1], flag, changed);
+    else
+      k_topo_detect<0><<<grid, 256, 0, s>>>(csr->row_ptr, csr->col_idx, n, rr, buf[cur ^ 1], flag, changed);
+    launches += 2;
+    CK(cudaGetLastError());
+    // the host reads `changed` every iteration (Alg. 4 l.22)
+    CK(cudaMemcpyAsync(hcnt, changed, 4, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    cnt = *hcnt;
+    cur ^= 1;
+    ++rr;
+  }
+  if (cur == 1)
+    CK(cudaMemcpyAsync(colors_out, buf[1], (size_t)n * 4, cudaMemcpyDeviceToDevice, s));
+  int32_t* dmax = changed;
+  CK(cudaMemsetAsync(dmax, 0, 4, s));
+  k_max_color<<<grid, 256, 0, s>>>(colors_out, n, dmax);
+  launches += 1;
+  CK(cudaEventRecord(e1, s));
+  int32_t mx = 0;
+  unsigned long long ed = 0;
+  CK(cudaMemcpyAsync(&mx, dmax, 4, cudaMemcpyDeviceToHost, s));
+  CK(cudaMemcpyAsync(&ed, edges, 8, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  const int32_t R = (int32_t)sizes.size();
+  if (r.round_sizes && r.round_cap > 0)
+    CK(cudaMemcpy(r.round_sizes, sizes.data(), (size_t)std::min(R, r.round_cap) * 4,
+                  cudaMemcpyHostToDevice));
+  if (stats) {
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, e0, e1);
+    stats->rounds = R;
+    stats->num_colors = mx;
+    int64_t vp = 0;
+    for (int32_t x : sizes) vp += x;
+    stats->vertices_processed = vp;
+    stats->edges_scanned = (int64_t)ed;
+    stats->entries_read = (int64_t)ed;
+    stats->elapsed_ms = ms;
+    stats->launches = launches;
+    stats->color_bits = 32;
+    // per iteration: every vertex's flag and X/T word, plus the detection pass over V
+    // (row pair, own color, every row entry and its color); the assignment of W_r reads
+    // its rows and their colors
+    stats->bytes_algorithmic = (int64_t)R * ((int64_t)n * (4 + 4 + 4 + 16 + 4) + nnz * 8) +
+                               (int64_t)ed * 8;
+    stats->grid_blocks = grid;
+  }
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  cudaFreeHost(hcnt);
+  cudaFreeAsync(ws, s);
+  cudaStreamSynchronize(s);
+  return status;
 }
 
 // ----- step entry points ------------------------------------------------------------------

@@ -362,3 +362,49 @@ def test_nccl_world1_color_dist():
         comm.close()
     finally:
         dist.destroy_process_group()
+
+
+# ------------------------------------------- topology-driven mapping (Algorithm 4, T-base)
+def check_topo(g, tb):
+    rp, ci = dev(g)
+    res = sgr.color_topo(rp, ci, RULE[tb], trace=True)
+    ref = oracle.jacobi(g, tb, nthreads=oracle.max_threads())
+    assert res.stats["rounds"] == ref.rounds, (g.name, res.stats["rounds"], ref.rounds)
+    assert np.array_equal(res.colors.cpu().numpy(), ref.colors), g.name
+    assert np.array_equal(res.round_sizes, ref.round_sizes), g.name
+    assert res.stats["num_colors"] == ref.num_colors
+    assert res.stats["vertices_processed"] == ref.vertices_processed
+    assert res.stats["edges_scanned"] == ref.edges_scanned
+    return res
+
+
+@pytest.mark.parametrize("seed", range(24))
+@pytest.mark.parametrize("tb", [LOW, PAP])
+def test_topology_driven_random_graphs(seed, tb):
+    check_topo(random_graph(seed), tb)
+
+
+@pytest.mark.parametrize("maker", [
+    lambda: gen.config(1),
+    lambda: gen.stencil3d(20, 20, 20, 27),
+    lambda: gen.er(1 << 14, 8 << 14, seed=5),
+    lambda: gen.rmat(14, 10, 0.45, 0.15, 0.15, seed=2),
+], ids=["cfg1", "s27-20", "er14", "rmat-g14"])
+@pytest.mark.parametrize("tb", [LOW, PAP])
+def test_topology_driven_families(maker, tb):
+    check_topo(maker(), tb)
+
+
+def test_topology_driven_equals_data_driven_and_edge_cases():
+    g = gen.rmat(16, 8, 0.57, 0.19, 0.19, seed=9)
+    rp, ci = dev(g)
+    a = sgr.color(rp, ci).colors
+    b = sgr.color_topo(rp, ci).colors
+    assert torch.equal(a, b)
+    # self-loops and duplicates (readings C7, C9), n = 1 with a loop, nnz = 0
+    r2 = raw_csr(4, [(0, 0), (0, 1), (0, 1), (1, 0), (1, 2), (2, 1), (2, 3), (3, 2), (3, 3)])
+    res = check_topo(r2, LOW)
+    assert res.stats["rounds"] >= 1
+    z = gen.from_edges(5, np.zeros((0, 2), np.int64))
+    res = sgr.color_topo(*dev(z))
+    assert res.colors.cpu().tolist() == [1] * 5 and res.stats["rounds"] == 1
