@@ -35,7 +35,8 @@ def parse():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", type=int, default=4, help="BASELINE.json config (1-based)")
+    ap.add_argument("--config", type=int, default=4,
+                    help="BASELINE.json config (1-based); 6-8: extra workloads (gen.config)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--tiebreak", default="lowid", choices=["lowid", "paper"])
     ap.add_argument("--no-cpu-baseline", action="store_true")

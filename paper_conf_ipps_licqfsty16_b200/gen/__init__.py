@@ -182,6 +182,13 @@ def config(idx: int) -> Graph:
         return rmat(24, 8, 0.57, 0.19, 0.19, seed=4)
     if idx == 5:
         return rmat(27, 8, 0.57, 0.19, 0.19, seed=5)
+    # extra workloads beyond BASELINE.json
+    if idx == 6:  # Table I rmat-er: R-MAT (.25,.25,.25,.25), 2^20 vertices, edge factor 10
+        return rmat(20, 10, 0.25, 0.25, 0.25, seed=6)
+    if idx == 7:  # Table I rmat-g: R-MAT (.45,.15,.15,.25), 2^20 vertices, edge factor 10
+        return rmat(20, 10, 0.45, 0.15, 0.15, seed=7)
+    if idx == 8:  # cfg4 with Graph500-style relabeling ("--permute")
+        return rmat(24, 8, 0.57, 0.19, 0.19, seed=4, permute=True)
     raise ValueError(idx)
 
 
@@ -191,4 +198,7 @@ CONFIG_NAMES = {
     3: "er-n2^24-pairs8n seed 3",
     4: "rmat-s24-ef8 (a=.57,b=c=.19) seed 4",
     5: "rmat-s27-ef8 (a=.57,b=c=.19) seed 5",
+    6: "rmat-er-s20-ef10 (a=b=c=.25, Table I) seed 6",
+    7: "rmat-g-s20-ef10 (a=.45,b=c=.15, Table I) seed 7",
+    8: "rmat-s24-ef8 (a=.57,b=c=.19) seed 4, permuted",
 }

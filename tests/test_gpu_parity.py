@@ -274,9 +274,10 @@ def test_compact_large_ragged():
 
 # ----------------------------------------------------------------------------- full size
 @pytest.mark.slow
-@pytest.mark.parametrize("cfg", [2, 3, 4])
+@pytest.mark.parametrize("cfg", [2, 3, 4, 6, 7, 8])
 def test_full_size_configs_bit_exact(cfg):
-    """BASELINE.json configs 2-4 at full size, in the launch configuration bench.py times
+    """BASELINE.json configs 2-4 and the extra workloads 6-8 (Table I shapes, permuted cfg4)
+    at full size, in the launch configuration bench.py times
     (default options), against the full oracle (OpenMP over each round's independent
     per-vertex loops; identical to the single-threaded oracle by construction)."""
     g = gen.config(cfg)
