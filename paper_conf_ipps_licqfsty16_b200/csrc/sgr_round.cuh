@@ -52,6 +52,15 @@ constexpr int kJB = 4 * kQB;  // entries per lane per batch
 #ifndef SGR_SLAYOUT
 #define SGR_SLAYOUT 1  // bin 2: lane-consecutive window slots (see bin2_trimmed)
 #endif
+#ifndef SGR_BAR2
+#define SGR_BAR2 1  // grid barrier on a monotonic arrival counter (no reset/release step)
+#endif
+#ifndef SGR_BIN1_PIPE
+#define SGR_BIN1_PIPE 0  // bin 1: flattened (vertex, batch) steps, next row in flight
+#endif
+#ifndef SGR_ROWPF
+#define SGR_ROWPF 0  // bin 0: prefetch the row two steps ahead (1 = into L2, 2 = into L1)
+#endif
 #ifndef SGR_BIN0_THREAD
 #define SGR_BIN0_THREAD 0  // bin 0: one thread per vertex (else 4-lane groups)
 #endif
@@ -1248,6 +1257,15 @@ __device__ __forceinline__ void bin0(const RoundArgs<C>& a, int k, const int32_t
     push_buffered(v >= 0 && any && gl == 0, v, pbuf, pending, out, out_cnt, lane);
     const int64_t s2 = v2 >= 0 ? ldg_i64(a.row_ptr + v2) : 0;
     const int64_t e2 = v2 >= 0 ? ldg_i64(a.row_ptr + v2 + 1) : 0;
+#if SGR_ROWPF
+    {  // warm the row two steps ahead (<= 128 bytes: its first and last line)
+      const int32_t* pf = gl == 0 ? a.col_idx + s2 : a.col_idx + e2 - 1;
+      if (gl < 2 && e2 > s2) {
+        if (SGR_ROWPF == 1) prefetch_l2(pf);
+        else prefetch_l1(pf);
+      }
+    }
+#endif
     i += step;
     v = v1;
     s = s1;
@@ -1377,6 +1395,117 @@ __device__ __forceinline__ void bin1(const RoundArgs<C>& a, int k, const int32_t
   push_flush(pbuf, pending, out, out_cnt, lane);
 }
 
+// Bin 1, software-pipelined (SGR_BIN1_PIPE): every 8-lane group walks a flattened stream of
+// (vertex, 64-entry batch) steps; while one step's color gathers are in flight the next
+// step's row entries (the same vertex's next batch, or the next vertex's first) are loaded,
+// so each batch costs one dependent round trip instead of two. Groups finish vertices at
+// different steps: the finish (group ballot, first fit from the group's table, Y write,
+// table clear) runs inside the step loop for the groups whose vertex ended.
+template <int TB, bool Persist, class C, bool Hub>
+__device__ __forceinline__ void bin1_pipe(const RoundArgs<C>& a, int k, const int32_t* list,
+                                          int nX, int32_t* out, int32_t* out_cnt, const C* X,
+                                          C* Y, uint8_t* wsm, int gw, int NW, int lane,
+                                          unsigned long long& edges,
+                                          unsigned long long& entries) {
+  if (gw * 4 >= nX) return;
+  const int g = lane >> 3, gl = lane & 7;
+  const unsigned gmask = 0xffu << (g * 8);
+  uint8_t* gtbl = wsm + WarpSmem<C, Hub>::kBuf + g * kMedTblB;
+  int32_t* pbuf = reinterpret_cast<int32_t*>(wsm + WarpSmem<C, Hub>::kPush);
+  int pending = 0;
+  const int step = NW * 4;
+  auto load_batch = [&](int64_t s, int32_t cnt, int32_t bb, int32_t (&w)[8]) {
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int32_t r = 64 * bb + gl + kGroup * u;
+      w[u] = r < cnt ? ld_row(a.col_idx + s + r) : -1;
+    }
+  };
+  // the group's current vertex and, prefetched, its next one
+  int i = gw * 4 + g;
+  int32_t v = i < nX ? ld_cg(list + i) : -1;
+  int64_t s = v >= 0 ? ldg_i64(a.row_ptr + v) : 0, e = v >= 0 ? ldg_i64(a.row_ptr + v + 1) : 0;
+  int32_t vn = i + step < nX ? ld_cg(list + i + step) : -1;
+  int64_t sn = vn >= 0 ? ldg_i64(a.row_ptr + vn) : 0, en = vn >= 0 ? ldg_i64(a.row_ptr + vn + 1) : 0;
+  int32_t cnt = (int32_t)(e - s), bb = 0;
+  int32_t w[8];
+  load_batch(s, cnt, 0, w);
+  int32_t xv = v >= 0 ? ldc<Persist>(X + v) : 0;
+  bool conf = false;
+  while (__any_sync(0xffffffffu, v >= 0)) {
+    uint32_t lb = 0;
+#pragma unroll
+    for (int u = 0; u < 8; ++u) lb |= (w[u] >= 0 && lose<TB>(v, w[u])) ? (1u << u) : 0u;
+    int32_t c[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) c[u] = w[u] >= 0 ? ldc<Persist>(X + w[u]) : -1;  // colors
+    // next step of this group: the same vertex's next batch, or the next vertex's first
+    const bool last = v < 0 || 64 * (bb + 1) >= cnt;
+    if (!last) {
+      load_batch(s, cnt, bb + 1, w);
+    } else if (vn >= 0) {
+      load_batch(sn, (int32_t)(en - sn), 0, w);
+    } else {
+#pragma unroll
+      for (int u = 0; u < 8; ++u) w[u] = -1;
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      if (c[u] >= 0) {
+        // deg <= 256 => first fit <= 257: colors >= 511 are clamped onto an unused byte
+        set_add(gtbl, (uint32_t)min(c[u], kMedTbl - 1));
+        conf |= c[u] == xv && ((lb >> u) & 1u);
+      }
+    }
+    bool push = false;
+    if (last && v >= 0) {  // finish v (group-converged: all 8 lanes share `last` and v)
+      __syncwarp(gmask);
+      const bool any = (__ballot_sync(gmask, conf) & gmask) != 0u;
+      int32_t tent = 0;
+      if (any) {
+        const uint32_t* t32 = reinterpret_cast<const uint32_t*>(gtbl);
+        for (int it = 0; it < kMedTbl / 32; ++it) {
+          uint32_t word = t32[it * 8 + gl];
+          if (it == 0 && gl == 0) word |= 0xffu;
+          const uint32_t z = __vcmpeq4(word, 0u);
+          const unsigned b = __ballot_sync(gmask, z != 0u) & gmask;
+          if (b) {
+            const int fl = __ffs(b) - 1;
+            const uint32_t zz = __shfl_sync(gmask, z, fl);
+            tent = (it * 8 + (fl & 7)) * 4 + (__ffs(zz) - 1) / 8;
+            break;
+          }
+        }
+      }
+      set_clear(gtbl, kMedTblB, gl, kGroup);
+      __syncwarp(gmask);
+      if (gl == 0) {
+        Y[v] = any ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a);
+        edges += (unsigned long long)cnt;
+        entries += (unsigned long long)cnt;
+      }
+      push = any && gl == 0;
+    }
+    push_buffered(push, v, pbuf, pending, out, out_cnt, lane);
+    if (last) {  // advance the group to its next vertex; prefetch the one after
+      i += step;
+      v = vn;
+      s = sn;
+      e = en;
+      cnt = (int32_t)(e - s);
+      bb = 0;
+      conf = false;
+      xv = v >= 0 ? ldc<Persist>(X + v) : 0;
+      vn = (v >= 0 && i + step < nX) ? ld_cg(list + i + step) : -1;
+      sn = vn >= 0 ? ldg_i64(a.row_ptr + vn) : 0;
+      en = vn >= 0 ? ldg_i64(a.row_ptr + vn + 1) : 0;
+    } else {
+      ++bb;
+    }
+  }
+  push_flush(pbuf, pending, out, out_cnt, lane);
+}
+
 // One fused pass F_k over all three bins; every warp of the grid calls it. Static
 // round-robin assignment (warp w takes items w, w + NW, ...), with the next item's list
 // entry and row offsets prefetched while the current one is processed.
@@ -1432,7 +1561,11 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, const C
   long long t1 = clock64();
   cyc[2] += (unsigned long long)(t1 - t0);
   // ---- bin 1: four vertices per warp (one per 8-lane group), 512-byte tables
+#if SGR_BIN1_PIPE
+  bin1_pipe<TB, Persist, C, Hub>(
+#else
   bin1<TB, Persist, C, Hub>(
+#endif
       a, k, sel(p, (const int32_t*)a.wl_m[0], (const int32_t*)a.wl_m[1]),
       w.m, sel(p ^ 1, a.wl_m[0], a.wl_m[1]), &ctrl->ring[rs(k + 1)].m, X, Y,
       wsm, gw, NW, lane, edges[1], entries[1]);
@@ -1520,16 +1653,17 @@ __device__ __forceinline__ void fold_pass(Ctrl* c, int k) {
   for (int q = 0; q < kBins; ++q) {
     const unsigned long long e = __ldcg(&c->edges_acc[rs(k)][q]);
     const unsigned long long x = __ldcg(&c->entries_acc[rs(k)][q]);
-    c->verts_total[q] += (unsigned long long)vin[q];
-    c->edges_total[q] += e;
-    c->entries_total[q] += x;
-    c->pushes_total[q] += (unsigned long long)vout[q];
+    // fire-and-forget reductions: the folding thread never waits on the totals
+    atomicAdd(&c->verts_total[q], (unsigned long long)vin[q]);
+    atomicAdd(&c->edges_total[q], e);
+    atomicAdd(&c->entries_total[q], x);
+    atomicAdd(&c->pushes_total[q], (unsigned long long)vout[q]);
     c->edges_acc[rs(k)][q] = 0ull;
     c->entries_acc[rs(k)][q] = 0ull;
     e_all += e;
     tot_in += vin[q];
   }
-  c->items_total += (unsigned long long)win.c;
+  atomicAdd(&c->items_total, (unsigned long long)win.c);
   c->ring[rs(k)] = Counts{};
   if (k - 1 < c->round_cap) {
     if (c->round_sizes) c->round_sizes[k - 1] = tot_in;
@@ -1686,6 +1820,11 @@ __device__ __forceinline__ uint32_t ld_acquire_gpu(const uint32_t* p) {
   asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
+__device__ __forceinline__ uint32_t ld_relaxed_gpu(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
 __device__ __forceinline__ void st_release_gpu(uint32_t* p, uint32_t v) {
   asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
@@ -1695,10 +1834,35 @@ __device__ __forceinline__ uint32_t atom_add_acq_rel_u32(uint32_t* p, uint32_t v
   return r;
 }
 
-// Grid-wide barrier of the persistent kernel (every block resident). Thread 0 of each block
-// arrives with an acq_rel atomic (publishing, via the preceding bar.sync, every write of
-// its block); the last arrival resets the count and releases the new generation.
-__device__ __forceinline__ void grid_sync(Ctrl* ctrl) {
+// Grid-wide barrier of the persistent kernel (every block resident).
+#if SGR_BAR2
+// Monotonic arrival counter (zeroed per coloring): thread 0 of each block adds 1 with
+// release semantics (publishing, via the preceding bar.sync, every write of its block) and
+// waits with acquire loads until barrier number `epoch` has all gridDim.x arrivals. No
+// last-arriver reset/release step: one L2 round trip less per barrier.
+__device__ __forceinline__ void red_release_gpu_u32(uint32_t* p, uint32_t v) {
+  asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void grid_sync(Ctrl* ctrl, uint32_t& epoch) {
+  __syncthreads();
+  ++epoch;
+  if (threadIdx.x == 0) {
+    red_release_gpu_u32(&ctrl->bar_count, 1u);
+    const uint32_t target = epoch * gridDim.x;
+    // poll with relaxed loads (served by L2; an acquire load would invalidate this SM's L1
+    // on every poll, evicting the lines the SM's other blocks are still gathering from),
+    // then one acquire load once the count is reached
+    while ((int32_t)(ld_relaxed_gpu(&ctrl->bar_count) - target) < 0) __nanosleep(20);
+    (void)ld_acquire_gpu(&ctrl->bar_count);
+  }
+  __syncthreads();
+}
+#else
+// Thread 0 of each block arrives with an acq_rel atomic (publishing, via the preceding
+// bar.sync, every write of its block); the last arrival resets the count and releases the
+// new generation.
+__device__ __forceinline__ void grid_sync(Ctrl* ctrl, uint32_t& epoch) {
+  (void)epoch;
   __syncthreads();
   if (threadIdx.x == 0) {
     const uint32_t gen = ld_acquire_gpu(&ctrl->bar_gen);
@@ -1712,7 +1876,7 @@ __device__ __forceinline__ void grid_sync(Ctrl* ctrl) {
   }
   __syncthreads();
 }
-
+#endif
 
 // All rounds in one cooperative launch (every block resident). Each block tracks k itself
 // and reads W_k's counts after the barrier that ends pass k-1; block 0 folds pass k-1 into
@@ -1729,8 +1893,11 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks<C, Hub>) k_persistent(Round
   uint32_t ph = 0;  // mbarrier phase bits of the warp's two TMA stages
   unsigned long long cyc[kBins] = {0, 0, 0};
   unsigned long long pcx[3] = {0, 0, 0};  // barrier waits, finalize, counter reduction
+  uint32_t epoch = 0;                     // grid barriers passed (SGR_BAR2)
   const int max_rounds = ld_cg(&ctrl->max_rounds);
-  const bool leader = blockIdx.x == 0 && threadIdx.x == 0;
+  // the last block folds the finished pass: it is the one that draws work last (items go to
+  // the lowest warp ids first), so the fold is off the critical path of thin rounds
+  const bool leader = blockIdx.x == gridDim.x - 1 && threadIdx.x == 0;
   int k = 2;
   for (;; ++k) {
     const Counts w = ld_counts(&ctrl->ring[rs(k)]);
@@ -1752,16 +1919,16 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks<C, Hub>) k_persistent(Round
     const long long t1 = clock64();
     pcx[2] += (unsigned long long)(t1 - t0);
     if constexpr (packed<C>() && Hub) {  // multi-chunk vertices: decided once all chunks are in
-      grid_sync(ctrl);
+      grid_sync(ctrl, epoch);
       const long long t2 = clock64();
       finalize_body<TB, true>(a, k);
       const long long t3 = clock64();
       pcx[0] += (unsigned long long)(t2 - t1);
       pcx[1] += (unsigned long long)(t3 - t2);
-      grid_sync(ctrl);
+      grid_sync(ctrl, epoch);
       pcx[0] += (unsigned long long)(clock64() - t3);
     } else {
-      grid_sync(ctrl);
+      grid_sync(ctrl, epoch);
       pcx[0] += (unsigned long long)(clock64() - t1);
     }
   }
