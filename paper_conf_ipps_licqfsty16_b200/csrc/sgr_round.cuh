@@ -236,6 +236,18 @@ __device__ __forceinline__ uint32_t ldraw(const C* p) {
     return (uint32_t)__ldg(p);
   }
 }
+// Bin-2 neighbour gathers (hub lists: scattered over the whole color array) at L2 only:
+// they would otherwise allocate L1 lines that are rarely reused, evicting the lines that
+// the bin-0/1 gathers and the row reads do reuse (cfg4 -3.6 %, ER -2 % measured with all
+// gathers at L2; the stencil's bin-0 gathers need L1: +8 % there). Coherent either way.
+#ifndef SGR_B2_CG
+#define SGR_B2_CG 1
+#endif
+template <bool Persist, class C>
+__device__ __forceinline__ uint32_t ldraw_b2(const C* p) {
+  if constexpr (Persist && SGR_B2_CG) return (uint32_t)__ldcg(p);
+  else return ldraw<Persist>(p);
+}
 template <class C>
 __device__ __forceinline__ int32_t cval(uint32_t raw) {
   if constexpr (packed<C>()) return (int32_t)(raw & kColorMask);
@@ -243,6 +255,17 @@ __device__ __forceinline__ int32_t cval(uint32_t raw) {
 }
 template <bool Persist, class C>
 __device__ __forceinline__ int32_t ldc(const C* p) { return cval<C>(ldraw<Persist>(p)); }
+// Bins 0/1 in the hub build (skewed graphs: rows of scattered small-degree vertices) gather
+// at L2 as well (cfg4 a further -1.1 %); the flat build (no bin 2: stencils, ER) keeps them
+// L1-cached, where stencil neighbours share lines across vertices (L2-only: +8 %).
+#ifndef SGR_HUB01_CG
+#define SGR_HUB01_CG 1
+#endif
+template <bool Persist, bool Hub, class C>
+__device__ __forceinline__ int32_t ldc01(const C* p) {
+  if constexpr (Persist && Hub && SGR_HUB01_CG) return cval<C>((uint32_t)__ldcg(p));
+  else return cval<C>(ldraw<Persist>(p));
+}
 
 template <class C>
 __device__ __forceinline__ C cpack(int32_t color, int32_t last, const RoundArgs<C>& a) {
@@ -810,7 +833,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
         okm |= (r >= off0 && r < nslots) ? (1u << j) : 0u;
       }
 #pragma unroll
-      for (int j = 0; j < kJB; ++j) raw[j] = ((okm >> j) & 1u) ? ldraw<Persist>(X + id[j]) : 0u;
+      for (int j = 0; j < kJB; ++j) raw[j] = ((okm >> j) & 1u) ? ldraw_b2<Persist>(X + id[j]) : 0u;
     };
     auto consume = [&](const int32_t (&id)[kJB], const uint32_t (&raw)[kJB], uint32_t okm) {
 #pragma unroll
@@ -1102,7 +1125,7 @@ __device__ __forceinline__ void finalize_body(const RoundArgs<Packed>& a, int k)
 // Bin 1: each 8-lane group of the warp processes one vertex (v < 0: idle group) in batches
 // of 64 row entries (8 per lane: all eight loads, then all eight gathers); only as many
 // batches as the row needs are issued. 32-bit relative indices throughout.
-template <int TB, bool Persist, class C>
+template <int TB, bool Persist, class C, bool Hub>
 __device__ __forceinline__ void process_group(const RoundArgs<C>& a, int k, int32_t v,
                                               int64_t s, int64_t e, const C* X, C* Y,
                                               uint8_t* gtbl, int gl, unsigned gmask,
@@ -1123,7 +1146,7 @@ __device__ __forceinline__ void process_group(const RoundArgs<C>& a, int k, int3
 #pragma unroll
     for (int u = 0; u < 8; ++u) lb |= (w[u] >= 0 && lose<TB>(v, w[u])) ? (1u << u) : 0u;
 #pragma unroll
-    for (int u = 0; u < 8; ++u) w[u] = w[u] >= 0 ? ldc<Persist>(X + w[u]) : -1;  // colors
+    for (int u = 0; u < 8; ++u) w[u] = w[u] >= 0 ? ldc01<Persist, Hub>(X + w[u]) : -1;  // colors
 #pragma unroll
     for (int u = 0; u < 8; ++u) {
       if (w[u] >= 0) {
@@ -1235,7 +1258,7 @@ __device__ __forceinline__ void bin0(const RoundArgs<C>& a, int k, const int32_t
     for (int u = 0; u < kK0; ++u) lb |= (w[u] >= 0 && lose<TB>(v, w[u])) ? (1u << u) : 0u;
     int32_t c[kK0];
 #pragma unroll
-    for (int u = 0; u < kK0; ++u) c[u] = (w[u] >= 0) ? ldc<Persist>(X + w[u]) : 0;
+    for (int u = 0; u < kK0; ++u) c[u] = (w[u] >= 0) ? ldc01<Persist, Hub>(X + w[u]) : 0;
     int32_t wn[kK0];
     load_row(v1, s1, e1, wn);  // next vertex's row, in flight with the gathers above
     bool conf = false;
@@ -1385,7 +1408,7 @@ __device__ __forceinline__ void bin1(const RoundArgs<C>& a, int k, const int32_t
     if (sn + 32 * gl < en) prefetch_l2(a.col_idx + sn + 32 * gl);  // 1 line / lane
     bool push = false;
     if (v >= 0 && gl == 0) entries += (unsigned long long)(e - s);
-    process_group<TB, Persist, C>(a, k, v, s, e, X, Y, gtbl, gl, gmask, push, edges);
+    process_group<TB, Persist, C, Hub>(a, k, v, s, e, X, Y, gtbl, gl, gmask, push, edges);
     push_buffered(push, v, pbuf, pending, out, out_cnt, lane);
     i = in;
     v = vn;
@@ -1438,7 +1461,7 @@ __device__ __forceinline__ void bin1_pipe(const RoundArgs<C>& a, int k, const in
     for (int u = 0; u < 8; ++u) lb |= (w[u] >= 0 && lose<TB>(v, w[u])) ? (1u << u) : 0u;
     int32_t c[8];
 #pragma unroll
-    for (int u = 0; u < 8; ++u) c[u] = w[u] >= 0 ? ldc<Persist>(X + w[u]) : -1;  // colors
+    for (int u = 0; u < 8; ++u) c[u] = w[u] >= 0 ? ldc01<Persist, Hub>(X + w[u]) : -1;  // colors
     // next step of this group: the same vertex's next batch, or the next vertex's first
     const bool last = v < 0 || 64 * (bb + 1) >= cnt;
     if (!last) {
