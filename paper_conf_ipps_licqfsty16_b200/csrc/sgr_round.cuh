@@ -52,6 +52,9 @@ constexpr int kJB = 4 * kQB;  // entries per lane per batch
 #ifndef SGR_SLAYOUT
 #define SGR_SLAYOUT 1  // bin 2: lane-consecutive window slots (see bin2_trimmed)
 #endif
+#ifndef SGR_SMALL_FIRST
+#define SGR_SMALL_FIRST 0  // pass order 0, 1, 2 instead of 2, 1, 0
+#endif
 #ifndef SGR_BAR2
 #define SGR_BAR2 1  // grid barrier on a monotonic arrival counter (no reset/release step)
 #endif
@@ -1055,7 +1058,13 @@ __device__ __forceinline__ void finalize_body(const RoundArgs<Packed>& a, int k)
   // vector loads issued together, first fit by a scan of the merged words, item pushes with
   // one aggregated atomicAdd per counter per warp
   const int B = min(32, (nF + NW - 1) / NW);
-  for (int base = gw * B; base < nF; base += NW * B) {
+  // every warp runs the same number of iterations (block-level aggregation below)
+  const int iters = nF > 0 ? (nF + NW * B - 1) / (NW * B) : 0;
+  __shared__ int32_t fin_tot[2][kWarps];   // per warp: items, vertices
+  __shared__ int32_t fin_base[kWarps];
+  const int wid = threadIdx.x >> 5;
+  for (int it = 0; it < iters; ++it) {
+    const int base = gw * B + it * NW * B;
     const int i = base + lane;
     const bool valid = lane < B && i < nF;
     const uint64_t f = valid ? (uint64_t)__ldcg(a.fin + i) : 0ull;
@@ -1096,11 +1105,27 @@ __device__ __forceinline__ void finalize_body(const RoundArgs<Packed>& a, int k)
     }
     const int32_t total = __shfl_sync(0xffffffffu, incl, 31);
     const unsigned cm = __ballot_sync(0xffffffffu, conf);
-    int32_t ob = 0;
+    // item slots: one atomicAdd per BLOCK and counter (every warp of the grid finalizes at
+    // the same moment, so per-warp atomics on two hot addresses would serialize)
     if (lane == 0) {
-      if (total) ob = atomicAdd(&ctrl->ring[rs(k + 1)].c, total);
-      if (cm) atomicAdd(&ctrl->ring[rs(k + 1)].cv, __popc(cm));
+      fin_tot[0][wid] = total;
+      fin_tot[1][wid] = (int32_t)__popc(cm);
     }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      int32_t run = 0, vs = 0;
+      for (int q = 0; q < kWarps; ++q) {
+        fin_base[q] = run;
+        run += fin_tot[0][q];
+        vs += fin_tot[1][q];
+      }
+      const int32_t b0 = run ? atomicAdd(&ctrl->ring[rs(k + 1)].c, run) : 0;
+      if (vs) atomicAdd(&ctrl->ring[rs(k + 1)].cv, vs);
+      for (int q = 0; q < kWarps; ++q) fin_base[q] += b0;
+    }
+    __syncthreads();
+    int32_t ob = 0;
+    if (lane == 0) ob = fin_base[wid];
     // first fits beyond the exact range of the table: warp rescans of the full rows (rare)
     unsigned rm = __ballot_sync(0xffffffffu, conf && (tent < 0 || tent >= kBigTbl - 1));
     while (rm) {
@@ -1547,63 +1572,86 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, const C
   C* Y = sel(k & 1, a.col[0], a.col[1]);
   uint8_t* wtbl = wsm + WarpSmem<C, Hub>::kBuf;
   (void)wtbl;
-  long long t0 = clock64();
-  // ---- bin 2 (Hub build only; the flat build runs when bin 2 is empty)
-  if constexpr (!Hub) {
-  } else if constexpr (packed<C>()) {
-    bin2_trimmed<TB, Persist>(a, k, p, X, Y, wsm, gw, NW, lane, w.c, edges[2], entries[2], ph);
-  } else {
-    const int nC = w.c;
-    const int64_t* items = sel(p, (const int64_t*)a.wl_c[0], (const int64_t*)a.wl_c[1]);
-    int64_t* out = sel(p ^ 1, a.wl_c[0], a.wl_c[1]);
-    int i = gw;
-    int64_t it = i < nC ? __ldcg(items + i) : 0;
-    int32_t v = (int32_t)((uint64_t)it >> 32);
-    int64_t s = i < nC ? ldg_i64(a.row_ptr + v) : 0, e = i < nC ? ldg_i64(a.row_ptr + v + 1) : 0;
-    while (i < nC) {
-      const int in = i + NW;
-      const int64_t itn = in < nC ? __ldcg(items + in) : 0;
-      const int32_t vn = (int32_t)((uint64_t)itn >> 32);
-      const int64_t sn = in < nC ? ldg_i64(a.row_ptr + vn) : 0;
-      const int64_t en = in < nC ? ldg_i64(a.row_ptr + vn + 1) : 0;
-      if (in < nC) {  // warm L2 with the next item's 4 KB window (one 128-byte line per lane)
-        const int64_t csn = sn + (int64_t)(int32_t)(uint32_t)itn * kChunk;
-        const int64_t ln = (csn & ~(int64_t)3) + 32 * lane;
-        if (ln < en) prefetch_l2(a.col_idx + ln);
+  auto run_bin2 = [&]() {
+    // ---- bin 2 (Hub build only; the flat build runs when bin 2 is empty)
+    if constexpr (!Hub) {
+    } else if constexpr (packed<C>()) {
+      bin2_trimmed<TB, Persist>(a, k, p, X, Y, wsm, gw, NW, lane, w.c, edges[2], entries[2], ph);
+    } else {
+      const int nC = w.c;
+      const int64_t* items = sel(p, (const int64_t*)a.wl_c[0], (const int64_t*)a.wl_c[1]);
+      int64_t* out = sel(p ^ 1, a.wl_c[0], a.wl_c[1]);
+      int i = gw;
+      int64_t it = i < nC ? __ldcg(items + i) : 0;
+      int32_t v = (int32_t)((uint64_t)it >> 32);
+      int64_t s = i < nC ? ldg_i64(a.row_ptr + v) : 0, e = i < nC ? ldg_i64(a.row_ptr + v + 1) : 0;
+      while (i < nC) {
+        const int in = i + NW;
+        const int64_t itn = in < nC ? __ldcg(items + in) : 0;
+        const int32_t vn = (int32_t)((uint64_t)itn >> 32);
+        const int64_t sn = in < nC ? ldg_i64(a.row_ptr + vn) : 0;
+        const int64_t en = in < nC ? ldg_i64(a.row_ptr + vn + 1) : 0;
+        if (in < nC) {  // warm L2 with the next item's 4 KB window (one 128-byte line per lane)
+          const int64_t csn = sn + (int64_t)(int32_t)(uint32_t)itn * kChunk;
+          const int64_t ln = (csn & ~(int64_t)3) + 32 * lane;
+          if (ln < en) prefetch_l2(a.col_idx + ln);
+        }
+        process_chunk_plain<TB, Persist, C>(a, k, v, (int32_t)(uint32_t)it, s, e, X, Y, out,
+                                            &ctrl->ring[rs(k + 1)].c, &ctrl->ring[rs(k + 1)].cv, wtbl,
+                                            lane, edges[2], entries[2]);
+        i = in;
+        it = itn;
+        v = vn;
+        s = sn;
+        e = en;
       }
-      process_chunk_plain<TB, Persist, C>(a, k, v, (int32_t)(uint32_t)it, s, e, X, Y, out,
-                                          &ctrl->ring[rs(k + 1)].c, &ctrl->ring[rs(k + 1)].cv, wtbl,
-                                          lane, edges[2], entries[2]);
-      i = in;
-      it = itn;
-      v = vn;
-      s = sn;
-      e = en;
     }
-  }
+  };
+  auto run_bin1 = [&]() {
+    // ---- bin 1: four vertices per warp (one per 8-lane group), 512-byte tables
+  #if SGR_BIN1_PIPE
+    bin1_pipe<TB, Persist, C, Hub>(
+  #else
+    bin1<TB, Persist, C, Hub>(
+  #endif
+        a, k, sel(p, (const int32_t*)a.wl_m[0], (const int32_t*)a.wl_m[1]),
+        w.m, sel(p ^ 1, a.wl_m[0], a.wl_m[1]), &ctrl->ring[rs(k + 1)].m, X, Y,
+        wsm, gw, NW, lane, edges[1], entries[1]);
+  };
+  auto run_bin0 = [&]() {
+    // ---- bin 0: eight vertices per warp, register masks
+  #if SGR_BIN0_THREAD
+    bin0_thread<TB, Persist, C, Hub>(
+  #else
+    bin0<TB, Persist, C, Hub>(
+  #endif
+        a, k, sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]),
+        w.t, sel(p ^ 1, a.wl_t[0], a.wl_t[1]), &ctrl->ring[rs(k + 1)].t, X, Y,
+        wsm, gw, NW, lane, edges[0], entries[0]);
+  };
+  // Order within the pass. Default 2, 1, 0: the large chunk items first (claimed from a
+  // cursor), the static small-vertex bins fill the tail. SGR_SMALL_FIRST: 0, 1, 2 (the
+  // dynamic bin-2 claims absorb the static bins' imbalance before the barrier).
+  long long t0 = clock64();
+#if SGR_SMALL_FIRST
+  run_bin0();
   long long t1 = clock64();
-  cyc[2] += (unsigned long long)(t1 - t0);
-  // ---- bin 1: four vertices per warp (one per 8-lane group), 512-byte tables
-#if SGR_BIN1_PIPE
-  bin1_pipe<TB, Persist, C, Hub>(
-#else
-  bin1<TB, Persist, C, Hub>(
-#endif
-      a, k, sel(p, (const int32_t*)a.wl_m[0], (const int32_t*)a.wl_m[1]),
-      w.m, sel(p ^ 1, a.wl_m[0], a.wl_m[1]), &ctrl->ring[rs(k + 1)].m, X, Y,
-      wsm, gw, NW, lane, edges[1], entries[1]);
+  cyc[0] += (unsigned long long)(t1 - t0);
+  run_bin1();
   long long t2 = clock64();
   cyc[1] += (unsigned long long)(t2 - t1);
-  // ---- bin 0: eight vertices per warp, register masks
-#if SGR_BIN0_THREAD
-  bin0_thread<TB, Persist, C, Hub>(
+  run_bin2();
+  cyc[2] += (unsigned long long)(clock64() - t2);
 #else
-  bin0<TB, Persist, C, Hub>(
-#endif
-      a, k, sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]),
-      w.t, sel(p ^ 1, a.wl_t[0], a.wl_t[1]), &ctrl->ring[rs(k + 1)].t, X, Y,
-      wsm, gw, NW, lane, edges[0], entries[0]);
+  run_bin2();
+  long long t1 = clock64();
+  cyc[2] += (unsigned long long)(t1 - t0);
+  run_bin1();
+  long long t2 = clock64();
+  cyc[1] += (unsigned long long)(t2 - t1);
+  run_bin0();
   cyc[0] += (unsigned long long)(clock64() - t2);
+#endif
 }
 
 // Block reduction of the per-thread counters, one atomicAdd each per block.
