@@ -52,6 +52,13 @@ constexpr int kJB = 4 * kQB;  // entries per lane per batch
 #ifndef SGR_SLAYOUT
 #define SGR_SLAYOUT 1  // bin 2: lane-consecutive window slots (see bin2_trimmed)
 #endif
+#ifndef SGR_LAZY
+#define SGR_LAZY 4  // bin 2 single-chunk lists: rewrite only if > cnt >> SGR_LAZY entries dropped
+#endif
+#ifndef SGR_CLRMAX
+#define SGR_CLRMAX 1  // bin 2: clear the chunk's tables only up to the largest color seen
+#endif
+static_assert(!SGR_CLRMAX || SGR_SLAYOUT, "SGR_CLRMAX tracks the largest color in the SLAYOUT batch loop");
 #ifndef SGR_SMALL_FIRST
 #define SGR_SMALL_FIRST 0  // pass order 0, 1, 2 instead of 2, 1, 0
 #endif
@@ -367,6 +374,24 @@ __device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t
 
 // Row entries of bins 0 and 1 (streamed once per pass). SGR_ROWNA: bypass L1 allocation,
 // leaving L1 to the color gathers.
+// Row entries in the flat build (no hubs: stencils, ER) with an L2 evict-last policy
+// (SGR_ROWEL): W stays close to V for many rounds on stencils, so the rows read in one pass
+// are read again in the next; evict-last keeps them in L2 ahead of streaming traffic.
+#ifndef SGR_ROWEL
+#define SGR_ROWEL 0
+#endif
+template <bool Hub>
+__device__ __forceinline__ int32_t ld_row_h(const int32_t* p) {
+  if constexpr (!Hub && SGR_ROWEL) {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    int32_t r;
+    asm volatile("ld.global.nc.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
+    return r;
+  } else {
+    return __ldg(p);
+  }
+}
 __device__ __forceinline__ int32_t ld_row(const int32_t* p) {
 #if SGR_ROWNA
   int32_t r;
@@ -822,6 +847,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
     int32_t* sbuf = bufs + st * (kStage / 4);
     bool conf = false;
     uint32_t lpos = 0;  // warp-uniform: live entries of the finished batches
+    uint32_t cmax = 0;  // SGR_CLRMAX: largest table index this lane set
     const unsigned lt_mask = (1u << lane) - 1u;
 #if SGR_SLAYOUT
     // batch bb: window slots 32 (kJB bb + j) + lane, j < kJB: consecutive lanes read
@@ -847,6 +873,9 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
           // recomputed exactly from the full row (warp_first_fit_rescan)
           const uint32_t ci = min(raw[j] & kColorMask, (uint32_t)(kBigTbl - 1));
           live = (raw[j] >> kRoundShift) == klive;
+#if SGR_CLRMAX
+          cmax = max(cmax, ci);
+#endif
           set_add(tbl_all, ci);
           if (!live) set_add(tbl_drop, ci);
           conf |= (int32_t)(raw[j] & kColorMask) == xv && lose<TB>(v, id[j]);
@@ -968,12 +997,16 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
         if (drop & ~fo) fx[lane] = fo | drop;
         // single chunk: the warp owns the whole list, so it is compacted in place, and not
         // rewritten at all when nothing was dropped (pass 2 read col_idx: always written)
-        if (k == 2 || live_total < (uint32_t)cnt) {
+        // SGR_LAZY > 0: keep the list (dead entries included) unless more than cnt >> SGR_LAZY
+        // entries dropped — listed dead neighbours are simply the untrimmed semantics
+        const bool rewrite = k == 2 || (SGR_LAZY ? (uint32_t)cnt - live_total > ((uint32_t)cnt >> SGR_LAZY)
+                                                 : live_total < (uint32_t)cnt);
+        if (rewrite) {
           write_live(lst_same + cur.s);
           lwrites += live_total;
         }
         if (lane == 0) {
-          len_nxt[v] = (int32_t)live_total;
+          len_nxt[v] = rewrite ? (int32_t)live_total : cnt;
           Y[v] = cpack<C>(tent, k + 1, a);
           // live <= kChunk: one chunk, the list stays in its buffer
           ibuf[ipend] = make_item(v, (int32_t)(cur.buf ? kBufBit : 0u));
@@ -1006,7 +1039,19 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
       if (lane == 0 && cur.c == 0)
         a.fin[fpos] = (int64_t)(((uint64_t)(uint32_t)slot << 32) | (uint32_t)v | (cur.buf ? kBufBit : 0u));
     }
+#if SGR_CLRMAX
+    {  // both sets, only the 16-byte groups up to the largest color set in this chunk
+      const uint32_t nq = (__reduce_max_sync(0xffffffffu, cmax) >> 4) + 1;
+      uint4* ta = reinterpret_cast<uint4*>(tbl_all);
+      uint4* td = reinterpret_cast<uint4*>(tbl_drop);
+      for (uint32_t q = lane; q < nq; q += 32) {
+        ta[q] = make_uint4(0u, 0u, 0u, 0u);
+        td[q] = make_uint4(0u, 0u, 0u, 0u);
+      }
+    }
+#else
     set_clear(tbl_all, kTblBytes, lane, 32);  // both sets
+#endif
     __syncwarp();
 #if !SGR_NO_TMA
     tq = clock64();
@@ -1165,7 +1210,7 @@ __device__ __forceinline__ void process_group(const RoundArgs<C>& a, int k, int3
 #pragma unroll
     for (int u = 0; u < 8; ++u) {
       const int32_t r = 64 * bb + gl + kGroup * u;
-      w[u] = r < cnt ? ld_row(row + r) : -1;
+      w[u] = r < cnt ? ld_row_h<Hub>(row + r) : -1;
     }
     uint32_t lb = 0;
 #pragma unroll
@@ -1266,7 +1311,7 @@ __device__ __forceinline__ void bin0(const RoundArgs<C>& a, int k, const int32_t
     const int32_t cnt = vv >= 0 ? (int32_t)(ee - ss) : 0;
     const int32_t* row = a.col_idx + ss;
 #pragma unroll
-    for (int u = 0; u < kK0; ++u) w[u] = (gl + G * u < cnt) ? ld_row(row + gl + G * u) : -1;
+    for (int u = 0; u < kK0; ++u) w[u] = (gl + G * u < cnt) ? ld_row_h<Hub>(row + gl + G * u) : -1;
   };
   int i = gw * VPW + g;
   int32_t v = i < nX ? ld_cg(list + i) : -1;
