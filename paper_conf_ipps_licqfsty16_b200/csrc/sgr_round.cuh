@@ -55,6 +55,9 @@ constexpr int kJB = 4 * kQB;  // entries per lane per batch
 #ifndef SGR_LAZY
 #define SGR_LAZY 4  // bin 2 single-chunk lists: rewrite only if > cnt >> SGR_LAZY entries dropped
 #endif
+#ifndef SGR_MCLAZY
+#define SGR_MCLAZY 1  // multi-chunk lists: keep uncompacted while <= 1/16 of entries are dead
+#endif
 #ifndef SGR_CLRMAX
 #define SGR_CLRMAX 1  // bin 2: clear the chunk's tables only up to the largest color seen
 #endif
@@ -313,6 +316,11 @@ __device__ __forceinline__ int64_t make_item(int32_t v, int32_t c) {
 // Bin-2 items of the trimmed mode carry the adjacency buffer holding the vertex's list in
 // bit 31 of the chunk field.
 constexpr uint32_t kBufBit = 0x80000000u;
+// Multi-chunk items of a list kept uncompacted this pass (SGR_MCLAZY): its chunks leave the
+// list where it is (dead entries included) and only count their live entries; the finalize
+// phase decides from the dead fraction whether the next pass compacts it.
+constexpr uint32_t kKeepBit = 0x40000000u;
+constexpr uint32_t kChunkMask = 0x3fffffffu;
 
 // Ticket increment with release+acquire semantics at GPU scope: every write this thread
 // (and, through the preceding __syncwarp, its warp) made is visible to whoever observes
@@ -701,7 +709,7 @@ __device__ __forceinline__ void process_chunk_plain(const RoundArgs<C>& a, int k
 // Bin 2, packed colors, trimmed lists (see the header comment). Per warp: a 2-stage TMA
 // pipeline over the warp's chunk items i, i + NW, i + 2 NW, ...
 struct ChunkHdr {
-  int32_t v, c, len, slot, buf;
+  int32_t v, c, len, slot, buf, keep;
   int64_t s, e;   // original row [s, e): list start in adj[*] and col_idx
   uint32_t fo;    // single-chunk vertex: this lane's word of its fixed set (prefetched)
   uint32_t xraw;  // X[v] word (prefetched; decoded at use, so the load is not waited for)
@@ -756,8 +764,9 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
   };
   auto finish_hdr = [&](int64_t it, ChunkHdr& h) {  // everything but the item itself
     h.v = (int32_t)((uint64_t)it >> 32);
-    h.c = (int32_t)((uint32_t)it & ~kBufBit);
+    h.c = (int32_t)((uint32_t)it & kChunkMask);
     h.buf = ((uint32_t)it & kBufBit) ? 1 : 0;
+    h.keep = ((uint32_t)it & kKeepBit) ? 1 : 0;
     h.s = ldg_i64(a.row_ptr + h.v);
     h.e = ldg_i64(a.row_ptr + h.v + 1);
     h.len = ld_cg(len_cur + h.v);
@@ -772,7 +781,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
     h.xraw = ldraw<Persist>(X + h.v);
   };
   auto zero_hdr = [](ChunkHdr& h) {
-    h.v = h.c = h.len = h.slot = h.buf = 0;
+    h.v = h.c = h.len = h.slot = h.buf = h.keep = 0;
     h.s = h.e = 0;
     h.fo = 0u;
     h.xraw = 0u;
@@ -1023,21 +1032,29 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
       // first fit once every chunk is in (no per-chunk fences or tickets)
       // (the atomics whose results are needed are issued first, consumed last)
       int32_t lbase = 0, fpos = 0;
+      const bool keep = cur.keep != 0;
       if (lane == 0) {
-        if (live_total) lbase = atomicAdd(len_nxt + v, (int32_t)live_total);
+        if (keep) {  // list stays: count live entries in the slot's accumulator (bits 32-63)
+          if (live_total) atomicAdd(a.acc_cnt + slot, (unsigned long long)live_total << 32);
+        } else if (live_total) {
+          lbase = atomicAdd(len_nxt + v, (int32_t)live_total);
+        }
         if (cur.c == 0) fpos = atomicAdd(&ctrl->ring[rs(k)].fin, 1);
-        if (any) atomicOr(a.acc_cnt + slot, 1ull);  // conflict flag
+        if (any) atomicOr(a.acc_cnt + slot, 1ull);  // conflict flag (bit 0)
       }
       uint32_t* accb = a.acc_bits + (int64_t)slot * 32;
       const uint32_t bits = tbl_bits32(tbl_all, lane);
       const uint32_t drop = tbl_bits32(tbl_drop, lane);
       if (bits) atomicOr(accb + lane, bits);
       if (drop) atomicOr(fx + lane, drop);
-      lbase = __shfl_sync(0xffffffffu, lbase, 0);
-      write_live(lst_other + cur.s + lbase);
-      lwrites += live_total;
+      if (!keep) {
+        lbase = __shfl_sync(0xffffffffu, lbase, 0);
+        write_live(lst_other + cur.s + lbase);
+        lwrites += live_total;
+      }
       if (lane == 0 && cur.c == 0)
-        a.fin[fpos] = (int64_t)(((uint64_t)(uint32_t)slot << 32) | (uint32_t)v | (cur.buf ? kBufBit : 0u));
+        a.fin[fpos] = (int64_t)(((uint64_t)(uint32_t)slot << 32) | (uint32_t)v |
+                                (cur.buf ? kBufBit : 0u) | (keep ? (1ull << 63) : 0ull));
     }
 #if SGR_CLRMAX
     {  // both sets, only the 16-byte groups up to the largest color set in this chunk
@@ -1114,9 +1131,10 @@ __device__ __forceinline__ void finalize_body(const RoundArgs<Packed>& a, int k)
     const bool valid = lane < B && i < nF;
     const uint64_t f = valid ? (uint64_t)__ldcg(a.fin + i) : 0ull;
     const int32_t v = (int32_t)((uint32_t)f & ~kBufBit);
-    const int32_t slot = (int32_t)(f >> 32);
-    bool conf = false;
-    int32_t nch2 = 0, tent = -1;
+    const int32_t slot = (int32_t)((f >> 32) & 0x7fffffffull);
+    const bool kept = (f >> 63) != 0ull;  // this pass left the list uncompacted
+    bool conf = false, keep_next = false;
+    int32_t nch2 = 0, tent = -1, len_list = 0;
     uint32_t xraw = 0u;
     uint4* accb = reinterpret_cast<uint4*>(a.acc_bits + (int64_t)slot * 32);
     if (valid) {
@@ -1127,10 +1145,17 @@ __device__ __forceinline__ void finalize_body(const RoundArgs<Packed>& a, int k)
         const uint4 x = __ldcg(accb + q), y = __ldcg(fxb + q);
         m[q] = make_uint4(x.x | y.x, x.y | y.y, x.z | y.z, x.w | y.w);
       }
-      conf = (__ldcg(a.acc_cnt + slot) & 1ull) != 0ull;
+      const unsigned long long cc = __ldcg(a.acc_cnt + slot);
+      conf = (cc & 1ull) != 0ull;
       xraw = ldraw<Persist>(X + v);
-      const int32_t ln = ld_cg(len_nxt + v);
-      nch2 = conf ? num_chunks(ln) : 0;
+      const int32_t lcur = ld_cg(len_cur + v);  // the list this pass read
+      const int32_t lnxt = ld_cg(len_nxt + v);  // compacting pass: live entries written
+      // next pass: the same list (kept) or the compacted one; keep it next pass too unless
+      // more than 1/16 of its entries are dead (kept) / were dropped this pass (compacted)
+      len_list = kept ? lcur : lnxt;
+      const int32_t dead = kept ? lcur - (int32_t)(cc >> 32) : lcur - lnxt;
+      keep_next = SGR_MCLAZY && dead <= (lcur >> 4);
+      nch2 = conf ? num_chunks(len_list) : 0;
       m[0].x |= 1u;  // color 0
 #pragma unroll
       for (int q = 7; q >= 0; --q) {  // lowest word with a zero bit
@@ -1185,8 +1210,10 @@ __device__ __forceinline__ void finalize_body(const RoundArgs<Packed>& a, int k)
     if (valid) {
       a.acc_cnt[slot] = 0ull;
       len_cur[v] = 0;  // consumed; the pass after next accumulates into it
+      if (conf && kept) len_nxt[v] = len_list;  // the same list again
       Y[v] = conf ? cpack<C>(tent, k + 1, a) : cpack<C>(cval<C>(xraw), k, a);
-      const uint32_t nbuf = ((uint32_t)f & kBufBit) ? 0u : kBufBit;  // the list moved buffers
+      const uint32_t obuf = (uint32_t)f & kBufBit;
+      const uint32_t nbuf = (kept ? obuf : (obuf ^ kBufBit)) | (keep_next ? kKeepBit : 0u);
       for (int32_t t = 0; t < nch2; ++t) out[ob + t] = make_item(v, (int32_t)(t | nbuf));
     }
   }
@@ -1842,7 +1869,7 @@ __global__ void k_pack(RoundArgs<C> a, uint2* send, int32_t cap) {
     else if (i < nT + nM) v = lm[i - nT];
     else if (i < total) {
       const int64_t it = lc[i - nT - nM];
-      if (((uint32_t)it & ~kBufBit) == 0u) v = (int32_t)((uint64_t)it >> 32);  // chunk 0
+      if (((uint32_t)it & kChunkMask) == 0u) v = (int32_t)((uint64_t)it >> 32);  // chunk 0
     }
     const unsigned m = __ballot_sync(0xffffffffu, v >= 0);
     if (m) {
