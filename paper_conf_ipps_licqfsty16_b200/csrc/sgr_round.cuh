@@ -58,6 +58,9 @@ constexpr int kJB = 4 * kQB;  // entries per lane per batch
 #ifndef SGR_MCLAZY
 #define SGR_MCLAZY 1  // multi-chunk lists: keep uncompacted while <= 1/16 of entries are dead
 #endif
+#ifndef SGR_MCLAZY_SHIFT
+#define SGR_MCLAZY_SHIFT 4  // dead-entry threshold: len >> SGR_MCLAZY_SHIFT
+#endif
 #ifndef SGR_CLRMAX
 #define SGR_CLRMAX 1  // bin 2: clear the chunk's tables only up to the largest color seen
 #endif
@@ -1154,7 +1157,7 @@ __device__ __forceinline__ void finalize_body(const RoundArgs<Packed>& a, int k)
       // more than 1/16 of its entries are dead (kept) / were dropped this pass (compacted)
       len_list = kept ? lcur : lnxt;
       const int32_t dead = kept ? lcur - (int32_t)(cc >> 32) : lcur - lnxt;
-      keep_next = SGR_MCLAZY && dead <= (lcur >> 4);
+      keep_next = SGR_MCLAZY && dead <= (lcur >> SGR_MCLAZY_SHIFT);
       nch2 = conf ? num_chunks(len_list) : 0;
       m[0].x |= 1u;  // color 0
 #pragma unroll
