@@ -61,6 +61,9 @@ constexpr int kJB = 4 * kQB;  // entries per lane per batch
 #ifndef SGR_MCLAZY_SHIFT
 #define SGR_MCLAZY_SHIFT 4  // dead-entry threshold: len >> SGR_MCLAZY_SHIFT
 #endif
+#ifndef SGR_DEFER_COMPACT
+#define SGR_DEFER_COMPACT 1  // bin 2: live bits per lane; compact the stage only when rewriting
+#endif
 #ifndef SGR_CLRMAX
 #define SGR_CLRMAX 1  // bin 2: clear the chunk's tables only up to the largest color seen
 #endif
@@ -876,7 +879,9 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
 #pragma unroll
       for (int j = 0; j < kJB; ++j) raw[j] = ((okm >> j) & 1u) ? ldraw_b2<Persist>(X + id[j]) : 0u;
     };
-    auto consume = [&](const int32_t (&id)[kJB], const uint32_t (&raw)[kJB], uint32_t okm) {
+    uint32_t lvb = 0;  // SGR_DEFER_COMPACT: live bit of slot 32 (kJB bb + j) + lane at kJB bb + j
+    auto consume = [&](int bb, const int32_t (&id)[kJB], const uint32_t (&raw)[kJB], uint32_t okm) {
+      (void)bb;
 #pragma unroll
       for (int j = 0; j < kJB; ++j) {
         bool live = false;
@@ -892,11 +897,15 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
           if (!live) set_add(tbl_drop, ci);
           conf |= (int32_t)(raw[j] & kColorMask) == xv && lose<TB>(v, id[j]);
         }
+#if SGR_DEFER_COMPACT
+        lvb |= live ? (1u << (kJB * bb + j)) : 0u;
+#else
         // compaction in window order (the list stays sorted): a live entry's position is
         // at most its own slot, and every lane already holds this batch's ids
         const unsigned bal = __ballot_sync(0xffffffffu, live);
         if (live) sbuf[lpos + __popc(bal & lt_mask)] = id[j];
         lpos += (uint32_t)__popc(bal);
+#endif
       }
     };
 #else
@@ -920,7 +929,8 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
 #pragma unroll
       for (int j = 0; j < kJB; ++j) raw[j] = ((okm >> j) & 1u) ? ldraw<Persist>(X + id[j]) : 0u;
     };
-    auto consume = [&](const int32_t (&id)[kJB], const uint32_t (&raw)[kJB], uint32_t okm) {
+    auto consume = [&](int bb, const int32_t (&id)[kJB], const uint32_t (&raw)[kJB], uint32_t okm) {
+      (void)bb;
       uint32_t lb = 0;  // live bits of this batch
 #pragma unroll
       for (int j = 0; j < kJB; ++j) {
@@ -959,7 +969,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
       fetch(0, id, raw, okm);
       for (int bb = 0; bb < nb; ++bb) {
         if (bb + 1 < nb) fetch(bb + 1, idn, rawn, okmn);
-        consume(id, raw, okm);
+        consume(bb, id, raw, okm);
 #pragma unroll
         for (int j = 0; j < kJB; ++j) {
           id[j] = idn[j];
@@ -974,7 +984,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
       uint32_t raw[kJB];
       uint32_t okm;
       fetch(bb, id, raw, okm);
-      consume(id, raw, okm);
+      consume(bb, id, raw, okm);
     }
 #endif
 #if !SGR_NO_TMA
@@ -987,9 +997,31 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
     }
     __syncwarp();
     const bool any = __any_sync(0xffffffffu, conf);
+#if SGR_DEFER_COMPACT && SGR_SLAYOUT
+    // live entries counted from the per-lane bits; the stage is compacted (in place, window
+    // order, one ballot per 32 slots) only when the list is actually rewritten
+    const uint32_t live_total = __reduce_add_sync(0xffffffffu, (uint32_t)__popc(lvb));
+    auto compact = [&]() {
+      uint32_t pos = 0;
+      for (int bb = 0; bb < nb; ++bb) {
+#pragma unroll
+        for (int j = 0; j < kJB; ++j) {
+          const bool lv = (lvb >> (kJB * bb + j)) & 1u;
+          const int32_t id = sbuf[32 * (kJB * bb + j) + lane];
+          const unsigned bal = __ballot_sync(0xffffffffu, lv);
+          if (lv) sbuf[pos + __popc(bal & lt_mask)] = id;  // <= its own slot: already read
+          pos += (uint32_t)__popc(bal);
+        }
+      }
+      __syncwarp();
+    };
+#else
     const uint32_t live_total = lpos;
+    auto compact = [&]() {};
+#endif
     // the compacted live list (front of the stage) to global memory, coalesced
     auto write_live = [&](int32_t* base) {
+      compact();
       for (uint32_t q = lane; q < live_total; q += 32) base[q] = sbuf[q];
     };
 
