@@ -80,6 +80,9 @@ static_assert(!SGR_CLRMAX || SGR_SLAYOUT, "SGR_CLRMAX tracks the largest color i
 #ifndef SGR_ROWPF
 #define SGR_ROWPF 0  // bin 0: prefetch the row two steps ahead (1 = into L2, 2 = into L1)
 #endif
+#ifndef SGR_HUB_B0T
+#define SGR_HUB_B0T 0  // hub build: thread-per-vertex bin 0
+#endif
 #ifndef SGR_BIN0_THREAD
 #define SGR_BIN0_THREAD 0  // bin 0: one thread per vertex (else 4-lane groups)
 #endif
@@ -1490,7 +1493,7 @@ __device__ __forceinline__ void bin0_thread(const RoundArgs<C>& a, int k, const 
       lb |= (((vm >> r) & 1ull) && lose<TB>(v, id[r])) ? (1ull << r) : 0ull;
     int32_t c[4 * kQ];
 #pragma unroll
-    for (int r = 0; r < 4 * kQ; ++r) c[r] = ((vm >> r) & 1ull) ? ldc<Persist>(X + id[r]) : 0;
+    for (int r = 0; r < 4 * kQ; ++r) c[r] = ((vm >> r) & 1ull) ? ldc01<Persist, Hub>(X + id[r]) : 0;
     const int64_t sn = vn >= 0 ? ldg_i64(a.row_ptr + vn) : 0;
     const int64_t en = vn >= 0 ? ldg_i64(a.row_ptr + vn + 1) : 0;
     bool conf = false;
@@ -1727,14 +1730,18 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, const C
   };
   auto run_bin0 = [&]() {
     // ---- bin 0: eight vertices per warp, register masks
-  #if SGR_BIN0_THREAD
-    bin0_thread<TB, Persist, C, Hub>(
-  #else
-    bin0<TB, Persist, C, Hub>(
-  #endif
-        a, k, sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]),
-        w.t, sel(p ^ 1, a.wl_t[0], a.wl_t[1]), &ctrl->ring[rs(k + 1)].t, X, Y,
-        wsm, gw, NW, lane, edges[0], entries[0]);
+    // thread per vertex (SGR_BIN0_THREAD; SGR_HUB_B0T: in the hub build only, where the
+    // small rows are scattered and short) or 4-lane groups
+    if constexpr (SGR_BIN0_THREAD || (Hub && SGR_HUB_B0T))
+      bin0_thread<TB, Persist, C, Hub>(
+          a, k, sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]),
+          w.t, sel(p ^ 1, a.wl_t[0], a.wl_t[1]), &ctrl->ring[rs(k + 1)].t, X, Y,
+          wsm, gw, NW, lane, edges[0], entries[0]);
+    else
+      bin0<TB, Persist, C, Hub>(
+          a, k, sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]),
+          w.t, sel(p ^ 1, a.wl_t[0], a.wl_t[1]), &ctrl->ring[rs(k + 1)].t, X, Y,
+          wsm, gw, NW, lane, edges[0], entries[0]);
   };
   // Order within the pass. Default 2, 1, 0: the large chunk items first (claimed from a
   // cursor), the static small-vertex bins fill the tail. SGR_SMALL_FIRST: 0, 1, 2 (the
