@@ -470,8 +470,33 @@ __global__ void __launch_bounds__(256) k_first(RoundArgs<C> a, int sorted) {
     }
     const int b = bin_of(e - s, a.small_max, a.med_max);
     Counts* w2 = &ctrl->ring[rs(2)];
-    warp_push(conflict && b == 0, v, a.wl_t[0], &w2->t);
-    warp_push(conflict && b == 1, v, a.wl_m[0], &w2->m);
+    {  // bins 0/1: one atomicAdd per BLOCK and bin (~40 % of all vertices enter W_2, so
+       // per-warp atomics on the two list counters serialize over the whole grid)
+      __shared__ int32_t fcnt[2][kWarps], fbase[2][kWarps];
+      const int wid = threadIdx.x >> 5;
+      const unsigned m0 = __ballot_sync(0xffffffffu, conflict && b == 0);
+      const unsigned m1 = __ballot_sync(0xffffffffu, conflict && b == 1);
+      if (lane == 0) {
+        fcnt[0][wid] = __popc(m0);
+        fcnt[1][wid] = __popc(m1);
+      }
+      __syncthreads();
+      if (threadIdx.x < 2) {
+        const int q = threadIdx.x;
+        int32_t run = 0;
+        for (int w = 0; w < (int)(blockDim.x >> 5); ++w) {
+          fbase[q][w] = run;
+          run += fcnt[q][w];
+        }
+        const int32_t b0 = run ? atomicAdd(q == 0 ? &w2->t : &w2->m, run) : 0;
+        for (int w = 0; w < (int)(blockDim.x >> 5); ++w) fbase[q][w] += b0;
+      }
+      __syncthreads();
+      const unsigned lt = (1u << lane) - 1u;
+      if (conflict && b == 0) a.wl_t[0][fbase[0][wid] + __popc(m0 & lt)] = v;
+      if (conflict && b == 1) a.wl_m[0][fbase[1][wid] + __popc(m1 & lt)] = v;
+      __syncthreads();  // fcnt / fbase are rewritten by the next iteration
+    }
     // bin 2: ceil(deg / kChunk) items per vertex and an accumulator slot
     const bool big = conflict && b == 2;
     const int32_t nch = big ? num_chunks(e - s) : 0;
