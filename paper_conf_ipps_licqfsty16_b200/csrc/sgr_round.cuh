@@ -16,9 +16,11 @@
 //          flight, u64 register mask per lane, OR-reduced in-group
 //   bin 1  deg <= med_max (<= 256): 8 lanes per vertex, <= 32 entries per lane, 512-byte
 //          forbidden table (one byte per color) in shared memory
-//   bin 2  larger rows, one warp per chunk of <= kChunk entries. A vertex with several
-//          chunks merges the chunks' 1024-bit partial sets with atomicOr and the last chunk
-//          to finish (atomic ticket) decides conflict and first fit.
+//   bin 2  larger rows, one warp per chunk of <= kChunk entries of the vertex's (trimmed)
+//          list, staged into shared memory by TMA; lane L gathers slots 32 j + L, so one
+//          gather instruction reads 32 consecutive (sorted) neighbours. A vertex with several
+//          chunks merges the chunks' 1024-bit partial sets with atomicOr and is decided in a
+//          finalize phase after a grid barrier (one lane per vertex).
 //
 // Live-neighbour trimming (bin 2, packed colors; DESIGN.md §3 proof (vii)): a neighbour
 // that has left the worklist never changes color again. Colors are stored as 16-bit words
@@ -30,7 +32,10 @@
 // of the neighbours it has dropped; every pass reads the current list, drops the neighbours
 // that are no longer live (their colors go to F), and writes the compacted list for the
 // next round. Conflict and first fit are computed from F ∪ {colors of the listed
-// neighbours}, exactly the colors of all neighbours. The chunk windows of the lists are
+// neighbours}, exactly the colors of all neighbours. Lists may also keep neighbours that
+// have left W (that is the untrimmed semantics), so they are only rewritten when more than
+// 1/16 of their entries are dead (single chunk: in place; several chunks: a keep bit per
+// item, decided in the finalize phase). The chunk windows of the lists are
 // staged into shared memory with TMA bulk copies (cp.async.bulk, mbarrier completion),
 // double-buffered per warp so the next chunk streams in while the current chunk's gathers
 // are in flight.
@@ -49,9 +54,6 @@ constexpr int kJB = 4 * kQB;  // entries per lane per batch
 #ifndef SGR_NO_TMA
 #define SGR_NO_TMA 0
 #endif
-#ifndef SGR_SLAYOUT
-#define SGR_SLAYOUT 1  // bin 2: lane-consecutive window slots (see bin2_trimmed)
-#endif
 #ifndef SGR_LAZY
 #define SGR_LAZY 4  // bin 2 single-chunk lists: rewrite only if > cnt >> SGR_LAZY entries dropped
 #endif
@@ -61,33 +63,17 @@ constexpr int kJB = 4 * kQB;  // entries per lane per batch
 #ifndef SGR_MCLAZY_SHIFT
 #define SGR_MCLAZY_SHIFT 4  // dead-entry threshold: len >> SGR_MCLAZY_SHIFT
 #endif
-#ifndef SGR_DEFER_COMPACT
-#define SGR_DEFER_COMPACT 1  // bin 2: live bits per lane; compact the stage only when rewriting
-#endif
 #ifndef SGR_CLRMAX
 #define SGR_CLRMAX 1  // bin 2: clear the chunk's tables only up to the largest color seen
 #endif
-static_assert(!SGR_CLRMAX || SGR_SLAYOUT, "SGR_CLRMAX tracks the largest color in the SLAYOUT batch loop");
 #ifndef SGR_SMALL_FIRST
 #define SGR_SMALL_FIRST 0  // pass order 0, 1, 2 instead of 2, 1, 0
-#endif
-#ifndef SGR_BAR2
-#define SGR_BAR2 1  // grid barrier on a monotonic arrival counter (no reset/release step)
-#endif
-#ifndef SGR_BIN1_PIPE
-#define SGR_BIN1_PIPE 0  // bin 1: flattened (vertex, batch) steps, next row in flight
-#endif
-#ifndef SGR_ROWPF
-#define SGR_ROWPF 0  // bin 0: prefetch the row two steps ahead (1 = into L2, 2 = into L1)
 #endif
 #ifndef SGR_HUB_B0T
 #define SGR_HUB_B0T 0  // hub build: thread-per-vertex bin 0
 #endif
 #ifndef SGR_BIN0_THREAD
 #define SGR_BIN0_THREAD 0  // bin 0: one thread per vertex (else 4-lane groups)
-#endif
-#ifndef SGR_XPIPE
-#define SGR_XPIPE 0  // bin 2: next batch's gathers in flight while this batch is consumed
 #endif
 
 namespace sgr {
@@ -403,24 +389,8 @@ __device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t
 
 // Row entries of bins 0 and 1 (streamed once per pass). SGR_ROWNA: bypass L1 allocation,
 // leaving L1 to the color gathers.
-// Row entries in the flat build (no hubs: stencils, ER) with an L2 evict-last policy
-// (SGR_ROWEL): W stays close to V for many rounds on stencils, so the rows read in one pass
-// are read again in the next; evict-last keeps them in L2 ahead of streaming traffic.
-#ifndef SGR_ROWEL
-#define SGR_ROWEL 0
-#endif
 template <bool Hub>
-__device__ __forceinline__ int32_t ld_row_h(const int32_t* p) {
-  if constexpr (!Hub && SGR_ROWEL) {
-    uint64_t pol;
-    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
-    int32_t r;
-    asm volatile("ld.global.nc.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
-    return r;
-  } else {
-    return __ldg(p);
-  }
-}
+__device__ __forceinline__ int32_t ld_row_h(const int32_t* p) { return __ldg(p); }
 __device__ __forceinline__ int32_t ld_row(const int32_t* p) {
 #if SGR_ROWNA
   int32_t r;
@@ -895,16 +865,12 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
     const long long tb = clock64();
     pc1 += (unsigned long long)(tb - ta);
 #endif
-    const int4* b4 = reinterpret_cast<const int4*>(bufs + st * (kStage / 4));
-    (void)b4;
     // live entries are compacted into the front of this stage as the batches go (a batch's
     // outputs land below its own slots, whose ids every lane already holds in registers)
     int32_t* sbuf = bufs + st * (kStage / 4);
     bool conf = false;
-    uint32_t lpos = 0;  // warp-uniform: live entries of the finished batches
     uint32_t cmax = 0;  // SGR_CLRMAX: largest table index this lane set
     const unsigned lt_mask = (1u << lane) - 1u;
-#if SGR_SLAYOUT
     // batch bb: window slots 32 (kJB bb + j) + lane, j < kJB: consecutive lanes read
     // consecutive (sorted) list entries, so neighbours close in id share a cache line
     // within one gather instruction
@@ -919,7 +885,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
 #pragma unroll
       for (int j = 0; j < kJB; ++j) raw[j] = ((okm >> j) & 1u) ? ldraw_b2<Persist>(X + id[j]) : 0u;
     };
-    uint32_t lvb = 0;  // SGR_DEFER_COMPACT: live bit of slot 32 (kJB bb + j) + lane at kJB bb + j
+    uint32_t lvb = 0;  // live bit of window slot 32 (kJB bb + j) + lane, at bit kJB bb + j
     auto consume = [&](int bb, const int32_t (&id)[kJB], const uint32_t (&raw)[kJB], uint32_t okm) {
       (void)bb;
 #pragma unroll
@@ -937,88 +903,9 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
           if (!live) set_add(tbl_drop, ci);
           conf |= (int32_t)(raw[j] & kColorMask) == xv && lose<TB>(v, id[j]);
         }
-#if SGR_DEFER_COMPACT
         lvb |= live ? (1u << (kJB * bb + j)) : 0u;
-#else
-        // compaction in window order (the list stays sorted): a live entry's position is
-        // at most its own slot, and every lane already holds this batch's ids
-        const unsigned bal = __ballot_sync(0xffffffffu, live);
-        if (live) sbuf[lpos + __popc(bal & lt_mask)] = id[j];
-        lpos += (uint32_t)__popc(bal);
-#endif
       }
     };
-#else
-    // batch bb: this lane's kJB window slots (kQB int4 of the stage) and their gathers
-    auto fetch = [&](int bb, int32_t (&id)[kJB], uint32_t (&raw)[kJB], uint32_t& okm) {
-      okm = 0;
-#pragma unroll
-      for (int qq = 0; qq < kQB; ++qq) {
-        const int q = kQB * bb + qq;
-        const int4 t4 = b4[lane + 32 * q];
-        id[4 * qq + 0] = t4.x;
-        id[4 * qq + 1] = t4.y;
-        id[4 * qq + 2] = t4.z;
-        id[4 * qq + 3] = t4.w;
-        {  // slots [r0, r0 + 4) of this int4 against the valid range [off0, nslots)
-          const int32_t r0 = 4 * (lane + 32 * q);
-          const int32_t lo = max(off0 - r0, 0), hi = min(nslots - r0, 4);
-          okm |= lo < hi ? (((1u << hi) - 1u) & ~((1u << lo) - 1u)) << (4 * qq) : 0u;
-        }
-      }
-#pragma unroll
-      for (int j = 0; j < kJB; ++j) raw[j] = ((okm >> j) & 1u) ? ldraw<Persist>(X + id[j]) : 0u;
-    };
-    auto consume = [&](int bb, const int32_t (&id)[kJB], const uint32_t (&raw)[kJB], uint32_t okm) {
-      (void)bb;
-      uint32_t lb = 0;  // live bits of this batch
-#pragma unroll
-      for (int j = 0; j < kJB; ++j) {
-        if ((okm >> j) & 1u) {
-          // colors >= 1023 are clamped onto byte 1023; a first fit of 1023 or more is
-          // recomputed exactly from the full row (warp_first_fit_rescan)
-          const uint32_t ci = min(raw[j] & kColorMask, (uint32_t)(kBigTbl - 1));
-          const bool live = (raw[j] >> kRoundShift) == klive;
-          set_add(tbl_all, ci);
-          if (!live) set_add(tbl_drop, ci);
-          conf |= (int32_t)(raw[j] & kColorMask) == xv && lose<TB>(v, id[j]);
-          lb |= live ? (1u << j) : 0u;
-        }
-      }
-      // positions: lane-major within the batch (the list is a set; order is free). They
-      // land below the batch's own slots, never on a later batch's.
-      const uint32_t c8 = (uint32_t)__popc(lb);
-      uint32_t incl = c8;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t t = __shfl_up_sync(0xffffffffu, incl, o);
-        if (lane >= o) incl += t;
-      }
-      uint32_t pos = lpos + incl - c8;
-#pragma unroll
-      for (int j = 0; j < kJB; ++j)
-        if ((lb >> j) & 1u) sbuf[pos++] = id[j];
-      lpos += __shfl_sync(0xffffffffu, incl, 31);
-    };
-#endif
-#if SGR_XPIPE
-    {  // the next batch's slots are read and its gathers issued before this batch is consumed
-      int32_t id[kJB], idn[kJB];
-      uint32_t raw[kJB], rawn[kJB];
-      uint32_t okm, okmn = 0;
-      fetch(0, id, raw, okm);
-      for (int bb = 0; bb < nb; ++bb) {
-        if (bb + 1 < nb) fetch(bb + 1, idn, rawn, okmn);
-        consume(bb, id, raw, okm);
-#pragma unroll
-        for (int j = 0; j < kJB; ++j) {
-          id[j] = idn[j];
-          raw[j] = rawn[j];
-        }
-        okm = okmn;
-      }
-    }
-#else
     for (int bb = 0; bb < nb; ++bb) {
       int32_t id[kJB];
       uint32_t raw[kJB];
@@ -1026,7 +913,6 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
       fetch(bb, id, raw, okm);
       consume(bb, id, raw, okm);
     }
-#endif
 #if !SGR_NO_TMA
     const long long tc = clock64();
     pc2 += (unsigned long long)(tc - tb);
@@ -1037,7 +923,6 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
     }
     __syncwarp();
     const bool any = __any_sync(0xffffffffu, conf);
-#if SGR_DEFER_COMPACT && SGR_SLAYOUT
     // live entries counted from the per-lane bits; the stage is compacted (in place, window
     // order, one ballot per 32 slots) only when the list is actually rewritten
     const uint32_t live_total = __reduce_add_sync(0xffffffffu, (uint32_t)__popc(lvb));
@@ -1055,10 +940,6 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
       }
       __syncwarp();
     };
-#else
-    const uint32_t live_total = lpos;
-    auto compact = [&]() {};
-#endif
     // the compacted live list (front of the stage) to global memory, coalesced
     auto write_live = [&](int32_t* base) {
       compact();
@@ -1453,15 +1334,6 @@ __device__ __forceinline__ void bin0(const RoundArgs<C>& a, int k, const int32_t
     push_buffered<kPushBufOf<Hub>>(v >= 0 && any && gl == 0, v, pbuf, pending, out, out_cnt, lane);
     const int64_t s2 = v2 >= 0 ? ldg_i64(a.row_ptr + v2) : 0;
     const int64_t e2 = v2 >= 0 ? ldg_i64(a.row_ptr + v2 + 1) : 0;
-#if SGR_ROWPF
-    {  // warm the row two steps ahead (<= 128 bytes: its first and last line)
-      const int32_t* pf = gl == 0 ? a.col_idx + s2 : a.col_idx + e2 - 1;
-      if (gl < 2 && e2 > s2) {
-        if (SGR_ROWPF == 1) prefetch_l2(pf);
-        else prefetch_l1(pf);
-      }
-    }
-#endif
     i += step;
     v = v1;
     s = s1;
@@ -1591,117 +1463,6 @@ __device__ __forceinline__ void bin1(const RoundArgs<C>& a, int k, const int32_t
   push_flush(pbuf, pending, out, out_cnt, lane);
 }
 
-// Bin 1, software-pipelined (SGR_BIN1_PIPE): every 8-lane group walks a flattened stream of
-// (vertex, 64-entry batch) steps; while one step's color gathers are in flight the next
-// step's row entries (the same vertex's next batch, or the next vertex's first) are loaded,
-// so each batch costs one dependent round trip instead of two. Groups finish vertices at
-// different steps: the finish (group ballot, first fit from the group's table, Y write,
-// table clear) runs inside the step loop for the groups whose vertex ended.
-template <int TB, bool Persist, class C, bool Hub>
-__device__ __forceinline__ void bin1_pipe(const RoundArgs<C>& a, int k, const int32_t* list,
-                                          int nX, int32_t* out, int32_t* out_cnt, const C* X,
-                                          C* Y, uint8_t* wsm, int gw, int NW, int lane,
-                                          unsigned long long& edges,
-                                          unsigned long long& entries) {
-  if (gw * 4 >= nX) return;
-  const int g = lane >> 3, gl = lane & 7;
-  const unsigned gmask = 0xffu << (g * 8);
-  uint8_t* gtbl = wsm + WarpSmem<C, Hub>::kBuf + g * kMedTblB;
-  int32_t* pbuf = reinterpret_cast<int32_t*>(wsm + WarpSmem<C, Hub>::kPush);
-  int pending = 0;
-  const int step = NW * 4;
-  auto load_batch = [&](int64_t s, int32_t cnt, int32_t bb, int32_t (&w)[8]) {
-#pragma unroll
-    for (int u = 0; u < 8; ++u) {
-      const int32_t r = 64 * bb + gl + kGroup * u;
-      w[u] = r < cnt ? ld_row(a.col_idx + s + r) : -1;
-    }
-  };
-  // the group's current vertex and, prefetched, its next one
-  int i = gw * 4 + g;
-  int32_t v = i < nX ? ld_cg(list + i) : -1;
-  int64_t s = v >= 0 ? ldg_i64(a.row_ptr + v) : 0, e = v >= 0 ? ldg_i64(a.row_ptr + v + 1) : 0;
-  int32_t vn = i + step < nX ? ld_cg(list + i + step) : -1;
-  int64_t sn = vn >= 0 ? ldg_i64(a.row_ptr + vn) : 0, en = vn >= 0 ? ldg_i64(a.row_ptr + vn + 1) : 0;
-  int32_t cnt = (int32_t)(e - s), bb = 0;
-  int32_t w[8];
-  load_batch(s, cnt, 0, w);
-  int32_t xv = v >= 0 ? ldc<Persist>(X + v) : 0;
-  bool conf = false;
-  while (__any_sync(0xffffffffu, v >= 0)) {
-    uint32_t lb = 0;
-#pragma unroll
-    for (int u = 0; u < 8; ++u) lb |= (w[u] >= 0 && lose<TB>(v, w[u])) ? (1u << u) : 0u;
-    int32_t c[8];
-#pragma unroll
-    for (int u = 0; u < 8; ++u) c[u] = w[u] >= 0 ? ldc01<Persist, Hub>(X + w[u]) : -1;  // colors
-    // next step of this group: the same vertex's next batch, or the next vertex's first
-    const bool last = v < 0 || 64 * (bb + 1) >= cnt;
-    if (!last) {
-      load_batch(s, cnt, bb + 1, w);
-    } else if (vn >= 0) {
-      load_batch(sn, (int32_t)(en - sn), 0, w);
-    } else {
-#pragma unroll
-      for (int u = 0; u < 8; ++u) w[u] = -1;
-    }
-#pragma unroll
-    for (int u = 0; u < 8; ++u) {
-      if (c[u] >= 0) {
-        // deg <= 256 => first fit <= 257: colors >= 511 are clamped onto an unused byte
-        set_add(gtbl, (uint32_t)min(c[u], kMedTbl - 1));
-        conf |= c[u] == xv && ((lb >> u) & 1u);
-      }
-    }
-    bool push = false;
-    if (last && v >= 0) {  // finish v (group-converged: all 8 lanes share `last` and v)
-      __syncwarp(gmask);
-      const bool any = (__ballot_sync(gmask, conf) & gmask) != 0u;
-      int32_t tent = 0;
-      if (any) {
-        const uint32_t* t32 = reinterpret_cast<const uint32_t*>(gtbl);
-        for (int it = 0; it < kMedTbl / 32; ++it) {
-          uint32_t word = t32[it * 8 + gl];
-          if (it == 0 && gl == 0) word |= 0xffu;
-          const uint32_t z = __vcmpeq4(word, 0u);
-          const unsigned b = __ballot_sync(gmask, z != 0u) & gmask;
-          if (b) {
-            const int fl = __ffs(b) - 1;
-            const uint32_t zz = __shfl_sync(gmask, z, fl);
-            tent = (it * 8 + (fl & 7)) * 4 + (__ffs(zz) - 1) / 8;
-            break;
-          }
-        }
-      }
-      set_clear(gtbl, kMedTblB, gl, kGroup);
-      __syncwarp(gmask);
-      if (gl == 0) {
-        Y[v] = any ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a);
-        edges += (unsigned long long)cnt;
-        entries += (unsigned long long)cnt;
-      }
-      push = any && gl == 0;
-    }
-    push_buffered<kPushBufOf<Hub>>(push, v, pbuf, pending, out, out_cnt, lane);
-    if (last) {  // advance the group to its next vertex; prefetch the one after
-      i += step;
-      v = vn;
-      s = sn;
-      e = en;
-      cnt = (int32_t)(e - s);
-      bb = 0;
-      conf = false;
-      xv = v >= 0 ? ldc<Persist>(X + v) : 0;
-      vn = (v >= 0 && i + step < nX) ? ld_cg(list + i + step) : -1;
-      sn = vn >= 0 ? ldg_i64(a.row_ptr + vn) : 0;
-      en = vn >= 0 ? ldg_i64(a.row_ptr + vn + 1) : 0;
-    } else {
-      ++bb;
-    }
-  }
-  push_flush(pbuf, pending, out, out_cnt, lane);
-}
-
 // One fused pass F_k over all three bins; every warp of the grid calls it. Static
 // round-robin assignment (warp w takes items w, w + NW, ...), with the next item's list
 // entry and row offsets prefetched while the current one is processed.
@@ -1757,11 +1518,7 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, const C
   };
   auto run_bin1 = [&]() {
     // ---- bin 1: four vertices per warp (one per 8-lane group), 512-byte tables
-  #if SGR_BIN1_PIPE
-    bin1_pipe<TB, Persist, C, Hub>(
-  #else
     bin1<TB, Persist, C, Hub>(
-  #endif
         a, k, sel(p, (const int32_t*)a.wl_m[0], (const int32_t*)a.wl_m[1]),
         w.m, sel(p ^ 1, a.wl_m[0], a.wl_m[1]), &ctrl->ring[rs(k + 1)].m, X, Y,
         wsm, gw, NW, lane, edges[1], entries[1]);
@@ -2058,7 +1815,6 @@ __device__ __forceinline__ uint32_t atom_add_acq_rel_u32(uint32_t* p, uint32_t v
 }
 
 // Grid-wide barrier of the persistent kernel (every block resident).
-#if SGR_BAR2
 // Monotonic arrival counter (zeroed per coloring): thread 0 of each block adds 1 with
 // release semantics (publishing, via the preceding bar.sync, every write of its block) and
 // waits with acquire loads until barrier number `epoch` has all gridDim.x arrivals. No
@@ -2080,26 +1836,6 @@ __device__ __forceinline__ void grid_sync(Ctrl* ctrl, uint32_t& epoch) {
   }
   __syncthreads();
 }
-#else
-// Thread 0 of each block arrives with an acq_rel atomic (publishing, via the preceding
-// bar.sync, every write of its block); the last arrival resets the count and releases the
-// new generation.
-__device__ __forceinline__ void grid_sync(Ctrl* ctrl, uint32_t& epoch) {
-  (void)epoch;
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    const uint32_t gen = ld_acquire_gpu(&ctrl->bar_gen);
-    const uint32_t arrived = atom_add_acq_rel_u32(&ctrl->bar_count, 1u);
-    if (arrived == gridDim.x - 1) {
-      ctrl->bar_count = 0u;
-      st_release_gpu(&ctrl->bar_gen, gen + 1u);
-    } else {
-      while (ld_acquire_gpu(&ctrl->bar_gen) == gen) __nanosleep(20);
-    }
-  }
-  __syncthreads();
-}
-#endif
 
 // All rounds in one cooperative launch (every block resident). Each block tracks k itself
 // and reads W_k's counts after the barrier that ends pass k-1; block 0 folds pass k-1 into
@@ -2116,7 +1852,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks<C, Hub>) k_persistent(Round
   uint32_t ph = 0;  // mbarrier phase bits of the warp's two TMA stages
   unsigned long long cyc[kBins] = {0, 0, 0};
   unsigned long long pcx[3] = {0, 0, 0};  // barrier waits, finalize, counter reduction
-  uint32_t epoch = 0;                     // grid barriers passed (SGR_BAR2)
+  uint32_t epoch = 0;                     // grid barriers passed
   const int max_rounds = ld_cg(&ctrl->max_rounds);
   // the last block folds the finished pass: it is the one that draws work last (items go to
   // the lowest warp ids first), so the fold is off the critical path of thin rounds
