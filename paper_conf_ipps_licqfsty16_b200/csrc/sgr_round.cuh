@@ -162,7 +162,8 @@ struct alignas(32) Counts {
   int32_t c;                 // bin 2 chunk items
   int32_t cv;                // bin 2 vertices
   int32_t fin;               // pass k: multi-chunk bin-2 vertices awaiting the finalize phase
-  int32_t pad[3];            // pad[0]: pass k's bin-2 work cursor
+  int32_t pad[3];            // pad[0]: pass k's bin-2 work cursor; pad[1]: multi-chunk
+                             // vertices in W_k (0: pass k needs no finalize phase)
 };
 // W_k's counts live in ring slot k % 3: pass k reads slot k % 3 and pushes W_{k+1} into
 // slot (k+1) % 3, while slot (k+2) % 3 (W_{k-1}, read by the finished pass k-1) is folded
@@ -499,9 +500,11 @@ __global__ void __launch_bounds__(256) k_first(RoundArgs<C> a, int sorted) {
       }
       const int total = __shfl_sync(0xffffffffu, incl, 31);
       int ib = 0;
+      const unsigned mmc = __ballot_sync(0xffffffffu, nch > 1);
       if (lane == 0) {
         ib = atomicAdd(&w2->c, total);
         atomicAdd(&w2->cv, __popc(mb));
+        if (mmc) atomicAdd(&w2->pad[1], __popc(mmc));
       }
       ib = __shfl_sync(0xffffffffu, ib, 0) + incl - nch;
       for (int32_t t = 0; t < nch; ++t) a.wl_c[0][ib + t] = make_item(v, t);
@@ -1078,7 +1081,7 @@ __device__ __forceinline__ void finalize_body(const RoundArgs<Packed>& a, int k)
   const int B = min(32, (nF + NW - 1) / NW);
   // every warp runs the same number of iterations (block-level aggregation below)
   const int iters = nF > 0 ? (nF + NW * B - 1) / (NW * B) : 0;
-  __shared__ int32_t fin_tot[2][kWarps];   // per warp: items, vertices
+  __shared__ int32_t fin_tot[3][kWarps];   // per warp: items, vertices, multi-chunk vertices
   __shared__ int32_t fin_base[kWarps];
   const int wid = threadIdx.x >> 5;
   for (int it = 0; it < iters; ++it) {
@@ -1133,20 +1136,24 @@ __device__ __forceinline__ void finalize_body(const RoundArgs<Packed>& a, int k)
     const unsigned cm = __ballot_sync(0xffffffffu, conf);
     // item slots: one atomicAdd per BLOCK and counter (every warp of the grid finalizes at
     // the same moment, so per-warp atomics on two hot addresses would serialize)
+    const unsigned mmc = __ballot_sync(0xffffffffu, nch2 > 1);  // multi-chunk next pass
     if (lane == 0) {
       fin_tot[0][wid] = total;
       fin_tot[1][wid] = (int32_t)__popc(cm);
+      fin_tot[2][wid] = (int32_t)__popc(mmc);
     }
     __syncthreads();
     if (threadIdx.x == 0) {
-      int32_t run = 0, vs = 0;
+      int32_t run = 0, vs = 0, mc = 0;
       for (int q = 0; q < kWarps; ++q) {
         fin_base[q] = run;
         run += fin_tot[0][q];
         vs += fin_tot[1][q];
+        mc += fin_tot[2][q];
       }
       const int32_t b0 = run ? atomicAdd(&ctrl->ring[rs(k + 1)].c, run) : 0;
       if (vs) atomicAdd(&ctrl->ring[rs(k + 1)].cv, vs);
+      if (mc) atomicAdd(&ctrl->ring[rs(k + 1)].pad[1], mc);
       for (int q = 0; q < kWarps; ++q) fin_base[q] += b0;
     }
     __syncthreads();
@@ -1877,10 +1884,14 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks<C, Hub>) k_persistent(Round
     block_add6(edges, entries, ctrl, k);
     const long long t1 = clock64();
     pcx[2] += (unsigned long long)(t1 - t0);
-    if constexpr (packed<C>() && Hub) {  // multi-chunk vertices: decided once all chunks are in
+    // multi-chunk vertices: decided once all chunks are in (no finalize phase, and no
+    // barrier for it, when W_k has none — most thin rounds of a skewed graph's tail)
+    bool fin_phase = false;
+    if constexpr (packed<C>() && Hub) fin_phase = w.pad[1] != 0;  // uniform over the grid
+    if (fin_phase) {
       grid_sync(ctrl, epoch);
       const long long t2 = clock64();
-      finalize_body<TB, true>(a, k);
+      if constexpr (packed<C>() && Hub) finalize_body<TB, true>(a, k);
       const long long t3 = clock64();
       pcx[0] += (unsigned long long)(t2 - t1);
       pcx[1] += (unsigned long long)(t3 - t2);
