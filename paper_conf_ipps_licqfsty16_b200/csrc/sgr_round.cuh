@@ -100,6 +100,8 @@ constexpr int kPushBufOf = Hub ? SGR_PUSHBUF : SGR_PUSHBUF_FLAT;
 constexpr int kPushBuf = SGR_PUSHBUF;
 constexpr int kK1 = 32;                 // entries per lane, bin 1 (8 x 32 = 256)
 constexpr int kMaxMed = kGroup * kK1;   // 256
+constexpr int kTile0 = 8;               // bin-0 tiles: <= 8 steps of 8 vertices
+constexpr int kTile1 = 4;               // bin-1 tiles: <= 4 steps of 4 vertices
 // Forbidden-color sets in shared memory: SGR_BITTBL = 1 one bit per color (shared atomicOr),
 // 0 one byte per color (plain byte stores). Bit sets leave more of the SM's unified
 // L1/shared storage to the L1 cache that serves the color gathers.
@@ -195,6 +197,7 @@ struct Ctrl {
   unsigned long long items_total;
   unsigned long long list_writes_total;   // compacted list entries written (bin 2, packed)
   unsigned long long bin_cycles[kBins];   // warp-cycles spent in each bin (SM clock)
+  int32_t tile_cur[3][2];                // per ring slot: bin-0 / bin-1 tile cursors
   unsigned long long phase_cycles[8];     // bin 2 (trimmed) phases: issue, wait, gather, post;
                                           // [4] grid barriers, [5] finalize, [6] counters
   int32_t* round_sizes;
@@ -1283,6 +1286,40 @@ __device__ __forceinline__ void push_flush(int32_t* pbuf, int& pending, int32_t*
   pending = 0;
 }
 
+// Step stream of a warp over a bin-0/1 list (flat build): tiles of kT steps of VPW list
+// positions; a warp's first tile is its own (gw), later ones come from a per-pass cursor,
+// each claimed one tile ahead (so the atomic's latency is never waited for). Warps that
+// spent long on bin 2 take fewer small-vertex tiles: the pass ends together.
+template <int VPW>
+struct StepStream {
+  int tile, j, next;   // warp-uniform except `next` (lane 0's claim, broadcast at use)
+  int ntiles, kT;
+  int* cursor;
+  int NW;
+  // tiles of kT <= kTmax steps; short lists get kT = 1 (one step per warp first, as many
+  // first tiles as warps) so thin passes spread over the grid
+  __device__ __forceinline__ void init(int gw, int nW, int nX, int kTmax, int* cur, int lane) {
+    NW = nW;
+    cursor = cur;
+    kT = max(1, min(kTmax, nX / (NW * VPW)));
+    ntiles = (nX + kT * VPW - 1) / (kT * VPW);
+    tile = gw;
+    j = 0;
+    next = ntiles;
+    if (lane == 0 && tile < ntiles) next = NW + atomicAdd(cursor, 1);
+  }
+  // list position of the current step's first vertex (0x7fffffff: done)
+  __device__ __forceinline__ int base() const { return tile < ntiles ? (tile * kT + j) * VPW : 0x7fffffff; }
+  __device__ __forceinline__ void advance(int lane) {
+    if (++j == kT) {
+      j = 0;
+      tile = __shfl_sync(0xffffffffu, next, 0);
+      next = ntiles;
+      if (lane == 0 && tile < ntiles) next = NW + atomicAdd(cursor, 1);
+    }
+  }
+};
+
 // Bin 0 driver: 4-lane groups, 8 vertices per warp per step; list entries and row offsets
 // prefetched two steps ahead, the row entries one step ahead (so they are in flight while
 // the current vertices' color gathers are), pushes buffered per warp.
@@ -1342,6 +1379,85 @@ __device__ __forceinline__ void bin0(const RoundArgs<C>& a, int k, const int32_t
     const int64_t s2 = v2 >= 0 ? ldg_i64(a.row_ptr + v2) : 0;
     const int64_t e2 = v2 >= 0 ? ldg_i64(a.row_ptr + v2 + 1) : 0;
     i += step;
+    v = v1;
+    s = s1;
+    e = e1;
+#pragma unroll
+    for (int u = 0; u < kK0; ++u) w[u] = wn[u];
+    v1 = v2;
+    s1 = s2;
+    e1 = e2;
+  }
+  push_flush(pbuf, pending, out, out_cnt, lane);
+}
+
+template <int TB, bool Persist, class C, bool Hub>
+__device__ __forceinline__ void bin0_tiled(const RoundArgs<C>& a, int k, const int32_t* list, int nX,
+                                           int* tile_cursor,
+                                     int32_t* out, int32_t* out_cnt, const C* X, C* Y,
+                                     uint8_t* wsm, int gw, int NW, int lane,
+                                     unsigned long long& edges, unsigned long long& entries) {
+  constexpr int G = kG0, VPW = 32 / kG0;
+  if (gw * VPW >= nX) return;
+  const int g = lane / G, gl = lane % G;
+  const unsigned gmask = ((1u << G) - 1u) << (g * G);
+  int32_t* pbuf = reinterpret_cast<int32_t*>(wsm + WarpSmem<C, Hub>::kPush);
+  int pending = 0;
+  const int step = NW * VPW;
+  auto load_row = [&](int32_t vv, int64_t ss, int64_t ee, int32_t (&w)[kK0]) {
+    const int32_t cnt = vv >= 0 ? (int32_t)(ee - ss) : 0;
+    const int32_t* row = a.col_idx + ss;
+#pragma unroll
+    for (int u = 0; u < kK0; ++u) w[u] = (gl + G * u < cnt) ? ld_row_h<Hub>(row + gl + G * u) : -1;
+  };
+  (void)step;
+  StepStream<VPW> gen;  // runs two steps ahead of the step being processed
+  gen.init(gw, NW, nX, kTile0, tile_cursor, lane);
+  auto pos = [&](int b) { return b < nX ? b + g : nX; };
+  int b0 = gen.base();
+  gen.advance(lane);
+  int b1 = gen.base();
+  int i = pos(b0);
+  int32_t v = i < nX ? ld_cg(list + i) : -1;
+  int64_t s = v >= 0 ? ldg_i64(a.row_ptr + v) : 0, e = v >= 0 ? ldg_i64(a.row_ptr + v + 1) : 0;
+  int32_t w[kK0];
+  load_row(v, s, e, w);
+  int32_t v1 = pos(b1) < nX ? ld_cg(list + pos(b1)) : -1;
+  int64_t s1 = v1 >= 0 ? ldg_i64(a.row_ptr + v1) : 0, e1 = v1 >= 0 ? ldg_i64(a.row_ptr + v1 + 1) : 0;
+  while (b0 < nX) {
+    gen.advance(lane);
+    const int b2 = gen.base();
+    const int32_t v2 = pos(b2) < nX ? ld_cg(list + pos(b2)) : -1;
+    const int32_t xv = v >= 0 ? ldc<Persist>(X + v) : 0;
+    uint32_t lb = 0;
+#pragma unroll
+    for (int u = 0; u < kK0; ++u) lb |= (w[u] >= 0 && lose<TB>(v, w[u])) ? (1u << u) : 0u;
+    int32_t c[kK0];
+#pragma unroll
+    for (int u = 0; u < kK0; ++u) c[u] = (w[u] >= 0) ? ldc01<Persist, Hub>(X + w[u]) : 0;
+    int32_t wn[kK0];
+    load_row(v1, s1, e1, wn);  // next vertex's row, in flight with the gathers above
+    bool conf = false;
+    uint32_t mask = 0;  // bit i = color i + 1 present (deg <= 32 => first fit <= 33)
+#pragma unroll
+    for (int u = 0; u < kK0; ++u) {
+      mask |= ((uint32_t)(c[u] - 1) < 32u) ? (1u << (c[u] - 1)) : 0u;
+      conf |= (c[u] == xv) & ((lb >> u) & 1u);
+    }
+#pragma unroll
+    for (int o = G / 2; o > 0; o >>= 1) mask |= __shfl_xor_sync(0xffffffffu, mask, o);
+    const bool any = (__ballot_sync(0xffffffffu, conf) & gmask) != 0u;
+    if (v >= 0 && gl == 0) {
+      const int32_t tent = ~mask ? __ffs(~mask) : 33;
+      Y[v] = any ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a);
+      edges += (unsigned long long)(e - s);
+      entries += (unsigned long long)(e - s);
+    }
+    push_buffered<kPushBufOf<Hub>>(v >= 0 && any && gl == 0, v, pbuf, pending, out, out_cnt, lane);
+    const int64_t s2 = v2 >= 0 ? ldg_i64(a.row_ptr + v2) : 0;
+    const int64_t e2 = v2 >= 0 ? ldg_i64(a.row_ptr + v2 + 1) : 0;
+    b0 = b1;
+    b1 = b2;
     v = v1;
     s = s1;
     e = e1;
@@ -1470,6 +1586,45 @@ __device__ __forceinline__ void bin1(const RoundArgs<C>& a, int k, const int32_t
   push_flush(pbuf, pending, out, out_cnt, lane);
 }
 
+template <int TB, bool Persist, class C, bool Hub>
+__device__ __forceinline__ void bin1_tiled(const RoundArgs<C>& a, int k, const int32_t* list, int nX,
+                                            int* tile_cursor,
+                                      int32_t* out, int32_t* out_cnt, const C* X, C* Y,
+                                      uint8_t* wsm, int gw, int NW, int lane,
+                                      unsigned long long& edges, unsigned long long& entries) {
+  const int g = lane >> 3, gl = lane & 7;
+  const unsigned gmask = 0xffu << (g * 8);
+  uint8_t* gtbl = wsm + WarpSmem<C, Hub>::kBuf + g * kMedTblB;
+  int32_t* pbuf = reinterpret_cast<int32_t*>(wsm + WarpSmem<C, Hub>::kPush);
+  int pending = 0;
+  if (gw * 4 >= nX) return;
+  StepStream<4> gen;  // one step ahead of the step being processed
+  gen.init(gw, NW, nX, kTile1, tile_cursor, lane);
+  int b0 = gen.base();
+  int i = b0 < nX ? b0 + g : nX;
+  int32_t v = i < nX ? ld_cg(list + i) : -1;
+  int64_t s = v >= 0 ? ldg_i64(a.row_ptr + v) : 0, e = v >= 0 ? ldg_i64(a.row_ptr + v + 1) : 0;
+  while (b0 < nX) {
+    gen.advance(lane);
+    const int b1 = gen.base();
+    const int in = b1 < nX ? b1 + g : nX;
+    const int32_t vn = in < nX ? ld_cg(list + in) : -1;
+    const int64_t sn = vn >= 0 ? ldg_i64(a.row_ptr + vn) : 0;
+    const int64_t en = vn >= 0 ? ldg_i64(a.row_ptr + vn + 1) : 0;
+    if (sn + 32 * gl < en) prefetch_l2(a.col_idx + sn + 32 * gl);  // 1 line / lane
+    bool push = false;
+    if (v >= 0 && gl == 0) entries += (unsigned long long)(e - s);
+    process_group<TB, Persist, C, Hub>(a, k, v, s, e, X, Y, gtbl, gl, gmask, push, edges);
+    push_buffered<kPushBufOf<Hub>>(push, v, pbuf, pending, out, out_cnt, lane);
+    b0 = b1;
+    i = in;
+    v = vn;
+    s = sn;
+    e = en;
+  }
+  push_flush(pbuf, pending, out, out_cnt, lane);
+}
+
 // One fused pass F_k over all three bins; every warp of the grid calls it. Static
 // round-robin assignment (warp w takes items w, w + NW, ...), with the next item's list
 // entry and row offsets prefetched while the current one is processed.
@@ -1525,10 +1680,18 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, const C
   };
   auto run_bin1 = [&]() {
     // ---- bin 1: four vertices per warp (one per 8-lane group), 512-byte tables
-    bin1<TB, Persist, C, Hub>(
-        a, k, sel(p, (const int32_t*)a.wl_m[0], (const int32_t*)a.wl_m[1]),
-        w.m, sel(p ^ 1, a.wl_m[0], a.wl_m[1]), &ctrl->ring[rs(k + 1)].m, X, Y,
-        wsm, gw, NW, lane, edges[1], entries[1]);
+    // flat build: tiles claimed from a per-pass cursor (ER -4.7 %); hub build: round-robin
+    // (tiles there: +0.4 % R-MAT s24, +4 % s16)
+    if constexpr (!Hub)
+      bin1_tiled<TB, Persist, C, Hub>(
+          a, k, sel(p, (const int32_t*)a.wl_m[0], (const int32_t*)a.wl_m[1]), w.m,
+          &ctrl->tile_cur[rs(k)][1], sel(p ^ 1, a.wl_m[0], a.wl_m[1]),
+          &ctrl->ring[rs(k + 1)].m, X, Y, wsm, gw, NW, lane, edges[1], entries[1]);
+    else
+      bin1<TB, Persist, C, Hub>(
+          a, k, sel(p, (const int32_t*)a.wl_m[0], (const int32_t*)a.wl_m[1]),
+          w.m, sel(p ^ 1, a.wl_m[0], a.wl_m[1]), &ctrl->ring[rs(k + 1)].m, X, Y,
+          wsm, gw, NW, lane, edges[1], entries[1]);
   };
   auto run_bin0 = [&]() {
     // ---- bin 0: eight vertices per warp, register masks
@@ -1539,6 +1702,11 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, const C
           a, k, sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]),
           w.t, sel(p ^ 1, a.wl_t[0], a.wl_t[1]), &ctrl->ring[rs(k + 1)].t, X, Y,
           wsm, gw, NW, lane, edges[0], entries[0]);
+    else if constexpr (!Hub)
+      bin0_tiled<TB, Persist, C, Hub>(
+          a, k, sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]), w.t,
+          &ctrl->tile_cur[rs(k)][0], sel(p ^ 1, a.wl_t[0], a.wl_t[1]),
+          &ctrl->ring[rs(k + 1)].t, X, Y, wsm, gw, NW, lane, edges[0], entries[0]);
     else
       bin0<TB, Persist, C, Hub>(
           a, k, sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]),
@@ -1652,6 +1820,8 @@ __device__ __forceinline__ void fold_pass(Ctrl* c, int k) {
   }
   atomicAdd(&c->items_total, (unsigned long long)win.c);
   c->ring[rs(k)] = Counts{};
+  c->tile_cur[rs(k)][0] = 0;
+  c->tile_cur[rs(k)][1] = 0;
   if (k - 1 < c->round_cap) {
     if (c->round_sizes) c->round_sizes[k - 1] = tot_in;
     if (c->round_edges) c->round_edges[k - 1] = (int64_t)e_all;
