@@ -160,25 +160,80 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
   for (int32_t c : cnt) total += c;
   if (total > 0) rounds = 2;
   vertices += total;
-  while (status == SGR_OK && total > 0) {
-    if (rounds > r.max_rounds) {
-      set_error("sgr_color_dist: max_rounds (%d) reached", r.max_rounds);
-      status = SGR_ENOCONV;
-      break;
+  // Passes k = 2, 3, ...: the host reads the per-rank counts of W_{k+1} with a lag of
+  // kLag passes (pinned slots + events) instead of blocking after every exchange. The
+  // all-gather capacity comes from the newest counts read so far: they bound every later
+  // round's counts because W only shrinks. Once some W_j is read to be empty no further
+  // passes are issued; the <= kLag already in flight run on empty worklists (no-ops), and
+  // R is taken from the counts, not from the passes issued.
+  constexpr int kLag = 2;
+  int32_t* slots = nullptr;  // [kLag + 1][world][2]
+  cudaEvent_t sev[kLag + 1];
+  for (int q = 0; q <= kLag; ++q) cudaEventCreateWithFlags(&sev[q], cudaEventDisableTiming);
+  if (status == SGR_OK) DCK(cudaMallocHost(&slots, sizeof(int32_t) * 2 * world * (kLag + 1)));
+  int32_t known_cap = status == SGR_OK ? *std::max_element(cnt.begin(), cnt.end()) : 0;
+  bool done = status != SGR_OK || total == 0 || overflow_seen;
+  int64_t issued = 0, consumed = 0;  // passes issued / whose counts were read
+  auto consume_one = [&]() {
+    const int q = (int)(consumed % (kLag + 1));
+    cudaEventSynchronize(sev[q]);
+    ++consumed;
+    if (done) return;  // passes after the end (or an overflow) are no-ops: ignore them
+    int64_t t = 0;
+    int32_t mx = 0;
+    for (int w = 0; w < world; ++w) {
+      t += slots[(q * world + w) * 2];
+      mx = std::max(mx, slots[(q * world + w) * 2]);
+      if (slots[(q * world + w) * 2 + 1]) overflow_seen = true;
     }
-    cap = *std::max_element(cnt.begin(), cnt.end());
+    if (overflow_seen) {  // stop; rerun with int32 words
+      done = true;
+      return;
+    }
+    known_cap = std::min(known_cap, mx);
+    vertices += t;
+    if (t > 0) ++rounds;
+    else done = true;
+  };
+  while (status == SGR_OK && !done) {
+    if (rounds + (issued - consumed) >= r.max_rounds + 1 && !done) {
+      // every pass in flight could still find W non-empty: drain before issuing more
+      while (consumed < issued) consume_one();
+      if (done) break;
+      if (rounds > r.max_rounds) {
+        set_error("sgr_color_dist: max_rounds (%d) reached", r.max_rounds);
+        status = SGR_ENOCONV;
+        break;
+      }
+    }
+    const int32_t cap_k = known_cap;
     for (int i = 0; i < P; ++i) {
       k_round<TB, C><<<grid, kBlock, round_smem<C>(), s>>>(args[i]);
       if constexpr (packed<C>()) k_finalize<TB, C><<<grid, kBlock, 0, s>>>(args[i]);
       k_advance<<<1, 32, 0, s>>>(args[i].ctrl, 0, 1);
+      DCK(cudaMemsetAsync(parts[i].send, 0, sizeof(uint2), s));
+      k_pack<C><<<first_grid(parts[i].hi - parts[i].lo + 1), 256, 0, s>>>(args[i], parts[i].send, cap_k);
     }
     DCK(cudaGetLastError());
-    status = exchange(cap, cnt);
-    total = 0;
-    for (int32_t c : cnt) total += c;
-    vertices += total;
-    if (total > 0) ++rounds;
+    status = gather(parts, recv, cap_k, s);
+    if (status != SGR_OK) break;
+    for (int i = 0; i < P; ++i)
+      k_apply<C><<<first_grid(cap_k), 256, 0, s>>>(args[i], recv, world, cap_k + 1, me0 + i);
+    DCK(cudaGetLastError());
+    const int q = (int)(issued % (kLag + 1));
+    DCK(cudaMemcpy2DAsync(slots + q * world * 2, sizeof(uint2), recv, (size_t)(cap_k + 1) * sizeof(uint2),
+                          sizeof(uint2), world, cudaMemcpyDeviceToHost, s));
+    DCK(cudaEventRecord(sev[q], s));
+    ++issued;
+    if (issued - consumed > kLag) consume_one();
   }
+  while (consumed < issued) consume_one();
+  if (status == SGR_OK && rounds > r.max_rounds) {
+    set_error("sgr_color_dist: max_rounds (%d) reached", r.max_rounds);
+    status = SGR_ENOCONV;
+  }
+  for (int q = 0; q <= kLag; ++q) cudaEventDestroy(sev[q]);
+  if (slots) cudaFreeHost(slots);
   cudaEventRecord(ev1, s);
   if (status == SGR_OK) {
     RoundArgs<C>& a0 = args[0];
