@@ -393,8 +393,21 @@ __device__ __forceinline__ void tma_load_1d(void* dst, const void* src, uint32_t
 
 // Row entries of bins 0 and 1 (streamed once per pass). SGR_ROWNA: bypass L1 allocation,
 // leaving L1 to the color gathers.
+// Row entries of bins 0/1. SGR_HUB_ROWNA: in the hub build (whose gathers bypass L1) read
+// them without allocating in L1 either.
+#ifndef SGR_HUB_ROWNA
+#define SGR_HUB_ROWNA 0
+#endif
 template <bool Hub>
-__device__ __forceinline__ int32_t ld_row_h(const int32_t* p) { return __ldg(p); }
+__device__ __forceinline__ int32_t ld_row_h(const int32_t* p) {
+  if constexpr (Hub && SGR_HUB_ROWNA) {
+    int32_t r;
+    asm volatile("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(r) : "l"(p));
+    return r;
+  } else {
+    return __ldg(p);
+  }
+}
 __device__ __forceinline__ int32_t ld_row(const int32_t* p) {
 #if SGR_ROWNA
   int32_t r;
