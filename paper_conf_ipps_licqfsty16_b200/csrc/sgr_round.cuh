@@ -47,7 +47,7 @@
 #include "sgr_common.cuh"
 
 #ifndef SGR_QB
-#define SGR_QB 2  // int4 slots per lane per batch (batch = 128 * SGR_QB window slots)
+#define SGR_QB 2  // bin-2 batch: kJB = 4 * SGR_QB window slots per lane (32 kJB per warp)
 #endif
 constexpr int kQB = SGR_QB;
 constexpr int kJB = 4 * kQB;  // entries per lane per batch
@@ -65,6 +65,9 @@ constexpr int kJB = 4 * kQB;  // entries per lane per batch
 #endif
 #ifndef SGR_CLRMAX
 #define SGR_CLRMAX 1  // bin 2: clear the chunk's tables only up to the largest color seen
+#endif
+#ifndef SGR_BARSLEEP
+#define SGR_BARSLEEP 20  // grid-barrier poll back-off (ns); 0 = spin
 #endif
 #ifndef SGR_SMALL_FIRST
 #define SGR_SMALL_FIRST 0  // pass order 0, 1, 2 instead of 2, 1, 0
@@ -2021,7 +2024,9 @@ __device__ __forceinline__ void grid_sync(Ctrl* ctrl, uint32_t& epoch) {
     // poll with relaxed loads (served by L2; an acquire load would invalidate this SM's L1
     // on every poll, evicting the lines the SM's other blocks are still gathering from),
     // then one acquire load once the count is reached
-    while ((int32_t)(ld_relaxed_gpu(&ctrl->bar_count) - target) < 0) __nanosleep(20);
+    while ((int32_t)(ld_relaxed_gpu(&ctrl->bar_count) - target) < 0) {
+      if (SGR_BARSLEEP) __nanosleep(SGR_BARSLEEP);
+    }
     (void)ld_acquire_gpu(&ctrl->bar_count);
   }
   __syncthreads();
