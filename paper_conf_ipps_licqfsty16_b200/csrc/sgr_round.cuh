@@ -69,6 +69,9 @@ constexpr int kJB = 4 * kQB;  // entries per lane per batch
 #ifndef SGR_BARSLEEP
 #define SGR_BARSLEEP 20  // grid-barrier poll back-off (ns); 0 = spin
 #endif
+#ifndef SGR_B1_BATCH_HUB
+#define SGR_B1_BATCH_HUB 8  // bin 1, hub build: row entries per lane per batch (8 or 16)
+#endif
 #ifndef SGR_SMALL_FIRST
 #define SGR_SMALL_FIRST 0  // pass order 0, 1, 2 instead of 2, 1, 0
 #endif
@@ -1213,21 +1216,22 @@ __device__ __forceinline__ void process_group(const RoundArgs<C>& a, int k, int3
   const int32_t* row = a.col_idx + s;
   const int32_t xv = v >= 0 ? ldc<Persist>(X + v) : 0;
   bool conf = false;
-  const int32_t nb = (cnt + 63) >> 6;
+  constexpr int B = Hub ? SGR_B1_BATCH_HUB : 8;  // entries per lane per batch
+  const int32_t nb = (cnt + 8 * B - 1) / (8 * B);
   for (int32_t bb = 0; bb < nb; ++bb) {
-    int32_t w[8];
+    int32_t w[B];
 #pragma unroll
-    for (int u = 0; u < 8; ++u) {
-      const int32_t r = 64 * bb + gl + kGroup * u;
+    for (int u = 0; u < B; ++u) {
+      const int32_t r = 8 * B * bb + gl + kGroup * u;
       w[u] = r < cnt ? ld_row_h<Hub>(row + r) : -1;
     }
     uint32_t lb = 0;
 #pragma unroll
-    for (int u = 0; u < 8; ++u) lb |= (w[u] >= 0 && lose<TB>(v, w[u])) ? (1u << u) : 0u;
+    for (int u = 0; u < B; ++u) lb |= (w[u] >= 0 && lose<TB>(v, w[u])) ? (1u << u) : 0u;
 #pragma unroll
-    for (int u = 0; u < 8; ++u) w[u] = w[u] >= 0 ? ldc01<Persist, Hub>(X + w[u]) : -1;  // colors
+    for (int u = 0; u < B; ++u) w[u] = w[u] >= 0 ? ldc01<Persist, Hub>(X + w[u]) : -1;  // colors
 #pragma unroll
-    for (int u = 0; u < 8; ++u) {
+    for (int u = 0; u < B; ++u) {
       if (w[u] >= 0) {
         // deg <= 256 => first fit <= 257: colors >= 511 are clamped onto an unused byte
         set_add(gtbl, (uint32_t)min(w[u], kMedTbl - 1));
