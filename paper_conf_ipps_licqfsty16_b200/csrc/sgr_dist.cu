@@ -18,7 +18,9 @@
 
 #include <algorithm>
 #include <cstring>
+#include <cstdlib>
 #include <functional>
+#include <map>
 #include <vector>
 
 #include "sgr.h"
@@ -174,6 +176,50 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
   int32_t known_cap = status == SGR_OK ? *std::max_element(cnt.begin(), cnt.end()) : 0;
   bool done = status != SGR_OK || total == 0 || overflow_seen;
   int64_t issued = 0, consumed = 0;  // passes issued / whose counts were read
+  // One pass = per partition: fused round, finalize, advance, pack; the exchange; apply.
+  auto enqueue_pass = [&](int32_t cap_k, cudaStream_t st) -> sgr_status {
+    for (int i = 0; i < P; ++i) {
+      k_round<TB, C><<<grid, kBlock, round_smem<C>(), st>>>(args[i]);
+      if constexpr (packed<C>()) k_finalize<TB, C><<<grid, kBlock, 0, st>>>(args[i]);
+      k_advance<<<1, 32, 0, st>>>(args[i].ctrl, 0, 1);
+      DCK(cudaMemsetAsync(parts[i].send, 0, sizeof(uint2), st));
+      // W_{k+1} is bounded by cap_k: size the grid by it, not by the range (a thin
+      // round's pack was ~9.5K blocks that found nothing to do)
+      k_pack<C><<<first_grid(std::min<int64_t>(cap_k, parts[i].hi - parts[i].lo) + 1), 256, 0, st>>>(
+          args[i], parts[i].send, cap_k);
+    }
+    DCK(cudaGetLastError());
+    const sgr_status gst = gather(parts, recv, cap_k, st);
+    if (gst != SGR_OK) return gst;
+    for (int i = 0; i < P; ++i)
+      k_apply<C><<<first_grid(cap_k), 256, 0, st>>>(args[i], recv, world, cap_k + 1, me0 + i);
+    DCK(cudaGetLastError());
+    return SGR_OK;
+  };
+  // The host-driven loop was launch-gap bound (7+ operations per round, ~40 us): each
+  // pass is captured once per all-gather capacity bucket into a CUDA graph (exchange
+  // included: NCCL collectives are capturable) and replayed. Capacities are rounded up to
+  // a quarter-octave (>= 4096 records, <= cap_max): the padding is at most 25 % of the
+  // records, and every rank derives the same bucket from the same counts. All state a
+  // pass reads (round number, ping-pong parity, worklist counts) lives on the device, so
+  // a replay is the same pass as a fresh launch. Opt-in (SGR_DIST_GRAPHS=1): on one B200
+  // (NCCL world 1) replay saved nothing per round and instantiation (one graph per bucket,
+  // per coloring) cost 0.3-0.5 ms (cfg1 2.97 -> 3.47 ms, cfg4 46.9 -> 47.2 ms).
+  const char* genv = getenv("SGR_DIST_GRAPHS");
+  const bool use_graphs = genv && genv[0] == '1';
+  std::map<int32_t, cudaGraphExec_t> graphs;
+  cudaStream_t gs = nullptr;  // capture stream (the caller's may be the legacy stream)
+  if (use_graphs && status == SGR_OK) DCK(cudaStreamCreateWithFlags(&gs, cudaStreamNonBlocking));
+  auto cap_bucket = [&](int32_t c) -> int32_t {
+    int64_t b = 4096;
+    if (c > 4096) {
+      int64_t p = 1;
+      while (p * 2 <= c) p *= 2;
+      const int64_t step = p / 4;
+      b = (c + step - 1) / step * step;
+    }
+    return (int32_t)std::min<int64_t>(b, cap_max);
+  };
   auto consume_one = [&]() {
     const int q = (int)(consumed % (kLag + 1));
     cudaEventSynchronize(sev[q]);
@@ -206,20 +252,31 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
         break;
       }
     }
-    const int32_t cap_k = known_cap;
-    for (int i = 0; i < P; ++i) {
-      k_round<TB, C><<<grid, kBlock, round_smem<C>(), s>>>(args[i]);
-      if constexpr (packed<C>()) k_finalize<TB, C><<<grid, kBlock, 0, s>>>(args[i]);
-      k_advance<<<1, 32, 0, s>>>(args[i].ctrl, 0, 1);
-      DCK(cudaMemsetAsync(parts[i].send, 0, sizeof(uint2), s));
-      k_pack<C><<<first_grid(parts[i].hi - parts[i].lo + 1), 256, 0, s>>>(args[i], parts[i].send, cap_k);
+    const int32_t cap_k = use_graphs ? cap_bucket(known_cap) : known_cap;
+    if (use_graphs) {
+      auto it = graphs.find(cap_k);
+      if (it == graphs.end()) {
+        cudaGraph_t g = nullptr;
+        DCK(cudaStreamBeginCapture(gs, cudaStreamCaptureModeThreadLocal));
+        const sgr_status cs = enqueue_pass(cap_k, gs);
+        const cudaError_t ce = cudaStreamEndCapture(gs, &g);
+        if (cs != SGR_OK) {
+          if (g) cudaGraphDestroy(g);
+          status = cs;
+          break;
+        }
+        DCK(ce);
+        cudaGraphExec_t ex = nullptr;
+        const cudaError_t ie = cudaGraphInstantiate(&ex, g, 0);
+        cudaGraphDestroy(g);
+        DCK(ie);
+        it = graphs.emplace(cap_k, ex).first;
+      }
+      DCK(cudaGraphLaunch(it->second, s));
+    } else {
+      status = enqueue_pass(cap_k, s);
+      if (status != SGR_OK) break;
     }
-    DCK(cudaGetLastError());
-    status = gather(parts, recv, cap_k, s);
-    if (status != SGR_OK) break;
-    for (int i = 0; i < P; ++i)
-      k_apply<C><<<first_grid(cap_k), 256, 0, s>>>(args[i], recv, world, cap_k + 1, me0 + i);
-    DCK(cudaGetLastError());
     const int q = (int)(issued % (kLag + 1));
     DCK(cudaMemcpy2DAsync(slots + q * world * 2, sizeof(uint2), recv, (size_t)(cap_k + 1) * sizeof(uint2),
                           sizeof(uint2), world, cudaMemcpyDeviceToHost, s));
@@ -233,6 +290,8 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
     status = SGR_ENOCONV;
   }
   for (int q = 0; q <= kLag; ++q) cudaEventDestroy(sev[q]);
+  for (auto& kv : graphs) cudaGraphExecDestroy(kv.second);
+  if (gs) cudaStreamDestroy(gs);
   if (slots) cudaFreeHost(slots);
   cudaEventRecord(ev1, s);
   if (status == SGR_OK) {

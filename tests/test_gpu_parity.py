@@ -314,6 +314,22 @@ def test_partitioned_equals_single_gpu(P, tb):
 
 
 @pytest.mark.parametrize("P", [1, 3])
+def test_partitioned_graph_replay(P, monkeypatch):
+    """SGR_DIST_GRAPHS=1: each pass (+ exchange) captured per capacity bucket and replayed;
+    the rounds, colors and counts are those of the eager loop and of the oracle (the
+    bucketed all-gather capacity pads records, the counts in the payload bound them)."""
+    monkeypatch.setenv("SGR_DIST_GRAPHS", "1")
+    for g in (gen.config(1), degree_boundary_graph(), gen.stencil3d(12, 12, 12)):
+        rp, ci = dev(g)
+        for tb in (LOW, PAP):
+            ref = oracle.jacobi(g, tb)
+            res = sgr.color_partitioned(rp, ci, P, tiebreak=RULE[tb])
+            assert np.array_equal(res.colors.cpu().numpy(), ref.colors), (g.name, P, tb)
+            assert res.stats["rounds"] == ref.rounds
+            assert res.stats["vertices_processed"] == ref.vertices_processed
+
+
+@pytest.mark.parametrize("P", [1, 3])
 def test_partitioned_color_overflow_rerun(P):
     """Partitions see a packed overflow in the same exchange and all redo the coloring
     with int32 words (color_cap lowered below K_300's colors by the test hook)."""
