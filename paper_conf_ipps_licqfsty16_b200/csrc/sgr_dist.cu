@@ -9,7 +9,8 @@
 //   3. an all-gather of the records (NCCL over NVLink between ranks, or device copies
 //      between partitions that share one GPU),
 //   4. k_apply: every replica writes the other partitions' records into both ping-pong
-//      buffers (a remote vertex is never written by the local pass).
+//      buffers (a remote vertex is never written by the local pass); the same launch
+//      advances the round (lockstep) and re-arms the send count.
 // Round k's records are a subset of W_k, so the largest count of the previous exchange is
 // a valid capacity for the padded all-gather: one collective per round (plus one counts
 // gather before the first). The result is bit-identical to one GPU: the passes read the
@@ -118,7 +119,8 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
     sgr_status st = gather(parts, recv, cap, s);
     if (st != SGR_OK) return st;
     for (int i = 0; i < P; ++i)
-      k_apply<C><<<first_grid(cap), 256, 0, s>>>(args[i], recv, world, cap + 1, me0 + i);
+      k_apply<C><<<first_grid(cap), 256, 0, s>>>(args[i], recv, world, cap + 1, me0 + i,
+                                                 parts[i].send, 0);
     DCK(cudaGetLastError());
     DCK(cudaMemcpy2DAsync(counts_host, sizeof(uint2), recv, (size_t)(cap + 1) * sizeof(uint2),
                           sizeof(uint2), world, cudaMemcpyDeviceToHost, s));
@@ -181,18 +183,18 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
     for (int i = 0; i < P; ++i) {
       k_round<TB, C><<<grid, kBlock, round_smem<C>(), st>>>(args[i]);
       if constexpr (packed<C>()) k_finalize<TB, C><<<grid, kBlock, 0, st>>>(args[i]);
-      k_advance<<<1, 32, 0, st>>>(args[i].ctrl, 0, 1);
-      DCK(cudaMemsetAsync(parts[i].send, 0, sizeof(uint2), st));
       // W_{k+1} is bounded by cap_k: size the grid by it, not by the range (a thin
-      // round's pack was ~9.5K blocks that found nothing to do)
+      // round's pack was ~9.5K blocks that found nothing to do). The pack runs before the
+      // advance (pre = 1), which k_apply carries, with the send-count reset.
       k_pack<C><<<first_grid(std::min<int64_t>(cap_k, parts[i].hi - parts[i].lo) + 1), 256, 0, st>>>(
-          args[i], parts[i].send, cap_k);
+          args[i], parts[i].send, cap_k, 1);
     }
     DCK(cudaGetLastError());
     const sgr_status gst = gather(parts, recv, cap_k, st);
     if (gst != SGR_OK) return gst;
     for (int i = 0; i < P; ++i)
-      k_apply<C><<<first_grid(cap_k), 256, 0, st>>>(args[i], recv, world, cap_k + 1, me0 + i);
+      k_apply<C><<<first_grid(cap_k), 256, 0, st>>>(args[i], recv, world, cap_k + 1, me0 + i,
+                                                    parts[i].send, 1);
     DCK(cudaGetLastError());
     return SGR_OK;
   };

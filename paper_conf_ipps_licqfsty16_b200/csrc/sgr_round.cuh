@@ -1882,9 +1882,11 @@ static __global__ void k_advance(Ctrl* ctrl, int first, int force = 0) {
 // owned part of W_{k+1}; every other replica needs those vertices' new color words.
 // Record = (v, word); slot 0 of a send buffer carries (count, 0).
 template <class C>
-__global__ void k_pack(RoundArgs<C> a, uint2* send, int32_t cap) {
+__global__ void k_pack(RoundArgs<C> a, uint2* send, int32_t cap, int pre = 0) {
   Ctrl* ctrl = a.ctrl;
-  const int k = ctrl->k;  // already advanced: W_k's lists are the new ones
+  // W_k's lists are the new ones: k = ctrl->k once advanced, ctrl->k + 1 when the pack runs
+  // before the advance (pre = 1; the round loop advances in k_apply)
+  const int k = ctrl->k + pre;
   const int p = k & 1;
   const C* Y = sel((k - 1) & 1, (const C*)a.col[0], (const C*)a.col[1]);
   const Counts w = ctrl->ring[rs(k)];
@@ -1923,7 +1925,14 @@ __global__ void k_pack(RoundArgs<C> a, uint2* send, int32_t cap) {
 // remote vertex is only ever written by these updates.
 template <class C>
 __global__ void k_apply(RoundArgs<C> a, const uint2* recv, int32_t parts, int32_t stride,
-                        int32_t me) {
+                        int32_t me, uint2* send_reset = nullptr, int adv = 0) {
+  // Round loop: this launch also carries the lockstep advance of pass k (the pack already
+  // read W_{k+1}) and re-arms the send count for the next pack (the all-gather has consumed
+  // it) — two fewer stream operations per round.
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    if (adv) advance_body(a.ctrl, false, true);
+    if (send_reset) send_reset[0].x = 0u;
+  }
   for (int q = 0; q < parts; ++q) {
     if (q == me) continue;
     const uint2* r = recv + (int64_t)q * stride;
