@@ -133,16 +133,16 @@ inline int round_grid(bool persistent) {
   if (!attr_set) {  // opt in to > 48 KB of dynamic shared memory
     cudaFuncSetAttribute(k_persistent<TB, C, Hub>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)round_smem<C, Hub>());
-    cudaFuncSetAttribute(k_round<TB, C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)round_smem<C>());
+    cudaFuncSetAttribute(k_round<TB, C, Hub>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)round_smem<C, Hub>());
     attr_set = true;
   }
   int per_sm = 0;
   cudaError_t e = persistent
       ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_persistent<TB, C, Hub>, kBlock,
                                                       round_smem<C, Hub>())
-      : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_round<TB, C>, kBlock,
-                                                      round_smem<C>());
+      : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_round<TB, C, Hub>, kBlock,
+                                                      round_smem<C, Hub>());
   if (e != cudaSuccess || per_sm <= 0) per_sm = 1;
   if (const char* env = getenv("SGR_BLOCKS_PER_SM")) {  // experiments: shrink the grid
     const int lim = atoi(env);

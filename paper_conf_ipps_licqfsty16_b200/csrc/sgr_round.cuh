@@ -1974,19 +1974,21 @@ __device__ __forceinline__ uint8_t* warp_smem_init(uint8_t* smem) {
   return wsm;
 }
 
-// One pass per launch (host / graph loop modes); k_advance follows it on the stream.
-template <int TB, class C>
-__global__ void __launch_bounds__(kBlock, kMinBlocks<C>) k_round(RoundArgs<C> a) {
+// One pass per launch (host / graph loop modes, distributed rounds); k_advance (or the
+// distributed k_apply) follows it on the stream. Hub = false is the flat build (bins 0/1
+// only), for colorings whose F_1 put no vertex into bin 2 (the caller reads big_count).
+template <int TB, class C, bool Hub = true>
+__global__ void __launch_bounds__(kBlock, kMinBlocks<C, Hub>) k_round(RoundArgs<C> a) {
   extern __shared__ __align__(16) uint8_t dsmem[];
   Ctrl* ctrl = a.ctrl;
   if (!ctrl->active) return;  // uniform across the grid
-  uint8_t* wsm = warp_smem_init<C>(dsmem);
+  uint8_t* wsm = warp_smem_init<C, Hub>(dsmem);
   unsigned long long edges[kBins] = {0, 0, 0}, entries[kBins] = {0, 0, 0};
   unsigned long long cyc[kBins] = {0, 0, 0};
   uint32_t ph = 0;
   const int k = ctrl->k;
   const Counts w = ctrl->ring[rs(k)];
-  round_body<TB, false, C, true>(a, k, w, wsm, edges, entries, ph, cyc);
+  round_body<TB, false, C, Hub>(a, k, w, wsm, edges, entries, ph, cyc);
   block_add6(edges, entries, ctrl, k);
   if ((threadIdx.x & 31) == 0)
     for (int q = 0; q < kBins; ++q) atomicAdd(&ctrl->bin_cycles[q], cyc[q]);
