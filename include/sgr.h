@@ -151,6 +151,21 @@ sgr_status sgr_color_host(const int64_t* row_ptr, const int32_t* col_idx, int64_
                           int64_t nnz, int32_t* colors_out, sgr_stats* stats,
                           const sgr_opts* opts);
 
+/* Pipelined end to end over `count` HOST graphs (the batch a user colors one after the
+ * other): graph i+1's row_ptr/col_idx upload and graph i-1's colors download run on two
+ * internal copy streams while graph i is colored (sgr_color_ex) on opts->stream, with two
+ * device buffer sets sized by the largest graph (stream-ordered allocator, released before
+ * return). Arguments are arrays of `count` entries: row_ptr[i] (n[i]+1 int64 offsets),
+ * col_idx[i] (nnz[i] int32 ids, may be NULL when nnz[i] == 0), colors_out[i] (n[i] int32);
+ * the same host buffers may appear more than once (read-only inputs; outputs should be
+ * distinct). Host buffers must be pinned for the copies to overlap the coloring (pageable
+ * memory makes them synchronous). stats: NULL or an array of `count` records, one per
+ * graph. Each colors_out[i] equals sgr_color_host's result for graph i. Returns at the
+ * first failing graph (its status; later graphs untouched); synchronizes all streams. */
+sgr_status sgr_color_host_batch(const int64_t* const* row_ptr, const int32_t* const* col_idx,
+                                const int64_t* n, const int64_t* nnz, int32_t* const* colors_out,
+                                int32_t count, sgr_stats* stats, const sgr_opts* opts);
+
 /* Topology-driven mapping of the same method: the paper's Algorithm 4 (T-base,
  * P:194-196) under the Jacobi reading. Every iteration visits all n vertices, one thread
  * per vertex: the uncolored ones take a first fit against the iteration's snapshot, then

@@ -26,7 +26,7 @@ from ._lib import Csr, Opts, Stats, check, load
 TIEBREAK = {"lowid": 0, "lowid_keeps": 0, "paper": 1}
 LOOP = {"auto": 0, "graph": 1, "persistent": 2, "host": 3}
 
-__all__ = ["color", "color_host", "color_topo", "color_partitioned", "color_dist", "assign", "commit",
+__all__ = ["color", "color_host", "color_host_batch", "color_topo", "color_partitioned", "color_dist", "assign", "commit",
            "detect", "compact", "validate_csr", "partition", "workspace_bytes", "gen",
            "ColorResult", "TIEBREAK"]
 
@@ -178,6 +178,38 @@ def color_host(row_ptr: np.ndarray, col_idx: np.ndarray, tiebreak="lowid", *, ou
                                 ptr(out) if n else None, ctypes.byref(st), ctypes.byref(opts)),
           "sgr_color_host")
     return ColorResult(out, st.as_dict())
+
+
+def color_host_batch(graphs, tiebreak="lowid", *, outs=None, stream=None, **opt_kw):
+    """Pipelined end to end over a list of HOST graphs [(row_ptr, col_idx), ...] (pinned
+    torch tensors or numpy arrays): graph i+1's upload and graph i-1's download overlap the
+    coloring of graph i, in the library (sgr_color_host_batch). Returns one ColorResult
+    per graph."""
+    ptr = (lambda a: a.data_ptr() if hasattr(a, "data_ptr") else a.ctypes.data)
+    size = (lambda a: a.numel() if hasattr(a, "numel") else len(a))
+    cnt = len(graphs)
+    keep, rps, cis, ns, nnzs = [], [], [], [], []
+    for rp, ci in graphs:
+        if isinstance(rp, np.ndarray):
+            rp = np.ascontiguousarray(rp, dtype=np.int64)
+        if isinstance(ci, np.ndarray):
+            ci = np.ascontiguousarray(ci, dtype=np.int32)
+        keep += [rp, ci]
+        ns.append(size(rp) - 1)
+        nnzs.append(size(ci))
+        rps.append(ptr(rp))
+        cis.append(ptr(ci) if nnzs[-1] else None)
+    if outs is None:
+        outs = [np.zeros(n, np.int32) for n in ns]
+    VP, I64 = ctypes.c_void_p, ctypes.c_int64
+    st = (Stats * max(cnt, 1))()
+    opts = make_opts(tiebreak, stream, **opt_kw)
+    check(load().sgr_color_host_batch((VP * max(cnt, 1))(*rps), (VP * max(cnt, 1))(*cis),
+                                      (I64 * max(cnt, 1))(*ns), (I64 * max(cnt, 1))(*nnzs),
+                                      (VP * max(cnt, 1))(*[ptr(o) if n else None for o, n in zip(outs, ns)]),
+                                      cnt, st, ctypes.byref(opts)),
+          "sgr_color_host_batch")
+    return [ColorResult(outs[i], st[i].as_dict()) for i in range(cnt)]
 
 
 def assign(row_ptr, col_idx, wl, colors_in, *, out=None, stream=None):

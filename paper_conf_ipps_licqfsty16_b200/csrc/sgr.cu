@@ -549,6 +549,89 @@ sgr_status sgr_color_host(const int64_t* row_ptr, const int32_t* col_idx, int64_
   return st;
 }
 
+// Pipelined end to end over a batch of host graphs: graph i+1's upload (stream `up`) and
+// graph i-1's download (stream `down`) run on the copy engines while graph i is colored on
+// the caller's stream. Two device buffer sets; the input set of graph i+1 was last read
+// by coloring i-1, which sgr_color_ex finished (it synchronizes) before the upload is
+// issued; the colors set of graph i waits for the download of graph i-2 (event).
+sgr_status sgr_color_host_batch(const int64_t* const* row_ptr, const int32_t* const* col_idx,
+                                const int64_t* n, const int64_t* nnz, int32_t* const* colors_out,
+                                int32_t count, sgr_stats* stats, const sgr_opts* opts) {
+  if (count < 0 || (count > 0 && (!row_ptr || !col_idx || !n || !nnz || !colors_out)))
+    return SGR_EINVAL;
+  int64_t max_n = 0, max_nnz = 1;
+  for (int32_t i = 0; i < count; ++i) {
+    if (n[i] < 0 || nnz[i] < 0 || n[i] >= ((int64_t)1 << 31) || !row_ptr[i] ||
+        (n[i] > 0 && !colors_out[i]) || (nnz[i] > 0 && !col_idx[i])) {
+      set_error("sgr_color_host_batch: graph %d: invalid sizes or null pointer", i);
+      return SGR_EINVAL;
+    }
+    max_n = std::max(max_n, n[i]);
+    max_nnz = std::max(max_nnz, nnz[i]);
+  }
+  if (stats) memset(stats, 0, sizeof(sgr_stats) * (size_t)count);
+  if (count == 0 || max_n == 0) return SGR_OK;
+  const Resolved r = resolve_opts(opts, max_n);
+  cudaStream_t s = r.stream, up = nullptr, down = nullptr;
+  keep_pool_memory();
+  CK(cudaStreamCreateWithFlags(&up, cudaStreamNonBlocking));
+  CK(cudaStreamCreateWithFlags(&down, cudaStreamNonBlocking));
+  cudaEvent_t ev_alloc, ev_up[2], ev_down[2];
+  CK(cudaEventCreateWithFlags(&ev_alloc, cudaEventDisableTiming));
+  for (int b = 0; b < 2; ++b) {
+    CK(cudaEventCreateWithFlags(&ev_up[b], cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&ev_down[b], cudaEventDisableTiming));
+  }
+  int64_t* d_rp[2] = {nullptr, nullptr};
+  int32_t* d_ci[2] = {nullptr, nullptr};
+  int32_t* d_col[2] = {nullptr, nullptr};
+  for (int b = 0; b < 2 && b < count; ++b) {
+    CK(cudaMallocAsync((void**)&d_rp[b], (size_t)(max_n + 1) * 8, s));
+    CK(cudaMallocAsync((void**)&d_ci[b], (size_t)max_nnz * 4, s));
+    CK(cudaMallocAsync((void**)&d_col[b], (size_t)max_n * 4, s));
+  }
+  CK(cudaEventRecord(ev_alloc, s));
+  CK(cudaStreamWaitEvent(up, ev_alloc, 0));
+  CK(cudaStreamWaitEvent(down, ev_alloc, 0));
+  auto upload = [&](int32_t i) -> sgr_status {
+    const int b = i & 1;
+    CK(cudaMemcpyAsync(d_rp[b], row_ptr[i], (size_t)(n[i] + 1) * 8, cudaMemcpyHostToDevice, up));
+    if (nnz[i] > 0)
+      CK(cudaMemcpyAsync(d_ci[b], col_idx[i], (size_t)nnz[i] * 4, cudaMemcpyHostToDevice, up));
+    CK(cudaEventRecord(ev_up[b], up));
+    return SGR_OK;
+  };
+  sgr_status st = upload(0);
+  for (int32_t i = 0; i < count && st == SGR_OK; ++i) {
+    const int b = i & 1;
+    if (i + 1 < count && (st = upload(i + 1)) != SGR_OK) break;
+    if (n[i] == 0) continue;
+    CK(cudaStreamWaitEvent(s, ev_up[b], 0));
+    if (i >= 2) CK(cudaStreamWaitEvent(s, ev_down[b], 0));  // graph i-2's colors are out
+    sgr_csr csr{d_rp[b], d_ci[b]};
+    st = sgr_color_ex(&csr, n[i], nnz[i], d_col[b], stats ? &stats[i] : nullptr, opts, nullptr, 0);
+    if (st != SGR_OK) break;
+    CK(cudaMemcpyAsync(colors_out[i], d_col[b], (size_t)n[i] * 4, cudaMemcpyDeviceToHost, down));
+    CK(cudaEventRecord(ev_down[b], down));
+  }
+  CK(cudaStreamSynchronize(up));
+  CK(cudaStreamSynchronize(down));
+  for (int b = 0; b < 2; ++b) {
+    if (d_rp[b]) cudaFreeAsync(d_rp[b], s);
+    if (d_ci[b]) cudaFreeAsync(d_ci[b], s);
+    if (d_col[b]) cudaFreeAsync(d_col[b], s);
+  }
+  CK(cudaStreamSynchronize(s));
+  cudaEventDestroy(ev_alloc);
+  for (int b = 0; b < 2; ++b) {
+    cudaEventDestroy(ev_up[b]);
+    cudaEventDestroy(ev_down[b]);
+  }
+  cudaStreamDestroy(up);
+  cudaStreamDestroy(down);
+  return st;
+}
+
 // ----- topology-driven mapping (Algorithm 4; sgr_topo.cuh) -------------------
 sgr_status sgr_color_topo(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* colors_out,
                           sgr_stats* stats, const sgr_opts* opts) {

@@ -218,6 +218,35 @@ def test_color_host_equals_device():
     assert np.array_equal(b, a)
 
 
+@pytest.mark.parametrize("tb", [LOW, PAP])
+def test_color_host_batch_pipelined(tb):
+    """sgr_color_host_batch: uploads/downloads overlapped with the colorings (two device
+    buffer sets, copy streams) give each graph the oracle's coloring — graphs of different
+    sizes (the buffer sets are reused across sizes), an empty one, an edgeless one, one
+    repeated, pinned torch and pageable numpy inputs mixed."""
+    gs = [gen.config(1), random_graph(3, n=300), gen.stencil3d(9, 9, 9), random_graph(5, n=1),
+          gen.config(1), degree_boundary_graph()]
+    empty = (np.zeros(1, np.int64), np.zeros(0, np.int32))
+    edgeless = (np.zeros(6, np.int64), np.zeros(0, np.int32))
+    host = []
+    for i, g in enumerate(gs):
+        if i % 2 == 0:
+            host.append((torch.from_numpy(g.row_ptr).pin_memory(), torch.from_numpy(g.col_idx).pin_memory()))
+        else:
+            host.append((g.row_ptr, g.col_idx))
+    host = host[:2] + [empty] + host[2:4] + [edgeless] + host[4:]
+    res = sgr.color_host_batch(host, RULE[tb])
+    assert len(res) == len(host)
+    assert res[2].colors.size == 0
+    assert np.array_equal(res[5].colors, np.ones(5, np.int32))
+    r = [x for i, x in enumerate(res) if i not in (2, 5)]
+    for g, x in zip(gs, r):
+        ref = oracle.jacobi(g, tb)
+        assert np.array_equal(x.colors, ref.colors), g.name
+        assert x.stats["rounds"] == ref.rounds
+    assert sgr.color_host_batch([], RULE[tb]) == []
+
+
 # ----------------------------------------------------------------------------- step API
 @pytest.mark.parametrize("seed", range(16))
 def test_step_entry_points(seed):
