@@ -1990,8 +1990,17 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks<C, Hub>) k_round(RoundArgs<
   const Counts w = ctrl->ring[rs(k)];
   round_body<TB, false, C, Hub>(a, k, w, wsm, edges, entries, ph, cyc);
   block_add6(edges, entries, ctrl, k);
+  // bin cycle stats: one atomic per block and bin (per-warp atomics were ~7K same-address
+  // reductions per launch, on every pass of the host-driven loops)
+  __shared__ unsigned long long cred[kBins][kWarps];
   if ((threadIdx.x & 31) == 0)
-    for (int q = 0; q < kBins; ++q) atomicAdd(&ctrl->bin_cycles[q], cyc[q]);
+    for (int q = 0; q < kBins; ++q) cred[q][threadIdx.x >> 5] = cyc[q];
+  __syncthreads();
+  if (threadIdx.x < kBins) {
+    unsigned long long z = 0;
+    for (int i = 0; i < kWarps; ++i) z += cred[threadIdx.x][i];
+    atomicAdd(&ctrl->bin_cycles[threadIdx.x], z);
+  }
 }
 
 // Finalize phase as its own launch (host / graph loop modes), between k_round and k_advance.
