@@ -54,23 +54,60 @@ def run(args):
     def step():
         return color_dist(comm, rp_d, ci_d, g.n, lo, hi, args.tiebreak)
 
+    import bench as _bench  # Clocks, peaks (repo root is on sys.path: bench.py runs us)
     for _ in range(max(args.warmup, 3)):
         res = step()
     torch.cuda.synchronize()
+    flush = torch.empty(2 * _bench.L2_BYTES // 4, dtype=torch.int32, device=dev)
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
           for _ in range(args.steps)]
+    clocks = _bench.Clocks(local)
     dist.barrier()
     torch.cuda.synchronize()
     for i in range(args.steps):
+        flush.fill_(i)  # L2 flushed between steps, outside the step events
         ev[i][0].record(stream)
         res = step()
         ev[i][1].record(stream)
     torch.cuda.synchronize()
     dist.barrier()
+    clk = clocks.stop()
     ms = statistics.mean(a.elapsed_time(b) for a, b in ev)
-    t = torch.tensor([ms], device=dev)
-    dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    ms_max = float(t.item())
+    t = torch.tensor([ms, float(res.stats.get("bytes_algorithmic", 0))], device=dev, dtype=torch.float64)
+    tm = t.clone()
+    dist.all_reduce(tm, op=dist.ReduceOp.MAX)
+    ms_max = float(tm[0].item())
+    dist.all_reduce(t, op=dist.ReduceOp.SUM)
+    alg_bytes = float(t[1].item())
+    clks = [None] * world
+    dist.all_gather_object(clks, clk)
+
+    # e2e: every step uploads the rank's owned rows from pinned host memory, colors, and
+    # reads its owned colors back; wall clock per step, max over ranks
+    e2e = None
+    if not args.no_e2e:
+        lrp_h = torch.from_numpy(lrp).pin_memory()
+        lci_h = torch.from_numpy(lci).pin_memory() if len(lci) else torch.zeros(4, dtype=torch.int32).pin_memory()
+        out_h = torch.empty(max(hi - lo, 1), dtype=torch.int32).pin_memory()
+        e_ms = []
+        for i in range(min(args.steps, 3)):
+            flush.fill_(i)
+            torch.cuda.synchronize()
+            dist.barrier()
+            t0 = time.perf_counter()
+            rp_e = lrp_h.to(dev, non_blocking=True)
+            ci_e = lci_h.to(dev, non_blocking=True)
+            r_e = color_dist(comm, rp_e, ci_e, g.n, lo, hi, args.tiebreak)
+            out_h[: hi - lo].copy_(r_e.colors[lo:hi], non_blocking=True)
+            torch.cuda.synchronize()
+            e_ms.append((time.perf_counter() - t0) * 1e3)
+        te = torch.tensor([statistics.mean(e_ms)], device=dev)
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        e_max = float(te.item())
+        e2e = {"value": g.nnz / (e_max * 1e-3) / 1e9, "unit": "GTEPS",
+               "h2d_bytes_per_step": int((g.n + world) * 8 + g.nnz * 4),
+               "d2h_bytes_per_step": int(g.n * 4), "ms_per_step": e_max,
+               "api": "sgr_color_dist per rank, owned rows uploaded and owned colors read back"}
     # every replica holds the full coloring: check ranks agree
     h = torch.tensor([int(res.colors.sum().item()), res.stats["rounds"]], device=dev, dtype=torch.int64)
     hs = [torch.zeros_like(h) for _ in range(world)]
@@ -88,7 +125,22 @@ def run(args):
                                           "NCCL all-gather of recolored vertices per round",
                            "ranges": [int(x) for x in ranges]},
                 "rounds": res.stats["rounds"], "num_colors": res.stats["num_colors"],
-                "replicas_agree": agree, "gpu_launches": res.stats["launches"] * args.steps}
+                "replicas_agree": agree, "gpu_launches": res.stats["launches"] * args.steps,
+                "e2e": e2e}
+        sm = [c["sm_mhz"] for c in clks if c and c.get("sm_mhz") is not None]
+        line["clocks"] = {"sm_mhz": min(sm) if sm else None,
+                          "sm_max_mhz": clks[0].get("sm_max_mhz") if clks[0] else None,
+                          "reasons": sorted({r for c in clks if c for r in c.get("reasons", [])}),
+                          "per_rank_sm_mhz": sm}
+        line["config"]["l2"] = "flushed between steps (outside the step events)"
+        peak, peak_src = _bench.peaks()
+        if alg_bytes > 0:
+            ach = alg_bytes / (ms_max * 1e-3) / 1e9
+            line["roofline"] = {"bound": "hbm", "kernel": "whole step (all ranks)", "achieved": ach,
+                                "peak": peak * world, "unit": "GB/s", "frac": ach / (peak * world),
+                                "traffic": None, "peak_source": f"{peak_src} x {world} GPUs"}
+        else:
+            line["roofline"] = None
         print(json.dumps(line), flush=True)
     comm.close()
     dist.destroy_process_group()
