@@ -65,6 +65,18 @@ def test_host_entry_points_without_gpu():
     st = sgr._lib.Stats()
     assert lib.sgr_color(None, 10, 0, None, ctypes.byref(st)) == -1
     assert lib.sgr_color_ex(None, -1, 0, None, None, None, None, 0) == -1
+    # batch entry point: count < 0, null arrays, a bad graph in the batch; count 0 is a no-op
+    assert lib.sgr_color_host_batch(None, None, None, None, None, -1, None, None) == -1
+    assert lib.sgr_color_host_batch(None, None, None, None, None, 1, None, None) == -1
+    assert lib.sgr_color_host_batch(None, None, None, None, None, 0, None, None) == 0
+    VP, I64 = ctypes.c_void_p, ctypes.c_int64
+    one = np.zeros(2, np.int64)
+    bad_n = lib.sgr_color_host_batch((VP * 1)(one.ctypes.data), (VP * 1)(None), (I64 * 1)(-1),
+                                     (I64 * 1)(0), (VP * 1)(None), 1, None, None)
+    assert bad_n == -1
+    no_ci = lib.sgr_color_host_batch((VP * 1)(one.ctypes.data), (VP * 1)(None), (I64 * 1)(1),
+                                     (I64 * 1)(3), (VP * 1)(one.ctypes.data), 1, None, None)
+    assert no_ci == -1  # nnz > 0 with a null col_idx
 
 
 def test_partition_balances_nnz():
