@@ -18,8 +18,10 @@
  * Graph input: CSR "R" (row offsets, n+1) and "C" (column indices, nnz), stored
  * "in the order they are defined" with no relabeling (reading C19). Contract:
  *   - row_ptr is int64, row_ptr[0] = 0, nondecreasing, row_ptr[n] = nnz;
- *   - col_idx is int32, 0 <= col_idx[e] < n, each row sorted ascending, and the col_idx
- *     pointer is 16-byte aligned (rows are read with 16-byte vector loads);
+ *   - col_idx is int32, 0 <= col_idx[e] < n, each row sorted ascending (or any order with
+ *     opts->unsorted_rows; sorted input without the flag is what F_1 relies on: unsorted
+ *     rows without it can give an improper coloring), and the col_idx pointer is 16-byte
+ *     aligned (rows are read with 16-byte vector loads);
  *   - the pattern is symmetric (w in adj(v) <=> v in adj(w)); asymmetric input is
  *     undefined (conflicts may go unseen);
  *   - self-loops and duplicate entries are allowed and provably never change the result;
@@ -104,6 +106,17 @@ typedef struct {
   int32_t color_cap;     /* test hook: 0 = 4095, the largest color a 16-bit word holds; a
                             smaller cap sends colorings whose colors exceed it down the
                             automatic 32-bit rerun path (results are unchanged) */
+  int32_t block_size;    /* threads per block (the paper's Fig. 8 parameter, P:267-273;
+                            performance only, never the result). 0 = 256. A multiple of 32:
+                            per-vertex kernels (F_1, steps, topology-driven, final) take
+                            32..1024; the fused round kernels 64..512 when the graph has
+                            rows of degree > bin_med_max (hub build), else 64..768.
+                            Anything else: SGR_EINVAL. */
+  int32_t unsorted_rows; /* != 0: rows may be in any order. F_1 then scans whole rows
+                            instead of reading the first / last entry (sorted rows are the
+                            default contract: with unsorted rows and this flag 0 the
+                            coloring can be improper). opts->validate reports unsorted rows
+                            (bit 4) only when this flag is 0. */
 } sgr_opts;
 
 /* Kernel classes (stats->kernel_*): F_1, the fused round pass(es), loop control, final. */
@@ -181,7 +194,9 @@ sgr_status sgr_color_topo(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* c
  * asynchronous on opts->stream; opts may be NULL) ---------------------------------------- */
 
 /* Alg. 5 l.4-10 against a snapshot: tent_out[i] = min{c > 0 : c != colors_in[w] for all
- * w in adj(wl[i])}. colors_in must not alias tent_out. */
+ * w in adj(wl[i])}. colors_in must not alias tent_out. The step is Alg. 5 l.5-6 literally:
+ * w ranges over every entry of the row, so a listed self-loop forbids v's own snapshot
+ * color (DESIGN.md §3 reading C7; inside sgr_color this never changes a result, proof v). */
 sgr_status sgr_assign(const sgr_csr* csr, int64_t n, const int32_t* wl, int64_t wl_len,
                       const int32_t* colors_in, int32_t* tent_out, const sgr_opts* opts);
 

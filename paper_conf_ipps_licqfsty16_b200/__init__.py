@@ -68,7 +68,8 @@ def _check_csr(row_ptr, col_idx):
 def make_opts(tiebreak="lowid", stream=None, max_rounds=0, loop_mode="auto", color_bits=0,
               bin_small_max=0, bin_med_max=0, validate=False, rounds_per_batch=0,
               profile=False, round_sizes=None, round_edges=None, round_cap=0,
-              round_ms=None, color_cap=0, round_ns=None) -> Opts:
+              round_ms=None, color_cap=0, round_ns=None, block_size=0,
+              unsorted_rows=False) -> Opts:
     o = Opts()
     load().sgr_opts_default(ctypes.byref(o))
     o.tiebreak = _tb(tiebreak)
@@ -87,6 +88,8 @@ def make_opts(tiebreak="lowid", stream=None, max_rounds=0, loop_mode="auto", col
     o.round_ms = round_ms.ctypes.data if round_ms is not None else None
     o.color_cap = int(color_cap)
     o.round_ns = round_ns.data_ptr() if round_ns is not None else None
+    o.block_size = int(block_size)
+    o.unsorted_rows = int(bool(unsorted_rows))
     return o
 
 
@@ -212,14 +215,14 @@ def color_host_batch(graphs, tiebreak="lowid", *, outs=None, stream=None, **opt_
     return [ColorResult(outs[i], st[i].as_dict()) for i in range(cnt)]
 
 
-def assign(row_ptr, col_idx, wl, colors_in, *, out=None, stream=None):
+def assign(row_ptr, col_idx, wl, colors_in, *, out=None, stream=None, **opt_kw):
     """Alg. 5 l.4-10 step: tent[i] = first-fit of wl[i] against the snapshot colors_in."""
     torch = _torch()
     _check_csr(row_ptr, col_idx)
     _require_cuda(wl, colors_in)
     tent = out if out is not None else torch.empty(wl.numel(), dtype=torch.int32, device=wl.device)
     csr = Csr(row_ptr.data_ptr(), col_idx.data_ptr() if col_idx.numel() else None)
-    o = make_opts(stream=stream)
+    o = make_opts(stream=stream, **opt_kw)
     check(load().sgr_assign(ctypes.byref(csr), row_ptr.numel() - 1,
                             wl.data_ptr() if wl.numel() else None, wl.numel(),
                             colors_in.data_ptr() if colors_in.numel() else None,
@@ -228,10 +231,10 @@ def assign(row_ptr, col_idx, wl, colors_in, *, out=None, stream=None):
     return tent
 
 
-def commit(wl, tent, colors, *, stream=None):
+def commit(wl, tent, colors, *, stream=None, **opt_kw):
     """Alg. 5 l.9 applied after the step: colors[wl[i]] = tent[i] (in place)."""
     _require_cuda(wl, tent, colors)
-    o = make_opts(stream=stream)
+    o = make_opts(stream=stream, **opt_kw)
     check(load().sgr_commit(wl.data_ptr() if wl.numel() else None,
                             tent.data_ptr() if tent.numel() else None, wl.numel(),
                             colors.data_ptr() if colors.numel() else None, ctypes.byref(o)),
@@ -239,14 +242,14 @@ def commit(wl, tent, colors, *, stream=None):
     return colors
 
 
-def detect(row_ptr, col_idx, wl, colors, tiebreak="lowid", *, out=None, stream=None):
+def detect(row_ptr, col_idx, wl, colors, tiebreak="lowid", *, out=None, stream=None, **opt_kw):
     """Alg. 5 l.13-14 step: uint8 flag per listed vertex (1 = v loses a conflict)."""
     torch = _torch()
     _check_csr(row_ptr, col_idx)
     _require_cuda(wl, colors)
     flags = out if out is not None else torch.empty(wl.numel(), dtype=torch.uint8, device=wl.device)
     csr = Csr(row_ptr.data_ptr(), col_idx.data_ptr() if col_idx.numel() else None)
-    o = make_opts(tiebreak, stream)
+    o = make_opts(tiebreak, stream, **opt_kw)
     check(load().sgr_detect(ctypes.byref(csr), row_ptr.numel() - 1,
                             wl.data_ptr() if wl.numel() else None, wl.numel(),
                             colors.data_ptr() if colors.numel() else None,

@@ -84,8 +84,13 @@ Resolved resolve_opts(const sgr_opts* o, int64_t n) {
   r.round_ms = o->round_ms;
   r.color_cap = (o->color_cap > 0 && o->color_cap < (int32_t)kColorMask) ? o->color_cap
                                                                          : (int32_t)kColorMask;
+  r.block = o->block_size > 0 ? o->block_size : kBlock;
+  r.sorted = o->unsorted_rows ? 0 : 1;
   return r;
 }
+
+// opts->block_size: a multiple of 32 within [lo, hi] (sgr.h).
+bool block_ok(int B, int lo, int hi) { return B % 32 == 0 && B >= lo && B <= hi; }
 
 // Pinned host slots for termination flags (reused across calls on this thread).
 static int32_t* pinned_flags() {
@@ -99,7 +104,7 @@ size_t ws_bytes(int64_t n, int64_t nnz, const Resolved& r) { return layout(n, nn
 // ----- CUDA-graph cache: one graph = `batch` round passes -----------------------------------
 struct GraphKey {
   unsigned char args[sizeof(RoundArgs<int32_t>)];
-  int tiebreak, bits, batch, dev, grid;
+  int tiebreak, bits, batch, dev, grid, block;
   bool operator==(const GraphKey& o) const { return memcmp(this, &o, sizeof(GraphKey)) == 0; }
 };
 
@@ -107,7 +112,7 @@ static std::mutex g_graph_mu;
 static std::vector<std::pair<GraphKey, cudaGraphExec_t>> g_graphs;
 
 template <int TB, class C>
-static sgr_status get_graph(const RoundArgs<C>& a, int grid, int batch, cudaGraphExec_t* out) {
+static sgr_status get_graph(const RoundArgs<C>& a, int grid, int B, int batch, cudaGraphExec_t* out) {
   GraphKey key;
   memset(&key, 0, sizeof(key));
   static_assert(sizeof(RoundArgs<C>) <= sizeof(key.args), "graph key");
@@ -116,6 +121,7 @@ static sgr_status get_graph(const RoundArgs<C>& a, int grid, int batch, cudaGrap
   key.bits = packed<C>() ? 16 : 32;
   key.batch = batch;
   key.grid = grid;
+  key.block = B;
   cudaGetDevice(&key.dev);
   std::lock_guard<std::mutex> lk(g_graph_mu);
   for (auto& e : g_graphs)
@@ -132,7 +138,7 @@ static sgr_status get_graph(const RoundArgs<C>& a, int grid, int batch, cudaGrap
     return cuda_fail(err, "cudaStreamBeginCapture", __LINE__);
   }
   for (int b = 0; b < batch; ++b) {
-    k_round<TB, C><<<grid, kBlock, round_smem<C>(), cs>>>(a);
+    k_round<TB, C><<<grid, B, round_smem<C>(B), cs>>>(a);
     if constexpr (packed<C>()) k_finalize<TB, C><<<grid, kBlock, 0, cs>>>(a);
     k_advance<<<1, 32, 0, cs>>>(a.ctrl, 0);
   }
@@ -207,12 +213,13 @@ void fill_stats(const Ctrl& c, int64_t n, int64_t nnz, sgr_stats* st, int cb) {
   st->entries_written = (int64_t)c.list_writes_total;
   b_round += 4 * (int64_t)c.list_writes_total;
   for (int q = 0; q < kBins; ++q) st->bin_warp_cycles[q] = (int64_t)c.bin_cycles[q];
-  if (const char* env = getenv("SGR_PHASES")) {  // experiments: bin-2 phase breakdown
-    (void)env;
+#if SGR_PHASE_CYCLES
+  if (getenv("SGR_PHASES")) {  // experiments: bin-2 phase breakdown
     fprintf(stderr, "sgr phases (warp-cycles): issue %llu wait %llu gather %llu post %llu | barrier %llu finalize %llu counters %llu\n",
             c.phase_cycles[0], c.phase_cycles[1], c.phase_cycles[2], c.phase_cycles[3],
             c.phase_cycles[4], c.phase_cycles[5], c.phase_cycles[6]);
   }
+#endif
   st->rounds = c.k - 1;
   st->num_colors = c.max_color;
   st->vertices_processed = n + vpass;
@@ -241,8 +248,17 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
   prof.on = r.profile != 0;
   int32_t launches = 0;
   const bool persistent = r.loop_mode == SGR_LOOP_PERSISTENT;
-  const int grid = round_grid<TB, C>(persistent);
-  const int grid_flat = persistent ? round_grid<TB, C, false>(true) : grid;
+  const int B = r.block;
+  // the block size must suit the build the coloring runs (hub: <= 512 threads when packed);
+  // the persistent path enqueues both builds, so both must accept it
+  if (!block_ok(B, 64, round_max_block<C, true>()) ||
+      (persistent && !block_ok(B, 64, round_max_block<C, false>()))) {
+    set_error("sgr_color: block_size %d not supported by the round kernels (64..%d, multiple of 32)",
+              B, round_max_block<C, true>());
+    return SGR_EINVAL;
+  }
+  const int grid = round_grid<TB, C>(persistent, B);
+  const int grid_flat = persistent ? round_grid<TB, C, false>(true, B) : grid;
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
   sgr_status status = SGR_OK;
   do {
@@ -271,7 +287,7 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
     cudaEventCreate(&ev1);
     cudaEventRecord(ev0, s);
 
-    prof.timed(SGR_K_FIRST, s, [&] { k_first<TB, C><<<first_grid(n), 256, 0, s>>>(a, 1); });
+    prof.timed(SGR_K_FIRST, s, [&] { k_first<TB, C><<<first_grid(n, B), B, 0, s>>>(a, r.sorted); });
     prof.timed(SGR_K_CTRL, s, [&] { k_advance<<<1, 32, 0, s>>>(a.ctrl, 1); });
     launches += 2;
     le = cudaGetLastError();
@@ -284,11 +300,11 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
       // both builds are enqueued; the one that does not match F_1's bins returns at once
       prof.timed(SGR_K_ROUND, s, [&] {
         void* args[] = {(void*)&a};
-        le = cudaLaunchCooperativeKernel((const void*)k_persistent<TB, C, true>, grid, kBlock,
-                                         args, round_smem<C, true>(), s);
+        le = cudaLaunchCooperativeKernel((const void*)k_persistent<TB, C, true>, grid, B,
+                                         args, round_smem<C, true>(B), s);
         if (le == cudaSuccess)
           le = cudaLaunchCooperativeKernel((const void*)k_persistent<TB, C, false>, grid_flat,
-                                           kBlock, args, round_smem<C, false>(), s);
+                                           B, args, round_smem<C, false>(B), s);
       });
       launches += 2;
       if (le != cudaSuccess) {
@@ -306,7 +322,7 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
       cudaEventCreateWithFlags(&done_ev[1], cudaEventDisableTiming);
       const bool use_graph = r.loop_mode == SGR_LOOP_GRAPH && !prof.on;
       cudaGraphExec_t gexec = nullptr;
-      if (use_graph) status = get_graph<TB, C>(a, grid, r.batch, &gexec);
+      if (use_graph) status = get_graph<TB, C>(a, grid, B, r.batch, &gexec);
       // Pipelined termination test: batch b's `active` flag is read after batch b+1 is
       // enqueued, so the GPU never waits for the host; surplus passes are no-ops.
       int64_t batches = 0;
@@ -317,7 +333,7 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
         } else {
           for (int b = 0; b < r.batch; ++b) {
             prof.timed(SGR_K_ROUND, s, [&] {
-              k_round<TB, C><<<grid, kBlock, round_smem<C>(), s>>>(a);
+              k_round<TB, C><<<grid, B, round_smem<C>(B), s>>>(a);
               if constexpr (packed<C>()) k_finalize<TB, C><<<grid, kBlock, 0, s>>>(a);
             });
             prof.timed(SGR_K_CTRL, s, [&] { k_advance<<<1, 32, 0, s>>>(a.ctrl, 0); });
@@ -345,9 +361,9 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
 
     prof.timed(SGR_K_FINAL, s, [&] {
       if constexpr (packed<C>())
-        k_unpack<<<reduce_grid(n), 256, 0, s>>>(a.col[0], colors_out, n, &a.ctrl->max_color);
+        k_unpack<<<reduce_grid(n, B), B, 0, s>>>(a.col[0], colors_out, n, &a.ctrl->max_color);
       else
-        k_max_color<<<reduce_grid(n), 256, 0, s>>>(colors_out, n, &a.ctrl->max_color);
+        k_max_color<<<reduce_grid(n, B), B, 0, s>>>(colors_out, n, &a.ctrl->max_color);
     });
     launches += 1;
     cudaEventRecord(ev1, s);
@@ -501,6 +517,7 @@ sgr_status sgr_color_ex(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* col
   if (r.validate) {
     int32_t viol = 0;
     status = run_validate(csr, n, nnz, &((Ctrl*)ws)->violations, s, &viol);
+    if (!r.sorted) viol &= ~4;  // any row order is accepted with opts->unsorted_rows
     if (status == SGR_OK && viol) {
       set_error("sgr_color: invalid CSR (violation mask %d)", viol);
       status = SGR_EINVAL;
@@ -661,13 +678,18 @@ sgr_status sgr_color_topo(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* c
   cudaEvent_t e0, e1;
   CK(cudaEventCreate(&e0));
   CK(cudaEventCreate(&e1));
-  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, (int64_t)num_sms() * 16));
+  const int B = r.block;
+  if (!block_ok(B, 32, kMaxBlockAny)) {
+    set_error("sgr_color_topo: block_size %d (32..1024, multiple of 32)", B);
+    return SGR_EINVAL;
+  }
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((n + B - 1) / B, (int64_t)num_sms() * 16 * 256 / B));
   std::vector<int32_t> sizes;
   sgr_status status = SGR_OK;
   int launches = 0;
   CK(cudaMemsetAsync(edges, 0, 8, s));
   CK(cudaEventRecord(e0, s));
-  k_topo_init<<<grid, 256, 0, s>>>(n, flag, buf[0]);
+  k_topo_init<<<grid, B, 0, s>>>(n, flag, buf[0]);
   ++launches;
   int32_t cnt = (int32_t)n;  // |W_1| = n
   int32_t rr = 1;
@@ -679,13 +701,13 @@ sgr_status sgr_color_topo(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* c
       break;
     }
     sizes.push_back(cnt);
-    k_topo_assign<<<grid, 256, 0, s>>>(csr->row_ptr, csr->col_idx, n, rr, flag, buf[cur],
+    k_topo_assign<<<grid, B, 0, s>>>(csr->row_ptr, csr->col_idx, n, rr, flag, buf[cur],
                                        buf[cur ^ 1], edges);
     CK(cudaMemsetAsync(changed, 0, 4, s));
     if (r.tiebreak)
-      k_topo_detect<1><<<grid, 256, 0, s>>>(csr->row_ptr, csr->col_idx, n, rr, buf[cur ^ 1], flag, changed);
+      k_topo_detect<1><<<grid, B, 0, s>>>(csr->row_ptr, csr->col_idx, n, rr, buf[cur ^ 1], flag, changed);
     else
-      k_topo_detect<0><<<grid, 256, 0, s>>>(csr->row_ptr, csr->col_idx, n, rr, buf[cur ^ 1], flag, changed);
+      k_topo_detect<0><<<grid, B, 0, s>>>(csr->row_ptr, csr->col_idx, n, rr, buf[cur ^ 1], flag, changed);
     launches += 2;
     CK(cudaGetLastError());
     // the host reads `changed` every iteration (Alg. 4 l.22)
@@ -699,7 +721,7 @@ sgr_status sgr_color_topo(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* c
     CK(cudaMemcpyAsync(colors_out, buf[1], (size_t)n * 4, cudaMemcpyDeviceToDevice, s));
   int32_t* dmax = changed;
   CK(cudaMemsetAsync(dmax, 0, 4, s));
-  k_max_color<<<grid, 256, 0, s>>>(colors_out, n, dmax);
+  k_max_color<<<grid, B, 0, s>>>(colors_out, n, dmax);
   launches += 1;
   CK(cudaEventRecord(e1, s));
   int32_t mx = 0;
@@ -740,9 +762,9 @@ sgr_status sgr_color_topo(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* c
 }
 
 // ----- step entry points ------------------------------------------------------------------
-static int grid_for(int64_t items, int per_block) {
+static int grid_for(int64_t items, int per_block, int B = 256) {
   const int64_t b = (items + per_block - 1) / per_block;
-  return (int)std::max<int64_t>(1, std::min<int64_t>(b, (int64_t)num_sms() * 16));
+  return (int)std::max<int64_t>(1, std::min<int64_t>(b, (int64_t)num_sms() * 16 * 256 / B));
 }
 
 sgr_status sgr_assign(const sgr_csr* csr, int64_t n, const int32_t* wl, int64_t wl_len,
@@ -755,7 +777,8 @@ sgr_status sgr_assign(const sgr_csr* csr, int64_t n, const int32_t* wl, int64_t 
     return SGR_EINVAL;
   }
   const Resolved r = resolve_opts(opts, n);
-  k_assign_step<<<grid_for(wl_len, 8), 256, 0, r.stream>>>(csr->row_ptr, csr->col_idx, wl, wl_len,
+  if (!block_ok(r.block, 32, kMaxBlockAny)) return SGR_EINVAL;
+  k_assign_step<<<grid_for(wl_len, r.block / 32, r.block), r.block, 0, r.stream>>>(csr->row_ptr, csr->col_idx, wl, wl_len,
                                                            colors_in, tent_out);
   CK(cudaGetLastError());
   return SGR_OK;
@@ -767,7 +790,8 @@ sgr_status sgr_commit(const int32_t* wl, const int32_t* tent, int64_t wl_len, in
   if (wl_len == 0) return SGR_OK;
   if (!wl || !tent || !colors) return SGR_EINVAL;
   const Resolved r = resolve_opts(opts, 0);
-  k_commit_step<<<grid_for(wl_len, 256), 256, 0, r.stream>>>(wl, tent, wl_len, colors);
+  if (!block_ok(r.block, 32, kMaxBlockAny)) return SGR_EINVAL;
+  k_commit_step<<<grid_for(wl_len, r.block, r.block), r.block, 0, r.stream>>>(wl, tent, wl_len, colors);
   CK(cudaGetLastError());
   return SGR_OK;
 }
@@ -778,12 +802,14 @@ sgr_status sgr_detect(const sgr_csr* csr, int64_t n, const int32_t* wl, int64_t 
   if (wl_len == 0) return SGR_OK;
   if (!csr->row_ptr || !wl || !colors || !conflict_out) return SGR_EINVAL;
   const Resolved r = resolve_opts(opts, n);
+  if (!block_ok(r.block, 32, kMaxBlockAny)) return SGR_EINVAL;
+  const int g = grid_for(wl_len, r.block / 32, r.block);
   if (r.tiebreak)
-    k_detect_step<1><<<grid_for(wl_len, 8), 256, 0, r.stream>>>(csr->row_ptr, csr->col_idx, wl,
-                                                               wl_len, colors, conflict_out);
+    k_detect_step<1><<<g, r.block, 0, r.stream>>>(csr->row_ptr, csr->col_idx, wl, wl_len, colors,
+                                                  conflict_out);
   else
-    k_detect_step<0><<<grid_for(wl_len, 8), 256, 0, r.stream>>>(csr->row_ptr, csr->col_idx, wl,
-                                                               wl_len, colors, conflict_out);
+    k_detect_step<0><<<g, r.block, 0, r.stream>>>(csr->row_ptr, csr->col_idx, wl, wl_len, colors,
+                                                  conflict_out);
   CK(cudaGetLastError());
   return SGR_OK;
 }

@@ -68,6 +68,11 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
                             int32_t* colors_out, sgr_stats* stats, const Gather& gather,
                             int64_t cap_hint, const Resolved& r, int* overflow_out) {
   cudaStream_t s = r.stream;
+  const int B = r.block;
+  if (!block_ok(B, 64, round_max_block<C, true>())) {
+    set_error("sgr_color_dist: block_size %d not supported by the round kernels", B);
+    return SGR_EINVAL;
+  }
   keep_pool_memory();
   const int P = (int)parts.size();
   std::vector<Layout> Ls;
@@ -97,12 +102,12 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
     DCK(cudaMemcpyAsync(args[i].ctrl, &hc, sizeof(Ctrl), cudaMemcpyHostToDevice, s));
     DCK(cudaMemsetAsync((char*)pt.ws + Ls[i].zero_begin, 0, Ls[i].zero_end - Ls[i].zero_begin, s));
     k_fill_c1<C><<<first_grid(n), 256, 0, s>>>(args[i]);
-    k_first<TB, C><<<first_grid(pt.hi - pt.lo), 256, 0, s>>>(args[i], 1);
+    k_first<TB, C><<<first_grid(pt.hi - pt.lo), 256, 0, s>>>(args[i], r.sorted);
     k_advance<<<1, 32, 0, s>>>(args[i].ctrl, 1, 0);
   }
   DCK(cudaGetLastError());
-  const int grid = round_grid<TB, C>(false);
-  const int grid_flat = round_grid<TB, C, false>(false);
+  const int grid = round_grid<TB, C>(false, B);
+  const int grid_flat = round_grid<TB, C, false>(false, B);
   std::vector<int32_t> big(P, 0);  // per part: F_1's bin-2 slots (0: flat build)
   uint2* recv = nullptr;
   DCK(cudaMallocAsync((void**)&recv, (size_t)world * (cap_max + 1) * sizeof(uint2), s));
@@ -188,9 +193,9 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
       // the build the persistent kernel would pick: the flat one (more L1, no finalize
       // phase) when F_1 put no vertex of this part into bin 2 (world-1 cfg2 31.3 -> 26.5 ms)
       if (big[i] == 0) {
-        k_round<TB, C, false><<<grid_flat, kBlock, round_smem<C, false>(), st>>>(args[i]);
+        k_round<TB, C, false><<<grid_flat, B, round_smem<C, false>(B), st>>>(args[i]);
       } else {
-        k_round<TB, C><<<grid, kBlock, round_smem<C>(), st>>>(args[i]);
+        k_round<TB, C><<<grid, B, round_smem<C>(B), st>>>(args[i]);
         if constexpr (packed<C>()) k_finalize<TB, C><<<grid, kBlock, 0, st>>>(args[i]);
       }
       // W_{k+1} is bounded by cap_k: size the grid by it, not by the range (a thin
@@ -322,6 +327,12 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
     DCK(cudaStreamSynchronize(s));
     int overflow = overflow_seen ? 1 : 0;
     for (int i = 0; i < P; ++i) overflow |= fin[i].overflow;
+    for (int i = 0; i < P; ++i)
+      if (fin[i].violations & 8) {
+        set_error("sgr_color_dist: a rank sent more records than its previous worklist "
+                  "held (asymmetric CSR?)");
+        status = SGR_EINVAL;
+      }
     if (overflow && !packed<C>()) {
       set_error("sgr_color_dist: 32-bit color overflow");
       status = SGR_EUNSUPPORTED;

@@ -3,6 +3,7 @@
 #pragma once
 #include <cuda_runtime.h>
 
+#include <atomic>
 #include <cstdlib>
 #include <cstring>
 
@@ -115,34 +116,47 @@ inline void build_args(RoundArgs<C>& a, const sgr_csr* csr, int64_t n, int64_t n
 
 // Streaming per-vertex kernels (F_1, unpack, max): one thread per vertex up to 64 blocks
 // per SM, so the dependent row_ptr -> col_idx loads of many vertices are in flight.
-inline int first_grid(int64_t n) {
-  return (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, (int64_t)num_sms() * 64));
+// (B = threads per block; the caps keep 64 x 256 / 8 x 256 threads per SM for any B.)
+inline int first_grid(int64_t n, int B = 256) {
+  return (int)std::max<int64_t>(1, std::min<int64_t>((n + B - 1) / B, (int64_t)num_sms() * 64 * 256 / B));
 }
 // Per-vertex kernels that end in one atomic per warp (unpack + max): 8 blocks per SM.
-inline int reduce_grid(int64_t n) {
-  return (int)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, (int64_t)num_sms() * 8));
+inline int reduce_grid(int64_t n, int B = 256) {
+  return (int)std::max<int64_t>(1, std::min<int64_t>((n + B - 1) / B, std::max<int64_t>(num_sms(), (int64_t)num_sms() * 8 * 256 / B)));
 }
 
+// Dynamic shared memory of a round-kernel block of `B` threads (per-warp slices).
 template <class C, bool Hub = true>
-constexpr size_t round_smem() { return (size_t)kWarps * WarpSmem<C, Hub>::kBytes; }
+constexpr size_t round_smem(int B = kBlock) { return (size_t)(B / 32) * WarpSmem<C, Hub>::kBytes; }
+// Largest block the round kernels of this build accept (their launch bounds).
+template <class C, bool Hub = true>
+constexpr int round_max_block() { return kMaxThreads<C, Hub>; }
 
 // Blocks of the round kernels: as many as are co-resident (persistent: required).
 template <int TB, class C, bool Hub = true>
-inline int round_grid(bool persistent) {
-  static bool attr_set = false;
-  if (!attr_set) {  // opt in to > 48 KB of dynamic shared memory
-    cudaFuncSetAttribute(k_persistent<TB, C, Hub>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)round_smem<C, Hub>());
-    cudaFuncSetAttribute(k_round<TB, C, Hub>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         (int)round_smem<C, Hub>());
-    attr_set = true;
+inline int round_grid(bool persistent, int B = kBlock) {
+  // The > 48 KB dynamic shared memory opt-in is a per-device function attribute: one bit
+  // per device (setting it twice from racing threads is harmless; the bit only skips the
+  // call once it has succeeded on that device).
+  static std::atomic<uint64_t> attr_set{0};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  const uint64_t bit = (dev >= 0 && dev < 64) ? (1ull << dev) : 0ull;
+  if (!bit || !(attr_set.load(std::memory_order_acquire) & bit)) {
+    // the opt-in covers the largest block the build accepts
+    const int smax = (int)round_smem<C, Hub>(round_max_block<C, Hub>());
+    const cudaError_t e1 = cudaFuncSetAttribute(
+        k_persistent<TB, C, Hub>, cudaFuncAttributeMaxDynamicSharedMemorySize, smax);
+    const cudaError_t e2 = cudaFuncSetAttribute(
+        k_round<TB, C, Hub>, cudaFuncAttributeMaxDynamicSharedMemorySize, smax);
+    if (e1 == cudaSuccess && e2 == cudaSuccess && bit) attr_set.fetch_or(bit, std::memory_order_acq_rel);
   }
   int per_sm = 0;
   cudaError_t e = persistent
-      ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_persistent<TB, C, Hub>, kBlock,
-                                                      round_smem<C, Hub>())
-      : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_round<TB, C, Hub>, kBlock,
-                                                      round_smem<C, Hub>());
+      ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_persistent<TB, C, Hub>, B,
+                                                      round_smem<C, Hub>(B))
+      : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_round<TB, C, Hub>, B,
+                                                      round_smem<C, Hub>(B));
   if (e != cudaSuccess || per_sm <= 0) per_sm = 1;
   if (const char* env = getenv("SGR_BLOCKS_PER_SM")) {  // experiments: shrink the grid
     const int lim = atoi(env);

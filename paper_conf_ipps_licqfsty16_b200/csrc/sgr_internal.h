@@ -28,13 +28,20 @@ struct Resolved {
   float* round_ms;
   int32_t color_cap;
   int64_t* round_ns;
+  int block;      // threads per block (opts->block_size; 0 -> 256)
+  int sorted;     // rows sorted ascending (F_1 reads one entry per row); 0: whole rows
 };
+
+// Threads-per-block limits (opts->block_size): per-vertex kernels, and the fused round
+// kernels (register budget fixed by their launch bounds: hub build 512, others 768).
+constexpr int kMaxBlockAny = 1024;
 
 void set_error(const char* fmt, ...);
 sgr_status cuda_fail(cudaError_t e, const char* what, int line);
 int num_sms();
 void keep_pool_memory();
 Resolved resolve_opts(const sgr_opts* o, int64_t n);
+bool block_ok(int B, int lo, int hi);
 size_t ws_bytes(int64_t n, int64_t nnz, const Resolved& r);
 void fill_stats(const Ctrl& c, int64_t n, int64_t nnz, sgr_stats* st, int cb);
 

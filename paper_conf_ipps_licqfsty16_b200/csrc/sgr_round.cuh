@@ -85,8 +85,9 @@ constexpr int kJB = 4 * kQB;  // entries per lane per batch
 namespace sgr {
 
 constexpr int kBins = 3;
-constexpr int kBlock = 256;             // threads per block (8 warps)
+constexpr int kBlock = 256;             // default threads per block (8 warps; opts->block_size)
 constexpr int kWarps = kBlock / 32;
+constexpr int kMaxWarps = 32;           // static per-warp arrays: any block up to 1024 threads
 constexpr int kGroup = 8;               // lanes per vertex in bins 0 and 1
 constexpr int kG0 = 4;                  // lanes per vertex in bin 0
 constexpr int kK0 = 8;                  // entries per lane, bin 0 (4 x 8 = 32 = max small)
@@ -155,6 +156,12 @@ constexpr int kStage = kWin * 4;        // bytes per TMA stage: one bin-2 window
 #endif
 template <class C, bool Hub = true>
 constexpr int kMinBlocks = (packed<C>() && Hub) ? SGR_MINB : (Hub ? 3 : SGR_FLATB);
+// Launch bounds of the round kernels: the register budget of kMinBlocks 256-thread blocks
+// per SM (packed hub build 2 -> 128 registers, the others 3 -> 85), expressed as ONE block
+// of up to kMaxThreads threads, so any block size up to that (opts->block_size, the
+// paper's Fig. 8 parameter) launches with the same per-thread register allocation.
+template <class C, bool Hub = true>
+constexpr int kMaxThreads = kBlock * kMinBlocks<C, Hub>;
 template <class C, bool Hub = true> struct WarpSmem {
   static constexpr int kBuf = (packed<C>() && Hub) ? 2 * kStage : 0;
   static constexpr int kPush = kBuf + kTblBytes;         // push buffer (kPushBuf int32)
@@ -325,6 +332,20 @@ __device__ __forceinline__ void prefetch_l2(const void* p) {
 }
 
 // Release / acquire fence at GPU scope (lighter than the fence.sc.gpu of __threadfence()).
+// Phase-cycle accounting (SM clock per bin / bin-2 phase; experiments only, stats
+// bin_warp_cycles): compiled out unless SGR_PHASE_CYCLES=1, so the production kernel
+// carries no clock reads or counter atomics for it.
+#ifndef SGR_PHASE_CYCLES
+#define SGR_PHASE_CYCLES 0
+#endif
+__device__ __forceinline__ long long pclock() {
+#if SGR_PHASE_CYCLES
+  return clock64();
+#else
+  return 0;
+#endif
+}
+
 __device__ __forceinline__ void fence_acq_rel_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
 
 __device__ __forceinline__ int64_t make_item(int32_t v, int32_t c) {
@@ -447,7 +468,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
 // Writes col[0] = C_1 (all 1), col[1] = C_2, and W_2 into the bins' lists [0]; bin-2
 // vertices of W_2 get a slot and (packed mode) their list length len[0][v] = deg(v).
 template <int TB, class C>
-__global__ void __launch_bounds__(256) k_first(RoundArgs<C> a, int sorted) {
+__global__ void __launch_bounds__(1024) k_first(RoundArgs<C> a, int sorted) {
   Ctrl* ctrl = a.ctrl;
   C* __restrict__ X = a.col[0];
   C* __restrict__ Y = a.col[1];
@@ -477,7 +498,7 @@ __global__ void __launch_bounds__(256) k_first(RoundArgs<C> a, int sorted) {
     Counts* w2 = &ctrl->ring[rs(2)];
     {  // bins 0/1: one atomicAdd per BLOCK and bin (~40 % of all vertices enter W_2, so
        // per-warp atomics on the two list counters serialize over the whole grid)
-      __shared__ int32_t fcnt[2][kWarps], fbase[2][kWarps];
+      __shared__ int32_t fcnt[2][kMaxWarps], fbase[2][kMaxWarps];
       const int wid = threadIdx.x >> 5;
       const unsigned m0 = __ballot_sync(0xffffffffu, conflict && b == 0);
       const unsigned m1 = __ballot_sync(0xffffffffu, conflict && b == 1);
@@ -837,7 +858,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
   int* cursor = &ctrl->ring[rs(k)].pad[0];
   unsigned long long lwrites = 0;  // warp-uniform
   unsigned long long pc0 = 0, pc1 = 0, pc2 = 0, pc3 = 0;  // phase cycles (lane 0 adds)
-  long long tq = clock64();
+  long long tq = pclock();
   int i = gw, in = gw + NW, inn = gw + 2 * NW, innn = gw + 3 * NW;
   ChunkHdr cur, nxt;
   load_hdr(i, cur);
@@ -883,11 +904,11 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
       __syncwarp();
     }
 #else
-    const long long ta = clock64();
+    const long long ta = pclock();
     pc0 += (unsigned long long)(ta - tq);
     mbar_wait(bars + st, (ph >> st) & 1u);
     ph ^= 1u << st;
-    const long long tb = clock64();
+    const long long tb = pclock();
     pc1 += (unsigned long long)(tb - ta);
 #endif
     // live entries are compacted into the front of this stage as the batches go (a batch's
@@ -939,7 +960,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
       consume(bb, id, raw, okm);
     }
 #if !SGR_NO_TMA
-    const long long tc = clock64();
+    const long long tc = pclock();
     pc2 += (unsigned long long)(tc - tb);
 #endif
     if (lane == 0) {
@@ -1052,7 +1073,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
 #endif
     __syncwarp();
 #if !SGR_NO_TMA
-    tq = clock64();
+    tq = pclock();
     pc3 += (unsigned long long)(tq - tc);
 #endif
     st ^= 1;
@@ -1069,7 +1090,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
   if (lane == 0 && lwrites) atomicAdd(&ctrl->list_writes_total, lwrites);
   // once per pass: this thread's list writes before the next pass's TMA (async-proxy) reads
   fence_proxy_async_global();
-  if (lane == 0) {
+  if (SGR_PHASE_CYCLES && lane == 0) {
     atomicAdd(&ctrl->phase_cycles[0], pc0);
     atomicAdd(&ctrl->phase_cycles[1], pc1);
     atomicAdd(&ctrl->phase_cycles[2], pc2);
@@ -1103,8 +1124,9 @@ __device__ __forceinline__ void finalize_body(const RoundArgs<Packed>& a, int k)
   const int B = min(32, (nF + NW - 1) / NW);
   // every warp runs the same number of iterations (block-level aggregation below)
   const int iters = nF > 0 ? (nF + NW * B - 1) / (NW * B) : 0;
-  __shared__ int32_t fin_tot[3][kWarps];   // per warp: items, vertices, multi-chunk vertices
-  __shared__ int32_t fin_base[kWarps];
+  __shared__ int32_t fin_tot[3][kMaxWarps];   // per warp: items, vertices, multi-chunk vertices
+  __shared__ int32_t fin_base[kMaxWarps];
+  const int nwb = (int)(blockDim.x >> 5);
   const int wid = threadIdx.x >> 5;
   for (int it = 0; it < iters; ++it) {
     const int base = gw * B + it * NW * B;
@@ -1167,7 +1189,7 @@ __device__ __forceinline__ void finalize_body(const RoundArgs<Packed>& a, int k)
     __syncthreads();
     if (threadIdx.x == 0) {
       int32_t run = 0, vs = 0, mc = 0;
-      for (int q = 0; q < kWarps; ++q) {
+      for (int q = 0; q < nwb; ++q) {
         fin_base[q] = run;
         run += fin_tot[0][q];
         vs += fin_tot[1][q];
@@ -1176,7 +1198,7 @@ __device__ __forceinline__ void finalize_body(const RoundArgs<Packed>& a, int k)
       const int32_t b0 = run ? atomicAdd(&ctrl->ring[rs(k + 1)].c, run) : 0;
       if (vs) atomicAdd(&ctrl->ring[rs(k + 1)].cv, vs);
       if (mc) atomicAdd(&ctrl->ring[rs(k + 1)].pad[1], mc);
-      for (int q = 0; q < kWarps; ++q) fin_base[q] += b0;
+      for (int q = 0; q < nwb; ++q) fin_base[q] += b0;
     }
     __syncthreads();
     int32_t ob = 0;
@@ -1736,32 +1758,32 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, const C
   // Order within the pass. Default 2, 1, 0: the large chunk items first (claimed from a
   // cursor), the static small-vertex bins fill the tail. SGR_SMALL_FIRST: 0, 1, 2 (the
   // dynamic bin-2 claims absorb the static bins' imbalance before the barrier).
-  long long t0 = clock64();
+  long long t0 = pclock();
 #if SGR_SMALL_FIRST
   run_bin0();
-  long long t1 = clock64();
+  long long t1 = pclock();
   cyc[0] += (unsigned long long)(t1 - t0);
   run_bin1();
-  long long t2 = clock64();
+  long long t2 = pclock();
   cyc[1] += (unsigned long long)(t2 - t1);
   run_bin2();
-  cyc[2] += (unsigned long long)(clock64() - t2);
+  cyc[2] += (unsigned long long)(pclock() - t2);
 #else
   run_bin2();
-  long long t1 = clock64();
+  long long t1 = pclock();
   cyc[2] += (unsigned long long)(t1 - t0);
   run_bin1();
-  long long t2 = clock64();
+  long long t2 = pclock();
   cyc[1] += (unsigned long long)(t2 - t1);
   run_bin0();
-  cyc[0] += (unsigned long long)(clock64() - t2);
+  cyc[0] += (unsigned long long)(pclock() - t2);
 #endif
 }
 
 // Block reduction of the per-thread counters, one atomicAdd each per block.
 __device__ __forceinline__ void block_add6(unsigned long long (&x)[kBins],
                                            unsigned long long (&y)[kBins], Ctrl* ctrl, int k) {
-  __shared__ unsigned long long red[2 * kBins][kWarps];
+  __shared__ unsigned long long red[2 * kBins][kMaxWarps];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
 #pragma unroll
   for (int q = 0; q < 2 * kBins; ++q) {
@@ -1774,7 +1796,7 @@ __device__ __forceinline__ void block_add6(unsigned long long (&x)[kBins],
   if (wid == 0) {
 #pragma unroll
     for (int q = 0; q < 2 * kBins; ++q) {
-      unsigned long long z = lane < kWarps ? red[q][lane] : 0ull;
+      unsigned long long z = lane < (int)(blockDim.x >> 5) ? red[q][lane] : 0ull;
 #pragma unroll
       for (int o = 16; o > 0; o >>= 1) z += __shfl_xor_sync(0xffffffffu, z, o);
       if (lane == 0 && z) {
@@ -1936,7 +1958,14 @@ __global__ void k_apply(RoundArgs<C> a, const uint2* recv, int32_t parts, int32_
   for (int q = 0; q < parts; ++q) {
     if (q == me) continue;
     const uint2* r = recv + (int64_t)q * stride;
-    const int32_t cnt = (int32_t)r[0].x;
+    int32_t cnt = (int32_t)r[0].x;
+    // A count above the slot capacity means W_{k+1} is not inside W_k on that rank, which
+    // the method guarantees for a symmetric CSR (DESIGN.md §3 proof ii): never read past
+    // the sender's block; flag it (bit 8 of violations, reported as SGR_EINVAL).
+    if (cnt > stride - 1 || cnt < 0) {
+      if (threadIdx.x == 0 && blockIdx.x == 0) atomicOr(&a.ctrl->violations, 8);
+      cnt = cnt < 0 ? 0 : stride - 1;
+    }
     for (int32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += gridDim.x * blockDim.x) {
       const uint2 rec = r[1 + i];
       a.col[0][rec.x] = (C)rec.y;
@@ -1978,7 +2007,7 @@ __device__ __forceinline__ uint8_t* warp_smem_init(uint8_t* smem) {
 // distributed k_apply) follows it on the stream. Hub = false is the flat build (bins 0/1
 // only), for colorings whose F_1 put no vertex into bin 2 (the caller reads big_count).
 template <int TB, class C, bool Hub = true>
-__global__ void __launch_bounds__(kBlock, kMinBlocks<C, Hub>) k_round(RoundArgs<C> a) {
+__global__ void __launch_bounds__(kMaxThreads<C, Hub>, 1) k_round(RoundArgs<C> a) {
   extern __shared__ __align__(16) uint8_t dsmem[];
   Ctrl* ctrl = a.ctrl;
   if (!ctrl->active) return;  // uniform across the grid
@@ -1992,13 +2021,14 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks<C, Hub>) k_round(RoundArgs<
   block_add6(edges, entries, ctrl, k);
   // bin cycle stats: one atomic per block and bin (per-warp atomics were ~7K same-address
   // reductions per launch, on every pass of the host-driven loops)
-  __shared__ unsigned long long cred[kBins][kWarps];
+  __shared__ unsigned long long cred[kBins][kMaxWarps];
+  if (!SGR_PHASE_CYCLES) return;
   if ((threadIdx.x & 31) == 0)
     for (int q = 0; q < kBins; ++q) cred[q][threadIdx.x >> 5] = cyc[q];
   __syncthreads();
   if (threadIdx.x < kBins) {
     unsigned long long z = 0;
-    for (int i = 0; i < kWarps; ++i) z += cred[threadIdx.x][i];
+    for (int i = 0; i < (int)(blockDim.x >> 5); ++i) z += cred[threadIdx.x][i];
     atomicAdd(&ctrl->bin_cycles[threadIdx.x], z);
   }
 }
@@ -2062,7 +2092,7 @@ __device__ __forceinline__ void grid_sync(Ctrl* ctrl, uint32_t& epoch) {
 // it is the right one for this coloring (Hub iff F_1 put a vertex into bin 2), so the
 // choice needs no host round trip.
 template <int TB, class C, bool Hub>
-__global__ void __launch_bounds__(kBlock, kMinBlocks<C, Hub>) k_persistent(RoundArgs<C> a) {
+__global__ void __launch_bounds__(kMaxThreads<C, Hub>, 1) k_persistent(RoundArgs<C> a) {
   extern __shared__ __align__(16) uint8_t dsmem[];
   Ctrl* ctrl = a.ctrl;
   if ((ld_cg(&ctrl->big_count) != 0) != Hub) return;  // uniform across the grid
@@ -2092,9 +2122,9 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks<C, Hub>) k_persistent(Round
     }
     unsigned long long edges[kBins] = {0, 0, 0}, entries[kBins] = {0, 0, 0};
     round_body<TB, true, C, Hub>(a, k, w, wsm, edges, entries, ph, cyc);
-    const long long t0 = clock64();
+    const long long t0 = pclock();
     block_add6(edges, entries, ctrl, k);
-    const long long t1 = clock64();
+    const long long t1 = pclock();
     pcx[2] += (unsigned long long)(t1 - t0);
     // multi-chunk vertices: decided once all chunks are in (no finalize phase, and no
     // barrier for it, when W_k has none — most thin rounds of a skewed graph's tail)
@@ -2102,19 +2132,19 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks<C, Hub>) k_persistent(Round
     if constexpr (packed<C>() && Hub) fin_phase = w.pad[1] != 0;  // uniform over the grid
     if (fin_phase) {
       grid_sync(ctrl, epoch);
-      const long long t2 = clock64();
+      const long long t2 = pclock();
       if constexpr (packed<C>() && Hub) finalize_body<TB, true>(a, k);
-      const long long t3 = clock64();
+      const long long t3 = pclock();
       pcx[0] += (unsigned long long)(t2 - t1);
       pcx[1] += (unsigned long long)(t3 - t2);
       grid_sync(ctrl, epoch);
-      pcx[0] += (unsigned long long)(clock64() - t3);
+      pcx[0] += (unsigned long long)(pclock() - t3);
     } else {
       grid_sync(ctrl, epoch);
-      pcx[0] += (unsigned long long)(clock64() - t1);
+      pcx[0] += (unsigned long long)(pclock() - t1);
     }
   }
-  if ((threadIdx.x & 31) == 0) {
+  if (SGR_PHASE_CYCLES && (threadIdx.x & 31) == 0) {
     for (int q = 0; q < kBins; ++q) atomicAdd(&ctrl->bin_cycles[q], cyc[q]);
     for (int q = 0; q < 3; ++q) atomicAdd(&ctrl->phase_cycles[4 + q], pcx[q]);
   }

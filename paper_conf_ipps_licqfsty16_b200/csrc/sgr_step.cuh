@@ -21,7 +21,7 @@ static __global__ void k_max_color(const int32_t* __restrict__ c, int64_t n, int
 // Step entry points (Algorithm 5 split line by line; not on the fused hot path).
 
 // Alg. 5 l.4-10: warp per listed vertex, exact for any degree.
-static __global__ void __launch_bounds__(256) k_assign_step(const int64_t* __restrict__ row_ptr,
+static __global__ void __launch_bounds__(1024) k_assign_step(const int64_t* __restrict__ row_ptr,
                                                      const int32_t* __restrict__ col_idx,
                                                      const int32_t* __restrict__ wl, int64_t len,
                                                      const int32_t* __restrict__ X,
@@ -47,7 +47,7 @@ static __global__ void k_commit_step(const int32_t* __restrict__ wl, const int32
 
 // Alg. 5 l.13-14: warp per listed vertex.
 template <int TB>
-__global__ void __launch_bounds__(256) k_detect_step(const int64_t* __restrict__ row_ptr,
+__global__ void __launch_bounds__(1024) k_detect_step(const int64_t* __restrict__ row_ptr,
                                                      const int32_t* __restrict__ col_idx,
                                                      const int32_t* __restrict__ wl, int64_t len,
                                                      const int32_t* __restrict__ C,

@@ -37,7 +37,7 @@ __device__ __forceinline__ int32_t thread_first_fit(const int32_t* __restrict__ 
 }
 
 // Alg. 4 l.4-13 for iteration r: T[v] = colored[v] ? X[v] : first fit against X.
-static __global__ void __launch_bounds__(256) k_topo_assign(const int64_t* __restrict__ row_ptr,
+static __global__ void __launch_bounds__(1024) k_topo_assign(const int64_t* __restrict__ row_ptr,
                                                             const int32_t* __restrict__ col_idx,
                                                             int64_t n, int32_t r,
                                                             const int32_t* __restrict__ flag,
@@ -61,7 +61,7 @@ static __global__ void __launch_bounds__(256) k_topo_assign(const int64_t* __res
 // Alg. 4 l.15-21 for iteration r over every vertex: a conflict makes v uncolored for
 // iteration r + 1 (flag[v] = r + 1) and counts towards `changed`.
 template <int TB>
-__global__ void __launch_bounds__(256) k_topo_detect(const int64_t* __restrict__ row_ptr,
+__global__ void __launch_bounds__(1024) k_topo_detect(const int64_t* __restrict__ row_ptr,
                                                      const int32_t* __restrict__ col_idx,
                                                      int64_t n, int32_t r,
                                                      const int32_t* __restrict__ T,

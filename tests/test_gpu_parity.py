@@ -201,8 +201,85 @@ def test_validate_rejects_bad_csr():
     assert sgr.validate_csr(rp, ci) & 4
     with pytest.raises(RuntimeError, match="invalid"):
         sgr.color(rp, ci, validate=True)
+    # unsorted rows are accepted (and colored exactly) with opts->unsorted_rows
+    sgr.color(rp, ci, validate=True, unsorted_rows=True)
     g = gen.config(1)
     assert sgr.validate_csr(*dev(g)) == 0
+
+
+def shuffled_rows(g, seed):
+    """Same graph, every row's entries in a random order (the contract's sorted order off)."""
+    rng = np.random.default_rng(seed)
+    ci = g.col_idx.copy()
+    for v in range(g.n):
+        a, b = int(g.row_ptr[v]), int(g.row_ptr[v + 1])
+        ci[a:b] = rng.permutation(ci[a:b])
+    return gen.Graph(g.n, g.nnz, g.row_ptr.copy(), ci, g.name + "-shuffled")
+
+
+@pytest.mark.parametrize("seed", range(6))
+@pytest.mark.parametrize("tb", [LOW, PAP])
+def test_unsorted_rows_flag(seed, tb):
+    """opts->unsorted_rows: F_1 scans whole rows; colors, R and |W_r| equal the oracle's
+    (which never depends on row order) for graphs whose rows are shuffled."""
+    g = random_graph(seed, n=300) if seed < 4 else gen.rmat(12, 8, 0.57, 0.19, 0.19, seed=seed)
+    h = shuffled_rows(g, seed)
+    rp, ci = dev(h)
+    ref = oracle.jacobi(h, tb)
+    for mode in ("persistent", "host"):
+        res = sgr.color(rp, ci, RULE[tb], trace=True, unsorted_rows=True, loop_mode=mode)
+        assert res.stats["rounds"] == ref.rounds
+        assert np.array_equal(res.colors.cpu().numpy(), ref.colors)
+        assert np.array_equal(res.round_sizes, ref.round_sizes)
+
+
+@pytest.mark.parametrize("B", [64, 96, 128, 256, 384, 512])
+@pytest.mark.parametrize("tb", [LOW, PAP])
+def test_block_size_never_changes_the_result(B, tb):
+    """opts->block_size (the paper's Fig. 8 parameter) is performance only: the
+    hub build (R-MAT with multi-chunk rows), the flat build (stencil) and both loop modes
+    give the oracle's colors, R and |W_r| at every supported size."""
+    for g in (gen.rmat(13, 8, 0.57, 0.19, 0.19, seed=2), gen.stencil3d(12, 11, 10, 27),
+              degree_boundary_graph()):
+        ref = oracle.jacobi(g, tb)
+        rp, ci = dev(g)
+        for mode in ("persistent", "host"):
+            res = sgr.color(rp, ci, RULE[tb], trace=True, block_size=B, loop_mode=mode)
+            assert res.stats["rounds"] == ref.rounds, (g.name, B, mode)
+            assert np.array_equal(res.colors.cpu().numpy(), ref.colors), (g.name, B, mode)
+            assert np.array_equal(res.round_sizes, ref.round_sizes)
+        res = sgr.color(rp, ci, RULE[tb], block_size=B, color_bits=32)
+        assert np.array_equal(res.colors.cpu().numpy(), ref.colors), (g.name, B, "int32")
+
+
+@pytest.mark.parametrize("B", [32, 64, 128, 256, 512, 1024])
+def test_block_size_topology_driven_and_steps(B):
+    """Per-vertex kernels take any multiple of 32 up to 1024: the topology-driven mapping
+    (Algorithm 4, the paper's thread-per-vertex kernel of Fig. 8) and the step entry points."""
+    g = gen.rmat(12, 8, 0.57, 0.19, 0.19, seed=3)
+    rp, ci = dev(g)
+    ref = oracle.jacobi(g, LOW)
+    res = sgr.color_topo(rp, ci, "lowid", block_size=B)
+    assert np.array_equal(res.colors.cpu().numpy(), ref.colors)
+    assert res.stats["rounds"] == ref.rounds
+    rng = np.random.default_rng(B)
+    snap = rng.integers(0, 9, g.n).astype(np.int32)
+    wl = np.sort(rng.choice(g.n, size=g.n // 3, replace=False)).astype(np.int32)
+    twl, tsnap = torch.from_numpy(wl).cuda(), torch.from_numpy(snap).cuda()
+    tent = sgr.assign(rp, ci, twl, tsnap, block_size=B)
+    assert np.array_equal(tent.cpu().numpy(), oracle.assign(g, wl, snap))
+    fl = sgr.detect(rp, ci, twl, tsnap, "paper", block_size=B)
+    assert np.array_equal(fl.cpu().numpy(), oracle.detect(g, wl, snap, PAP))
+
+
+def test_block_size_rejected():
+    g = gen.rmat(10, 8, 0.57, 0.19, 0.19, seed=1)
+    rp, ci = dev(g)
+    for B in (33, 16, 2048, 1024):  # 1024 exceeds the fused round kernels' launch bounds
+        with pytest.raises(RuntimeError, match="invalid argument"):
+            sgr.color(rp, ci, block_size=B)
+    with pytest.raises(RuntimeError, match="invalid argument"):
+        sgr.color_topo(rp, ci, block_size=48)
 
 
 def test_color_host_equals_device():
@@ -272,6 +349,28 @@ def test_step_entry_points(seed):
     assert np.array_equal(colors.cpu().numpy(), exp)
 
 
+@pytest.mark.parametrize("seed", range(8))
+def test_step_assign_with_self_loops(seed):
+    """Reading C7 on the step API: sgr_assign is Alg. 5 l.5-6 literally, so a listed
+    self-loop forbids v's own snapshot color; GPU and oracle agree on graphs with self-loops
+    and duplicate entries under arbitrary snapshots (and detection never flags a loop)."""
+    rng = np.random.default_rng(100 + seed)
+    h = with_loops_and_dups(random_graph(seed, n=int(rng.integers(2, 300))), seed)
+    rp, ci = dev(h)
+    snap = rng.integers(0, 7, h.n).astype(np.int32)
+    wl = np.arange(h.n, dtype=np.int32)
+    twl, tsnap = torch.from_numpy(wl).cuda(), torch.from_numpy(snap).cuda()
+    assert np.array_equal(sgr.assign(rp, ci, twl, tsnap).cpu().numpy(), oracle.assign(h, wl, snap))
+    for tb in (LOW, PAP):
+        assert np.array_equal(sgr.detect(rp, ci, twl, tsnap, RULE[tb]).cpu().numpy(),
+                              oracle.detect(h, wl, snap, tb))
+    # one vertex with a self-loop, snapshot color 1: l.6 forbids 1, so the first fit is 2
+    one = raw_csr(1, [(0, 0)])
+    t = sgr.assign(*dev(one), torch.zeros(1, dtype=torch.int32, device="cuda"),
+                   torch.ones(1, dtype=torch.int32, device="cuda"))
+    assert t.cpu().tolist() == [2]
+
+
 def test_step_loop_reproduces_algorithm5():
     """Driving assign -> commit -> detect -> compact from Python = the fused library path."""
     g = gen.rmat(13, 8, 0.57, 0.19, 0.19, seed=6)
@@ -314,16 +413,19 @@ def test_full_size_configs_bit_exact(cfg):
 
 
 @pytest.mark.slow
-@pytest.mark.skipif(os.environ.get("SGR_TEST_CFG5") != "1",
-                    reason="cfg5 (R-MAT s27, 2.1 G entries): ~10 min; set SGR_TEST_CFG5=1")
 def test_cfg5_full_size():
-    """BASELINE config 5 (R-MAT scale 27, nnz 2.13e9, int64 offsets) on one GPU against the
-    full oracle (OpenMP), plus the partitioned protocol on 2 partitions of the same device."""
+    """BASELINE config 5 (R-MAT scale 27, nnz 2.13e9 > 2^31: the int64-offset path, reading
+    C17) on one GPU against the full oracle (OpenMP), element by element (colors, R, |W_r|,
+    sum deg(W_r)), plus the partitioned protocol on 2 partitions of the same device. Runs in
+    the default -m gpu suite (a few minutes: generation + the OpenMP oracle dominate)."""
     g = gen.config(5)
+    assert g.nnz > 2 ** 31 and int(g.row_ptr[g.n // 2]) < 2 ** 31 < int(g.row_ptr[-1])
     res, ref = check_full(g, LOW)
+    assert res.stats["color_bits"] == 16
     rp, ci = dev(g)
     part = sgr.color_partitioned(rp, ci, 2)
     assert np.array_equal(part.colors.cpu().numpy(), ref.colors)
+    assert part.stats["rounds"] == ref.rounds
 
 
 # ----------------------------------------------------------------------------- multi-GPU path

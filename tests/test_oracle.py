@@ -273,6 +273,24 @@ def test_step_functions(seed):
             assert bool(fl[i]) == exp
 
 
+def test_step_assign_self_loop_reading_c7():
+    """Reading C7 on the step API: oracle_assign is Alg. 5 l.5-6 literally —
+    w ranges over every listed entry, so a self-loop forbids v's own snapshot color. Hand
+    values: a lone vertex with a loop and snapshot color 1 gets 2 (without the loop: 1); a
+    duplicated entry changes nothing; detection never flags a loop (l.14: v < v is false)."""
+    loop = raw_csr(1, [(0, 0)])
+    assert oracle.assign(loop, [0], [1]).tolist() == [2]
+    assert oracle.assign(loop, [0], [3]).tolist() == [1]
+    bare = raw_csr(1, [])
+    assert oracle.assign(bare, [0], [1]).tolist() == [1]
+    # path 0-1 with a loop on 1 and a duplicated (0,1): snapshot [1, 2]
+    g = raw_csr(2, [(0, 1), (0, 1), (1, 0), (1, 0), (1, 1)])
+    assert oracle.assign(g, [0, 1], [1, 2]).tolist() == [1, 3]
+    assert oracle.detect(g, [0, 1], [2, 2], LOW).tolist() == [0, 1]
+    assert oracle.detect(loop, [0], [1], LOW).tolist() == [0]
+    assert oracle.detect(loop, [0], [1], PAP).tolist() == [0]
+
+
 def test_rmat_s16_quality_and_rule_asymmetry():
     """cfg1: lowid uses about as many colors as Algorithm 1 (north_star: within 10%),
     the paper rule noticeably more on unpermuted R-MAT (SURVEY exec. summary item 3)."""
