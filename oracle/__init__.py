@@ -51,6 +51,7 @@ def _load():
     lib.oracle_assign.argtypes = [vp, vp, i64, vp, i64, vp, vp]
     lib.oracle_detect.argtypes = [vp, vp, i64, vp, i64, vp, i32, vp]
     lib.oracle_jacobi_partitioned.argtypes = [vp, vp, i64, i32, i32, vp, vp, vp]
+    lib.oracle_gauss_seidel.argtypes = [vp, vp, i64, i32, i64, i32, i64, vp, vp, i64, vp]
     lib.oracle_max_threads.argtypes = []
     _lib = lib
     return lib
@@ -118,6 +119,28 @@ def jacobi(g, tiebreak: int = TIEBREAK_LOWID_KEEPS, detect_over_v: bool = False,
                                       nthreads, max_rounds, _ptr(color),
                                       ctypes.cast(trace, ctypes.c_void_p), cap,
                                       ctypes.byref(rounds)), "jacobi")
+    r = rounds.value
+    dt = np.dtype([("w_size", np.int64), ("w_edges", np.int64), ("next_size", np.int64),
+                   ("max_color", np.int32), ("pad", np.int32)])
+    tr = np.frombuffer(trace, dtype=dt, count=min(r, cap)).copy()
+    return JacobiResult(color, r, tr, rc == 0)
+
+
+def gauss_seidel(g, substeps: int, partition: int = 0, tiebreak: int = TIEBREAK_LOWID_KEEPS,
+                 max_rounds: int = 0, trace_cap: int | None = None) -> JacobiResult:
+    """O3 — K-sub-step Gauss-Seidel rounds; partition 0 = strided
+    (v mod K), 1 = blocked (floor(v K / n)). See oracle/sgr_oracle.h."""
+    rp, ci, n = _csr(g)
+    color = np.zeros(n, np.int32)
+    cap = (n + 1) if trace_cap is None else trace_cap
+    if max_rounds > 0:
+        cap = min(cap, max_rounds)
+    trace = (Round * max(cap, 1))()
+    rounds = ctypes.c_int64(0)
+    rc = _check(_load().oracle_gauss_seidel(_ptr(rp), _ptr(ci), n, tiebreak, int(substeps),
+                                            int(partition), max_rounds, _ptr(color),
+                                            ctypes.cast(trace, ctypes.c_void_p), cap,
+                                            ctypes.byref(rounds)), "gauss_seidel")
     r = rounds.value
     dt = np.dtype([("w_size", np.int64), ("w_edges", np.int64), ("next_size", np.int64),
                    ("max_color", np.int32), ("pad", np.int32)])

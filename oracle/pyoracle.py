@@ -52,3 +52,23 @@ def jacobi(n, adj, rule=LOWID_KEEPS):
         W = [v for v in W if any(color[w] == color[v] and loses(rule, v, w) for w in adj[v])]
         history.append(list(color))
     return color, len(worklists), worklists, history
+
+
+def gauss_seidel(n, adj, K, partition=0, rule=LOWID_KEEPS):
+    """K-sub-step rounds: the round's vertices go in K groups, in
+    order; a group sees the colors the earlier groups of the round gave. Returns
+    (colors, rounds, [sorted W_r])."""
+    def part(v):
+        return (v * K) // n if partition == 1 else v % K
+    color = [0] * n
+    W = list(range(n))
+    worklists = []
+    while W:
+        worklists.append(sorted(W))
+        for j in range(K):
+            seen = dict(enumerate(color))
+            for v in W:
+                if part(v) == j:
+                    color[v] = mex_positive({seen[w] for w in adj[v]})
+        W = [v for v in W if any(color[w] == color[v] and loses(rule, v, w) for w in adj[v])]
+    return color, len(worklists), worklists

@@ -190,6 +190,78 @@ int oracle_jacobi(const int64_t* row_ptr, const int32_t* col_idx, int64_t n, int
   return status;
 }
 
+/* ---------------------------------------------------------------------------------------
+ * O3 — K-sub-step Gauss-Seidel rounds (reading C20).
+ * The paper's kernels write color[v] in place inside the parallel loop of Alg. 5 l.4-10
+ * (P:169), so later threads may read earlier threads' new colors. O3 makes
+ * that deterministic: the loop runs as K sub-steps in a fixed order, each one Jacobi
+ * against the colors left by the sub-steps before it.
+ * ------------------------------------------------------------------------------------- */
+static int64_t gs_part(int64_t v, int64_t n, int64_t K, int partition) {
+  return partition == 1 ? (int64_t)(((__int128)v * K) / n) : v % K;
+}
+
+int oracle_gauss_seidel(const int64_t* row_ptr, const int32_t* col_idx, int64_t n, int tiebreak,
+                        int64_t K, int partition, int64_t max_rounds, int32_t* color,
+                        oracle_round* trace, int64_t trace_cap, int64_t* rounds_out) {
+  if (n < 0 || !row_ptr || (n > 0 && (!color || (!col_idx && row_ptr[n] > 0)))) return -1;
+  if (tiebreak != ORACLE_TIEBREAK_PAPER && tiebreak != ORACLE_TIEBREAK_LOWID_KEEPS) return -1;
+  if (K < 1 || (partition != 0 && partition != 1)) return -1;
+  const int64_t masklen = max_degree(row_ptr, n) + 2;
+  const size_t nn = (size_t)(n > 0 ? n : 1);
+  int32_t* W_in = (int32_t*)malloc(nn * sizeof(int32_t));
+  int32_t* W_out = (int32_t*)malloc(nn * sizeof(int32_t));
+  int32_t* snapshot = (int32_t*)malloc(nn * sizeof(int32_t));
+  int64_t* colorMask = (int64_t*)malloc((size_t)masklen * sizeof(int64_t));
+  if (!W_in || !W_out || !snapshot || !colorMask) {
+    free(W_in); free(W_out); free(snapshot); free(colorMask);
+    return -2;
+  }
+  for (int64_t i = 0; i < masklen; ++i) colorMask[i] = -1;      /* a not in V       */
+  for (int64_t v = 0; v < n; ++v) color[v] = 0;
+  int64_t w_len = n;                                             /* l.2 W_in <- V    */
+  for (int64_t v = 0; v < n; ++v) W_in[v] = (int32_t)v;
+  int64_t r = 0, label = 0;
+  int status = 0;
+  while (w_len > 0) {                                            /* l.3              */
+    if (max_rounds > 0 && r == max_rounds) {
+      status = 1;
+      break;
+    }
+    ++r;
+    int64_t w_edges = 0;
+    for (int64_t j = 0; j < K; ++j) {                            /* sub-steps in order */
+      /* sub-step j reads the colors as the previous sub-steps left them (Jacobi inside) */
+      memcpy(snapshot, color, (size_t)n * sizeof(int32_t));
+      for (int64_t i = 0; i < w_len; ++i) {                      /* l.4 v in W_in    */
+        const int64_t v = W_in[i];
+        if (gs_part(v, n, K, partition) != j) continue;
+        color[v] = first_fit(row_ptr, col_idx, v, snapshot, colorMask, label++); /* l.5-9 */
+        w_edges += row_ptr[v + 1] - row_ptr[v];
+      }
+    }
+    int64_t out_len = 0;                                         /* l.11-18 over W_in */
+    for (int64_t i = 0; i < w_len; ++i)
+      if (has_conflict(row_ptr, col_idx, W_in[i], color, tiebreak)) W_out[out_len++] = W_in[i];
+    if (trace && r - 1 < trace_cap) {
+      int32_t mc = 0;
+      for (int64_t v = 0; v < n; ++v) mc = color[v] > mc ? color[v] : mc;
+      trace[r - 1].w_size = w_len;
+      trace[r - 1].w_edges = w_edges;
+      trace[r - 1].next_size = out_len;
+      trace[r - 1].max_color = mc;
+      trace[r - 1].pad = 0;
+    }
+    int32_t* t = W_in;                                           /* l.19             */
+    W_in = W_out;
+    W_out = t;
+    w_len = out_len;
+  }
+  if (rounds_out) *rounds_out = r;
+  free(W_in); free(W_out); free(snapshot); free(colorMask);
+  return status;
+}
+
 int oracle_assign(const int64_t* row_ptr, const int32_t* col_idx, int64_t n, const int32_t* wl,
                   int64_t wl_len, const int32_t* snapshot, int32_t* tent) {
   if (n < 0 || wl_len < 0 || !row_ptr || (wl_len > 0 && (!wl || !snapshot || !tent))) return -1;

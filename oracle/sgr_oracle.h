@@ -73,6 +73,19 @@ int oracle_jacobi_partitioned(const int64_t* row_ptr, const int32_t* col_idx, in
                               int tiebreak, int P, const int64_t* ranges, int32_t* color,
                               int64_t* rounds_out);
 
+/* O3 — reduced-round variant (DESIGN.md §3 reading C20): Algorithm 5
+ * with each round's assignment loop (l.4-10) split into K sub-steps taken in order
+ * j = 0..K-1. Vertex v belongs to sub-step part(v) = v mod K (partition 0, "strided") or
+ * floor(v * K / n) (partition 1, "blocked", ids in order). Sub-step j assigns its members of
+ * W_in against the colors as the previous sub-step left them — the in-place writes of
+ * Alg. 5 l.9 become visible between sub-steps — and, within the sub-step,
+ * against that sub-step's snapshot (Jacobi). Detection (l.12-18) follows the K sub-steps
+ * as in O2. K = 1 is O2; K = n, blocked, is Algorithm 1 in one round. Same trace, return
+ * values and max_rounds meaning as oracle_jacobi; single-threaded. */
+int oracle_gauss_seidel(const int64_t* row_ptr, const int32_t* col_idx, int64_t n, int tiebreak,
+                        int64_t K, int partition, int64_t max_rounds, int32_t* color,
+                        oracle_round* trace, int64_t trace_cap, int64_t* rounds_out);
+
 /* Number of worker threads oracle_jacobi would use for nthreads <= 0 (OpenMP max). */
 int oracle_max_threads(void);
 

@@ -301,3 +301,81 @@ def test_rmat_s16_quality_and_rule_asymmetry():
     assert abs(lo.num_colors - a1) <= 0.10 * a1
     assert pa.num_colors > lo.num_colors
     assert is_proper(g, lo.colors) and is_proper(g, pa.colors)
+
+
+# ----------------------------------------------------------------------------- O3 (§8(f) item 4)
+def path(n):
+    return gen.from_edges(n, np.stack([np.arange(n - 1), np.arange(1, n)], 1).astype(np.int64))
+
+
+@pytest.mark.parametrize("seed", range(12))
+@pytest.mark.parametrize("part", [0, 1])
+def test_gs_one_substep_is_jacobi(seed, part):
+    """K = 1: one sub-step per round is O2 exactly (colors, R, the whole trace)."""
+    g = random_graph(seed) if seed < 10 else gen.rmat(11, 8, 0.57, 0.19, 0.19, seed=seed)
+    for tb in (LOW, PAP):
+        a = oracle.gauss_seidel(g, 1, part, tb)
+        b = oracle.jacobi(g, tb)
+        assert np.array_equal(a.colors, b.colors) and a.rounds == b.rounds
+        assert np.array_equal(a.trace, b.trace)
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_gs_n_substeps_is_algorithm1(seed):
+    """K = n: every vertex is its own sub-step, taken in id order (blocked, and strided since
+    v mod n = v), i.e. Algorithm 1 in natural order — pinned to networkx's greedy_color —
+    finished in one round (a sequential greedy coloring has no conflict)."""
+    g = random_graph(seed, n=40)
+    G = to_nx(g)
+    nxc = nx.greedy_color(G, strategy=lambda G_, c: list(range(g.n)))
+    ref = np.array([nxc[v] + 1 for v in range(g.n)], np.int32)
+    for part in (0, 1):
+        for tb in (LOW, PAP):
+            r = oracle.gauss_seidel(g, max(g.n, 1), part, tb)
+            assert np.array_equal(r.colors, ref) and r.rounds == (1 if g.n else 0)
+
+
+def test_gs_hand_traces():
+    """Hand-derived. P4 = 0-1-2-3:
+    K=2 strided, lowid: sub-step {0,2} against all-0 -> [1,0,1,0]; {1,3} -> [1,2,1,2]; proper, R=1.
+    K=2 blocked ({0,1},{2,3}), lowid: {0,1} -> [1,1,0,0]; {2,3} against it: 2 -> mex{1,0}=2,
+      3 -> mex{0}=1 -> [1,1,2,1]; 1 loses to 0 -> W2={1}; round 2: 1 -> mex{1,2}=3 -> [1,3,2,1], R=2.
+    K=2 blocked, paper rule: same round 1; 0 loses to 1 (0 < 1) -> W2={0}; 0 -> mex{1}=2 -> [2,1,2,1].
+    K3, K=3 strided: 0 -> 1; 1 -> mex{1,0}=2; 2 -> mex{1,2}=3 -> [1,2,3], R=1."""
+    p4 = path(4)
+    r = oracle.gauss_seidel(p4, 2, 0, LOW)
+    assert r.colors.tolist() == [1, 2, 1, 2] and r.rounds == 1
+    r = oracle.gauss_seidel(p4, 2, 1, LOW)
+    assert r.colors.tolist() == [1, 3, 2, 1] and r.rounds == 2
+    assert r.round_sizes.tolist() == [4, 1]
+    r = oracle.gauss_seidel(p4, 2, 1, PAP)
+    assert r.colors.tolist() == [2, 1, 2, 1] and r.rounds == 2
+    k3 = gen.from_edges(3, np.array([[0, 1], [1, 2], [0, 2]], np.int64))
+    r = oracle.gauss_seidel(k3, 3, 0, LOW)
+    assert r.colors.tolist() == [1, 2, 3] and r.rounds == 1
+
+
+@pytest.mark.parametrize("n", [2, 5, 64, 1001])
+def test_gs_path_two_strided_substeps_closed_form(n):
+    """A natural-order path with K = 2 strided: evens take 1, then odds take 2 -> Algorithm 1
+    (alternating 1, 2) in one round, against O2's n rounds (test_path_rounds_closed_form)."""
+    r = oracle.gauss_seidel(path(n), 2, 0, LOW)
+    assert r.rounds == 1 and r.colors.tolist() == [1 + (v & 1) for v in range(n)]
+
+
+@pytest.mark.parametrize("seed", range(24))
+def test_gs_c_equals_python_twin_and_invariants(seed):
+    g = random_graph(seed)
+    adj = adjacency(g)
+    rng = np.random.default_rng(seed)
+    K = int(rng.integers(2, 7))
+    for part in (0, 1):
+        for tb, rule in ((LOW, pyoracle.LOWID_KEEPS), (PAP, pyoracle.PAPER)):
+            r = oracle.gauss_seidel(g, K, part, tb)
+            col, R, wls = pyoracle.gauss_seidel(g.n, adj, K, part, rule)
+            assert r.colors.tolist() == col and r.rounds == R
+            assert r.round_sizes.tolist() == [len(w) for w in wls]
+            assert is_proper(g, r.colors)
+            assert np.all(r.colors <= g.degrees + 1) and (g.n == 0 or r.colors.min() >= 1)
+            for a, b in zip(wls, wls[1:]):  # W strictly shrinking, W_{r+1} inside W_r
+                assert len(b) < len(a) and set(b) <= set(a)
