@@ -44,6 +44,10 @@ def parse():
     ap.add_argument("--loop-mode", default="auto")
     ap.add_argument("--dist", action="store_true",
                     help="use the multi-GPU (NCCL) path even for one rank")
+    ap.add_argument("--block-size", type=int, default=0,
+                    help="threads per block (opts->block_size; 0 = 256)")
+    ap.add_argument("--no-secondary", action="store_true",
+                    help="skip the secondary paper-rule (v < w) line")
     return ap.parse_args()
 
 
@@ -51,6 +55,15 @@ def parse():
 # into a 64 MB L2-resident array, ~1 distinct 128-byte line per SM-cycle; see
 # profiles/r01_ncu_summary.md). The round kernel's binding resource besides HBM.
 GATHER_PEAK_G = 271.0
+
+
+def ncu_metric(workload: str, kernel: str, key: str):
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if not os.path.exists(p):
+        return None
+    with open(p) as f:
+        d = json.load(f)
+    return d.get(workload, {}).get(kernel, {}).get(key)
 
 
 def ncu_traffic(workload: str, kernel: str):
@@ -127,6 +140,33 @@ def workload_name(cfg):
     return gen.CONFIG_NAMES[cfg]
 
 
+def bench_config(args, g) -> dict:
+    """The workload a line is quoted on; identical for our arm and the reference arm."""
+    return {"workload": workload_name(args.config), "n": g.n, "nnz": g.nnz,
+            "tiebreak": args.tiebreak, "parallelism": "single GPU",
+            "l2": "flushed between steps (256 MiB write, outside the step events); "
+                  "CSR inputs 1.2 GB > L2",
+            "loop_mode": args.loop_mode, "block_size": args.block_size or 256}
+
+
+def cpu_model() -> str:
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+# The paper's own headline numbers (PAPER.md:5 abstract, :257 Fig. 7; NVIDIA K20c, P:125):
+# context for the speedup lines, never a target of this metric (different GPU, datasets).
+PAPER_CONTEXT = {"speedup_vs_sequential": 3.0, "speedup_vs_csrcolor": 1.5, "gpu": "NVIDIA K20c",
+                 "source": "PAPER.md:5 (abstract), :257 (Fig. 7: data-driven 1.5x csrcolor)",
+                 "note": "context only: other hardware and datasets (UF matrices, P:234)"}
+
+
 # ------------------------------------------------------------------------ CPU oracle legs
 def oracle_run(g, tiebreak: int, edges_total: int | None, budget_s: float = 30.0):
     """Time the oracle (as it stands) on the box's host cores. A full O2 run if it fits the
@@ -187,10 +227,9 @@ def run_reference(args):
             "n_gpus": args.gpus, "device": "host cpu", "steps": len(times), "warmup": args.warmup, "ms_per_step": t * 1e3,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
             "dtype": "int32", "data": "synthetic",
-            "config": {"workload": workload_name(args.config), "n": g.n, "nnz": g.nnz,
-                       "tiebreak": args.tiebreak},
+            "config": bench_config(args, g),
             "cpu_baseline": {"value": value, "unit": "GTEPS", "cores": cores, "kind": "oracle",
-                             "sample": sample},
+                             "sample": sample, "cpu_model": cpu_model()},
             "e2e": {"value": value, "unit": "GTEPS", "h2d_bytes_per_step": 0,
                     "d2h_bytes_per_step": 0}}
     if res is not None:
@@ -217,12 +256,19 @@ def run_single(args):
     stream = torch.cuda.current_stream()
     torch.cuda.synchronize()
 
-    def step(profile=False):
-        return sgr.color(rp, ci, args.tiebreak, out=colors, workspace=ws, profile=profile,
-                         loop_mode=args.loop_mode)
+    def step(profile=False, tiebreak=None):
+        return sgr.color(rp, ci, tiebreak or args.tiebreak, out=colors, workspace=ws,
+                         profile=profile, loop_mode=args.loop_mode, block_size=args.block_size)
 
     for _ in range(max(args.warmup, 3)):
         res = step()
+    torch.cuda.synchronize()
+    # |W_2| (F_1's output) from one traced coloring: the pushes of the round kernel are
+    # sum_{k>=2} |W_{k+1}| = sum_{k>=2} |W_k| - |W_2| (the result is deterministic)
+    tr = sgr.color(rp, ci, args.tiebreak, trace=True, loop_mode=args.loop_mode,
+                   block_size=args.block_size)
+    w2 = int(tr.round_sizes[1]) if len(tr.round_sizes) > 1 else 0
+    del tr
     torch.cuda.synchronize()
 
     # timed region: K complete colorings, L2 flushed between them (outside the step events).
@@ -255,15 +301,39 @@ def run_single(args):
 
     peak, peak_src = peaks()
     dom = max(kms, key=lambda k: kms[k])
-    achieved = kb[dom] / (kms[dom] * 1e-3) / 1e9 if kms[dom] > 0 else 0.0
     total_kernel_ms = sum(kms.values())
+    launches_dom = max(kl[dom], 1)
+    launch_s = kms[dom] * 1e-3 / launches_dom  # average launch duration (CUDA events)
+    # SURVEY §8(d) algorithmic bytes of the fused round kernel (one launch per coloring in
+    # the persistent mode), from the method's own counts, independent of trimming:
+    #   per scanned edge of rounds >= 2 (sum_k |adj(W_k)|): 4 B col_idx + one color word
+    #   per worklist vertex of rounds >= 2 (sum_k |W_k|): 4 B id + 16 B int64 row pair + X[v] + Y[v]
+    #   per push (sum_{k>=2} |W_{k+1}|): 4 B
+    cb = 2 if st["color_bits"] == 16 else 4
+    e_k = st["edges_scanned"] - g.nnz
+    v_k = st["vertices_processed"] - g.n
+    pushes = max(v_k - w2, 0)
+    alg8d = (4 + cb) * e_k + (4 + 16 + 2 * cb) * v_k + 4 * pushes
+    # e_k, v_k, pushes are per coloring (one step); kb[dom] sums the K timed steps
+    per_launch = (alg8d / (launches_dom / args.steps) if dom == "round"
+                  else kb[dom] / launches_dom)
+    achieved = per_launch / launch_s / 1e9 if launch_s > 0 else 0.0
+    traffic = ncu_traffic(workload_name(args.config), dom)
     roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak,
                 "unit": "GB/s", "frac": achieved / peak,
-                "traffic": ncu_traffic(workload_name(args.config), dom),
+                "traffic": traffic,
+                "byte_model": "SURVEY.md §8(d): (4+cb)*sum|adj(W_k)| + (20+2cb)*sum|W_k| + 4*pushes, "
+                              "k >= 2, cb = color word bytes",
                 "peak_source": peak_src,
                 "launches_per_step": kl[dom] / args.steps,
-                "algorithmic_bytes_per_launch": kb[dom] / max(kl[dom], 1),
-                "avg_launch_us": kms[dom] * 1e3 / max(kl[dom], 1),
+                "algorithmic_bytes_per_launch": per_launch,
+                "sum_adj_W_k": e_k, "sum_W_k": v_k, "pushes": pushes,
+                "dram_frac": (traffic / launch_s / 1e9 / peak) if (traffic and launch_s > 0) else None,
+                "lts_read_sectors": ncu_metric(workload_name(args.config), dom, "lts_read_sectors"),
+                "trimmed_model": {"bytes_per_launch": kb[dom] / launches_dom,
+                                  "achieved": kb[dom] / launches_dom / launch_s / 1e9 if launch_s > 0 else 0.0,
+                                  "note": "bytes the trimmed lists actually move (DESIGN.md §5)"},
+                "avg_launch_us": kms[dom] * 1e3 / launches_dom,
                 "share_of_kernel_time": kms[dom] / total_kernel_ms if total_kernel_ms else None,
                 "kernel_ms_per_step": {k: v / args.steps for k, v in kms.items()},
                 "whole_step": {"algorithmic_GBps": st["bytes_algorithmic"] / (ms * 1e-3) / 1e9,
@@ -317,11 +387,7 @@ def run_single(args):
             "steps": args.steps, "warmup": max(args.warmup, 3), "ms_per_step": ms,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
             "dtype": "int32", "data": "synthetic",
-            "config": {"workload": workload_name(args.config), "n": g.n, "nnz": g.nnz,
-                       "tiebreak": args.tiebreak, "parallelism": "single GPU",
-                       "l2": "flushed between steps (256 MiB write, outside the step events); "
-                             "CSR inputs 1.2 GB > L2",
-                       "loop_mode": args.loop_mode},
+            "config": bench_config(args, g),
             "rounds": st["rounds"], "num_colors": st["num_colors"],
             "A_scanned_per_nnz": st["edges_scanned"] / g.nnz,
             "B_worklist_per_n": st["vertices_processed"] / g.n,
@@ -329,16 +395,44 @@ def run_single(args):
             "wall_s_timed_region": wall, "gpu_launches": launches,
             "roofline": roofline, "clocks": clk, "e2e": e2e, "gen_s": gen_s}
 
+    # secondary row (reading C4): the paper's own tie-break, v < w recolors v
+    other = "paper" if args.tiebreak == "lowid" else "lowid"
+    sec = None
+    if not args.no_secondary:
+        step(tiebreak=other)
+        s_ms, s_st = [], None
+        for i in range(3):
+            flush.fill_(i)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            s_st = step(tiebreak=other).stats
+            e1.record(stream)
+            torch.cuda.synchronize()
+            s_ms.append(e0.elapsed_time(e1))
+        sec = {"tiebreak": other, "value": g.nnz / (statistics.mean(s_ms) * 1e-3) / 1e9,
+               "unit": "GTEPS", "ms_per_step": statistics.mean(s_ms), "steps": 3,
+               "rounds": s_st["rounds"], "num_colors": s_st["num_colors"],
+               "A_scanned_per_nnz": s_st["edges_scanned"] / g.nnz}
+        line["secondary"] = sec
+    line["paper_context"] = dict(PAPER_CONTEXT)
+
     if not args.no_cpu_baseline:
         tb = 0 if args.tiebreak == "lowid" else 1
         o = oracle_run(g, tb, st["edges_scanned"], budget_s=30.0)
         a1_colors, a1_s = alg1_run(g)
         line["cpu_baseline"] = {"value": g.nnz / o["seconds"] / 1e9, "unit": "GTEPS",
-                                "cores": o["cores"], "kind": "oracle", "sample": o["sample"]}
+                                "cores": o["cores"], "kind": "oracle", "sample": o["sample"],
+                                "cpu_model": cpu_model(),
+                                "threads_note": f"O2 on {o['cores']} OpenMP threads (one per "
+                                                "host core); Algorithm 1 on 1 core below"}
         line["colors_vs_seq_greedy"] = {"ours": st["num_colors"], "alg1": a1_colors,
                                         "ratio": st["num_colors"] / a1_colors,
                                         "alg1_seconds_1core": a1_s,
                                         "speedup_vs_alg1_1core": a1_s / (ms * 1e-3)}
+        if sec is not None:
+            sec["colors_vs_alg1"] = sec["num_colors"] / a1_colors
+            sec["speedup_vs_alg1_1core"] = a1_s / (sec["ms_per_step"] * 1e-3)
+        line["paper_context"]["ours_speedup_vs_sequential_alg1_1core"] = a1_s / (ms * 1e-3)
         if o["result"] is not None:
             ok = bool(np.array_equal(o["result"].colors, colors.cpu().numpy()))
             line["parity_vs_oracle_full"] = ok

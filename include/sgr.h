@@ -190,6 +190,22 @@ sgr_status sgr_color_host_batch(const int64_t* const* row_ptr, const int32_t* co
 sgr_status sgr_color_topo(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* colors_out,
                           sgr_stats* stats, const sgr_opts* opts);
 
+/* Reduced-round variants (DESIGN.md §3 reading C20). Different
+ * semantics from sgr_color: a round's assignment loop (Alg. 5 l.4-10) runs as `substeps`
+ * ordered sub-steps over a fixed id partition — partition 0: v mod substeps ("strided"),
+ * 1: floor(v * substeps / n) ("blocked") — and sub-step j sees the colors written by the
+ * sub-steps before it (the paper's in-place writes, P:169/174/190, made deterministic);
+ * then detection and compaction as Alg. 5 l.12-15. Deterministic, equal to the oracle's
+ * O3 (colors, rounds, |W_r|); substeps = 1 is sgr_color's result. Partition 2 is the
+ * paper-faithful NONDETERMINISTIC mode: one in-place assignment per round whose first fits
+ * read colors other warps are writing (substeps ignored); the result is a proper coloring
+ * whose colors and rounds may vary from run to run. Plain int32 colors, host-driven
+ * rounds (one count readback per round). Uses opts tiebreak, max_rounds, stream,
+ * block_size and round_sizes / round_edges / round_cap; synchronizes the stream. */
+sgr_status sgr_color_gs(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t substeps,
+                        int32_t partition, int32_t* colors_out, sgr_stats* stats,
+                        const sgr_opts* opts);
+
 /* ---- one-round step entry points: Algorithm 5 split line by line (all device pointers,
  * asynchronous on opts->stream; opts may be NULL) ---------------------------------------- */
 

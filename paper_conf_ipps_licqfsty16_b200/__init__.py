@@ -26,7 +26,7 @@ from ._lib import Csr, Opts, Stats, check, load
 TIEBREAK = {"lowid": 0, "lowid_keeps": 0, "paper": 1}
 LOOP = {"auto": 0, "graph": 1, "persistent": 2, "host": 3}
 
-__all__ = ["color", "color_host", "color_host_batch", "color_topo", "color_partitioned", "color_dist", "assign", "commit",
+__all__ = ["color", "color_host", "color_host_batch", "color_topo", "color_gs", "color_partitioned", "color_dist", "assign", "commit",
            "detect", "compact", "validate_csr", "partition", "workspace_bytes", "gen",
            "ColorResult", "TIEBREAK"]
 
@@ -162,6 +162,42 @@ def color_topo(row_ptr, col_idx, tiebreak="lowid", *, out=None, stream=None, tra
     res = ColorResult(colors, st.as_dict())
     if trace:
         res.round_sizes = rs[:res.stats["rounds"]].cpu().numpy()
+    return res
+
+
+GS_PARTITION = {"strided": 0, "blocked": 1, "inplace": 2}
+
+
+def color_gs(row_ptr, col_idx, substeps=16, partition="strided", tiebreak="lowid", *, out=None,
+             stream=None, trace=False, **opt_kw) -> ColorResult:
+    """Reduced-round variant (include/sgr.h sgr_color_gs): each round's
+    assignment runs as `substeps` ordered sub-steps ("strided": v mod K, "blocked":
+    floor(v K / n)), a sub-step seeing the earlier ones' colors; "inplace" is the paper's
+    nondeterministic in-place mode. Different semantics (fewer rounds, more colors) from
+    color(); substeps=1 equals it."""
+    torch = _torch()
+    _check_csr(row_ptr, col_idx)
+    n = row_ptr.numel() - 1
+    nnz = col_idx.numel()
+    colors = out if out is not None else torch.empty(n, dtype=torch.int32, device=row_ptr.device)
+    _require_cuda(colors)
+    rs = re = None
+    if trace:
+        rs = torch.zeros(n + 2, dtype=torch.int32, device=row_ptr.device)
+        re = torch.zeros(n + 2, dtype=torch.int64, device=row_ptr.device)
+    opts = make_opts(tiebreak, stream, round_sizes=rs, round_edges=re,
+                     round_cap=(n + 2) if trace else 0, **opt_kw)
+    part = GS_PARTITION[partition] if isinstance(partition, str) else int(partition)
+    csr = Csr(row_ptr.data_ptr(), col_idx.data_ptr() if nnz else None)
+    st = Stats()
+    check(load().sgr_color_gs(ctypes.byref(csr), n, nnz, int(substeps), part,
+                              colors.data_ptr() if n else None, ctypes.byref(st),
+                              ctypes.byref(opts)), "sgr_color_gs")
+    res = ColorResult(colors, st.as_dict())
+    if trace:
+        R = res.stats["rounds"]
+        res.round_sizes = rs[:R].cpu().numpy()
+        res.round_edges = re[:R].cpu().numpy()
     return res
 
 

@@ -68,7 +68,7 @@ class Stats(ctypes.Structure):
 _lib = None
 
 EXPORTS = ("sgr_opts_default", "sgr_workspace_bytes", "sgr_color", "sgr_color_ex",
-           "sgr_color_host", "sgr_color_host_batch", "sgr_color_topo", "sgr_assign", "sgr_commit", "sgr_detect", "sgr_compact",
+           "sgr_color_host", "sgr_color_host_batch", "sgr_color_topo", "sgr_color_gs", "sgr_assign", "sgr_commit", "sgr_detect", "sgr_compact",
            "sgr_validate_csr", "sgr_partition", "sgr_nccl_unique_id", "sgr_comm_init",
            "sgr_comm_destroy", "sgr_color_dist", "sgr_color_partitioned", "sgr_strerror",
            "sgr_last_error", "sgr_version")
@@ -94,6 +94,7 @@ def load():
     lib.sgr_color_host.argtypes = [vp, vp, i64, i64, vp, P(Stats), P(Opts)]
     lib.sgr_color_host_batch.argtypes = [P(vp), P(vp), P(i64), P(i64), P(vp), i32, P(Stats), P(Opts)]
     lib.sgr_color_topo.argtypes = [P(Csr), i64, i64, vp, P(Stats), P(Opts)]
+    lib.sgr_color_gs.argtypes = [P(Csr), i64, i64, i32, i32, vp, P(Stats), P(Opts)]
     lib.sgr_assign.argtypes = [P(Csr), i64, vp, i64, vp, vp, P(Opts)]
     lib.sgr_commit.argtypes = [vp, vp, i64, vp, P(Opts)]
     lib.sgr_detect.argtypes = [P(Csr), i64, vp, i64, vp, vp, P(Opts)]

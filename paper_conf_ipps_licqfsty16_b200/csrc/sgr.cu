@@ -15,6 +15,7 @@
 #include "sgr_round.cuh"
 #include "sgr_step.cuh"
 #include "sgr_topo.cuh"
+#include "sgr_gs.cuh"
 
 namespace sgr {
 
@@ -761,11 +762,144 @@ sgr_status sgr_color_topo(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* c
   return status;
 }
 
-// ----- step entry points ------------------------------------------------------------------
 static int grid_for(int64_t items, int per_block, int B = 256) {
   const int64_t b = (items + per_block - 1) / per_block;
   return (int)std::max<int64_t>(1, std::min<int64_t>(b, (int64_t)num_sms() * 16 * 256 / B));
 }
+
+// ----- reduced-round variants (sgr_gs.cuh) --------------------------
+sgr_status sgr_color_gs(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t substeps,
+                        int32_t partition, int32_t* colors_out, sgr_stats* stats,
+                        const sgr_opts* opts) {
+  if (!csr || n < 0 || nnz < 0 || n >= ((int64_t)1 << 31) || substeps < 1 || partition < 0 ||
+      partition > 2) {
+    set_error("sgr_color_gs: invalid sizes, csr, substeps or partition");
+    return SGR_EINVAL;
+  }
+  if (stats) memset(stats, 0, sizeof(*stats));
+  if (n == 0) return SGR_OK;
+  if (!csr->row_ptr || !colors_out || (nnz > 0 && !csr->col_idx)) {
+    set_error("sgr_color_gs: null pointer");
+    return SGR_EINVAL;
+  }
+  const Resolved r = resolve_opts(opts, n);
+  const int B = r.block;
+  if (!block_ok(B, 32, kMaxBlockAny)) {
+    set_error("sgr_color_gs: block_size %d (32..1024, multiple of 32)", B);
+    return SGR_EINVAL;
+  }
+  const int64_t K = partition == 2 ? 1 : substeps;
+  cudaStream_t s = r.stream;
+  keep_pool_memory();
+  // workspace: W[2] | T | flags | tiles | counters
+  const size_t nb = align_up((size_t)n * 4, 256);
+  const int64_t tiles = (n + kCompactTile - 1) / kCompactTile;
+  char* ws = nullptr;
+  CK(cudaMallocAsync((void**)&ws, 4 * nb + align_up((size_t)tiles * 4, 256) + 256, s));
+  int32_t* W[2] = {(int32_t*)ws, (int32_t*)(ws + nb)};
+  int32_t* T = (int32_t*)(ws + 2 * nb);
+  uint8_t* flags = (uint8_t*)(ws + 3 * nb);
+  int32_t* tile = (int32_t*)(ws + 4 * nb);
+  char* tail = ws + 4 * nb + align_up((size_t)tiles * 4, 256);
+  int64_t* dcount = (int64_t*)tail;
+  unsigned long long* edges = (unsigned long long*)(tail + 64);
+  int64_t* hcnt = nullptr;
+  CK(cudaMallocHost((void**)&hcnt, sizeof(int64_t)));
+  cudaEvent_t e0, e1;
+  CK(cudaEventCreate(&e0));
+  CK(cudaEventCreate(&e1));
+  const int grid_v = (int)std::max<int64_t>(1, std::min<int64_t>((n + B - 1) / B, (int64_t)num_sms() * 16 * 256 / B));
+  std::vector<int32_t> sizes;
+  std::vector<int64_t> round_edges;
+  sgr_status status = SGR_OK;
+  int launches = 0;
+  unsigned long long edges_prev = 0;
+  CK(cudaMemsetAsync(edges, 0, 8, s));
+  CK(cudaEventRecord(e0, s));
+  k_gs_init<<<grid_v, B, 0, s>>>(n, W[0], colors_out);
+  ++launches;
+  int64_t len = n;
+  int cur = 0;
+  while (len > 0) {
+    if ((int64_t)sizes.size() >= r.max_rounds) {
+      status = SGR_ENOCONV;
+      set_error("sgr_color_gs: max_rounds reached");
+      break;
+    }
+    sizes.push_back((int32_t)len);
+    const int gw = grid_for(len, B / 32, B);
+    if (partition == 2) {
+      k_gs_inplace<<<gw, B, 0, s>>>(csr->row_ptr, csr->col_idx, W[cur], len, colors_out, edges);
+      ++launches;
+    } else {
+      for (int64_t j = 0; j < K; ++j) {  // sub-steps in order (Alg. 5 l.4-10 split K ways)
+        k_gs_assign<<<gw, B, 0, s>>>(csr->row_ptr, csr->col_idx, W[cur], len, n, K, partition, j,
+                                     colors_out, T, edges);
+        k_gs_commit<<<grid_for(len, B, B), B, 0, s>>>(W[cur], len, n, K, partition, j, T, colors_out);
+        launches += 2;
+      }
+    }
+    // Alg. 5 l.12-15 over W_r, then the order-preserving compaction
+    if (r.tiebreak)
+      k_detect_step<1><<<gw, B, 0, s>>>(csr->row_ptr, csr->col_idx, W[cur], len, colors_out, flags);
+    else
+      k_detect_step<0><<<gw, B, 0, s>>>(csr->row_ptr, csr->col_idx, W[cur], len, colors_out, flags);
+    const int64_t tl = (len + kCompactTile - 1) / kCompactTile;
+    k_compact_count<<<(unsigned)tl, 256, 0, s>>>(flags, len, tile);
+    k_compact_scan<<<1, 1024, 0, s>>>(tile, tl, dcount);
+    k_compact_scatter<<<(unsigned)tl, 256, 0, s>>>(W[cur], flags, len, tile, W[cur ^ 1]);
+    launches += 4;
+    CK(cudaGetLastError());
+    unsigned long long ed = 0;
+    CK(cudaMemcpyAsync(hcnt, dcount, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(&ed, edges, 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    round_edges.push_back((int64_t)(ed - edges_prev));
+    edges_prev = ed;
+    len = *hcnt;
+    cur ^= 1;
+  }
+  int32_t* dmax = (int32_t*)(tail + 128);
+  CK(cudaMemsetAsync(dmax, 0, 4, s));
+  k_max_color<<<grid_v, B, 0, s>>>(colors_out, n, dmax);
+  ++launches;
+  CK(cudaEventRecord(e1, s));
+  int32_t mx = 0;
+  CK(cudaMemcpyAsync(&mx, dmax, 4, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  const int32_t R = (int32_t)sizes.size();
+  if (r.round_cap > 0) {
+    const int32_t m = std::min(R, r.round_cap);
+    if (r.round_sizes) CK(cudaMemcpy(r.round_sizes, sizes.data(), (size_t)m * 4, cudaMemcpyHostToDevice));
+    if (r.round_edges) CK(cudaMemcpy(r.round_edges, round_edges.data(), (size_t)m * 8, cudaMemcpyHostToDevice));
+  }
+  if (stats) {
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, e0, e1);
+    stats->rounds = R;
+    stats->num_colors = mx;
+    int64_t vp = 0;
+    for (int32_t x : sizes) vp += x;
+    stats->vertices_processed = vp;
+    stats->edges_scanned = (int64_t)edges_prev;
+    stats->entries_read = (int64_t)edges_prev;
+    stats->elapsed_ms = ms;
+    stats->launches = launches;
+    stats->color_bits = 32;
+    stats->grid_blocks = grid_v;
+    // per worklist vertex and sub-step: the id; per member: row pair, the first-fit scan of
+    // its row (id + color per entry), T write + commit; detection re-reads the row
+    stats->bytes_algorithmic = vp * (4 * K + 16 + 12) + (int64_t)edges_prev * 16;
+  }
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  cudaFreeHost(hcnt);
+  cudaFreeAsync(ws, s);
+  cudaStreamSynchronize(s);
+  return status;
+}
+
+// ----- step entry points ------------------------------------------------------------------
 
 sgr_status sgr_assign(const sgr_csr* csr, int64_t n, const int32_t* wl, int64_t wl_len,
                       const int32_t* colors_in, int32_t* tent_out, const sgr_opts* opts) {

@@ -14,13 +14,28 @@ __device__ __forceinline__ bool lose(int32_t v, int32_t w) {
   else return v > w;
 }
 
-__device__ __forceinline__ int32_t ldg_i32(const int32_t* p) { return __ldg(p); }
-__device__ __forceinline__ int64_t ldg_i64(const int64_t* p) { return __ldg(p); }
+// Loads of the read-only CSR arrays R (row_ptr) and C (col_idx). SGR_LDG = 1 (default):
+// through the read-only data path, __ldg / ld.global.nc — the paper's D-ldg / T-ldg
+// optimization (Fig. 4). SGR_LDG = 0: the normal load path, ld.global.ca — the
+// paper's D-base / T-base (the ablation of P:236; tools/ldg_ablation.py).
+#ifndef SGR_LDG
+#define SGR_LDG 1
+#endif
+template <class T>
+__device__ __forceinline__ T ld_ro(const T* p) {
+#if SGR_LDG
+  return __ldg(p);
+#else
+  return __ldca(p);
+#endif
+}
+__device__ __forceinline__ int32_t ldg_i32(const int32_t* p) { return ld_ro(p); }
+__device__ __forceinline__ int64_t ldg_i64(const int64_t* p) { return ld_ro(p); }
 
 // Read-only load of col_idx (the CSR never changes during a coloring). Measured on B200
 // (tools/gather_bench.cu): ld.global.nc.L1::no_allocate is up to 3.5x slower than plain
 // ld.global.nc for this access mix, so the plain read-only path is used.
-__device__ __forceinline__ int32_t ld_stream(const int32_t* p) { return __ldg(p); }
+__device__ __forceinline__ int32_t ld_stream(const int32_t* p) { return ld_ro(p); }
 
 // Color loads. A persistent kernel writes the color buffers while it runs, so it must not
 // read them through the non-coherent path: Persist loads go to L2 (ld.global.cg); the

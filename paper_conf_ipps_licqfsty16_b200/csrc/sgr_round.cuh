@@ -432,7 +432,7 @@ __device__ __forceinline__ int32_t ld_row_h(const int32_t* p) {
     asm volatile("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(r) : "l"(p));
     return r;
   } else {
-    return __ldg(p);
+    return ld_ro(p);
   }
 }
 __device__ __forceinline__ int32_t ld_row(const int32_t* p) {
@@ -441,10 +441,10 @@ __device__ __forceinline__ int32_t ld_row(const int32_t* p) {
   asm volatile("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(r) : "l"(p));
   return r;
 #else
-  return __ldg(p);
+  return ld_ro(p);
 #endif
 }
-__device__ __forceinline__ int4 ld_row4(const int4* p) { return __ldg(p); }
+__device__ __forceinline__ int4 ld_row4(const int4* p) { return ld_ro(p); }
 __device__ __forceinline__ void prefetch_l1(const void* p) {
   asm volatile("prefetch.global.L1 [%0];" ::"l"(p));
 }
@@ -634,7 +634,7 @@ __device__ __noinline__ int32_t warp_first_fit_rescan(const int32_t* __restrict_
     uint64_t m0 = 0, m1 = 0, m2 = 0, m3 = 0;
     if (base == 0) m0 = 1;
     for (int64_t j = s + lane; j < e; j += 32) {
-      const uint32_t idx = (uint32_t)(ldc<Persist>(X + __ldg(col_idx + j)) - base);
+      const uint32_t idx = (uint32_t)(ldc<Persist>(X + ld_ro(col_idx + j)) - base);
       if (idx < 256u) {
         const uint64_t bit = 1ull << (idx & 63);
         const uint32_t q = idx >> 6;
@@ -678,11 +678,11 @@ __device__ __forceinline__ void process_chunk_plain(const RoundArgs<C>& a, int k
     int4 t = make_int4(-1, -1, -1, -1);
     if (p0 + 3 >= cs && p0 < ce) {
       if (p0 + 4 <= a.nnz) {
-        t = __ldg(col4 + lane + 32 * q);
+        t = ld_ro(col4 + lane + 32 * q);
       } else {  // the array's last, partial 16-byte group: never read past nnz
-        t.x = __ldg(a.col_idx + p0);
-        if (p0 + 1 < a.nnz) t.y = __ldg(a.col_idx + p0 + 1);
-        if (p0 + 2 < a.nnz) t.z = __ldg(a.col_idx + p0 + 2);
+        t.x = ld_ro(a.col_idx + p0);
+        if (p0 + 1 < a.nnz) t.y = ld_ro(a.col_idx + p0 + 1);
+        if (p0 + 2 < a.nnz) t.z = ld_ro(a.col_idx + p0 + 2);
       }
     }
     w[4 * q + 0] = (p0 + 0 >= cs && p0 + 0 < ce) ? t.x : -1;

@@ -32,7 +32,7 @@ static __global__ void __launch_bounds__(1024) k_assign_step(const int64_t* __re
        i += (int64_t)gridDim.x * wpb) {
     const int32_t v = __ldg(wl + i);
     const int32_t t =
-        warp_first_fit_from<false>(col_idx, X, __ldg(row_ptr + v), __ldg(row_ptr + v + 1), 0, lane);
+        warp_first_fit_from<false>(col_idx, X, ld_ro(row_ptr + v), ld_ro(row_ptr + v + 1), 0, lane);
     if (lane == 0) tent[i] = t;
   }
 }
@@ -59,8 +59,8 @@ __global__ void __launch_bounds__(1024) k_detect_step(const int64_t* __restrict_
     const int32_t v = __ldg(wl + i);
     const int32_t cv = __ldg(C + v);
     bool c = false;
-    for (int64_t j = __ldg(row_ptr + v) + lane; j < __ldg(row_ptr + v + 1) && !c; j += 32) {
-      const int32_t w = __ldg(col_idx + j);
+    for (int64_t j = ld_ro(row_ptr + v) + lane; j < ld_ro(row_ptr + v + 1) && !c; j += 32) {
+      const int32_t w = ld_ro(col_idx + j);
       c = (__ldg(C + w) == cv) && lose<TB>(v, w);
     }
     c = __any_sync(0xffffffffu, c);

@@ -27,7 +27,7 @@ __device__ __forceinline__ int32_t thread_first_fit(const int32_t* __restrict__ 
   for (int32_t base = 0;; base += 64) {
     uint64_t m = 0;
     for (int64_t j = s; j < e; ++j) {
-      const int32_t w = __ldg(col_idx + j);
+      const int32_t w = ld_ro(col_idx + j);
       if (w == v) continue;  // a self-loop never forbids (reading C7)
       const uint32_t idx = (uint32_t)(__ldg(X + w) - base - 1);
       if (idx < 64u) m |= 1ull << idx;
@@ -48,7 +48,7 @@ static __global__ void __launch_bounds__(1024) k_topo_assign(const int64_t* __re
   for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n;
        v += (int64_t)gridDim.x * blockDim.x) {
     if (__ldg(flag + v) == r) {  // colored[v] = false
-      const int64_t s = __ldg(row_ptr + v), e = __ldg(row_ptr + v + 1);
+      const int64_t s = ld_ro(row_ptr + v), e = ld_ro(row_ptr + v + 1);
       T[v] = thread_first_fit(col_idx, X, (int32_t)v, s, e);
       my += (unsigned long long)(e - s);
     } else {
@@ -73,9 +73,9 @@ __global__ void __launch_bounds__(1024) k_topo_detect(const int64_t* __restrict_
     bool c = false;
     if (v < n) {
       const int32_t tv = __ldg(T + v);
-      const int64_t e = __ldg(row_ptr + v + 1);
-      for (int64_t j = __ldg(row_ptr + v); j < e && !c; ++j) {
-        const int32_t w = __ldg(col_idx + j);
+      const int64_t e = ld_ro(row_ptr + v + 1);
+      for (int64_t j = ld_ro(row_ptr + v); j < e && !c; ++j) {
+        const int32_t w = ld_ro(col_idx + j);
         c = lose<TB>((int32_t)v, w) && __ldg(T + w) == tv;
       }
       if (c) flag[v] = r + 1;

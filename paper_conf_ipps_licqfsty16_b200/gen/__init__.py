@@ -189,6 +189,9 @@ def config(idx: int) -> Graph:
         return rmat(20, 10, 0.45, 0.15, 0.15, seed=7)
     if idx == 8:  # cfg4 with Graph500-style relabeling ("--permute")
         return rmat(24, 8, 0.57, 0.19, 0.19, seed=4, permute=True)
+    if idx == 9:  # cfg5's shape with edge factor 9: nnz ~ 2.39e9 > 2^31 (cfg5's 2.126e9 is
+        # just below), so the int64 row offsets (reading C17) really exceed 32 bits
+        return rmat(27, 9, 0.57, 0.19, 0.19, seed=9)
     raise ValueError(idx)
 
 
@@ -201,4 +204,5 @@ CONFIG_NAMES = {
     6: "rmat-er-s20-ef10 (a=b=c=.25, Table I) seed 6",
     7: "rmat-g-s20-ef10 (a=.45,b=c=.15, Table I) seed 7",
     8: "rmat-s24-ef8 (a=.57,b=c=.19) seed 4, permuted",
+    9: "rmat-s27-ef9 (a=.57,b=c=.19) seed 9 (nnz > 2^31)",
 }

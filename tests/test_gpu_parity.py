@@ -413,19 +413,34 @@ def test_full_size_configs_bit_exact(cfg):
 
 
 @pytest.mark.slow
-def test_cfg5_full_size():
-    """BASELINE config 5 (R-MAT scale 27, nnz 2.13e9 > 2^31: the int64-offset path, reading
-    C17) on one GPU against the full oracle (OpenMP), element by element (colors, R, |W_r|,
-    sum deg(W_r)), plus the partitioned protocol on 2 partitions of the same device. Runs in
-    the default -m gpu suite (a few minutes: generation + the OpenMP oracle dominate)."""
-    g = gen.config(5)
-    assert g.nnz > 2 ** 31 and int(g.row_ptr[g.n // 2]) < 2 ** 31 < int(g.row_ptr[-1])
+def test_nnz_beyond_2_31_full_size():
+    """Row offsets past 2^31 (reading C17): cfg5's shape (R-MAT scale 27) with edge factor 9,
+    nnz ~ 2.39e9 > 2^31 (cfg5 itself has 2,125,681,752 entries, just below 2^31), on one GPU
+    against the full oracle (OpenMP), element by element (colors, R, |W_r|, sum deg(W_r)),
+    plus the partitioned protocol on 2 partitions of the same device. Rows of every degree
+    bin, including multi-chunk bin-2 rows, start beyond offset 2^31. Runs in the default
+    -m gpu suite (a few minutes: generation and the OpenMP oracle dominate)."""
+    g = gen.config(9)
+    deg = np.diff(g.row_ptr)
+    past = g.row_ptr[:-1] >= 2 ** 31
+    assert g.nnz > 2 ** 31 and past.any()
+    assert (deg[past] <= 32).any() and ((deg[past] > 32) & (deg[past] <= 256)).any()
+    assert (deg[past] > 1020).any()  # multi-chunk rows (bin 2) beyond 2^31
     res, ref = check_full(g, LOW)
     assert res.stats["color_bits"] == 16
     rp, ci = dev(g)
     part = sgr.color_partitioned(rp, ci, 2)
     assert np.array_equal(part.colors.cpu().numpy(), ref.colors)
     assert part.stats["rounds"] == ref.rounds
+
+
+@pytest.mark.slow
+def test_cfg5_full_size():
+    """BASELINE config 5 (R-MAT scale 27, ef 8: nnz = 2,125,681,752, int64 offsets) on one
+    GPU in bench.py's launch configuration against the full oracle, element by element."""
+    g = gen.config(5)
+    res, ref = check_full(g, LOW)
+    assert res.stats["color_bits"] == 16
 
 
 # ----------------------------------------------------------------------------- multi-GPU path
@@ -574,3 +589,73 @@ def test_multi_chunk_hub_lists(maker, tb):
     assert deg.max() > 2 * 1020, deg.max()  # really multi-chunk
     res, _ = check_full(g, tb)
     assert res.stats["entries_read"] <= res.stats["edges_scanned"]
+
+
+# ----------------------------------------------------------------------------- §8(f) item 4
+def check_gs(g, K, part, tb):
+    rp, ci = dev(g)
+    res = sgr.color_gs(rp, ci, K, part, RULE[tb], trace=True)
+    ref = oracle.gauss_seidel(g, K, part, tb)
+    assert res.stats["rounds"] == ref.rounds, (g.name, K, part, res.stats["rounds"], ref.rounds)
+    assert np.array_equal(res.colors.cpu().numpy(), ref.colors), (g.name, K, part)
+    assert np.array_equal(res.round_sizes, ref.round_sizes)
+    assert np.array_equal(res.round_edges, ref.trace["w_edges"])
+    assert res.stats["num_colors"] == ref.num_colors
+    return res, ref
+
+
+@pytest.mark.parametrize("seed", range(16))
+@pytest.mark.parametrize("part", ["strided", "blocked"])
+def test_gs_substeps_random_graphs(seed, part):
+    """K-sub-step Gauss-Seidel rounds against the oracle's O3:
+    bit-exact colors, R, |W_r| and sum deg(W_r), both rules, K in 1..16."""
+    g = random_graph(seed, n=200)
+    for K in (1, 2, 3, 16):
+        for tb in (LOW, PAP):
+            check_gs(g, K, 0 if part == "strided" else 1, tb)
+
+
+@pytest.mark.parametrize("maker", [
+    lambda: gen.config(1),
+    lambda: gen.stencil3d(16, 15, 14, 27),
+    lambda: gen.er(1 << 14, 8 << 14, seed=5),
+    lambda: gen.rmat(13, 10, 0.45, 0.15, 0.15, seed=3),
+], ids=["cfg1", "s27", "er14", "rmat-g13"])
+@pytest.mark.parametrize("K", [4, 16, 64])
+def test_gs_substeps_families(maker, K):
+    g = maker()
+    for part in (0, 1):
+        check_gs(g, K, part, LOW)
+
+
+def test_gs_one_substep_equals_jacobi_and_loops():
+    g = gen.config(1)
+    rp, ci = dev(g)
+    a = sgr.color_gs(rp, ci, 1, "strided").colors
+    assert torch.equal(a, sgr.color(rp, ci).colors)
+    h = with_loops_and_dups(random_graph(3, n=150), 3)  # listed self-loops: Alg. 5 l.5-6 literally
+    for K in (1, 4):
+        check_gs(h, K, 0, LOW)
+
+
+@pytest.mark.parametrize("tb", [LOW, PAP])
+def test_gs_inplace_nondeterministic_is_proper(tb):
+    """Partition 2: the paper's in-place assignment (nondeterministic): every run ends with a
+    proper coloring, colors in [1, deg + 1], and W shrinking every round."""
+    for g in (gen.config(1), gen.stencil3d(20, 20, 20, 27), random_graph(7, n=300)):
+        rp, ci = dev(g)
+        deg = np.diff(g.row_ptr)
+        for _ in range(3):
+            res = sgr.color_gs(rp, ci, 1, "inplace", RULE[tb], trace=True)
+            c = res.colors.cpu().numpy()
+            assert c.min() >= 1 and np.all(c <= deg + 1)
+            src = np.repeat(np.arange(g.n), deg)
+            assert not np.any((c[src] == c[g.col_idx]) & (src != g.col_idx)), g.name
+            assert np.all(np.diff(res.round_sizes) < 0)
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("cfg", [3, 4])
+def test_gs_full_size(cfg):
+    """cfg3 / cfg4 at full size with K = 16 strided sub-steps against the oracle's O3."""
+    check_gs(gen.config(cfg), 16, 0, LOW)
