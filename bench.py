@@ -192,6 +192,13 @@ def oracle_run(g, tiebreak: int, edges_total: int | None, budget_s: float = 30.0
             "result": None}
 
 
+def oracle_parity(g, colors, rounds, tiebreak) -> bool:
+    """Rank 0 of the multi-GPU line: the replica's colors and R equal the oracle's (O2)."""
+    import oracle
+    ref = oracle.jacobi(g, 0 if tiebreak == "lowid" else 1, nthreads=oracle.max_threads())
+    return bool(np.array_equal(ref.colors, colors)) and ref.rounds == rounds
+
+
 def alg1_run(g):
     import oracle
     t0 = time.perf_counter()
@@ -446,7 +453,7 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     if world > 1 or args.gpus > 1 or args.dist:
         from paper_conf_ipps_licqfsty16_b200 import benchdist
-        return benchdist.run(args)
+        return benchdist.run(args, check=oracle_parity)
     return run_single(args)
 
 

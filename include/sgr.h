@@ -142,7 +142,19 @@ typedef struct {
   int32_t grid_blocks;               /* blocks of the round kernel                        */
   int32_t color_bits;                /* width the coloring finished with (16 or 32)       */
   int64_t entries_written;           /* compacted neighbour-list entries written (bin 2)  */
+  int32_t transport;                 /* partitioned / multi-GPU colorings: how replicas were
+                                        kept equal — SGR_XCHG_* below; 0 otherwise         */
 } sgr_stats;
+
+/* stats->transport of sgr_color_partitioned / sgr_color_dist. */
+enum {
+  SGR_XCHG_NONE = 0,        /* single part: nothing to exchange                          */
+  SGR_XCHG_DEVICE = 1,      /* one cooperative launch, every color word stored into all
+                               replicas (parts of one device, or NVLink peer memory), device
+                               barrier across parts (k_persistent_dist)                     */
+  SGR_XCHG_ALLGATHER = 2    /* host-driven rounds, padded all-gather of (v, color) records
+                               per round (NCCL between GPUs, device copies on one GPU)      */
+};
 
 void sgr_opts_default(sgr_opts* opts);
 

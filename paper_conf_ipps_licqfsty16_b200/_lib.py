@@ -46,7 +46,8 @@ class Stats(ctypes.Structure):
                 ("bin_vertices", ctypes.c_int64 * 3), ("bin_edges", ctypes.c_int64 * 3),
                 ("chunk_items", ctypes.c_int64), ("bin_warp_cycles", ctypes.c_int64 * 3),
                 ("grid_blocks", ctypes.c_int32),
-                ("color_bits", ctypes.c_int32), ("entries_written", ctypes.c_int64)]
+                ("color_bits", ctypes.c_int32), ("entries_written", ctypes.c_int64),
+                ("transport", ctypes.c_int32)]
 
     def as_dict(self) -> dict:
         d = {k: getattr(self, k) for k in ("rounds", "num_colors", "vertices_processed",
@@ -62,6 +63,7 @@ class Stats(ctypes.Structure):
         d["grid_blocks"] = self.grid_blocks
         d["entries_written"] = self.entries_written
         d["color_bits"] = self.color_bits
+        d["transport"] = ("none", "device", "allgather")[self.transport] if 0 <= self.transport < 3 else self.transport
         return d
 
 

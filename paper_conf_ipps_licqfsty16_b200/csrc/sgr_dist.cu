@@ -365,6 +365,7 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
       stats->vertices_processed = vertices;
       stats->grid_blocks = grid;
       stats->color_bits = packed<C>() ? 16 : 32;
+      stats->transport = world > 1 ? SGR_XCHG_ALLGATHER : SGR_XCHG_NONE;
       cudaEventElapsedTime(&stats->elapsed_ms, ev0, ev1);
     }
   }
@@ -379,6 +380,255 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
   }
   cudaStreamSynchronize(s);
   return status;
+}
+
+// ---------------------------------------------------------------------------------------
+// Device-side exchange (k_persistent_dist): every part writes its color words straight into
+// all replicas and the rounds run in one cooperative launch per device, with a barrier
+// across parts. Parts on one device share the launch (block groups); on several GPUs
+// each rank is one part and the other replicas are NVLink peer memory (CUDA IPC), with
+// `xsync` ordering the setup steps across ranks (an NCCL all-reduce; nullptr on one device).
+struct DevPart {
+  int64_t lo = 0, hi = 0, nnz = 0;
+  sgr_csr csr{};          // owned rows: local offsets, global column ids
+  void* ws = nullptr;     // workspace of layout(n, nnz)
+  int32_t* colors = nullptr;
+  bool own_colors = false;
+};
+struct PeerView {         // multi-GPU: the other ranks' workspaces (IPC-mapped), by rank
+  std::vector<void*> ws;  // ws[me] = own
+  int me = 0;
+};
+using XSync = std::function<sgr_status(cudaStream_t, int32_t* dflag, int op_max)>;
+
+template <int TB, class C, bool Hub>
+static int dist_grid(int B) {
+  const int smax = (int)round_smem<C, Hub>(round_max_block<C, Hub>());
+  cudaFuncSetAttribute(k_persistent_dist<TB, C, Hub>, cudaFuncAttributeMaxDynamicSharedMemorySize, smax);
+  int per_sm = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_persistent_dist<TB, C, Hub>, B,
+                                                    round_smem<C, Hub>(B)) != cudaSuccess ||
+      per_sm <= 0)
+    per_sm = 1;
+  return per_sm * num_sms();
+}
+
+template <int TB, class C>
+static sgr_status run_dev(std::vector<DevPart>& parts, int nranks, int me0, int64_t n,
+                          int32_t* colors_out, sgr_stats* stats, const PeerView* peers,
+                          const XSync& xsync, const Resolved& r, int* overflow_out) {
+  cudaStream_t s = r.stream;
+  const int B = r.block;
+  if (peers && !packed<C>()) {  // int32 replicas are not in the peer-mapped workspace
+    set_error("sgr_color_dist: device exchange needs 16-bit words");
+    return SGR_EUNSUPPORTED;
+  }
+  if (!block_ok(B, 64, round_max_block<C, true>())) {
+    set_error("sgr_color_dist: block_size %d not supported by the round kernels", B);
+    return SGR_EINVAL;
+  }
+  keep_pool_memory();
+  const int P = (int)parts.size();
+  std::vector<Layout> Ls;
+  std::vector<RoundArgs<C>> args(P);
+  for (int i = 0; i < P; ++i) {
+    DevPart& pt = parts[i];
+    Ls.push_back(layout(n, pt.nnz, r));
+    if (!pt.ws) DCK(cudaMallocAsync(&pt.ws, Ls[i].total, s));
+    if (!packed<C>() && (i > 0 || !colors_out)) {
+      DCK(cudaMallocAsync((void**)&pt.colors, (size_t)n * 4, s));
+      pt.own_colors = true;
+    } else {
+      pt.colors = colors_out;
+    }
+    sgr_csr shifted{pt.csr.row_ptr - pt.lo, pt.csr.col_idx};
+    build_args<C>(args[i], &shifted, n, pt.nnz, pt.colors, pt.ws, Ls[i], r);
+    args[i].v_begin = (int32_t)pt.lo;
+    args[i].v_end = (int32_t)pt.hi;
+    Ctrl hc;
+    memset(&hc, 0, sizeof(hc));
+    hc.k = 1;
+    hc.max_rounds = r.max_rounds;
+    DCK(cudaMemcpyAsync(args[i].ctrl, &hc, sizeof(Ctrl), cudaMemcpyHostToDevice, s));
+    DCK(cudaMemsetAsync((char*)pt.ws + Ls[i].zero_begin, 0, Ls[i].zero_end - Ls[i].zero_begin, s));
+  }
+  // pointer tables: every part's (col[0], col[1]) of the OTHER replicas, all Ctrl, all
+  // cross counters. Plain colors: replica i's col[0] is its colors buffer (not in ws), so
+  // on several GPUs only packed words (both buffers in the workspace) can be peer-mapped.
+  auto col_of = [&](int rank, int b) -> C* {
+    if (peers) {
+      char* w = (char*)peers->ws[rank];
+      const size_t cb = align_up((size_t)n * sizeof(C), 256);
+      return (C*)(w + Ls[0].off_col + (b ? cb : 0));
+    }
+    return args[rank].col[b];
+  };
+  auto ctrl_of = [&](int rank) -> Ctrl* {
+    return peers ? (Ctrl*)peers->ws[rank] : args[rank].ctrl;
+  };
+  const int per = 2 * (nranks - 1) + 2 * nranks;  // pointers per part
+  std::vector<void*> tab((size_t)per * P);
+  for (int i = 0; i < P; ++i) {
+    const int me = me0 + i;
+    void** t = tab.data() + (size_t)per * i;
+    int q = 0;
+    for (int j = 0; j < nranks; ++j)
+      if (j != me) {
+        t[2 * q] = col_of(j, 0);
+        t[2 * q + 1] = col_of(j, 1);
+        ++q;
+      }
+    for (int j = 0; j < nranks; ++j) {
+      t[2 * (nranks - 1) + j] = ctrl_of(j);
+      t[2 * (nranks - 1) + nranks + j] = &ctrl_of(j)->xbar;
+    }
+  }
+  void** dtab = nullptr;
+  RoundArgs<C>* dargs = nullptr;
+  int32_t* dflag = nullptr;
+  DCK(cudaMallocAsync((void**)&dtab, tab.size() * sizeof(void*), s));
+  DCK(cudaMallocAsync((void**)&dargs, sizeof(RoundArgs<C>) * P, s));
+  DCK(cudaMallocAsync((void**)&dflag, 64, s));
+  DCK(cudaMemcpyAsync(dtab, tab.data(), tab.size() * sizeof(void*), cudaMemcpyHostToDevice, s));
+  for (int i = 0; i < P; ++i) {
+    void** t = dtab + (size_t)per * i;
+    args[i].rep = (C* const*)t;
+    args[i].nrep = nranks - 1;
+    args[i].rctrl = (Ctrl* const*)(t + 2 * (nranks - 1));
+    args[i].xbar = (uint32_t* const*)(t + 2 * (nranks - 1) + nranks);
+    args[i].nranks = nranks;
+    args[i].me = me0 + i;
+  }
+  sgr_status status = SGR_OK;
+  // C_1 in both buffers of every replica, before any part broadcasts C_2 into it
+  for (int i = 0; i < P; ++i) k_fill_c1<C><<<first_grid(n), 256, 0, s>>>(args[i]);
+  DCK(cudaGetLastError());
+  if (xsync && (status = xsync(s, dflag, 0)) != SGR_OK) return status;
+  // F_1 per part (its C_2 words go into every replica), then the first advance
+  for (int i = 0; i < P; ++i) {
+    k_first<TB, C><<<first_grid(parts[i].hi - parts[i].lo), 256, 0, s>>>(args[i], r.sorted);
+    k_advance<<<1, 32, 0, s>>>(args[i].ctrl, 1, 0);
+  }
+  DCK(cudaGetLastError());
+  // the build every part runs: hub if any part put a vertex into bin 2 (all ranks agree)
+  std::vector<int32_t> big(P, 0);
+  for (int i = 0; i < P; ++i)
+    DCK(cudaMemcpyAsync(&big[i], &args[i].ctrl->big_count, 4, cudaMemcpyDeviceToHost, s));
+  DCK(cudaStreamSynchronize(s));
+  int32_t hub = 0;
+  for (int32_t b : big) hub |= b != 0;
+  if (xsync) {  // max over ranks; also orders every rank's F_1 broadcast before the rounds
+    DCK(cudaMemcpyAsync(dflag, &hub, 4, cudaMemcpyHostToDevice, s));
+    if ((status = xsync(s, dflag, 1)) != SGR_OK) return status;
+    DCK(cudaMemcpyAsync(&hub, dflag, 4, cudaMemcpyDeviceToHost, s));
+    DCK(cudaStreamSynchronize(s));
+  }
+  const int gmax = hub ? dist_grid<TB, C, true>(B) : dist_grid<TB, C, false>(B);
+  const int gB = std::max(1, gmax / P);  // blocks per part
+  const int grid = gB * P;
+  for (int i = 0; i < P; ++i) {
+    args[i].gfirst = gB * i;
+    args[i].gnum = gB;
+  }
+  DCK(cudaMemcpyAsync(dargs, args.data(), sizeof(RoundArgs<C>) * P, cudaMemcpyHostToDevice, s));
+  cudaEvent_t ev0, ev1;
+  cudaEventCreate(&ev0);
+  cudaEventCreate(&ev1);
+  cudaEventRecord(ev0, s);
+  {
+    const RoundArgs<C>* pa = dargs;
+    int np = P;
+    void* kargs[] = {(void*)&pa, (void*)&np};
+    const cudaError_t le = hub
+        ? cudaLaunchCooperativeKernel((const void*)k_persistent_dist<TB, C, true>, grid, B, kargs,
+                                      round_smem<C, true>(B), s)
+        : cudaLaunchCooperativeKernel((const void*)k_persistent_dist<TB, C, false>, grid, B, kargs,
+                                      round_smem<C, false>(B), s);
+    if (le != cudaSuccess) return cuda_fail(le, "cooperative launch of k_persistent_dist", __LINE__);
+  }
+  cudaEventRecord(ev1, s);
+  RoundArgs<C>& a0 = args[0];
+  if constexpr (packed<C>()) {
+    k_unpack<<<reduce_grid(n), 256, 0, s>>>(a0.col[0], colors_out, n, &a0.ctrl->max_color);
+  } else {
+    if (a0.col[0] != (C*)colors_out)
+      DCK(cudaMemcpyAsync(colors_out, a0.col[0], (size_t)n * 4, cudaMemcpyDeviceToDevice, s));
+    k_max_color<<<reduce_grid(n), 256, 0, s>>>(colors_out, n, &a0.ctrl->max_color);
+  }
+  DCK(cudaGetLastError());
+  std::vector<Ctrl> fin(P);
+  for (int i = 0; i < P; ++i)
+    DCK(cudaMemcpyAsync(&fin[i], args[i].ctrl, sizeof(Ctrl), cudaMemcpyDeviceToHost, s));
+  DCK(cudaStreamSynchronize(s));
+  // no rank may release its workspace while another can still read its counters
+  if (xsync && (status = xsync(s, dflag, 0)) != SGR_OK) return status;
+  int overflow = 0;
+  for (int i = 0; i < P; ++i) overflow |= fin[i].overflow;
+  if (overflow && !packed<C>()) {
+    set_error("sgr_color_dist: 32-bit color overflow");
+    status = SGR_EUNSUPPORTED;
+  }
+  if (overflow && packed<C>()) *overflow_out = 1;
+  if (fin[0].status == 1 && !overflow) {
+    set_error("sgr_color_dist: max_rounds (%d) reached", r.max_rounds);
+    status = SGR_ENOCONV;
+  }
+  if (stats && status == SGR_OK) {
+    memset(stats, 0, sizeof(*stats));
+    int64_t nnz_parts = 0, verts = 0;
+    for (int i = 0; i < P; ++i) {
+      sgr_stats t;
+      memset(&t, 0, sizeof(t));
+      fill_stats(fin[i], 0, 0, &t, (int)sizeof(C));
+      stats->edges_scanned += t.edges_scanned;
+      stats->entries_read += t.entries_read;
+      stats->entries_written += t.entries_written;
+      stats->bytes_algorithmic += t.bytes_algorithmic;
+      stats->chunk_items += t.chunk_items;
+      verts += t.vertices_processed;
+      for (int q = 0; q < 3; ++q) {
+        stats->bin_vertices[q] += t.bin_vertices[q];
+        stats->bin_edges[q] += t.bin_edges[q];
+      }
+      nnz_parts += parts[i].nnz;
+    }
+    stats->edges_scanned += nnz_parts;  // round 1 (this device's parts)
+    stats->vertices_processed = verts + n * P / std::max(nranks, 1);
+    stats->rounds = fin[0].k - 1;
+    stats->num_colors = fin[0].max_color;
+    stats->launches = 3 * P + 2;
+    stats->grid_blocks = grid;
+    stats->color_bits = packed<C>() ? 16 : 32;
+    stats->transport = nranks > 1 ? SGR_XCHG_DEVICE : SGR_XCHG_NONE;
+    cudaEventElapsedTime(&stats->elapsed_ms, ev0, ev1);
+  }
+  cudaEventDestroy(ev0);
+  cudaEventDestroy(ev1);
+  cudaFreeAsync(dtab, s);
+  cudaFreeAsync(dargs, s);
+  cudaFreeAsync(dflag, s);
+  for (auto& pt : parts) {
+    if (!peers) cudaFreeAsync(pt.ws, s);
+    pt.ws = peers ? pt.ws : nullptr;
+    if (pt.own_colors) cudaFreeAsync(pt.colors, s);
+    pt.own_colors = false;
+  }
+  cudaStreamSynchronize(s);
+  return status;
+}
+
+template <class... A>
+static sgr_status dispatch_dev(const Resolved& r, A&&... args) {
+  int overflow = 0;
+  if (r.color_bits == 16) {
+    const sgr_status st = r.tiebreak ? run_dev<1, Packed>(args..., r, &overflow)
+                                     : run_dev<0, Packed>(args..., r, &overflow);
+    if (st != SGR_OK || !overflow) return st;
+  }
+  Resolved r32 = r;
+  r32.color_bits = 32;
+  return r.tiebreak ? run_dev<1, int32_t>(args..., r32, &overflow)
+                    : run_dev<0, int32_t>(args..., r32, &overflow);
 }
 
 // Packed (16-bit) words first; if any partition's first fit exceeded the color cap, every
@@ -396,6 +646,89 @@ static sgr_status dispatch(const Resolved& r, A&&... args) {
   return r.tiebreak ? run_parts<1, int32_t>(args..., r32, &overflow)
                     : run_parts<0, int32_t>(args..., r32, &overflow);
 }
+
+#if SGR_HAVE_NCCL
+// Device-side exchange across GPUs (k_persistent_dist, one part per rank): the workspaces
+// (replicas, counters) are cudaMalloc'd, their IPC handles all-gathered over NCCL and
+// mapped into every rank (NVLink peer memory), so each rank's pass stores its color words
+// straight into all replicas and the ranks meet at a device-side barrier. SGR_EUNSUPPORTED
+// (the caller then uses the NCCL all-gather transport) when a peer cannot be mapped.
+static sgr_status color_dist_device(DistComm* c, const sgr_csr* local, int64_t n, int64_t v_begin,
+                                    int64_t v_end, int64_t nnz_local, int32_t* colors_out,
+                                    sgr_stats* stats, const Resolved& r) {
+  cudaStream_t s = r.stream;
+  Resolved r16 = r;
+  r16.color_bits = 16;
+  const Layout L = layout(n, nnz_local, r16);
+  std::vector<DevPart> dp(1);
+  dp[0].lo = v_begin;
+  dp[0].hi = v_end;
+  dp[0].nnz = nnz_local;
+  dp[0].csr = *local;
+  if (c->world == 1) {  // no other replica: the rounds of one part, no exchange at all
+    return dispatch_dev(r, dp, 1, 0, n, colors_out, stats, (const PeerView*)nullptr, XSync());
+  }
+  if (r.color_bits == 32) return SGR_EUNSUPPORTED;  // the same on every rank (same opts)
+  void* ws = nullptr;
+  DCK(cudaMalloc(&ws, L.total));  // IPC needs a cudaMalloc allocation
+  cudaIpcMemHandle_t h;
+  DCK(cudaIpcGetMemHandle(&h, ws));
+  char* dh = nullptr;
+  DCK(cudaMalloc((void**)&dh, sizeof(h) * (c->world + 1)));
+  DCK(cudaMemcpy(dh + sizeof(h) * c->world, &h, sizeof(h), cudaMemcpyHostToDevice));
+  ncclResult_t rc = ncclAllGather(dh + sizeof(h) * c->world, dh, sizeof(h), ncclChar, c->comm, s);
+  std::vector<cudaIpcMemHandle_t> hs(c->world);
+  if (rc == ncclSuccess) DCK(cudaMemcpyAsync(hs.data(), dh, sizeof(h) * c->world, cudaMemcpyDeviceToHost, s));
+  DCK(cudaStreamSynchronize(s));
+  cudaFree(dh);
+  if (rc != ncclSuccess) {
+    cudaFree(ws);
+    set_error("ncclAllGather (IPC handles): %s", ncclGetErrorString(rc));
+    return SGR_ENCCL;
+  }
+  PeerView pv;
+  pv.me = c->rank;
+  pv.ws.assign(c->world, nullptr);
+  pv.ws[c->rank] = ws;
+  bool mapped = true;
+  for (int q = 0; q < c->world && mapped; ++q) {
+    if (q == c->rank) continue;
+    if (cudaIpcOpenMemHandle(&pv.ws[q], hs[q], cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+      cudaGetLastError();
+      mapped = false;
+    }
+  }
+  // every rank must take the same path: agree on the mapping outcome
+  int32_t* dflag = nullptr;
+  DCK(cudaMalloc((void**)&dflag, 4));
+  int32_t ok = mapped ? 1 : 0;
+  DCK(cudaMemcpy(dflag, &ok, 4, cudaMemcpyHostToDevice));
+  rc = ncclAllReduce(dflag, dflag, 1, ncclInt32, ncclMin, c->comm, s);
+  DCK(cudaMemcpyAsync(&ok, dflag, 4, cudaMemcpyDeviceToHost, s));
+  DCK(cudaStreamSynchronize(s));
+  cudaFree(dflag);
+  sgr_status st = SGR_EUNSUPPORTED;
+  if (rc == ncclSuccess && ok) {
+    dp[0].ws = ws;
+    XSync xs = [c](cudaStream_t st2, int32_t* f, int op_max) -> sgr_status {
+      const ncclResult_t e = ncclAllReduce(f, f, 1, ncclInt32, op_max ? ncclMax : ncclSum, c->comm, st2);
+      if (e != ncclSuccess) {
+        set_error("ncclAllReduce: %s", ncclGetErrorString(e));
+        return SGR_ENCCL;
+      }
+      return SGR_OK;
+    };
+    int overflow = 0;
+    st = r.tiebreak ? run_dev<1, Packed>(dp, c->world, c->rank, n, colors_out, stats, &pv, xs, r16, &overflow)
+                    : run_dev<0, Packed>(dp, c->world, c->rank, n, colors_out, stats, &pv, xs, r16, &overflow);
+    if (st == SGR_OK && overflow) st = SGR_EUNSUPPORTED;  // every rank saw it: int32 via NCCL
+  }
+  for (int q = 0; q < c->world; ++q)
+    if (q != c->rank && pv.ws[q]) cudaIpcCloseMemHandle(pv.ws[q]);
+  cudaFree(ws);
+  return st;
+}
+#endif
 
 }  // namespace sgr
 
@@ -457,14 +790,30 @@ sgr_status sgr_color_partitioned(const sgr_csr* csr, int64_t n, int64_t nnz, int
     DCK(cudaStreamSynchronize(s));  // lrp is a host temporary
     pt.csr = sgr_csr{local_rp[p], local_ci[p]};
   }
-  // the all-gather between partitions that share this device: device copies
-  Gather gather = [](std::vector<Part>& ps, uint2* recv, int32_t cap, cudaStream_t st) -> sgr_status {
-    for (size_t q = 0; q < ps.size(); ++q)
-      DCK(cudaMemcpyAsync(recv + q * (size_t)(cap + 1), ps[q].send, (size_t)(cap + 1) * sizeof(uint2),
-                          cudaMemcpyDeviceToDevice, st));
-    return SGR_OK;
-  };
-  const sgr_status st = dispatch(r, parts, P, 0, n, colors_out, stats, gather, (int64_t)0);
+  sgr_status st;
+  const char* hl = getenv("SGR_DIST_HOSTLOOP");
+  if (!(hl && hl[0] == '1')) {
+    // device-side exchange: one cooperative launch, a block group per partition, every
+    // color word stored into all replicas (k_persistent_dist)
+    std::vector<DevPart> dp(P);
+    for (int p = 0; p < P; ++p) {
+      dp[p].lo = parts[p].lo;
+      dp[p].hi = parts[p].hi;
+      dp[p].nnz = parts[p].nnz;
+      dp[p].csr = parts[p].csr;
+    }
+    st = dispatch_dev(r, dp, P, 0, n, colors_out, stats, (const PeerView*)nullptr, XSync());
+  } else {
+    // host-driven rounds with an explicit all-gather (the NCCL transport's protocol) done by
+    // device copies between the partitions of this device
+    Gather gather = [](std::vector<Part>& ps, uint2* recv, int32_t cap, cudaStream_t st2) -> sgr_status {
+      for (size_t q = 0; q < ps.size(); ++q)
+        DCK(cudaMemcpyAsync(recv + q * (size_t)(cap + 1), ps[q].send, (size_t)(cap + 1) * sizeof(uint2),
+                            cudaMemcpyDeviceToDevice, st2));
+      return SGR_OK;
+    };
+    st = dispatch(r, parts, P, 0, n, colors_out, stats, gather, (int64_t)0);
+  }
   for (int p = 0; p < P; ++p) {
     cudaFreeAsync(local_rp[p], s);
     cudaFreeAsync(local_ci[p], s);
@@ -543,6 +892,13 @@ sgr_status sgr_color_dist(void* comm, const sgr_csr* local, int64_t n_global, in
 #if SGR_HAVE_NCCL
   DistComm* c = (DistComm*)comm;
   const Resolved r = resolve_opts(opts, n_global);
+  const char* tr = getenv("SGR_DIST_TRANSPORT");  // "nccl": the host-driven all-gather path
+  if (!(tr && strcmp(tr, "nccl") == 0)) {
+    const sgr_status ds = color_dist_device(c, local, n_global, v_begin, v_end, nnz_local,
+                                            colors_out, stats, r);
+    if (ds != SGR_EUNSUPPORTED) return ds;
+    // no peer access between the ranks' GPUs (or int32 words needed): NCCL transport below
+  }
   std::vector<Part> parts(1);
   parts[0].lo = v_begin;
   parts[0].hi = v_end;

@@ -199,7 +199,8 @@ struct Ctrl {
   int32_t big_count;         // slots handed to bin-2 vertices by F_1
   int32_t max_color;
   int32_t violations;
-  int32_t pad[5];
+  uint32_t xbar;             // cross-part barrier counter (k_persistent_dist; other parts add)
+  int32_t pad[4];
   Counts ring[3];
   unsigned long long edges_acc[3][kBins];    // per ring slot: sum of deg(v) over the pass's
   unsigned long long entries_acc[3][kBins];  // vertices / list entries actually read
@@ -242,7 +243,25 @@ struct RoundArgs {
   int32_t v_begin;            // owned vertex range [v_begin, v_end) (multi-GPU: a partition)
   int32_t v_end;
   int32_t color_cap;          // packed mode: largest color a 16-bit word holds (<= 4095)
+  // Device-side exchange (k_persistent_dist): every color word this part
+  // writes for its own vertices is also stored into the other replicas (other partitions
+  // of this device, or NVLink peer memory of other GPUs), so no exchange step exists.
+  C* const* rep;              // [2 * nrep]: replica q's (col[0], col[1]); nullptr: none
+  int32_t nrep;
+  int32_t gfirst, gnum;       // this part's block group in a multi-part launch (gnum 0: grid)
+  int32_t nranks, me;         // parts / ranks taking part in the coloring, this one's index
+  Ctrl* const* rctrl;         // [nranks] every part's Ctrl (own included): global counts
+  uint32_t* const* xbar;      // [nranks] every part's cross-part barrier counter
 };
+
+// This part's block group: the whole grid, or (multi-part launch) blocks
+// [gfirst, gfirst + gnum).
+template <class C>
+__device__ __forceinline__ int grp_block(const RoundArgs<C>& a) {
+  return a.gnum ? (int)blockIdx.x - a.gfirst : (int)blockIdx.x;
+}
+template <class C>
+__device__ __forceinline__ int grp_size(const RoundArgs<C>& a) { return a.gnum ? a.gnum : (int)gridDim.x; }
 
 // Parameter-struct selects without dynamic indexing (which would spill it to the stack).
 template <class T>
@@ -316,6 +335,17 @@ __device__ __forceinline__ C cpack(int32_t color, int32_t last, const RoundArgs<
     (void)last;
     (void)a;
     return (C)color;
+  }
+}
+
+// Y[v] = word, and the same word into every other replica's buffer of that parity (pass
+// k writes col[k & 1]; F_1's C_2 is parity 1). Other parts never write v (only its owner
+// does) and read that buffer only as the NEXT pass's snapshot, after the pass barrier.
+template <class C>
+__device__ __forceinline__ void put_y(const RoundArgs<C>& a, C* Y, int k, int32_t v, C word) {
+  Y[v] = word;
+  if (a.nrep) {
+    for (int q = 0; q < a.nrep; ++q) a.rep[2 * q + (k & 1)][v] = word;
   }
 }
 
@@ -492,7 +522,7 @@ __global__ void __launch_bounds__(1024) k_first(RoundArgs<C> a, int sorted) {
         }
       }
       X[v] = cpack<C>(1, 1, a);
-      Y[v] = cpack<C>(conflict ? 2 : 1, conflict ? 2 : 1, a);
+      put_y<C>(a, Y, 1, v, cpack<C>(conflict ? 2 : 1, conflict ? 2 : 1, a));
     }
     const int b = bin_of(e - s, a.small_max, a.med_max);
     Counts* w2 = &ctrl->ring[rs(2)];
@@ -553,6 +583,7 @@ __global__ void __launch_bounds__(1024) k_first(RoundArgs<C> a, int sorted) {
       for (int32_t t = 0; t < nch; ++t) a.wl_c[0][ib + t] = make_item(v, t);
     }
   }
+  if (a.nrep) __threadfence_system();  // C_2 stores into peer replicas: visible system-wide
 }
 
 // ---------------------------------------------------------------------------------------
@@ -719,7 +750,7 @@ __device__ __forceinline__ void process_chunk_plain(const RoundArgs<C>& a, int k
       if (tent < 0) tent = warp_first_fit_rescan<Persist>(a.col_idx, X, s, e, kBigTbl, lane);
     }
     if (lane == 0) {
-      Y[v] = any ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a);
+      put_y<C>(a, Y, k, v, any ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a));
       if (any) {
         out[atomicAdd(out_cnt, 1)] = make_item(v, 0);
         atomicAdd(out_vcnt, 1);
@@ -751,7 +782,7 @@ __device__ __forceinline__ void process_chunk_plain(const RoundArgs<C>& a, int k
       }
       int32_t ob = 0;
       if (lane == 0) {
-        Y[v] = conf_all ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a);
+        put_y<C>(a, Y, k, v, conf_all ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a));
         if (conf_all) {
           ob = atomicAdd(out_cnt, nch);
           atomicAdd(out_vcnt, 1);
@@ -1018,7 +1049,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
         }
         if (lane == 0) {
           len_nxt[v] = rewrite ? (int32_t)live_total : cnt;
-          Y[v] = cpack<C>(tent, k + 1, a);
+          put_y<C>(a, Y, k, v, cpack<C>(tent, k + 1, a));
           // live <= kChunk: one chunk, the list stays in its buffer
           ibuf[ipend] = make_item(v, (int32_t)(cur.buf ? kBufBit : 0u));
         }
@@ -1026,7 +1057,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
         ++vpend;
         if (ipend == 32) iflush();
       } else if (lane == 0) {
-        Y[v] = cpack<C>(xv, k, a);
+        put_y<C>(a, Y, k, v, cpack<C>(xv, k, a));
       }
     } else {
       // several chunks: publish this chunk's partial forbidden set, dropped colors and
@@ -1109,8 +1140,8 @@ __device__ __forceinline__ void finalize_body(const RoundArgs<Packed>& a, int k)
   Ctrl* ctrl = a.ctrl;
   const int p = k & 1;
   const int lane = threadIdx.x & 31;
-  const int gw = (int)((blockIdx.x * blockDim.x + threadIdx.x) >> 5);
-  const int NW = (int)((gridDim.x * blockDim.x) >> 5);
+  const int gw = (int)((grp_block(a) * blockDim.x + threadIdx.x) >> 5);
+  const int NW = (int)((grp_size(a) * blockDim.x) >> 5);
   const int nF = ld_cg(&ctrl->ring[rs(k)].fin);
   const C* X = sel((k - 1) & 1, (const C*)a.col[0], (const C*)a.col[1]);
   C* Y = sel(k & 1, a.col[0], a.col[1]);
@@ -1218,7 +1249,7 @@ __device__ __forceinline__ void finalize_body(const RoundArgs<Packed>& a, int k)
       a.acc_cnt[slot] = 0ull;
       len_cur[v] = 0;  // consumed; the pass after next accumulates into it
       if (conf && kept) len_nxt[v] = len_list;  // the same list again
-      Y[v] = conf ? cpack<C>(tent, k + 1, a) : cpack<C>(cval<C>(xraw), k, a);
+      put_y<C>(a, Y, k, v, conf ? cpack<C>(tent, k + 1, a) : cpack<C>(cval<C>(xraw), k, a));
       const uint32_t obuf = (uint32_t)f & kBufBit;
       const uint32_t nbuf = (kept ? obuf : (obuf ^ kBufBit)) | (keep_next ? kKeepBit : 0u);
       for (int32_t t = 0; t < nch2; ++t) out[ob + t] = make_item(v, (int32_t)(t | nbuf));
@@ -1293,7 +1324,7 @@ __device__ __forceinline__ void process_group(const RoundArgs<C>& a, int k, int3
   }
   set_clear(gtbl, kMedTblB, gl, kGroup);
   __syncwarp();
-  if (v >= 0 && gl == 0) Y[v] = any ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a);
+  if (v >= 0 && gl == 0) put_y<C>(a, Y, k, v, any ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a));
   push = (v >= 0) && any && gl == 0;
 }
 
@@ -1413,7 +1444,7 @@ __device__ __forceinline__ void bin0(const RoundArgs<C>& a, int k, const int32_t
     const bool any = (__ballot_sync(0xffffffffu, conf) & gmask) != 0u;
     if (v >= 0 && gl == 0) {
       const int32_t tent = ~mask ? __ffs(~mask) : 33;
-      Y[v] = any ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a);
+      put_y<C>(a, Y, k, v, any ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a));
       edges += (unsigned long long)(e - s);
       entries += (unsigned long long)(e - s);
     }
@@ -1491,7 +1522,7 @@ __device__ __forceinline__ void bin0_tiled(const RoundArgs<C>& a, int k, const i
     const bool any = (__ballot_sync(0xffffffffu, conf) & gmask) != 0u;
     if (v >= 0 && gl == 0) {
       const int32_t tent = ~mask ? __ffs(~mask) : 33;
-      Y[v] = any ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a);
+      put_y<C>(a, Y, k, v, any ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a));
       edges += (unsigned long long)(e - s);
       entries += (unsigned long long)(e - s);
     }
@@ -1580,7 +1611,7 @@ __device__ __forceinline__ void bin0_thread(const RoundArgs<C>& a, int k, const 
     }
     if (v >= 0) {
       const int32_t tent = ~mask ? __ffs(~mask) : 33;
-      Y[v] = conf ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a);
+      put_y<C>(a, Y, k, v, conf ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a));
       edges += (unsigned long long)cnt;
       entries += (unsigned long long)cnt;
     }
@@ -1679,8 +1710,8 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, const C
   Ctrl* ctrl = a.ctrl;
   const int p = k & 1;
   const int lane = threadIdx.x & 31;
-  const int gw = (int)((blockIdx.x * blockDim.x + threadIdx.x) >> 5);
-  const int NW = (int)((gridDim.x * blockDim.x) >> 5);
+  const int gw = (int)((grp_block(a) * blockDim.x + threadIdx.x) >> 5);
+  const int NW = (int)((grp_size(a) * blockDim.x) >> 5);
   const C* X = sel((k - 1) & 1, (const C*)a.col[0], (const C*)a.col[1]);
   C* Y = sel(k & 1, a.col[0], a.col[1]);
   uint8_t* wtbl = wsm + WarpSmem<C, Hub>::kBuf;
@@ -2147,6 +2178,142 @@ __global__ void __launch_bounds__(kMaxThreads<C, Hub>, 1) k_persistent(RoundArgs
   if (SGR_PHASE_CYCLES && (threadIdx.x & 31) == 0) {
     for (int q = 0; q < kBins; ++q) atomicAdd(&ctrl->bin_cycles[q], cyc[q]);
     for (int q = 0; q < 3; ++q) atomicAdd(&ctrl->phase_cycles[4 + q], pcx[q]);
+  }
+}
+
+// ---------------------------------------------------------------------------------------
+// Multi-part persistent kernel: the distributed rounds with the exchange done
+// on the device. Each part (a vertex range with its own rows, worklists and a full color
+// replica) runs the same fused pass as k_persistent in its own block group; put_y stores
+// every color word the part writes into all replicas as well (other parts of this device,
+// or NVLink peer memory when each GPU holds one part), so after the pass barrier every
+// replica holds C_{k+1} and no exchange step, host round trip or collective launch remains.
+// The pass barrier spans all parts: a group barrier on the part's own counter, then the
+// group's first block signals every other part's cross counter (red.release.sys) and waits
+// for all of theirs (ld.acquire.sys), then a second group barrier. Loop decisions use the
+// counts of ALL parts (termination, color overflow, the finalize phase), read after it.
+__device__ __forceinline__ uint32_t ld_acquire_sys(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint32_t ld_relaxed_sys(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.relaxed.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ int32_t ld_relaxed_sys_i32(const int32_t* p) {
+  int32_t v;
+  asm volatile("ld.relaxed.sys.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void red_release_sys_u32(uint32_t* p, uint32_t v) {
+  asm volatile("red.release.sys.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// Barrier of one block group (nblk blocks) on `ctrl->bar_count` (as grid_sync).
+__device__ __forceinline__ void group_sync(Ctrl* ctrl, uint32_t& epoch, int nblk) {
+  __syncthreads();
+  ++epoch;
+  if (threadIdx.x == 0) {
+    red_release_gpu_u32(&ctrl->bar_count, 1u);
+    const uint32_t target = epoch * (uint32_t)nblk;
+    while ((int32_t)(ld_relaxed_gpu(&ctrl->bar_count) - target) < 0) {
+      if (SGR_BARSLEEP) __nanosleep(SGR_BARSLEEP);
+    }
+    (void)ld_acquire_gpu(&ctrl->bar_count);
+  }
+  __syncthreads();
+}
+
+template <class C>
+__device__ __forceinline__ void part_sync(const RoundArgs<C>& a, uint32_t& epoch, uint32_t& xepoch) {
+  const int nblk = grp_size(a);
+  group_sync(a.ctrl, epoch, nblk);
+  if (a.nranks > 1) {
+    if (grp_block(a) == 0 && threadIdx.x == 0) {
+      ++xepoch;
+      for (int q = 0; q < a.nranks; ++q)
+        if (q != a.me) red_release_sys_u32(a.xbar[q], 1u);
+      const uint32_t target = xepoch * (uint32_t)(a.nranks - 1);
+      uint32_t* mine = a.xbar[a.me];
+      while ((int32_t)(ld_relaxed_sys(mine) - target) < 0) {
+        if (SGR_BARSLEEP) __nanosleep(SGR_BARSLEEP);
+      }
+      (void)ld_acquire_sys(mine);
+    } else {
+      ++xepoch;
+    }
+    group_sync(a.ctrl, epoch, nblk);
+  }
+}
+
+// Counts of pass k over all parts (thread 0 reads them, the block shares them).
+struct GlobalCounts {
+  int64_t items;
+  int32_t overflow;
+  int32_t multi;  // multi-chunk bin-2 vertices anywhere (the finalize phase is global)
+};
+template <class C>
+__device__ __forceinline__ GlobalCounts global_counts(const RoundArgs<C>& a, int k) {
+  __shared__ GlobalCounts gc;
+  if (threadIdx.x == 0) {
+    GlobalCounts g{0, 0, 0};
+    for (int q = 0; q < a.nranks; ++q) {
+      const Counts* r = &a.rctrl[q]->ring[rs(k)];
+      g.items += (int64_t)ld_relaxed_sys_i32(&r->t) + ld_relaxed_sys_i32(&r->m) + ld_relaxed_sys_i32(&r->c);
+      g.multi |= ld_relaxed_sys_i32(&r->pad[1]) != 0;
+      g.overflow |= ld_relaxed_sys_i32(&a.rctrl[q]->overflow);
+    }
+    gc = g;
+  }
+  __syncthreads();
+  const GlobalCounts g = gc;
+  __syncthreads();  // gc is rewritten by the next call
+  return g;
+}
+
+template <int TB, class C, bool Hub>
+__global__ void __launch_bounds__(kMaxThreads<C, Hub>, 1) k_persistent_dist(const RoundArgs<C>* __restrict__ parts,
+                                                                        int nparts) {
+  extern __shared__ __align__(16) uint8_t dsmem[];
+  const int gB = (int)gridDim.x / nparts;
+  const int p = min((int)blockIdx.x / gB, nparts - 1);
+  const RoundArgs<C> a = parts[p];
+  Ctrl* ctrl = a.ctrl;
+  uint8_t* wsm = warp_smem_init<C, Hub>(dsmem);
+  uint32_t ph = 0;
+  unsigned long long cyc[kBins] = {0, 0, 0};
+  uint32_t epoch = 0, xepoch = 0;
+  const int max_rounds = ld_cg(&ctrl->max_rounds);
+  const bool leader = grp_block(a) == grp_size(a) - 1 && threadIdx.x == 0;
+  // every part's F_1 (and its broadcast of C_2) finished before this launch (stream order /
+  // the host's cross-rank sync), so pass 2 can start at once
+  int k = 2;
+  for (;; ++k) {
+    const Counts w = ld_counts(&ctrl->ring[rs(k)]);
+    const GlobalCounts g = global_counts(a, k);
+    if (leader && k > 2) fold_pass(ctrl, k - 1);
+    const bool active = g.items > 0 && !g.overflow;
+    if (!active || k > max_rounds) {  // uniform over all parts
+      if (leader) {
+        ctrl->k = k;
+        ctrl->active = 0;
+        if (active) ctrl->status = 1;
+        if (g.overflow) ctrl->overflow = 1;  // every part reruns with int32 words
+      }
+      break;
+    }
+    unsigned long long edges[kBins] = {0, 0, 0}, entries[kBins] = {0, 0, 0};
+    round_body<TB, true, C, Hub>(a, k, w, wsm, edges, entries, ph, cyc);
+    block_add6(edges, entries, ctrl, k);
+    bool fin_phase = false;
+    if constexpr (packed<C>() && Hub) fin_phase = g.multi != 0;  // uniform over all parts
+    if (fin_phase) {  // a part's multi-chunk vertices are all its own: a group barrier
+      group_sync(ctrl, epoch, grp_size(a));
+      if constexpr (packed<C>() && Hub) finalize_body<TB, true>(a, k);
+    }
+    part_sync(a, epoch, xepoch);
   }
 }
 

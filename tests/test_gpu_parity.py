@@ -446,10 +446,16 @@ def test_cfg5_full_size():
 # ----------------------------------------------------------------------------- multi-GPU path
 @pytest.mark.parametrize("P", [1, 2, 3, 5, 8])
 @pytest.mark.parametrize("tb", [LOW, PAP])
-def test_partitioned_equals_single_gpu(P, tb):
-    """The distributed exchange protocol (sgr_dist.cu: pack -> padded all-gather -> apply into
-    both replica buffers, lockstep advance) on P partitions of one device is bit-exact."""
-    for g in (gen.config(1), degree_boundary_graph(), random_graph(7, n=300)):
+@pytest.mark.parametrize("transport", ["device", "hostloop"])
+def test_partitioned_equals_single_gpu(P, tb, transport, monkeypatch):
+    """The distributed protocol on P partitions of one device is bit-exact, with both
+    transports: the device-side exchange (k_persistent_dist: color words stored into every
+    replica, barrier across parts, one cooperative launch) and the host-driven rounds with
+    a padded all-gather (pack -> gather -> apply, lockstep advance)."""
+    if transport == "hostloop":
+        monkeypatch.setenv("SGR_DIST_HOSTLOOP", "1")
+    for g in (gen.config(1), degree_boundary_graph(), random_graph(7, n=300),
+              gen.stencil3d(14, 13, 12, 27)):
         rp, ci = dev(g)
         ref = oracle.jacobi(g, tb)
         res = sgr.color_partitioned(rp, ci, P, tiebreak=RULE[tb])
@@ -457,6 +463,8 @@ def test_partitioned_equals_single_gpu(P, tb):
         assert res.stats["rounds"] == ref.rounds
         assert res.stats["vertices_processed"] == ref.vertices_processed
         assert res.stats["num_colors"] == ref.num_colors
+        if P > 1:
+            assert res.stats["transport"] == ("device" if transport == "device" else "allgather")
 
 
 @pytest.mark.parametrize("P", [1, 3])
@@ -465,6 +473,7 @@ def test_partitioned_graph_replay(P, monkeypatch):
     the rounds, colors and counts are those of the eager loop and of the oracle (the
     bucketed all-gather capacity pads records, the counts in the payload bound them)."""
     monkeypatch.setenv("SGR_DIST_GRAPHS", "1")
+    monkeypatch.setenv("SGR_DIST_HOSTLOOP", "1")
     for g in (gen.config(1), degree_boundary_graph(), gen.stencil3d(12, 12, 12)):
         rp, ci = dev(g)
         for tb in (LOW, PAP):
@@ -476,9 +485,12 @@ def test_partitioned_graph_replay(P, monkeypatch):
 
 
 @pytest.mark.parametrize("P", [1, 3])
-def test_partitioned_color_overflow_rerun(P):
+@pytest.mark.parametrize("transport", ["device", "hostloop"])
+def test_partitioned_color_overflow_rerun(P, transport, monkeypatch):
     """Partitions see a packed overflow in the same exchange and all redo the coloring
     with int32 words (color_cap lowered below K_300's colors by the test hook)."""
+    if transport == "hostloop":
+        monkeypatch.setenv("SGR_DIST_HOSTLOOP", "1")
     g = degree_boundary_graph()
     rp, ci = dev(g)
     for tb in (LOW, PAP):
@@ -502,13 +514,16 @@ def test_partitioned_random_ranges_and_widths(bits):
         assert torch.equal(res.colors, ref), (P, ranges)
 
 
-def test_nccl_world1_color_dist():
+@pytest.mark.parametrize("transport", ["device", "nccl"])
+def test_nccl_world1_color_dist(transport, monkeypatch):
     """sgr_comm_init + sgr_color_dist over a one-rank NCCL communicator (the box has one
     GPU; multi-rank NCCL is exercised by bench.py under torchrun on a multi-GPU node)."""
     import socket
 
     import torch.distributed as dist
     from paper_conf_ipps_licqfsty16_b200.dist import Comm, color_dist
+    if transport == "nccl":
+        monkeypatch.setenv("SGR_DIST_TRANSPORT", "nccl")
     with socket.socket() as s:
         s.bind(("127.0.0.1", 0))
         port = s.getsockname()[1]
