@@ -263,8 +263,11 @@ def run_single(args):
     stream = torch.cuda.current_stream()
     torch.cuda.synchronize()
 
+    colors_sec = torch.empty(g.n, dtype=torch.int32, device=dev)  # secondary-rule output
+
     def step(profile=False, tiebreak=None):
-        return sgr.color(rp, ci, tiebreak or args.tiebreak, out=colors, workspace=ws,
+        return sgr.color(rp, ci, tiebreak or args.tiebreak,
+                         out=colors_sec if tiebreak else colors, workspace=ws,
                          profile=profile, loop_mode=args.loop_mode, block_size=args.block_size)
 
     for _ in range(max(args.warmup, 3)):

@@ -85,6 +85,9 @@ static sgr_status run_parts(std::vector<Part>& parts, int world, int me0, int64_
     Ls.push_back(layout(n, pt.nnz, r));
     DCK(cudaMallocAsync(&pt.ws, Ls[i].total, s));
     DCK(cudaMallocAsync((void**)&pt.send, (size_t)(cap_max + 1) * sizeof(uint2), s));
+    // the padded all-gather copies whole slots; records past a rank's count are never
+    // read, but start them defined (compute-sanitizer initcheck)
+    DCK(cudaMemsetAsync(pt.send, 0, (size_t)(cap_max + 1) * sizeof(uint2), s));
     if (!packed<C>() && (i > 0 || !colors_out)) {
       DCK(cudaMallocAsync((void**)&pt.colors, (size_t)n * 4, s));
       pt.own_colors = true;

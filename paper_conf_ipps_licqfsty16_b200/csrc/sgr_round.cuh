@@ -66,6 +66,13 @@ constexpr int kJB = 4 * kQB;  // entries per lane per batch
 #ifndef SGR_CLRMAX
 #define SGR_CLRMAX 1  // bin 2: clear the chunk's tables only up to the largest color seen
 #endif
+// Small-color passes: pass k reads C_k, whose colors are <= k (round 1 colors everything 1
+// and a first fit is at most one above the largest neighbour color), so for k <= 62 every
+// forbidden set fits a 64-bit register mask: bins 1 and 2 OR bits into registers and
+// reduce them across lanes instead of storing bytes into shared tables and scanning them.
+#ifndef SGR_SMALLMASK
+#define SGR_SMALLMASK 1
+#endif
 #ifndef SGR_BARSLEEP
 #define SGR_BARSLEEP 20  // grid-barrier poll back-off (ns); 0 = spin
 #endif
@@ -794,6 +801,7 @@ __device__ __forceinline__ void process_chunk_plain(const RoundArgs<C>& a, int k
       }
     }
   }
+  __syncwarp();  // every lane's table reads (first-fit scan) before any lane clears
   set_clear(tbl, kBigTblB, lane, 32);
   __syncwarp();
 }
@@ -851,9 +859,24 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
     const int64_t cs = h.s + (int64_t)h.c * kChunk;
     const int64_t ce = min(h.s + (int64_t)h.len, cs + kChunk);
     const int64_t w0 = cs & ~(int64_t)3;
-    const uint32_t bytes = (uint32_t)(((ce - w0 + 3) >> 2) << 4);
+    int64_t wend = (ce + 3) & ~(int64_t)3;  // 16-byte-aligned window [w0, wend)
+    int32_t* dst = bufs + st * (kStage / 4);
+    const int32_t* src = list_src(h.buf);
     fence_proxy_async();  // generic-proxy reads of this stage happen-before the async write
-    tma_load_1d(bufs + st * (kStage / 4), list_src(h.buf) + w0, bytes, bars + st);
+    if (k == 2 && wend > a.nnz) {
+      // pass 2 reads col_idx, which holds exactly nnz entries (the adjacency buffers are
+      // padded): the array's last partial 16-byte group is copied by plain loads, so the
+      // bulk copy never reads past nnz (compute-sanitizer memcheck, round 2)
+      const int64_t full = max(a.nnz & ~(int64_t)3, w0);
+      for (int64_t q = full; q < ce; ++q) dst[q - w0] = ld_ro(src + q);
+      wend = full;
+    }
+    const uint32_t bytes = (uint32_t)((wend - w0) * 4);
+    if (bytes) {
+      tma_load_1d(dst, src + w0, bytes, bars + st);
+    } else {  // nothing left for the bulk copy: complete the phase with a plain arrival
+      asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(bars + st)) : "memory");
+    }
   };
   auto finish_hdr = [&](int64_t it, ChunkHdr& h) {  // everything but the item itself
     h.v = (int32_t)((uint64_t)it >> 32);
@@ -948,6 +971,8 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
     bool conf = false;
     uint32_t cmax = 0;  // SGR_CLRMAX: largest table index this lane set
     const unsigned lt_mask = (1u << lane) - 1u;
+    const bool small = SGR_SMALLMASK && k <= 62;  // uniform: every color of X is <= k
+    uint64_t mall = 0, mdrop = 0;                 // small passes: colors seen / dropped
     // batch bb: window slots 32 (kJB bb + j) + lane, j < kJB: consecutive lanes read
     // consecutive (sorted) list entries, so neighbours close in id share a cache line
     // within one gather instruction
@@ -971,13 +996,19 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
         if ((okm >> j) & 1u) {
           // colors >= 1023 are clamped onto byte 1023; a first fit of 1023 or more is
           // recomputed exactly from the full row (warp_first_fit_rescan)
-          const uint32_t ci = min(raw[j] & kColorMask, (uint32_t)(kBigTbl - 1));
           live = (raw[j] >> kRoundShift) == klive;
+          if (small) {
+            const uint64_t bit = 1ull << (raw[j] & 63u);
+            mall |= bit;
+            mdrop |= live ? 0ull : bit;
+          } else {
+            const uint32_t ci = min(raw[j] & kColorMask, (uint32_t)(kBigTbl - 1));
 #if SGR_CLRMAX
-          cmax = max(cmax, ci);
+            cmax = max(cmax, ci);
 #endif
-          set_add(tbl_all, ci);
-          if (!live) set_add(tbl_drop, ci);
+            set_add(tbl_all, ci);
+            if (!live) set_add(tbl_drop, ci);
+          }
           conf |= (int32_t)(raw[j] & kColorMask) == xv && lose<TB>(v, id[j]);
         }
         lvb |= live ? (1u << (kJB * bb + j)) : 0u;
@@ -1000,6 +1031,12 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
     }
     __syncwarp();
     const bool any = __any_sync(0xffffffffu, conf);
+    // this lane's 32-bit word of the chunk's color set / dropped set (colors [32 lane, +32))
+    auto set_word = [&](const uint8_t* tbl, uint64_t m) -> uint32_t {
+      if (!small) return tbl_bits32(tbl, lane);
+      const uint64_t w = warp_or64(m);
+      return lane == 0 ? (uint32_t)w : (lane == 1 ? (uint32_t)(w >> 32) : 0u);
+    };
     // live entries counted from the per-lane bits; the stage is compacted (in place, window
     // order, one ballot per 32 slots) only when the list is actually rewritten
     const uint32_t live_total = __reduce_add_sync(0xffffffffu, (uint32_t)__popc(lvb));
@@ -1030,12 +1067,12 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
     if (nch == 1) {
       if (any) {
         const uint32_t fo = cur.fo;
-        const uint32_t word = tbl_bits32(tbl_all, lane) | fo | (lane == 0 ? 1u : 0u);
+        const uint32_t word = set_word(tbl_all, mall) | fo | (lane == 0 ? 1u : 0u);
         int32_t tent = bits_first_free(word);
         if (tent < 0 || tent >= kBigTbl - 1) {  // beyond the exact range of the table
           tent = warp_first_fit_rescan<Persist>(a.col_idx, X, cur.s, cur.e, kBigTbl - 1, lane);
         }
-        const uint32_t drop = tbl_bits32(tbl_drop, lane);
+        const uint32_t drop = set_word(tbl_drop, mdrop);
         if (drop & ~fo) fx[lane] = fo | drop;
         // single chunk: the warp owns the whole list, so it is compacted in place, and not
         // rewritten at all when nothing was dropped (pass 2 read col_idx: always written)
@@ -1076,8 +1113,8 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
         if (any) atomicOr(a.acc_cnt + slot, 1ull);  // conflict flag (bit 0)
       }
       uint32_t* accb = a.acc_bits + (int64_t)slot * 32;
-      const uint32_t bits = tbl_bits32(tbl_all, lane);
-      const uint32_t drop = tbl_bits32(tbl_drop, lane);
+      const uint32_t bits = set_word(tbl_all, mall);
+      const uint32_t drop = set_word(tbl_drop, mdrop);
       if (bits) atomicOr(accb + lane, bits);
       if (drop) atomicOr(fx + lane, drop);
       if (!keep) {
@@ -1089,8 +1126,9 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
         a.fin[fpos] = (int64_t)(((uint64_t)(uint32_t)slot << 32) | (uint32_t)v |
                                 (cur.buf ? kBufBit : 0u) | (keep ? (1ull << 63) : 0ull));
     }
+    __syncwarp();  // every lane's table reads before the clear
 #if SGR_CLRMAX
-    {  // both sets, only the 16-byte groups up to the largest color set in this chunk
+    if (!small) {  // both sets, only the 16-byte groups up to the largest color set in this chunk
       const uint32_t nq = (__reduce_max_sync(0xffffffffu, cmax) >> 4) + 1;
       uint4* ta = reinterpret_cast<uint4*>(tbl_all);
       uint4* td = reinterpret_cast<uint4*>(tbl_drop);
@@ -1100,7 +1138,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
       }
     }
 #else
-    set_clear(tbl_all, kTblBytes, lane, 32);  // both sets
+    if (!small) set_clear(tbl_all, kTblBytes, lane, 32);  // both sets
 #endif
     __syncwarp();
 #if !SGR_NO_TMA
@@ -1269,6 +1307,8 @@ __device__ __forceinline__ void process_group(const RoundArgs<C>& a, int k, int3
   const int32_t* row = a.col_idx + s;
   const int32_t xv = v >= 0 ? ldc<Persist>(X + v) : 0;
   bool conf = false;
+  const bool small = SGR_SMALLMASK && k <= 62;  // uniform: colors of X are <= k < 64
+  uint64_t msk = 0;
   constexpr int B = Hub ? SGR_B1_BATCH_HUB : 8;  // entries per lane per batch
   const int32_t nb = (cnt + 8 * B - 1) / (8 * B);
   for (int32_t bb = 0; bb < nb; ++bb) {
@@ -1287,7 +1327,8 @@ __device__ __forceinline__ void process_group(const RoundArgs<C>& a, int k, int3
     for (int u = 0; u < B; ++u) {
       if (w[u] >= 0) {
         // deg <= 256 => first fit <= 257: colors >= 511 are clamped onto an unused byte
-        set_add(gtbl, (uint32_t)min(w[u], kMedTbl - 1));
+        if (small) msk |= 1ull << (w[u] & 63);
+        else set_add(gtbl, (uint32_t)min(w[u], kMedTbl - 1));
         conf |= w[u] == xv && ((lb >> u) & 1u);
       }
     }
@@ -1296,7 +1337,11 @@ __device__ __forceinline__ void process_group(const RoundArgs<C>& a, int k, int3
   __syncwarp();
   const bool any = (__ballot_sync(0xffffffffu, conf) & gmask) != 0u;
   int32_t tent = 0;
-  if (v >= 0 && any) {  // the group scans its table 32 bytes (8 words) per step
+  if (small) {  // OR the group's masks (xor butterfly inside the 8-lane group)
+#pragma unroll
+    for (int o = 4; o > 0; o >>= 1) msk |= __shfl_xor_sync(0xffffffffu, msk, o);
+    tent = __ffsll((long long)~(msk | 1ull)) - 1;  // bit c = color c; color 0 never free
+  } else if (v >= 0 && any) {  // the group scans its table 32 bytes (8 words) per step
     const uint32_t* t32 = reinterpret_cast<const uint32_t*>(gtbl);
 #if SGR_BITTBL
     {  // 512 bits = 16 words, two per lane of the group
@@ -1322,7 +1367,8 @@ __device__ __forceinline__ void process_group(const RoundArgs<C>& a, int k, int3
     }
 #endif
   }
-  set_clear(gtbl, kMedTblB, gl, kGroup);
+  __syncwarp();  // the group's table reads (first-fit scan) before any lane clears
+  if (!small) set_clear(gtbl, kMedTblB, gl, kGroup);
   __syncwarp();
   if (v >= 0 && gl == 0) put_y<C>(a, Y, k, v, any ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a));
   push = (v >= 0) && any && gl == 0;

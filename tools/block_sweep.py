@@ -24,6 +24,9 @@ from paper_conf_ipps_licqfsty16_b200 import gen  # noqa: E402
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--configs", type=int, nargs="+", default=[4, 1, 3, 7])
+    ap.add_argument("--topo-configs", type=int, nargs="+", default=[1, 3, 7],
+                    help="configs for the topology-driven sweep (T-base on cfg4 takes ~28 s "
+                         "per coloring: a hub row is one thread's serial loop)")
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--out", default=None)
     args = ap.parse_args()
@@ -34,6 +37,8 @@ def main():
         rp = torch.from_numpy(g.row_ptr).cuda()
         ci = torch.from_numpy(g.col_idx).cuda()
         for mapping in ("data-driven", "topology-driven"):
+            if mapping == "topology-driven" and cfg not in args.topo_configs:
+                continue
             fn = sgr.color if mapping == "data-driven" else sgr.color_topo
             ref = fn(rp, ci, "lowid").colors.clone()
             sizes = [64, 96, 128, 192, 256, 384, 512] if mapping == "data-driven" else \
@@ -60,6 +65,7 @@ def main():
                 print(json.dumps(rec), flush=True)
                 if out:
                     out.write(json.dumps(rec) + "\n")
+                    out.flush()
         del rp, ci
         torch.cuda.empty_cache()
 
