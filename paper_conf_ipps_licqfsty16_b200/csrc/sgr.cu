@@ -791,11 +791,12 @@ sgr_status sgr_color_gs(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t subs
   const int64_t K = partition == 2 ? 1 : substeps;
   cudaStream_t s = r.stream;
   keep_pool_memory();
-  // workspace: W[2] | T | flags | tiles | counters
+  // workspace: W[2] | T | flags | seg | tiles | counters | K counts / offsets / cursors
   const size_t nb = align_up((size_t)n * 4, 256);
   const int64_t tiles = (n + kCompactTile - 1) / kCompactTile;
+  const size_t kb = align_up((size_t)(K + 1) * 4, 256);
   char* ws = nullptr;
-  CK(cudaMallocAsync((void**)&ws, 4 * nb + align_up((size_t)tiles * 4, 256) + 256, s));
+  CK(cudaMallocAsync((void**)&ws, 5 * nb + align_up((size_t)tiles * 4, 256) + 256 + 3 * kb, s));
   int32_t* W[2] = {(int32_t*)ws, (int32_t*)(ws + nb)};
   int32_t* T = (int32_t*)(ws + 2 * nb);
   uint8_t* flags = (uint8_t*)(ws + 3 * nb);
@@ -803,6 +804,10 @@ sgr_status sgr_color_gs(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t subs
   char* tail = ws + 4 * nb + align_up((size_t)tiles * 4, 256);
   int64_t* dcount = (int64_t*)tail;
   unsigned long long* edges = (unsigned long long*)(tail + 64);
+  int32_t* seg = (int32_t*)(tail + 256);
+  int32_t* kcnt = (int32_t*)(tail + 256 + nb);
+  int32_t* koff = (int32_t*)(tail + 256 + nb + kb);
+  int32_t* kcur = (int32_t*)(tail + 256 + nb + 2 * kb);
   int64_t* hcnt = nullptr;
   CK(cudaMallocHost((void**)&hcnt, sizeof(int64_t)));
   cudaEvent_t e0, e1;
@@ -832,10 +837,18 @@ sgr_status sgr_color_gs(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t subs
       k_gs_inplace<<<gw, B, 0, s>>>(csr->row_ptr, csr->col_idx, W[cur], len, colors_out, edges);
       ++launches;
     } else {
+      // the round's members split once into K contiguous sub-step segments
+      const int gl = grid_for(len, B, B);
+      CK(cudaMemsetAsync(kcnt, 0, (size_t)K * 4, s));
+      k_gs_hist<<<gl, B, 0, s>>>(W[cur], len, n, K, partition, kcnt);
+      k_gs_scan<<<1, 32, 0, s>>>(kcnt, K, koff, kcur);
+      k_gs_scatter<<<gl, B, 0, s>>>(W[cur], len, n, K, partition, kcur, seg);
+      launches += 3;
+      const int gseg = grid_for((len + K - 1) / K, B, B);  // a sub-step's expected share
       for (int64_t j = 0; j < K; ++j) {  // sub-steps in order (Alg. 5 l.4-10 split K ways)
-        k_gs_assign<<<gw, B, 0, s>>>(csr->row_ptr, csr->col_idx, W[cur], len, n, K, partition, j,
-                                     colors_out, T, edges);
-        k_gs_commit<<<grid_for(len, B, B), B, 0, s>>>(W[cur], len, n, K, partition, j, T, colors_out);
+        k_gs_assign_seg<<<gseg, B, 0, s>>>(csr->row_ptr, csr->col_idx, seg, koff, j, colors_out, T,
+                                           edges);
+        k_gs_commit_seg<<<gseg, B, 0, s>>>(seg, koff, j, T, colors_out);
         launches += 2;
       }
     }

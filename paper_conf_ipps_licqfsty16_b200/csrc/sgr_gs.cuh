@@ -6,7 +6,7 @@
 // other threads of the same round already changed. Here that becomes
 // deterministic: a round's worklist is split by a fixed id partition into K sub-steps run
 // in order; sub-step j assigns its members against the colors left by sub-steps < j
-// (Jacobi within the sub-step: k_gs_assign reads C, k_gs_commit writes it afterwards).
+// (Jacobi within the sub-step: k_gs_assign_seg reads C, k_gs_commit_seg writes it after).
 // Detection and compaction after the K sub-steps reuse the step kernels (Alg. 5 l.12-15).
 // Partition 2 is the paper-faithful nondeterministic mode: one in-place sub-step whose
 // first fits read C while other warps write it (only properness and color counts are
@@ -23,44 +23,6 @@ namespace sgr {
 __device__ __forceinline__ int64_t gs_part(int64_t v, int64_t n, int64_t K, int partition) {
   return partition == 1 ? (int64_t)(((unsigned __int128)v * (unsigned long long)K) / (unsigned long long)n)
                         : v % K;
-}
-
-// Sub-step j of a round: T[i] = first fit of wl[i] against C for the members of part j
-// (one warp per listed vertex; C is not written while this kernel runs). Sum of degrees of
-// the members into *edges (one atomic per block).
-static __global__ void __launch_bounds__(1024) k_gs_assign(const int64_t* __restrict__ row_ptr,
-                                                           const int32_t* __restrict__ col_idx,
-                                                           const int32_t* __restrict__ wl, int64_t len,
-                                                           int64_t n, int64_t K, int partition,
-                                                           int64_t j, const int32_t* __restrict__ C,
-                                                           int32_t* __restrict__ T,
-                                                           unsigned long long* edges) {
-  const int lane = threadIdx.x & 31;
-  const int64_t wpb = blockDim.x >> 5;
-  unsigned long long my = 0;
-  for (int64_t i = (int64_t)blockIdx.x * wpb + (threadIdx.x >> 5); i < len;
-       i += (int64_t)gridDim.x * wpb) {
-    const int32_t v = __ldg(wl + i);
-    if (gs_part(v, n, K, partition) != j) continue;  // warp-uniform
-    const int64_t s = ld_ro(row_ptr + v), e = ld_ro(row_ptr + v + 1);
-    const int32_t t = warp_first_fit_from<false>(col_idx, C, s, e, 0, lane);
-    if (lane == 0) {
-      T[i] = t;
-      my += (unsigned long long)(e - s);
-    }
-  }
-  block_add(my, edges);
-}
-
-// Sub-step j's writes become visible to the next sub-step: C[wl[i]] = T[i] for part j.
-static __global__ void k_gs_commit(const int32_t* __restrict__ wl, int64_t len, int64_t n, int64_t K,
-                                   int partition, int64_t j, const int32_t* __restrict__ T,
-                                   int32_t* __restrict__ C) {
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < len;
-       i += (int64_t)gridDim.x * blockDim.x) {
-    const int32_t v = wl[i];
-    if (gs_part(v, n, K, partition) == j) C[v] = T[i];
-  }
 }
 
 // Paper-faithful in-place assignment (nondeterministic): one warp per listed vertex reads
@@ -84,6 +46,94 @@ static __global__ void __launch_bounds__(1024) k_gs_inplace(const int64_t* __res
     }
   }
   block_add(my, edges);
+}
+
+// ---- bucketed sub-steps: each round's worklist is split once into its K sub-step
+// segments (a histogram, an exclusive scan and a scatter), so a sub-step touches only its
+// own members; low-degree members take their first fit one thread each, the others one warp.
+static __global__ void k_gs_hist(const int32_t* __restrict__ wl, int64_t len, int64_t n, int64_t K,
+                                 int partition, int32_t* __restrict__ cnt) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < len;
+       i += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(cnt + gs_part(wl[i], n, K, partition), 1);
+}
+
+// Exclusive scan of the K counts (one block; K <= a few thousand), cnt -> off[0..K], and
+// the scatter cursors reset to the offsets.
+static __global__ void k_gs_scan(const int32_t* __restrict__ cnt, int64_t K, int32_t* __restrict__ off,
+                                 int32_t* __restrict__ cur) {
+  if (threadIdx.x == 0) {
+    int32_t run = 0;
+    for (int64_t j = 0; j < K; ++j) {
+      off[j] = run;
+      cur[j] = run;
+      run += cnt[j];
+    }
+    off[K] = run;
+  }
+}
+
+static __global__ void k_gs_scatter(const int32_t* __restrict__ wl, int64_t len, int64_t n, int64_t K,
+                                    int partition, int32_t* __restrict__ cur, int32_t* __restrict__ seg) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < len;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t v = wl[i];
+    seg[atomicAdd(cur + gs_part(v, n, K, partition), 1)] = v;
+  }
+}
+
+// Sub-step j over its segment seg[off[j] .. off[j+1]): T[i] = first fit against C. Lane L of
+// a warp takes entry 32 w + L; members of degree <= 64 are done by their own thread (64-color
+// register windows, rescanning the row per window), larger ones by the whole warp in turn.
+static __global__ void __launch_bounds__(1024) k_gs_assign_seg(const int64_t* __restrict__ row_ptr,
+                                                               const int32_t* __restrict__ col_idx,
+                                                               const int32_t* __restrict__ seg,
+                                                               const int32_t* __restrict__ off, int64_t j,
+                                                               const int32_t* __restrict__ C,
+                                                               int32_t* __restrict__ T,
+                                                               unsigned long long* edges) {
+  const int lane = threadIdx.x & 31;
+  const int64_t b = __ldg(off + j), e_ = __ldg(off + j + 1);
+  const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);
+  unsigned long long my = 0;
+  for (int64_t base = b + (((int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) << 5); base < e_;
+       base += nw << 5) {
+    const int64_t i = base + lane;
+    const bool ok = i < e_;
+    const int32_t v = ok ? __ldg(seg + i) : 0;
+    const int64_t s = ok ? ld_ro(row_ptr + v) : 0, e = ok ? ld_ro(row_ptr + v + 1) : 0;
+    const bool small = ok && e - s <= 64;
+    if (small) {
+      int32_t t = 0;
+      for (int32_t wb = 0; t == 0; wb += 64) {  // colors (wb, wb + 64]
+        uint64_t m = 0;
+        for (int64_t q = s; q < e; ++q) {
+          const uint32_t idx = (uint32_t)(__ldg(C + ld_ro(col_idx + q)) - wb - 1);
+          if (idx < 64u) m |= 1ull << idx;
+        }
+        if (~m) t = wb + __ffsll((long long)~m);
+      }
+      T[i] = t;
+    }
+    if (ok) my += (unsigned long long)(e - s);
+    unsigned big = __ballot_sync(0xffffffffu, ok && !small);
+    while (big) {
+      const int l = __ffs(big) - 1;
+      big &= big - 1u;
+      const int64_t sl = __shfl_sync(0xffffffffu, s, l), el = __shfl_sync(0xffffffffu, e, l);
+      const int32_t t = warp_first_fit_from<false>(col_idx, C, sl, el, 0, lane);
+      if (lane == l) T[i] = t;
+    }
+  }
+  block_add(my, edges);
+}
+
+static __global__ void k_gs_commit_seg(const int32_t* __restrict__ seg, const int32_t* __restrict__ off,
+                                       int64_t j, const int32_t* __restrict__ T, int32_t* __restrict__ C) {
+  const int64_t b = __ldg(off + j), e = __ldg(off + j + 1);
+  for (int64_t i = b + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < e;
+       i += (int64_t)gridDim.x * blockDim.x)
+    C[seg[i]] = T[i];
 }
 
 static __global__ void k_gs_init(int64_t n, int32_t* __restrict__ wl, int32_t* __restrict__ C) {
