@@ -90,6 +90,23 @@ Resolved resolve_opts(const sgr_opts* o, int64_t n) {
   return r;
 }
 
+// Bytes of the L2 persisting carve-out for the color buffers (0: off). Experiment switch
+// SGR_L2PERSIST=1, read once per process; sets the device's persisting-L2 limit once.
+static size_t l2_persist_bytes() {
+  static size_t bytes = [] {
+    const char* e = getenv("SGR_L2PERSIST");
+    if (!(e && e[0] == '1')) return (size_t)0;
+    int dev = 0, mx = 0, win = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&mx, cudaDevAttrMaxPersistingL2CacheSize, dev);
+    cudaDeviceGetAttribute(&win, cudaDevAttrMaxAccessPolicyWindowSize, dev);
+    if (mx <= 0 || win <= 0) return (size_t)0;
+    cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)mx);
+    return (size_t)std::min(mx, win);
+  }();
+  return bytes;
+}
+
 // opts->block_size: a multiple of 32 within [lo, hi] (sgr.h).
 bool block_ok(int B, int lo, int hi) { return B % 32 == 0 && B >= lo && B <= hi; }
 
@@ -300,12 +317,37 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
     if (persistent) {
       // both builds are enqueued; the one that does not match F_1's bins returns at once
       prof.timed(SGR_K_ROUND, s, [&] {
-        void* args[] = {(void*)&a};
-        le = cudaLaunchCooperativeKernel((const void*)k_persistent<TB, C, true>, grid, B,
-                                         args, round_smem<C, true>(B), s);
-        if (le == cudaSuccess)
-          le = cudaLaunchCooperativeKernel((const void*)k_persistent<TB, C, false>, grid_flat,
-                                           B, args, round_smem<C, false>(B), s);
+        // cooperative launches; optionally with an L2 persisting window over the two color
+        // buffers (SGR_L2PERSIST=1, experiment: the gathers' working set kept resident
+        // against the streaming lists)
+        cudaLaunchAttribute at[2];
+        at[0].id = cudaLaunchAttributeCooperative;
+        at[0].val.cooperative = 1;
+        int nat = 1;
+        // packed: both color buffers are adjacent in the workspace; plain: the workspace one
+        const size_t colb = packed<C>() ? 2 * align_up((size_t)n * sizeof(C), 256) : (size_t)n * 4;
+        if (l2_persist_bytes() > 0) {
+          at[1].id = cudaLaunchAttributeAccessPolicyWindow;
+          at[1].val.accessPolicyWindow.base_ptr = (void*)a.col[packed<C>() ? 0 : 1];
+          at[1].val.accessPolicyWindow.num_bytes = std::min(colb, l2_persist_bytes());
+          at[1].val.accessPolicyWindow.hitRatio = 1.0f;
+          at[1].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+          at[1].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+          nat = 2;
+        }
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3(grid);
+        cfg.blockDim = dim3(B);
+        cfg.dynamicSmemBytes = round_smem<C, true>(B);
+        cfg.stream = s;
+        cfg.attrs = at;
+        cfg.numAttrs = nat;
+        le = cudaLaunchKernelEx(&cfg, k_persistent<TB, C, true>, a);
+        if (le == cudaSuccess) {
+          cfg.gridDim = dim3(grid_flat);
+          cfg.dynamicSmemBytes = round_smem<C, false>(B);
+          le = cudaLaunchKernelEx(&cfg, k_persistent<TB, C, false>, a);
+        }
       });
       launches += 2;
       if (le != cudaSuccess) {

@@ -45,7 +45,8 @@ for cfg in args.configs:
     rp = torch.from_numpy(g.row_ptr).cuda()
     ci = torch.from_numpy(g.col_idx).cuda()
     base_ms, base = timed(lambda: sgr.color(rp, ci))
-    rows = [{"config": gen.CONFIG_NAMES[cfg], "path": "sgr_color (single part)", "ms": base_ms}]
+    rows = [{"config": gen.CONFIG_NAMES[cfg], "path": "sgr_color (single part)", "ms": base_ms,
+             "rounds_ms": base.stats["elapsed_ms"]}]
     for P in args.parts:
         ranges = sgr.partition(g.row_ptr, P)
         for tr in ("device", "hostloop"):
@@ -54,8 +55,10 @@ for cfg in args.configs:
             else:
                 os.environ.pop("SGR_DIST_HOSTLOOP", None)
             ms, r = timed(lambda: sgr.color_partitioned(rp, ci, P, ranges=ranges))
+            # ms: the whole call (host-side split of the CSR into local rows, allocations,
+            # F_1, rounds); rounds_ms: device time of the rounds (library CUDA events)
             rows.append({"config": gen.CONFIG_NAMES[cfg], "path": f"partitioned P={P} {tr}",
-                         "ms": ms, "transport": r.stats["transport"],
+                         "ms": ms, "rounds_ms": r.stats["elapsed_ms"], "transport": r.stats["transport"],
                          "bit_exact_vs_sgr_color": bool(torch.equal(r.colors, base.colors)),
                          "rounds": r.stats["rounds"]})
     os.environ.pop("SGR_DIST_HOSTLOOP", None)
