@@ -838,7 +838,7 @@ sgr_status sgr_color_gs(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t subs
   const int64_t tiles = (n + kCompactTile - 1) / kCompactTile;
   const size_t kb = align_up((size_t)(K + 1) * 4, 256);
   char* ws = nullptr;
-  CK(cudaMallocAsync((void**)&ws, 5 * nb + align_up((size_t)tiles * 4, 256) + 256 + 3 * kb, s));
+  CK(cudaMallocAsync((void**)&ws, 6 * nb + align_up((size_t)tiles * 4, 256) + 256 + 4 * kb, s));
   int32_t* W[2] = {(int32_t*)ws, (int32_t*)(ws + nb)};
   int32_t* T = (int32_t*)(ws + 2 * nb);
   uint8_t* flags = (uint8_t*)(ws + 3 * nb);
@@ -850,6 +850,8 @@ sgr_status sgr_color_gs(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t subs
   int32_t* kcnt = (int32_t*)(tail + 256 + nb);
   int32_t* koff = (int32_t*)(tail + 256 + nb + kb);
   int32_t* kcur = (int32_t*)(tail + 256 + nb + 2 * kb);
+  int32_t* kbig = (int32_t*)(tail + 256 + nb + 3 * kb);  // per sub-step: members of degree > 64
+  int32_t* bigl = (int32_t*)(tail + 256 + nb + 4 * kb);
   int64_t* hcnt = nullptr;
   CK(cudaMallocHost((void**)&hcnt, sizeof(int64_t)));
   cudaEvent_t e0, e1;
@@ -882,16 +884,22 @@ sgr_status sgr_color_gs(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t subs
       // the round's members split once into K contiguous sub-step segments
       const int gl = grid_for(len, B, B);
       CK(cudaMemsetAsync(kcnt, 0, (size_t)K * 4, s));
+      CK(cudaMemsetAsync(kbig, 0, (size_t)K * 4, s));
       k_gs_hist<<<gl, B, 0, s>>>(W[cur], len, n, K, partition, kcnt);
       k_gs_scan<<<1, 32, 0, s>>>(kcnt, K, koff, kcur);
       k_gs_scatter<<<gl, B, 0, s>>>(W[cur], len, n, K, partition, kcur, seg);
       launches += 3;
-      const int gseg = grid_for((len + K - 1) / K, B, B);  // a sub-step's expected share
+      // a sub-step's share is unknown on the host: size for the whole round (blocks past
+      // the segment exit at once); the big members get one warp each, at least a wave
+      const int gseg = std::max(grid_for(len, B, B), num_sms());
+      const int gbig = num_sms() * 8 * 256 / B;
       for (int64_t j = 0; j < K; ++j) {  // sub-steps in order (Alg. 5 l.4-10 split K ways)
         k_gs_assign_seg<<<gseg, B, 0, s>>>(csr->row_ptr, csr->col_idx, seg, koff, j, colors_out, T,
-                                           edges);
+                                           bigl, kbig + j, edges);
+        k_gs_assign_big<<<gbig, B, 0, s>>>(csr->row_ptr, csr->col_idx, seg, bigl, kbig + j, colors_out,
+                                           T, edges);
         k_gs_commit_seg<<<gseg, B, 0, s>>>(seg, koff, j, T, colors_out);
-        launches += 2;
+        launches += 3;
       }
     }
     // Alg. 5 l.12-15 over W_r, then the order-preserving compaction

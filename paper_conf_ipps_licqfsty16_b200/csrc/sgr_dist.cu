@@ -404,12 +404,12 @@ struct PeerView {         // multi-GPU: the other ranks' workspaces (IPC-mapped)
 };
 using XSync = std::function<sgr_status(cudaStream_t, int32_t* dflag, int op_max)>;
 
-template <int TB, class C, bool Hub>
+template <int TB, class C, bool Hub, bool Multi>
 static int dist_grid(int B) {
   const int smax = (int)round_smem<C, Hub>(round_max_block<C, Hub>());
-  cudaFuncSetAttribute(k_persistent_dist<TB, C, Hub>, cudaFuncAttributeMaxDynamicSharedMemorySize, smax);
+  cudaFuncSetAttribute(k_persistent_dist<TB, C, Hub, Multi>, cudaFuncAttributeMaxDynamicSharedMemorySize, smax);
   int per_sm = 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_persistent_dist<TB, C, Hub>, B,
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_persistent_dist<TB, C, Hub, Multi>, B,
                                                     round_smem<C, Hub>(B)) != cudaSuccess ||
       per_sm <= 0)
     per_sm = 1;
@@ -526,7 +526,9 @@ static sgr_status run_dev(std::vector<DevPart>& parts, int nranks, int me0, int6
     DCK(cudaMemcpyAsync(&hub, dflag, 4, cudaMemcpyDeviceToHost, s));
     DCK(cudaStreamSynchronize(s));
   }
-  const int gmax = hub ? dist_grid<TB, C, true>(B) : dist_grid<TB, C, false>(B);
+  const bool multi = P > 1;
+  const int gmax = hub ? (multi ? dist_grid<TB, C, true, true>(B) : dist_grid<TB, C, true, false>(B))
+                       : (multi ? dist_grid<TB, C, false, true>(B) : dist_grid<TB, C, false, false>(B));
   const int gB = std::max(1, gmax / P);  // blocks per part
   const int grid = gB * P;
   for (int i = 0; i < P; ++i) {
@@ -539,14 +541,16 @@ static sgr_status run_dev(std::vector<DevPart>& parts, int nranks, int me0, int6
   cudaEventCreate(&ev1);
   cudaEventRecord(ev0, s);
   {
+    RoundArgs<C> a0 = args[0];
     const RoundArgs<C>* pa = dargs;
     int np = P;
-    void* kargs[] = {(void*)&pa, (void*)&np};
-    const cudaError_t le = hub
-        ? cudaLaunchCooperativeKernel((const void*)k_persistent_dist<TB, C, true>, grid, B, kargs,
-                                      round_smem<C, true>(B), s)
-        : cudaLaunchCooperativeKernel((const void*)k_persistent_dist<TB, C, false>, grid, B, kargs,
-                                      round_smem<C, false>(B), s);
+    void* kargs[] = {(void*)&a0, (void*)&pa, (void*)&np};
+    const void* fn = hub ? (multi ? (const void*)k_persistent_dist<TB, C, true, true>
+                                  : (const void*)k_persistent_dist<TB, C, true, false>)
+                         : (multi ? (const void*)k_persistent_dist<TB, C, false, true>
+                                  : (const void*)k_persistent_dist<TB, C, false, false>);
+    const cudaError_t le = cudaLaunchCooperativeKernel(fn, grid, B, kargs,
+                                                       hub ? round_smem<C, true>(B) : round_smem<C, false>(B), s);
     if (le != cudaSuccess) return cuda_fail(le, "cooperative launch of k_persistent_dist", __LINE__);
   }
   cudaEventRecord(ev1, s);

@@ -83,14 +83,17 @@ static __global__ void k_gs_scatter(const int32_t* __restrict__ wl, int64_t len,
 }
 
 // Sub-step j over its segment seg[off[j] .. off[j+1]): T[i] = first fit against C. Lane L of
-// a warp takes entry 32 w + L; members of degree <= 64 are done by their own thread (64-color
-// register windows, rescanning the row per window), larger ones by the whole warp in turn.
+// a warp takes entry 32 w + L; a member of degree <= 64 is done by its own thread (64-color
+// register windows, rescanning the row per window); larger ones are appended to big[] (one
+// atomic per warp) for k_gs_assign_big, one warp each.
 static __global__ void __launch_bounds__(1024) k_gs_assign_seg(const int64_t* __restrict__ row_ptr,
                                                                const int32_t* __restrict__ col_idx,
                                                                const int32_t* __restrict__ seg,
                                                                const int32_t* __restrict__ off, int64_t j,
                                                                const int32_t* __restrict__ C,
                                                                int32_t* __restrict__ T,
+                                                               int32_t* __restrict__ big,
+                                                               int32_t* __restrict__ nbig,
                                                                unsigned long long* edges) {
   const int lane = threadIdx.x & 31;
   const int64_t b = __ldg(off + j), e_ = __ldg(off + j + 1);
@@ -114,15 +117,40 @@ static __global__ void __launch_bounds__(1024) k_gs_assign_seg(const int64_t* __
         if (~m) t = wb + __ffsll((long long)~m);
       }
       T[i] = t;
+      my += (unsigned long long)(e - s);
     }
-    if (ok) my += (unsigned long long)(e - s);
-    unsigned big = __ballot_sync(0xffffffffu, ok && !small);
-    while (big) {
-      const int l = __ffs(big) - 1;
-      big &= big - 1u;
-      const int64_t sl = __shfl_sync(0xffffffffu, s, l), el = __shfl_sync(0xffffffffu, e, l);
-      const int32_t t = warp_first_fit_from<false>(col_idx, C, sl, el, 0, lane);
-      if (lane == l) T[i] = t;
+    const unsigned bm = __ballot_sync(0xffffffffu, ok && !small);
+    if (bm) {
+      int o = 0;
+      if (lane == 0) o = atomicAdd(nbig, __popc(bm));
+      o = __shfl_sync(0xffffffffu, o, 0);
+      if (ok && !small) big[o + __popc(bm & ((1u << lane) - 1u))] = (int32_t)i;
+    }
+  }
+  block_add(my, edges);
+}
+
+// The sub-step's members of degree > 64 (positions in seg), one warp each.
+static __global__ void __launch_bounds__(1024) k_gs_assign_big(const int64_t* __restrict__ row_ptr,
+                                                               const int32_t* __restrict__ col_idx,
+                                                               const int32_t* __restrict__ seg,
+                                                               const int32_t* __restrict__ big,
+                                                               const int32_t* __restrict__ nbig,
+                                                               const int32_t* __restrict__ C,
+                                                               int32_t* __restrict__ T,
+                                                               unsigned long long* edges) {
+  const int lane = threadIdx.x & 31;
+  const int64_t wpb = blockDim.x >> 5;
+  const int64_t cnt = __ldg(nbig);
+  unsigned long long my = 0;
+  for (int64_t q = (int64_t)blockIdx.x * wpb + (threadIdx.x >> 5); q < cnt; q += (int64_t)gridDim.x * wpb) {
+    const int32_t i = __ldg(big + q);
+    const int32_t v = __ldg(seg + i);
+    const int64_t s = ld_ro(row_ptr + v), e = ld_ro(row_ptr + v + 1);
+    const int32_t t = warp_first_fit_from<false>(col_idx, C, s, e, 0, lane);
+    if (lane == 0) {
+      T[i] = t;
+      my += (unsigned long long)(e - s);
     }
   }
   block_add(my, edges);

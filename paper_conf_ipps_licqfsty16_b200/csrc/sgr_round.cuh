@@ -2320,12 +2320,7 @@ __device__ __forceinline__ GlobalCounts global_counts(const RoundArgs<C>& a, int
 }
 
 template <int TB, class C, bool Hub>
-__global__ void __launch_bounds__(kMaxThreads<C, Hub>, 1) k_persistent_dist(const RoundArgs<C>* __restrict__ parts,
-                                                                        int nparts) {
-  extern __shared__ __align__(16) uint8_t dsmem[];
-  const int gB = (int)gridDim.x / nparts;
-  const int p = min((int)blockIdx.x / gB, nparts - 1);
-  const RoundArgs<C> a = parts[p];
+__device__ __forceinline__ void dist_body(const RoundArgs<C>& a, uint8_t* dsmem) {
   Ctrl* ctrl = a.ctrl;
   uint8_t* wsm = warp_smem_init<C, Hub>(dsmem);
   uint32_t ph = 0;
@@ -2360,6 +2355,26 @@ __global__ void __launch_bounds__(kMaxThreads<C, Hub>, 1) k_persistent_dist(cons
       if constexpr (packed<C>() && Hub) finalize_body<TB, true>(a, k);
     }
     part_sync(a, epoch, xepoch);
+  }
+}
+
+// Multi = false: one part per launch (each GPU of a multi-GPU coloring, or one partition):
+// its arguments stay kernel parameters. Multi = true: `nparts` block groups on this device,
+// each block copying its part's arguments from `parts`.
+template <int TB, class C, bool Hub, bool Multi>
+__global__ void __launch_bounds__(kMaxThreads<C, Hub>, 1) k_persistent_dist(RoundArgs<C> a0,
+                                                                        const RoundArgs<C>* __restrict__ parts,
+                                                                        int nparts) {
+  extern __shared__ __align__(16) uint8_t dsmem[];
+  if constexpr (Multi) {
+    const int gB = (int)gridDim.x / nparts;
+    const int p = min((int)blockIdx.x / gB, nparts - 1);
+    const RoundArgs<C> a = parts[p];
+    dist_body<TB, C, Hub>(a, dsmem);
+  } else {
+    (void)parts;
+    (void)nparts;
+    dist_body<TB, C, Hub>(a0, dsmem);
   }
 }
 
