@@ -41,7 +41,6 @@
 // are in flight.
 // Worklist pushes: warp ballot + popc + one atomicAdd per warp.
 #pragma once
-#include <climits>
 #include <cstdint>
 #include <cuda_runtime.h>
 
@@ -88,9 +87,6 @@ constexpr int kJB = 4 * kQB;  // entries per lane per batch
 #endif
 #ifndef SGR_BIN0_THREAD
 #define SGR_BIN0_THREAD 0  // bin 0: one thread per vertex (else 4-lane groups)
-#endif
-#ifndef SGR_B0_STAGE
-#define SGR_B0_STAGE 1  // flat build, bin 0: a step's 8 rows read as one coalesced segment
 #endif
 
 namespace sgr {
@@ -1534,61 +1530,6 @@ __device__ __forceinline__ void bin0_tiled(const RoundArgs<C>& a, int k, const i
     for (int u = 0; u < kK0; ++u) w[u] = (gl + G * u < cnt) ? ld_row_h<Hub>(row + gl + G * u) : -1;
   };
   (void)step;
-  // SGR_B0_STAGE: the step's 8 rows usually lie in one short stretch of col_idx (stencils, and
-  // early rounds of graphs whose worklists are nearly V in id order): load its 16-byte-aligned
-  // window with two coalesced int4 loads per lane, issued while the current step's gathers
-  // are in flight, then hand every lane its entries through the warp's (otherwise unused in
-  // bin 0) shared table area; rows spread wider than the stage take the per-lane loads.
-  constexpr int kStageE = 256;  // entries: 8 rows of <= 32, window alignment included
-  int32_t* stage = reinterpret_cast<int32_t*>(wsm + WarpSmem<C, Hub>::kBuf);
-  static_assert(kStageE * 4 <= kTblBytes, "bin-0 stage fits the warp's tables");
-  int4 q0 = make_int4(0, 0, 0, 0), q1 = make_int4(0, 0, 0, 0);
-  int64_t sg0 = 0;
-  bool staged = false;  // warp-uniform
-  auto span_of = [&](int64_t ss, int64_t ee, bool has) {  // warp-wide [min s, max e)
-    long long lo = has ? ss : LLONG_MAX, hi = has ? ee : LLONG_MIN;
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-      lo = min(lo, (long long)__shfl_xor_sync(0xffffffffu, lo, o));
-      hi = max(hi, (long long)__shfl_xor_sync(0xffffffffu, hi, o));
-    }
-    return make_longlong2(lo, hi);
-  };
-  auto stage_issue = [&](int64_t ss, int64_t ee, bool has) {  // global int4 loads in flight
-    const longlong2 sp = span_of(ss, ee, has);
-    staged = false;
-    if (SGR_B0_STAGE && !Hub && sp.x <= sp.y && sp.y - (sp.x & ~3ll) <= kStageE) {
-      staged = true;
-      sg0 = sp.x & ~3ll;
-      const int64_t nq = (sp.y - sg0 + 3) >> 2;
-      auto ld4 = [&](int64_t qi) -> int4 {
-        const int64_t p0 = sg0 + 4 * qi;
-        if (qi >= nq) return make_int4(0, 0, 0, 0);
-        if (p0 + 4 <= a.nnz) return ld_ro(reinterpret_cast<const int4*>(a.col_idx + p0));
-        int4 t = make_int4(0, 0, 0, 0);  // the array's last partial group: never past nnz
-        t.x = ld_ro(a.col_idx + p0);
-        if (p0 + 1 < a.nnz) t.y = ld_ro(a.col_idx + p0 + 1);
-        if (p0 + 2 < a.nnz) t.z = ld_ro(a.col_idx + p0 + 2);
-        return t;
-      };
-      q0 = ld4(lane);
-      q1 = ld4(lane + 32);
-    }
-  };
-  auto stage_take = [&](int32_t vv, int64_t ss, int64_t ee, int32_t (&w)[kK0]) {
-    if (!staged) {
-      load_row(vv, ss, ee, w);
-      return;
-    }
-    __syncwarp();  // the previous step's reads of the stage are done
-    reinterpret_cast<int4*>(stage)[lane] = q0;
-    reinterpret_cast<int4*>(stage)[lane + 32] = q1;
-    __syncwarp();
-    const int32_t cnt = vv >= 0 ? (int32_t)(ee - ss) : 0;
-    const int32_t o = (int32_t)(ss - sg0);
-#pragma unroll
-    for (int u = 0; u < kK0; ++u) w[u] = (gl + G * u < cnt) ? stage[o + gl + G * u] : -1;
-  };
   StepStream<VPW> gen;  // runs two steps ahead of the step being processed
   gen.init(gw, NW, nX, kTile0, tile_cursor, lane);
   auto pos = [&](int b) { return b < nX ? b + g : nX; };
@@ -1614,7 +1555,7 @@ __device__ __forceinline__ void bin0_tiled(const RoundArgs<C>& a, int k, const i
 #pragma unroll
     for (int u = 0; u < kK0; ++u) c[u] = (w[u] >= 0) ? ldc01<Persist, Hub>(X + w[u]) : 0;
     int32_t wn[kK0];
-    stage_issue(s1, e1, v1 >= 0);  // next step's rows, in flight with the gathers above
+    load_row(v1, s1, e1, wn);  // next vertex's row, in flight with the gathers above
     bool conf = false;
     uint32_t mask = 0;  // bit i = color i + 1 present (deg <= 32 => first fit <= 33)
 #pragma unroll
@@ -1632,7 +1573,6 @@ __device__ __forceinline__ void bin0_tiled(const RoundArgs<C>& a, int k, const i
       entries += (unsigned long long)(e - s);
     }
     push_buffered<kPushBufOf<Hub>>(v >= 0 && any && gl == 0, v, pbuf, pending, out, out_cnt, lane);
-    stage_take(v1, s1, e1, wn);
     const int64_t s2 = v2 >= 0 ? ldg_i64(a.row_ptr + v2) : 0;
     const int64_t e2 = v2 >= 0 ? ldg_i64(a.row_ptr + v2 + 1) : 0;
     b0 = b1;
@@ -1647,12 +1587,6 @@ __device__ __forceinline__ void bin0_tiled(const RoundArgs<C>& a, int k, const i
     e1 = e2;
   }
   push_flush(pbuf, pending, out, out_cnt, lane);
-  if (SGR_B0_STAGE && !Hub) {  // bin 1 of the next pass expects zeroed tables
-    __syncwarp();
-    reinterpret_cast<int4*>(stage)[lane] = make_int4(0, 0, 0, 0);
-    reinterpret_cast<int4*>(stage)[lane + 32] = make_int4(0, 0, 0, 0);
-    __syncwarp();
-  }
 }
 
 // Bin 0, one thread per vertex (SGR_BIN0_THREAD): lane L of the warp takes list position
