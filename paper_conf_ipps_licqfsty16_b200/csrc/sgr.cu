@@ -1,6 +1,7 @@
 // sgr.cu — host side of libsgr.so: the C ABI of include/sgr.h (single GPU + step entry
 // points). Multi-GPU lives in sgr_dist.cu. DESIGN.md §5 describes the round loop.
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include <cstdarg>
 #include <cstdio>
@@ -177,6 +178,17 @@ static sgr_status get_graph(const RoundArgs<C>& a, int grid, int B, int batch, c
   return SGR_OK;
 }
 
+// NVTX range for the scope (balanced on every exit path).
+struct NvtxRange {
+  bool open = true;
+  explicit NvtxRange(const char* m) { nvtxRangePushA(m); }
+  void end() {
+    if (open) nvtxRangePop();
+    open = false;
+  }
+  ~NvtxRange() { end(); }
+};
+
 // ----- profiling (opts->profile): CUDA events around launches ------------------------------
 struct Prof {
   bool on = false;
@@ -305,8 +317,13 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
     cudaEventCreate(&ev1);
     cudaEventRecord(ev0, s);
 
-    prof.timed(SGR_K_FIRST, s, [&] { k_first<TB, C><<<first_grid(n, B), B, 0, s>>>(a, r.sorted); });
-    prof.timed(SGR_K_CTRL, s, [&] { k_advance<<<1, 32, 0, s>>>(a.ctrl, 1); });
+    // NVTX ranges (SURVEY §5 tracing): host-side enqueue phases, visible to ncu
+    // (--nvtx --nvtx-include) and nsys; one range per round batch in the host/graph loops
+    {
+      NvtxRange nr("sgr F1");
+      prof.timed(SGR_K_FIRST, s, [&] { k_first<TB, C><<<first_grid(n, B), B, 0, s>>>(a, r.sorted); });
+      prof.timed(SGR_K_CTRL, s, [&] { k_advance<<<1, 32, 0, s>>>(a.ctrl, 1); });
+    }
     launches += 2;
     le = cudaGetLastError();
     if (le != cudaSuccess) {
@@ -314,6 +331,7 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
       break;
     }
 
+    NvtxRange nr_rounds(persistent ? "sgr rounds (persistent)" : "sgr rounds (host loop)");
     if (persistent) {
       // both builds are enqueued; the one that does not match F_1's bins returns at once
       prof.timed(SGR_K_ROUND, s, [&] {
@@ -371,6 +389,7 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
       int64_t batches = 0;
       bool finished = status != SGR_OK;
       while (!finished) {
+        NvtxRange nr_batch("sgr round batch");
         if (use_graph) {
           le = cudaGraphLaunch(gexec, s);
         } else {
@@ -402,6 +421,7 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
       if (status != SGR_OK) break;
     }
 
+    nr_rounds.end();
     prof.timed(SGR_K_FINAL, s, [&] {
       if constexpr (packed<C>())
         k_unpack<<<reduce_grid(n, B), B, 0, s>>>(a.col[0], colors_out, n, &a.ctrl->max_color);

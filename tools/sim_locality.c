@@ -58,6 +58,7 @@ int main(int argc, char** argv) {
   for (int64_t i = 0; i < wl; ++i) { Y[W[i]] = 2; inW[W[i]] = 1; }
   int64_t S = 0; /* epoch size */
   double tot_g[3] = {0}, tot_lo[3] = {0}, tot_ld[3] = {0}, tot_skip[3] = {0};
+  double hot[4] = {0};  /* bin-2 gathers with id < 2^12, 2^14, 2^16, 2^18 */
   printf("k |W| | g0 l0 | g1 l1 live1 | g2 l2orig l2dense | epoch\n");
   for (int k = 2; wl > 0; ++k) {
     /* snapshot X = C_k */
@@ -71,7 +72,8 @@ int main(int argc, char** argv) {
     double g[3] = {0}, lo[3] = {0}, ld[3] = {0}, skip[3] = {0};
     /* bins 0/1: instruction groups over the ascending worklist */
     int64_t nw2 = 0;
-#pragma omp parallel for schedule(dynamic, 4096) reduction(+ : g[:3], lo[:3], ld[:3], skip[:3])
+    double hotl[4] = {0};
+#pragma omp parallel for schedule(dynamic, 4096) reduction(+ : g[:3], lo[:3], ld[:3], skip[:3], hotl[:4])
     for (int64_t i = 0; i < wl; ++i) {
       const int32_t v = W[i];
       const int64_t d = R[v + 1] - R[v];
@@ -94,6 +96,7 @@ int main(int argc, char** argv) {
         for (int64_t j = R[v]; j < R[v + 1]; ++j) {
           const int32_t w = C[j];
           if (!inW[w]) continue;
+          for (int h = 0; h < 4; ++h) hotl[h] += w < (1 << (12 + 2 * h)) ? 1 : 0;
           a[m] = (uint32_t)w >> shift;
           b[m] = (uint32_t)rank[w] >> shift;
           if (++m == 32) {
@@ -166,12 +169,15 @@ int main(int argc, char** argv) {
     printf("%d %lld | %.0f %.0f | %.0f %.0f %.0f | %.0f %.0f %.0f | %lld\n", k, (long long)wl, g[0],
            lo[0], g[1], lo[1], ld[1], g[2], lo[2], ld[2], (long long)S);
     for (int q = 0; q < 3; ++q) { tot_g[q] += g[q]; tot_lo[q] += lo[q]; tot_ld[q] += ld[q]; tot_skip[q] += skip[q]; }
+    for (int h = 0; h < 4; ++h) hot[h] += hotl[h];
+    if (k < 40) printf("   hot %.3f %.3f %.3f %.3f of bin2\n", hotl[0] / (g[2] + 1e-9), hotl[1] / (g[2] + 1e-9), hotl[2] / (g[2] + 1e-9), hotl[3] / (g[2] + 1e-9));
     if (k < 40) printf("   skip %.0f %.0f %.0f\n", skip[0], skip[1], skip[2]);
     int32_t* tw = W; W = W2; W2 = tw;
     wl = nw2;
   }
   printf("TOTAL gathers bin0 %.3g bin1 %.3g (live %.3g) bin2 %.3g | lines bin0 %.3g bin1 %.3g bin2 orig %.3g dense %.3g\n",
          tot_g[0], tot_g[1], tot_ld[1], tot_g[2], tot_lo[0], tot_lo[1], tot_lo[2], tot_ld[2]);
+  printf("HOT bin-2 gathers with id < 2^12/14/16/18: %.3f %.3f %.3f %.3f\n", hot[0] / tot_g[2], hot[1] / tot_g[2], hot[2] / tot_g[2], hot[3] / tot_g[2]);
   printf("SKIPPABLE (conflict-first) bin0 %.3g bin1 %.3g bin2 %.3g\n", tot_skip[0], tot_skip[1], tot_skip[2]);
   return 0;
 }
