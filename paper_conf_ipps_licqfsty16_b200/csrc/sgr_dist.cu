@@ -400,6 +400,7 @@ struct DevPart {
 };
 struct PeerView {         // multi-GPU: the other ranks' workspaces (IPC-mapped), by rank
   std::vector<void*> ws;  // ws[me] = own
+  std::vector<int64_t> ranges;  // nranks + 1 vertex-range boundaries of all ranks
   int me = 0;
 };
 using XSync = std::function<sgr_status(cudaStream_t, int32_t* dflag, int op_max)>;
@@ -503,6 +504,27 @@ static sgr_status run_dev(std::vector<DevPart>& parts, int nranks, int me0, int6
     args[i].me = me0 + i;
   }
   sgr_status status = SGR_OK;
+  // every part's vertex range (host); boundary masks when <= 8 parts (SURVEY §8(e)
+  // boundary filtering: a color word goes only to the replicas that read it)
+  std::vector<int64_t> rg;
+  if (peers) {
+    rg = peers->ranges;
+  } else {
+    rg.push_back(parts[0].lo);
+    for (auto& pt : parts) rg.push_back(pt.hi);
+  }
+  std::vector<uint8_t*> masks(P, nullptr);
+  int64_t* dranges = nullptr;
+  if (nranks > 1 && nranks <= 8) {
+    DCK(cudaMallocAsync((void**)&dranges, rg.size() * 8, s));
+    DCK(cudaMemcpyAsync(dranges, rg.data(), rg.size() * 8, cudaMemcpyHostToDevice, s));
+    for (int i = 0; i < P; ++i) {
+      DCK(cudaMallocAsync((void**)&masks[i], (size_t)std::max<int64_t>(parts[i].hi - parts[i].lo, 1), s));
+      k_remote_mask<C><<<first_grid(parts[i].hi - parts[i].lo), 256, 0, s>>>(args[i], dranges, masks[i]);
+      args[i].rmask = masks[i];
+    }
+    DCK(cudaGetLastError());
+  }
   // C_1 in both buffers of every replica, before any part broadcasts C_2 into it
   for (int i = 0; i < P; ++i) k_fill_c1<C><<<first_grid(n), 256, 0, s>>>(args[i]);
   DCK(cudaGetLastError());
@@ -555,13 +577,22 @@ static sgr_status run_dev(std::vector<DevPart>& parts, int nranks, int me0, int6
   }
   cudaEventRecord(ev1, s);
   RoundArgs<C>& a0 = args[0];
-  if constexpr (packed<C>()) {
-    k_unpack<<<reduce_grid(n), 256, 0, s>>>(a0.col[0], colors_out, n, &a0.ctrl->max_color);
-  } else {
-    if (a0.col[0] != (C*)colors_out)
-      DCK(cudaMemcpyAsync(colors_out, a0.col[0], (size_t)n * 4, cudaMemcpyDeviceToDevice, s));
-    k_max_color<<<reduce_grid(n), 256, 0, s>>>(colors_out, n, &a0.ctrl->max_color);
+  // every vertex's final color is exact in its owner's replica (other replicas only hold
+  // the boundary vertices they read): assemble colors_out range by range, from the local
+  // parts' replicas and (several GPUs) the peers' mapped ones
+  for (int j = 0; j < nranks; ++j) {
+    const int64_t lo = rg[j], len = rg[j + 1] - rg[j];
+    if (len <= 0) continue;
+    const int i = j - me0;  // local part index, if this device owns rank j
+    const C* src = (i >= 0 && i < P) ? args[i].col[0] : col_of(j, 0);
+    if constexpr (packed<C>()) {
+      k_unpack<<<reduce_grid(len), 256, 0, s>>>(src + lo, colors_out + lo, len, &a0.ctrl->max_color);
+    } else {
+      if (src != (const C*)colors_out)
+        DCK(cudaMemcpyAsync(colors_out + lo, src + lo, (size_t)len * 4, cudaMemcpyDeviceToDevice, s));
+    }
   }
+  if constexpr (!packed<C>()) k_max_color<<<reduce_grid(n), 256, 0, s>>>(colors_out, n, &a0.ctrl->max_color);
   DCK(cudaGetLastError());
   std::vector<Ctrl> fin(P);
   for (int i = 0; i < P; ++i)
@@ -614,6 +645,9 @@ static sgr_status run_dev(std::vector<DevPart>& parts, int nranks, int me0, int6
   cudaFreeAsync(dtab, s);
   cudaFreeAsync(dargs, s);
   cudaFreeAsync(dflag, s);
+  if (dranges) cudaFreeAsync(dranges, s);
+  for (auto* m : masks)
+    if (m) cudaFreeAsync(m, s);
   for (auto& pt : parts) {
     if (!peers) cudaFreeAsync(pt.ws, s);
     pt.ws = peers ? pt.ws : nullptr;
@@ -695,6 +729,32 @@ static sgr_status color_dist_device(DistComm* c, const sgr_csr* local, int64_t n
   }
   PeerView pv;
   pv.me = c->rank;
+  {  // every rank's [v_begin, v_end): the ranges for the masks and the final assembly
+    int64_t* dr = nullptr;
+    DCK(cudaMalloc((void**)&dr, 16 * (size_t)(c->world + 1)));
+    const int64_t mine[2] = {v_begin, v_end};
+    DCK(cudaMemcpy(dr + 2 * c->world, mine, 16, cudaMemcpyHostToDevice));
+    const ncclResult_t e = ncclAllGather(dr + 2 * c->world, dr, 2, ncclInt64, c->comm, s);
+    std::vector<int64_t> all(2 * (size_t)c->world);
+    if (e == ncclSuccess) DCK(cudaMemcpyAsync(all.data(), dr, 16 * (size_t)c->world, cudaMemcpyDeviceToHost, s));
+    DCK(cudaStreamSynchronize(s));
+    cudaFree(dr);
+    if (e != ncclSuccess) {
+      cudaFree(ws);
+      set_error("ncclAllGather (ranges): %s", ncclGetErrorString(e));
+      return SGR_ENCCL;
+    }
+    // the device path needs rank-ordered contiguous ranges covering V (what sgr_partition
+    // gives); anything else takes the all-gather transport (every rank sees the same data)
+    bool contiguous = all[0] == 0 && all[2 * (c->world - 1) + 1] == n;
+    for (int q = 0; q + 1 < c->world; ++q) contiguous &= all[2 * q + 1] == all[2 * q + 2];
+    if (!contiguous) {
+      cudaFree(ws);
+      return SGR_EUNSUPPORTED;
+    }
+    pv.ranges.push_back(all[0]);
+    for (int q = 0; q < c->world; ++q) pv.ranges.push_back(all[2 * q + 1]);
+  }
   pv.ws.assign(c->world, nullptr);
   pv.ws[c->rank] = ws;
   bool mapped = true;

@@ -259,6 +259,10 @@ struct RoundArgs {
   int32_t nranks, me;         // parts / ranks taking part in the coloring, this one's index
   Ctrl* const* rctrl;         // [nranks] every part's Ctrl (own included): global counts
   uint32_t* const* xbar;      // [nranks] every part's cross-part barrier counter
+  // Boundary filtering: bit q of rmask[v - v_begin] is set iff part q owns a
+  // neighbour of v, i.e. replica q will ever read v's color; interior vertices (mask 0) are
+  // written to the own replica only. nullptr: broadcast to every replica (> 8 parts).
+  const uint8_t* rmask;
 };
 
 // This part's block group: the whole grid, or (multi-part launch) blocks
@@ -352,7 +356,29 @@ template <class C>
 __device__ __forceinline__ void put_y(const RoundArgs<C>& a, C* Y, int k, int32_t v, C word) {
   Y[v] = word;
   if (a.nrep) {
-    for (int q = 0; q < a.nrep; ++q) a.rep[2 * q + (k & 1)][v] = word;
+    const uint32_t mk = a.rmask ? (uint32_t)a.rmask[v - a.v_begin] : 0xffffffffu;
+    for (int q = 0; q < a.nrep; ++q) {
+      const int rank = q < a.me ? q : q + 1;  // rep[] skips this part's own replica
+      if ((mk >> rank) & 1u) a.rep[2 * q + (k & 1)][v] = word;
+    }
+  }
+}
+
+// rmask of the owned vertices: OR over each row of the bit of the part owning the neighbour
+// (ranges: nranks + 1 boundaries, device memory), the own part excluded.
+template <class C>
+__global__ void k_remote_mask(RoundArgs<C> a, const int64_t* __restrict__ ranges, uint8_t* mask) {
+  for (int64_t v = (int64_t)a.v_begin + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < a.v_end;
+       v += (int64_t)gridDim.x * blockDim.x) {
+    uint32_t m = 0;
+    const int64_t e = ldg_i64(a.row_ptr + v + 1);
+    for (int64_t j = ldg_i64(a.row_ptr + v); j < e; ++j) {
+      const int64_t w = ld_ro(a.col_idx + j);
+      int q = 0;
+      while (q + 1 < a.nranks && ranges[q + 1] <= w) ++q;  // <= 8 parts: linear
+      m |= 1u << q;
+    }
+    mask[v - a.v_begin] = (uint8_t)(m & ~(1u << a.me));
   }
 }
 
