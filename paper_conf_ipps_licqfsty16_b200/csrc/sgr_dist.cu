@@ -516,14 +516,25 @@ static sgr_status run_dev(std::vector<DevPart>& parts, int nranks, int me0, int6
   std::vector<uint8_t*> masks(P, nullptr);
   int64_t* dranges = nullptr;
   if (nranks > 1 && nranks <= 8) {
-    DCK(cudaMallocAsync((void**)&dranges, rg.size() * 8, s));
+    // a part uses its masks only when at most half of its vertices are boundary vertices
+    // (slab partitions of meshes): on skewed graphs nearly every vertex has remote
+    // neighbours, and the per-store mask load would cost more than the stores it saves
+    DCK(cudaMallocAsync((void**)&dranges, rg.size() * 8 + 8 * (size_t)P, s));
+    unsigned long long* dbound = (unsigned long long*)(dranges + rg.size());
     DCK(cudaMemcpyAsync(dranges, rg.data(), rg.size() * 8, cudaMemcpyHostToDevice, s));
+    DCK(cudaMemsetAsync(dbound, 0, 8 * (size_t)P, s));
     for (int i = 0; i < P; ++i) {
-      DCK(cudaMallocAsync((void**)&masks[i], (size_t)std::max<int64_t>(parts[i].hi - parts[i].lo, 1), s));
-      k_remote_mask<C><<<first_grid(parts[i].hi - parts[i].lo), 256, 0, s>>>(args[i], dranges, masks[i]);
-      args[i].rmask = masks[i];
+      const int64_t own = parts[i].hi - parts[i].lo;
+      DCK(cudaMallocAsync((void**)&masks[i], (size_t)std::max<int64_t>(own, 1), s));
+      const int gm = (int)std::max<int64_t>(1, std::min<int64_t>((own + 7) / 8, (int64_t)num_sms() * 16));
+      k_remote_mask<C><<<gm, 256, 0, s>>>(args[i], dranges, masks[i], dbound + i);
     }
     DCK(cudaGetLastError());
+    std::vector<unsigned long long> bound(P, 0);
+    DCK(cudaMemcpyAsync(bound.data(), dbound, 8 * (size_t)P, cudaMemcpyDeviceToHost, s));
+    DCK(cudaStreamSynchronize(s));
+    for (int i = 0; i < P; ++i)
+      if (2 * (int64_t)bound[i] <= parts[i].hi - parts[i].lo) args[i].rmask = masks[i];
   }
   // C_1 in both buffers of every replica, before any part broadcasts C_2 into it
   for (int i = 0; i < P; ++i) k_fill_c1<C><<<first_grid(n), 256, 0, s>>>(args[i]);

@@ -365,21 +365,31 @@ __device__ __forceinline__ void put_y(const RoundArgs<C>& a, C* Y, int k, int32_
 }
 
 // rmask of the owned vertices: OR over each row of the bit of the part owning the neighbour
-// (ranges: nranks + 1 boundaries, device memory), the own part excluded.
+// (ranges: nranks + 1 boundaries, device memory), the own part excluded; one warp per
+// vertex (hub rows are long). *boundary counts the owned vertices with a nonzero mask.
 template <class C>
-__global__ void k_remote_mask(RoundArgs<C> a, const int64_t* __restrict__ ranges, uint8_t* mask) {
-  for (int64_t v = (int64_t)a.v_begin + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < a.v_end;
-       v += (int64_t)gridDim.x * blockDim.x) {
+__global__ void k_remote_mask(RoundArgs<C> a, const int64_t* __restrict__ ranges, uint8_t* mask,
+                              unsigned long long* boundary) {
+  const int lane = threadIdx.x & 31;
+  const int64_t wpb = blockDim.x >> 5;
+  unsigned long long cnt = 0;
+  for (int64_t v = a.v_begin + (int64_t)blockIdx.x * wpb + (threadIdx.x >> 5); v < a.v_end;
+       v += (int64_t)gridDim.x * wpb) {
     uint32_t m = 0;
     const int64_t e = ldg_i64(a.row_ptr + v + 1);
-    for (int64_t j = ldg_i64(a.row_ptr + v); j < e; ++j) {
+    for (int64_t j = ldg_i64(a.row_ptr + v) + lane; j < e; j += 32) {
       const int64_t w = ld_ro(a.col_idx + j);
       int q = 0;
-      while (q + 1 < a.nranks && ranges[q + 1] <= w) ++q;  // <= 8 parts: linear
+      while (q + 1 < a.nranks && __ldg(ranges + q + 1) <= w) ++q;  // <= 8 parts: linear
       m |= 1u << q;
     }
-    mask[v - a.v_begin] = (uint8_t)(m & ~(1u << a.me));
+    m = __reduce_or_sync(0xffffffffu, m) & ~(1u << a.me);
+    if (lane == 0) {
+      mask[v - a.v_begin] = (uint8_t)m;
+      cnt += m ? 1ull : 0ull;
+    }
   }
+  block_add(cnt, boundary);
 }
 
 __device__ __forceinline__ int bin_of(int64_t d, int small_max, int med_max) {
