@@ -167,8 +167,11 @@ constexpr int kMinBlocks = (packed<C>() && Hub) ? SGR_MINB : (Hub ? 3 : SGR_FLAT
 // per SM (packed hub build 2 -> 128 registers, the others 3 -> 85), expressed as ONE block
 // of up to kMaxThreads threads, so any block size up to that (opts->block_size, the
 // paper's Fig. 8 parameter) launches with the same per-thread register allocation.
+#ifndef SGR_HUB_MAXT
+#define SGR_HUB_MAXT 0  // experiments: override the packed hub build's threads-per-SM budget
+#endif
 template <class C, bool Hub = true>
-constexpr int kMaxThreads = kBlock * kMinBlocks<C, Hub>;
+constexpr int kMaxThreads = (SGR_HUB_MAXT && packed<C>() && Hub) ? SGR_HUB_MAXT : kBlock * kMinBlocks<C, Hub>;
 template <class C, bool Hub = true> struct WarpSmem {
   static constexpr int kBuf = (packed<C>() && Hub) ? 2 * kStage : 0;
   static constexpr int kPush = kBuf + kTblBytes;         // push buffer (kPushBuf int32)
