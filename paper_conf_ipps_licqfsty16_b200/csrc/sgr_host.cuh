@@ -150,6 +150,7 @@ inline int round_grid(bool persistent, int B = kBlock) {
     const cudaError_t e2 = cudaFuncSetAttribute(
         k_round<TB, C, Hub>, cudaFuncAttributeMaxDynamicSharedMemorySize, smax);
     if (e1 == cudaSuccess && e2 == cudaSuccess && bit) attr_set.fetch_or(bit, std::memory_order_acq_rel);
+    if (e1 != cudaSuccess || e2 != cudaSuccess) cudaGetLastError();  // do not leak into later checks
   }
   int per_sm = 0;
   cudaError_t e = persistent
