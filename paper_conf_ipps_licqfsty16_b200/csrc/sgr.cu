@@ -274,6 +274,7 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
   cudaStream_t s = r.stream;
   RoundArgs<C> a;
   build_args<C>(a, csr, n, nnz, colors_out, ws, L, r);
+  if (r.loop_mode == SGR_LOOP_PERSISTENT) set_bitmaps<C>(a, ws, L, n);  // dense flat passes
   Prof prof;
   prof.on = r.profile != 0;
   int32_t launches = 0;
@@ -289,6 +290,7 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
   }
   const int grid = round_grid<TB, C>(persistent, B);
   const int grid_flat = persistent ? round_grid<TB, C, false>(true, B) : grid;
+  const int grid_dense = persistent && a.bm[0] ? dense_grid<TB, C>(B) : 0;
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
   sgr_status status = SGR_OK;
   do {
@@ -361,13 +363,20 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
         cfg.attrs = at;
         cfg.numAttrs = nat;
         le = cudaLaunchKernelEx(&cfg, k_persistent<TB, C, true>, a);
+        if (le == cudaSuccess && grid_dense > 0) {  // dense passes (flat build, meshes)
+          cfg.gridDim = dim3(grid_dense);
+          cfg.dynamicSmemBytes = round_smem<C, false>(B);
+          le = cudaLaunchKernelEx(&cfg, k_dense<TB, C>, a);
+          if (le == cudaSuccess)  // k_persistent's grid barrier starts from zero again
+            le = cudaMemsetAsync(&a.ctrl->bar_count, 0, sizeof(uint32_t), s);
+        }
         if (le == cudaSuccess) {
           cfg.gridDim = dim3(grid_flat);
           cfg.dynamicSmemBytes = round_smem<C, false>(B);
           le = cudaLaunchKernelEx(&cfg, k_persistent<TB, C, false>, a);
         }
       });
-      launches += 2;
+      launches += grid_dense > 0 ? 3 : 2;
       if (le != cudaSuccess) {
         status = cuda_fail(le, "cooperative launch of k_persistent", __LINE__);
         break;

@@ -24,7 +24,7 @@ struct Layout {
   bool packed;
   int64_t cap_m, cap_c, cap_big;
   size_t off_col, off_t, off_m, off_c, off_big, off_accb, off_accc, off_fixed, off_len, off_adj,
-      off_fin;
+      off_fin, off_bm;
   size_t zero_begin, zero_end, total;
 };
 
@@ -62,6 +62,9 @@ inline Layout layout(int64_t n, int64_t nnz, const Resolved& r) {
   L.zero_end = o;  // accumulators, fixed sets and list lengths start at zero
   L.off_fin = o;
   o += align_up((size_t)L.cap_big * 8, 256);
+  // worklist membership bitmaps (dense passes of the flat build): 2 x ceil(n / 32) words
+  L.off_bm = o;
+  o += 2 * align_up((size_t)((n + 31) / 32) * 4, 256);
   if (L.packed) {
     L.off_adj = o;
     o += 2 * align_up((size_t)(nnz + 16) * 4, 256);
@@ -70,6 +73,15 @@ inline Layout layout(int64_t n, int64_t nnz, const Resolved& r) {
   return L;
 }
 
+
+// The dense passes' bitmaps (single-GPU colorings only: F_1 writes W_2's when set).
+template <class C>
+inline void set_bitmaps(RoundArgs<C>& a, void* ws, const Layout& L, int64_t n) {
+  char* b = (char*)ws;
+  const size_t bmb = align_up((size_t)((n + 31) / 32) * 4, 256);
+  a.bm[0] = (uint32_t*)(b + L.off_bm);
+  a.bm[1] = (uint32_t*)(b + L.off_bm + bmb);
+}
 
 template <class C>
 inline void build_args(RoundArgs<C>& a, const sgr_csr* csr, int64_t n, int64_t nnz,
@@ -163,6 +175,27 @@ inline int round_grid(bool persistent, int B = kBlock) {
     const int lim = atoi(env);
     if (lim > 0 && lim < per_sm) per_sm = lim;
   }
+  return per_sm * num_sms();
+}
+
+// Blocks of k_dense (its own register allocation; the flat build's shared memory).
+template <int TB, class C>
+inline int dense_grid(int B = kBlock) {
+  static std::atomic<uint64_t> attr_set{0};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  const uint64_t bit = (dev >= 0 && dev < 64) ? (1ull << dev) : 0ull;
+  if (!bit || !(attr_set.load(std::memory_order_acquire) & bit)) {
+    const cudaError_t e1 = cudaFuncSetAttribute(k_dense<TB, C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                (int)round_smem<C, false>(round_max_block<C, false>()));
+    if (e1 == cudaSuccess && bit) attr_set.fetch_or(bit, std::memory_order_acq_rel);
+    if (e1 != cudaSuccess) cudaGetLastError();
+  }
+  int per_sm = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_dense<TB, C>, B, round_smem<C, false>(B)) !=
+          cudaSuccess ||
+      per_sm <= 0)
+    per_sm = 1;
   return per_sm * num_sms();
 }
 

@@ -172,12 +172,19 @@ constexpr int kMinBlocks = (packed<C>() && Hub) ? SGR_MINB : (Hub ? 3 : SGR_FLAT
 #endif
 template <class C, bool Hub = true>
 constexpr int kMaxThreads = (SGR_HUB_MAXT && packed<C>() && Hub) ? SGR_HUB_MAXT : kBlock * kMinBlocks<C, Hub>;
+// Dense passes of the flat build stage a warp step's 32 rows in the warp's shared memory
+// (its tables and push buffer, unused by those passes): at least this many entries, so 32
+// rows of the small bin (<= 32 entries each, 16-byte window alignment included) fit.
+#ifndef SGR_DENSE_CAP
+#define SGR_DENSE_CAP 1056
+#endif
 template <class C, bool Hub = true> struct WarpSmem {
   static constexpr int kBuf = (packed<C>() && Hub) ? 2 * kStage : 0;
   static constexpr int kPush = kBuf + kTblBytes;         // push buffer (kPushBuf int32)
   static constexpr int kItems = kPush + kPushBufOf<Hub> * 4;  // bin-2 item buffer (32 int64)
   static constexpr int kBars = kItems + (Hub ? 32 * 8 : 0);  // 2 mbarriers
-  static constexpr int kBytes = kBars + (Hub ? 16 : 0);
+  static constexpr int kUsed = kBars + (Hub ? 16 : 0);
+  static constexpr int kBytes = Hub ? kUsed : (kUsed > 4 * SGR_DENSE_CAP ? kUsed : 4 * SGR_DENSE_CAP);
 };
 
 // Work counts of one worklist W_k (32 bytes: one pair of vector loads).
@@ -210,7 +217,9 @@ struct Ctrl {
   int32_t max_color;
   int32_t violations;
   uint32_t xbar;             // cross-part barrier counter (k_persistent_dist; other parts add)
-  int32_t pad[4];
+  int32_t cmp_cnt[2];        // bitmap -> worklist compaction (dense -> sparse): bin cursors
+  int32_t pad[2];
+  unsigned long long span_sum;  // F_1: sum over rows of (last - first entry) — row locality
   Counts ring[3];
   unsigned long long edges_acc[3][kBins];    // per ring slot: sum of deg(v) over the pass's
   unsigned long long entries_acc[3][kBins];  // vertices / list entries actually read
@@ -245,6 +254,8 @@ struct RoundArgs {
   uint32_t* fixed;            // [slot][32] colors of dropped (finalized) neighbours
   int64_t* fin;               // finalize list: multi-chunk vertices of the pass
                               // (slot << 32 | buf << 31 | v)
+  uint32_t* bm[2];            // worklist membership bitmaps (flat build's dense passes): W_k
+                              // in bm[k & 1], bit v & 31 of word v >> 5
   Ctrl* ctrl;
   int64_t nnz;
   int32_t n;
@@ -550,19 +561,23 @@ __global__ void __launch_bounds__(1024) k_first(RoundArgs<C> a, int sorted) {
   C* __restrict__ Y = a.col[1];
   const int lane = threadIdx.x & 31;
   const int64_t n = a.v_end;
+  unsigned long long span_acc = 0;  // this thread's rows: sum of widths (dense-pass decision)
   for (int64_t base = (int64_t)a.v_begin + (int64_t)blockIdx.x * blockDim.x; base < n;
        base += (int64_t)gridDim.x * blockDim.x) {
     const int64_t vi = base + threadIdx.x;
     bool conflict = false;
     int64_t s = 0, e = 0;
     const int32_t v = (int32_t)vi;
+    uint32_t span = 0;  // last - first entry of the row: its width in id space
     if (vi < n) {
       s = ldg_i64(a.row_ptr + v);
       e = ldg_i64(a.row_ptr + v + 1);
       if (e > s) {
         if (sorted) {
-          if constexpr (TB == 1) conflict = ldg_i32(a.col_idx + e - 1) > v;
-          else conflict = ldg_i32(a.col_idx + s) < v;
+          const int32_t first = ldg_i32(a.col_idx + s), last = ldg_i32(a.col_idx + e - 1);
+          if constexpr (TB == 1) conflict = last > v;
+          else conflict = first < v;
+          span = (uint32_t)max(last - first, 0);
         } else {
           for (int64_t j = s; j < e && !conflict; ++j) conflict = lose<TB>(v, ldg_i32(a.col_idx + j));
         }
@@ -572,6 +587,11 @@ __global__ void __launch_bounds__(1024) k_first(RoundArgs<C> a, int sorted) {
     }
     const int b = bin_of(e - s, a.small_max, a.med_max);
     Counts* w2 = &ctrl->ring[rs(2)];
+    if (a.bm[0]) {  // W_2's membership bitmap (single GPU: v_begin = 0, warps word-aligned)
+      const unsigned mw = __ballot_sync(0xffffffffu, conflict);
+      if (lane == 0 && base + threadIdx.x < n) a.bm[0][(base + threadIdx.x) >> 5] = mw;
+      span_acc += span;  // row locality: summed per block at the end (one atomic each)
+    }
     {  // bins 0/1: one atomicAdd per BLOCK and bin (~40 % of all vertices enter W_2, so
        // per-warp atomics on the two list counters serialize over the whole grid)
       __shared__ int32_t fcnt[2][kMaxWarps], fbase[2][kMaxWarps];
@@ -630,6 +650,7 @@ __global__ void __launch_bounds__(1024) k_first(RoundArgs<C> a, int sorted) {
     }
   }
   if (a.nrep) __threadfence_system();  // C_2 stores into peer replicas: visible system-wide
+  if (a.bm[0]) block_add(span_acc, &ctrl->span_sum);
 }
 
 // ---------------------------------------------------------------------------------------
@@ -1896,6 +1917,179 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, const C
 #endif
 }
 
+// ---------------------------------------------------------------------------------------
+// Dense passes (flat build, single GPU). While |W_k| > n / SGR_DENSE_DIV (stencils: W = V
+// for ~100 of 314 rounds; ER's first rounds) the grid walks V in id order instead of the
+// worklists: a warp takes one 32-vertex word of the membership bitmap bm[k & 1] per step,
+// one thread per vertex. The 32 rows are one contiguous col_idx segment: the warp copies its
+// 16-byte-aligned window into shared memory with asynchronous 16-byte copies (all in flight
+// at once), then every lane issues ALL gathers of its row together (a row of <= 32 entries:
+// up to 32 loads in flight per lane, 1024 per warp), and the j-th gathers of the 32 lanes
+// are the 32 consecutive vertices' j-th neighbours (one or two lines on a stencil). The pass
+// writes Y for members, the next bitmap word (ballot of the members that conflict; no
+// worklist reads or pushes) and W_{k+1}'s per-bin counts: the sparse pass's exact results.
+// When the next pass is sparse, a compaction phase first turns its bitmap into worklists.
+#ifndef SGR_DENSE
+#define SGR_DENSE 1
+#endif
+#ifndef SGR_DENSE_DIV
+#define SGR_DENSE_DIV 2
+#endif
+#ifndef SGR_DENSE_SPAN
+#define SGR_DENSE_SPAN 16  // dense passes only if the mean row width is below n / 16
+#endif
+
+template <int TB, bool Persist, class C>
+__device__ __forceinline__ void dense_body(const RoundArgs<C>& a, int k, const C* X, C* Y,
+                                           uint8_t* wsm, unsigned long long (&edges)[kBins],
+                                           unsigned long long (&entries)[kBins],
+                                           int32_t (&nxt)[2]) {
+  const int lane = threadIdx.x & 31;
+  const int gw = (int)((blockIdx.x * blockDim.x + threadIdx.x) >> 5);
+  const int NW = (int)((gridDim.x * blockDim.x) >> 5);
+  const uint32_t* bcur = a.bm[k & 1];
+  uint32_t* bnxt = a.bm[(k + 1) & 1];
+  int32_t* stage = reinterpret_cast<int32_t*>(wsm);  // the warp's tables + push buffer
+  constexpr int kCap = WarpSmem<C, false>::kBytes / 4;
+  const int nwords = (a.n + 31) >> 5;
+  for (int g = gw; g < nwords; g += NW) {
+    const uint32_t word = __ldcg(bcur + g);
+    uint32_t out = 0u;
+    if (word) {
+      const int32_t v = (g << 5) + lane;
+      const bool inr = v < a.n;
+      const int64_t s = inr ? ldg_i64(a.row_ptr + v) : a.nnz;
+      const int64_t e = inr ? ldg_i64(a.row_ptr + v + 1) : a.nnz;
+      // the 32 rows are one contiguous segment: its 16-byte-aligned window (capped at the
+      // stage) by asynchronous 16-byte copies, all in flight at once, zero-filled past nnz
+      const int64_t seg0 = __shfl_sync(0xffffffffu, s, 0) & ~(int64_t)3;
+      const int64_t seg1 = __shfl_sync(0xffffffffu, e, 31);
+      const int32_t nq = (int32_t)min((seg1 - seg0 + 3) >> 2, (int64_t)(kCap / 4));
+      const int32_t len = 4 * nq;  // staged entries [seg0, seg0 + len)
+      __syncwarp();
+      for (int32_t q = lane; q < nq; q += 32) {
+        const int64_t p0 = seg0 + 4 * q;
+        const uint32_t bytes = (uint32_t)min((int64_t)16, (a.nnz - p0) * 4);
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_addr(stage + 4 * q)),
+                     "l"(a.col_idx + p0), "r"(bytes)
+                     : "memory");
+      }
+      asm volatile("cp.async.commit_group;\n cp.async.wait_group 0;" ::: "memory");
+      __syncwarp();
+      const bool mem = (word >> lane) & 1u;
+      bool conf = false;
+      if (mem) {
+        const int32_t xv = ldc<Persist>(X + v);
+        const int32_t d = (int32_t)(e - s);
+        const int32_t off = (int32_t)(s - seg0);
+        int32_t tent;
+        if (d <= 32 && off + d <= len) {  // the whole row is staged: every gather at once
+          int32_t c[32];
+#pragma unroll
+          for (int j = 0; j < 32; ++j) c[j] = j < d ? ldc<Persist>(X + stage[off + j]) : 0;
+          uint32_t m = 0;  // bit c - 1 = color c present (first fit <= 33)
+#pragma unroll
+          for (int j = 0; j < 32; ++j) {
+            const uint32_t ci = (uint32_t)(c[j] - 1);
+            m |= ci < 32u ? (1u << ci) : 0u;
+            if (c[j] == xv && j < d) conf |= lose<TB>(v, stage[off + j]);
+          }
+          tent = ~m ? __ffs(~m) : 33;
+        } else {  // long or unstaged row: batches of 8, 4 x 64-bit masks (deg <= 256)
+          uint64_t m0 = 0, m1 = 0, m2 = 0, m3 = 0;
+          for (int32_t j = 0; j < d; j += 8) {
+            int32_t w[8], c[8];
+#pragma unroll
+            for (int u = 0; u < 8; ++u) {
+              const int32_t q = off + j + u;
+              w[u] = j + u < d ? (q < len ? stage[q] : ld_row(a.col_idx + s + j + u)) : -1;
+            }
+#pragma unroll
+            for (int u = 0; u < 8; ++u) c[u] = w[u] >= 0 ? ldc<Persist>(X + w[u]) : 0;
+#pragma unroll
+            for (int u = 0; u < 8; ++u) {
+              const uint32_t ci = (uint32_t)(c[u] - 1);
+              const uint64_t bit = 1ull << (ci & 63u);
+              m0 |= ci < 64u ? bit : 0ull;
+              m1 |= ci - 64u < 64u ? bit : 0ull;
+              m2 |= ci - 128u < 64u ? bit : 0ull;
+              m3 |= ci - 192u < 64u ? bit : 0ull;
+              conf |= w[u] >= 0 && c[u] == xv && lose<TB>(v, w[u]);
+            }
+          }
+          tent = 257;
+          if (~m3) tent = 192 + __ffsll((long long)~m3);
+          if (~m2) tent = 128 + __ffsll((long long)~m2);
+          if (~m1) tent = 64 + __ffsll((long long)~m1);
+          if (~m0) tent = __ffsll((long long)~m0);
+        }
+        put_y<C>(a, Y, k, v, conf ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a));
+        const int b = d <= a.small_max ? 0 : 1;
+        edges[b] += (unsigned long long)d;
+        entries[b] += (unsigned long long)d;
+        nxt[b] += conf ? 1 : 0;
+      }
+      out = __ballot_sync(0xffffffffu, mem && conf);
+    }
+    if (lane == 0) bnxt[g] = out;
+  }
+  __syncwarp();
+}
+
+// W_k's bin worklists from its bitmap (the first sparse pass after dense ones, once per
+// coloring): members in id order, pushed with one atomicAdd per warp and bin; the counts
+// were produced by the dense pass. The warp's shared tables are re-zeroed (the dense passes
+// used them as row stages).
+template <class C>
+__device__ __forceinline__ void dense_to_lists(const RoundArgs<C>& a, int k, uint8_t* wsm) {
+  const int lane = threadIdx.x & 31;
+  const int gw = (int)((blockIdx.x * blockDim.x + threadIdx.x) >> 5);
+  const int NW = (int)((gridDim.x * blockDim.x) >> 5);
+  set_clear(wsm + WarpSmem<C, false>::kBuf, kTblBytes, lane, 32);
+  const uint32_t* bm = a.bm[k & 1];
+  int32_t* lt = sel(k & 1, a.wl_t[0], a.wl_t[1]);
+  int32_t* lm = sel(k & 1, a.wl_m[0], a.wl_m[1]);
+  const int nwords = (a.n + 31) >> 5;
+  for (int g = gw; g < nwords; g += NW) {
+    const uint32_t word = __ldcg(bm + g);
+    if (!word) continue;  // warp-uniform
+    const int32_t v = (g << 5) + lane;
+    const bool mem = (word >> lane) & 1u;
+    const int64_t d = mem ? ldg_i64(a.row_ptr + v + 1) - ldg_i64(a.row_ptr + v) : 0;
+    const bool b0 = mem && d <= a.small_max, b1 = mem && d > a.small_max;
+    const unsigned m0 = __ballot_sync(0xffffffffu, b0), m1 = __ballot_sync(0xffffffffu, b1);
+    int o0 = 0, o1 = 0;
+    if (lane == 0) {
+      if (m0) o0 = atomicAdd(&a.ctrl->cmp_cnt[0], __popc(m0));
+      if (m1) o1 = atomicAdd(&a.ctrl->cmp_cnt[1], __popc(m1));
+    }
+    o0 = __shfl_sync(0xffffffffu, o0, 0);
+    o1 = __shfl_sync(0xffffffffu, o1, 0);
+    const unsigned lt_mask = (1u << lane) - 1u;
+    if (b0) lt[o0 + __popc(m0 & lt_mask)] = v;
+    if (b1) lm[o1 + __popc(m1 & lt_mask)] = v;
+  }
+  __syncwarp();
+}
+
+// Block sum of two per-thread counts, added to *d0 / *d1 with one atomic each.
+__device__ __forceinline__ void block_add2(int32_t (&x)[2], int32_t* d0, int32_t* d1) {
+  __shared__ int32_t red2[2][kMaxWarps];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int32_t a0 = __reduce_add_sync(0xffffffffu, x[0]);
+  const int32_t a1 = __reduce_add_sync(0xffffffffu, x[1]);
+  if (lane == 0) {
+    red2[0][wid] = a0;
+    red2[1][wid] = a1;
+  }
+  __syncthreads();
+  if (threadIdx.x < 2) {
+    int32_t t = 0;
+    for (int q = 0; q < (int)(blockDim.x >> 5); ++q) t += red2[threadIdx.x][q];
+    if (t) atomicAdd(threadIdx.x == 0 ? d0 : d1, t);
+  }
+}
+
 // Block reduction of the per-thread counters, one atomicAdd each per block.
 __device__ __forceinline__ void block_add6(unsigned long long (&x)[kBins],
                                            unsigned long long (&y)[kBins], Ctrl* ctrl, int k) {
@@ -2222,7 +2416,8 @@ __global__ void __launch_bounds__(kMaxThreads<C, Hub>, 1) k_persistent(RoundArgs
   // the last block folds the finished pass: it is the one that draws work last (items go to
   // the lowest warp ids first), so the fold is off the critical path of thin rounds
   const bool leader = blockIdx.x == gridDim.x - 1 && threadIdx.x == 0;
-  int k = 2;
+  // pass 2, or the first sparse pass after k_dense's dense passes (it sets ctrl->k)
+  int k = ld_cg(&ctrl->k);
   for (;; ++k) {
     const Counts w = ld_counts(&ctrl->ring[rs(k)]);
     const int overflow = ld_cg(&ctrl->overflow);
@@ -2415,6 +2610,47 @@ __global__ void __launch_bounds__(kMaxThreads<C, Hub>, 1) k_persistent_dist(Roun
     (void)nparts;
     dist_body<TB, C, Hub>(a0, dsmem);
   }
+}
+
+// The dense passes as their own cooperative launch (between the two builds of
+// k_persistent), so the sparse kernel's register allocation is not shaped by the dense
+// code: it runs passes 2, 3, ... while they qualify (flat graph, bitmaps present, mean row
+// width below n / SGR_DENSE_SPAN, |W_k| > n / SGR_DENSE_DIV), builds the first sparse
+// pass's worklists from its bitmap and leaves ctrl->k there; the host zeroes the barrier
+// counter before k_persistent starts.
+// Dense passes pay only where consecutive vertices have neighbours close in id (meshes):
+// their thread-per-vertex gathers then share lines. 27-point stencil: mean row width ~2 N^2
+// = n / 52 at N = 104; on ER (mean width ~0.9 n) dense passes measured 6.3 -> 7.2 ms.
+template <int TB, class C>
+__global__ void __launch_bounds__(kMaxThreads<C, false>, 1) k_dense(RoundArgs<C> a) {
+  extern __shared__ __align__(16) uint8_t dsmem[];
+  Ctrl* ctrl = a.ctrl;
+  if (!SGR_DENSE || a.bm[0] == nullptr) return;
+  if (ld_cg(&ctrl->big_count) != 0 || !ld_cg(&ctrl->active)) return;  // uniform
+  if (__ldcg(&ctrl->span_sum) > (unsigned long long)a.n * (unsigned long long)a.n / SGR_DENSE_SPAN)
+    return;
+  uint8_t* wsm = warp_smem_init<C, false>(dsmem);
+  uint32_t epoch = 0;
+  const int max_rounds = ld_cg(&ctrl->max_rounds);
+  const bool leader = blockIdx.x == gridDim.x - 1 && threadIdx.x == 0;
+  int k = 2;
+  for (;; ++k) {
+    const Counts w = ld_counts(&ctrl->ring[rs(k)]);
+    const bool dense = items_of(w) > 0 && !ld_cg(&ctrl->overflow) && k <= max_rounds &&
+                       (int64_t)(w.t + w.m) * SGR_DENSE_DIV > (int64_t)a.n;
+    if (!dense) break;  // uniform; k_persistent folds pass k - 1 and goes on from k
+    if (leader && k > 2) fold_pass(ctrl, k - 1);
+    const C* X = sel((k - 1) & 1, (const C*)a.col[0], (const C*)a.col[1]);
+    C* Y = sel(k & 1, a.col[0], a.col[1]);
+    unsigned long long edges[kBins] = {0, 0, 0}, entries[kBins] = {0, 0, 0};
+    int32_t nx[2] = {0, 0};
+    dense_body<TB, true, C>(a, k, X, Y, wsm, edges, entries, nx);
+    block_add2(nx, &ctrl->ring[rs(k + 1)].t, &ctrl->ring[rs(k + 1)].m);
+    block_add6(edges, entries, ctrl, k);
+    grid_sync(ctrl, epoch);
+  }
+  if (k > 2) dense_to_lists(a, k, wsm);  // W_k's lists (in bm[k & 1]) for the sparse passes
+  if (leader) ctrl->k = k;
 }
 
 // Final colors (packed words) into the caller's int32 output, and their maximum.

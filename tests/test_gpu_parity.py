@@ -676,3 +676,41 @@ def test_gs_inplace_nondeterministic_is_proper(tb):
 def test_gs_full_size(cfg):
     """cfg3 / cfg4 at full size with K = 16 strided sub-steps against the oracle's O3."""
     check_gs(gen.config(cfg), 16, 0, LOW)
+
+
+# ----------------------------------------------------------------------------- dense passes
+def local_long_rows(nx, ny, every=997, width=120):
+    """A 9-point grid plus, every `every` vertices, edges to the next `width` ids: rows of
+    33..256 entries (bin 1) that stay local in id space, so the flat build's dense passes
+    take their long-row path."""
+    g = gen.stencil2d(nx, ny, 9)
+    src = np.repeat(np.arange(g.n), np.diff(g.row_ptr))
+    e = [np.stack([src, g.col_idx], 1)]
+    for v in range(0, g.n - width - 1, every):
+        e.append(np.stack([np.full(width, v), np.arange(v + 1, v + 1 + width)], 1))
+    return gen.from_edges(g.n, np.concatenate(e).astype(np.int64))
+
+
+@pytest.mark.parametrize("maker", [
+    lambda: gen.stencil3d(40, 40, 40, 27),
+    lambda: gen.stencil3d(37, 35, 33, 7),
+    lambda: gen.stencil2d(401, 299, 5),
+    lambda: gen.stencil2d(250, 250, 9),
+    lambda: local_long_rows(300, 301),
+], ids=["s27-40", "s7-odd", "s5-odd", "s9-250", "long-rows"])
+@pytest.mark.parametrize("tb", [LOW, PAP])
+def test_dense_passes_of_the_flat_build(maker, tb):
+    """Graphs with local rows (mean row width < n/16) run their first rounds as dense passes
+    (bitmap worklists, thread per vertex, staged rows) and switch to sparse passes through
+    the bitmap -> worklist compaction: colors, R, |W_r| and sum deg(W_r) equal the oracle's,
+    in both color widths, and equal the host loop (which never uses dense passes)."""
+    g = maker()
+    rp, ci = dev(g)
+    ref = oracle.jacobi(g, tb)
+    for bits in (16, 32):
+        res, _ = check_full(g, tb, color_bits=bits)
+        host = sgr.color(rp, ci, RULE[tb], loop_mode="host", color_bits=bits)
+        assert torch.equal(res.colors, host.colors)
+    for B in (64, 192, 512):
+        res = sgr.color(rp, ci, RULE[tb], block_size=B)
+        assert np.array_equal(res.colors.cpu().numpy(), ref.colors), B
