@@ -493,15 +493,114 @@ static sgr_status run_any(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t* c
   return st;
 }
 
-}  // namespace sgr
-
-using namespace sgr;
-
 #define CK(call)                                                  \
   do {                                                            \
     cudaError_t e_ = (call);                                      \
     if (e_ != cudaSuccess) return cuda_fail(e_, #call, __LINE__); \
   } while (0)
+
+// K sub-steps per round in one cooperative launch (gsp::k_gs_persistent, a grid barrier per
+// sub-step); partitions 0 (strided) and 1 (blocked).
+template <int TB>
+static sgr_status color_gs_persistent(const sgr_csr* csr, int64_t n, int64_t nnz, int64_t K,
+                                      int32_t partition, int32_t* colors_out, sgr_stats* stats,
+                                      const Resolved& r) {
+  cudaStream_t s = r.stream;
+  const size_t nb = align_up((size_t)n * 4, 256);
+  const size_t kb = align_up((size_t)(K + 1) * 4, 256);
+  const size_t cb2 = align_up((size_t)4 * K * 4, 256);
+  char* ws = nullptr;
+  CK(cudaMallocAsync((void**)&ws, 3 * nb + cb2 + 2 * kb + 256, s));
+  gsp::Args a;
+  memset(&a, 0, sizeof(a));
+  a.row_ptr = csr->row_ptr;
+  a.col_idx = csr->col_idx;
+  a.C[0] = colors_out;
+  a.C[1] = (int32_t*)ws;
+  a.L[0] = (int32_t*)(ws + nb);
+  a.L[1] = (int32_t*)(ws + 2 * nb);
+  a.cnt = (int32_t*)(ws + 3 * nb);
+  int32_t* poff = (int32_t*)(ws + 3 * nb + cb2);
+  int32_t* pcur = (int32_t*)(ws + 3 * nb + cb2 + kb);
+  a.poff = poff;
+  a.ctrl = (gsp::Ctrl*)(ws + 3 * nb + cb2 + 2 * kb);
+  a.n = n;
+  a.K = K;
+  a.partition = partition;
+  a.max_rounds = r.max_rounds;
+  a.round_sizes = r.round_sizes;
+  a.round_edges = r.round_edges;
+  a.round_cap = r.round_cap;
+  a.tiebreak = TB;
+  CK(cudaMemsetAsync(a.C[0], 0, (size_t)n * 4, s));  // 0 = not yet colored
+  CK(cudaMemsetAsync(a.C[1], 0, (size_t)n * 4, s));
+  CK(cudaMemsetAsync(a.cnt, 0, cb2, s));
+  CK(cudaMemsetAsync(a.ctrl, 0, sizeof(gsp::Ctrl), s));
+  // list regions: part j's members, counted and scanned
+  int32_t* hist = a.cnt;  // scratch for the histogram (re-zeroed below)
+  gsp::k_part_hist<<<std::max(1, (int)std::min<int64_t>((n + 255) / 256, num_sms() * 8)), 256, 0, s>>>(
+      n, K, partition, hist);
+  k_gs_scan<<<1, 32, 0, s>>>(hist, K, poff, pcur);
+  CK(cudaMemsetAsync(a.cnt, 0, cb2, s));
+  int per_sm = 0;
+  const void* fn = (const void*)gsp::k_gs_persistent<TB>;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, gsp::k_gs_persistent<TB>, 256, 0) != cudaSuccess ||
+      per_sm <= 0)
+    per_sm = 1;
+  const int grid = per_sm * num_sms();
+  cudaEvent_t e0, e1;
+  CK(cudaEventCreate(&e0));
+  CK(cudaEventCreate(&e1));
+  CK(cudaEventRecord(e0, s));
+  void* args[] = {(void*)&a};
+  cudaError_t le = cudaLaunchCooperativeKernel(fn, grid, 256, args, 0, s);
+  if (le != cudaSuccess) {
+    cudaFreeAsync(ws, s);
+    return cuda_fail(le, "cooperative launch of k_gs_persistent", __LINE__);
+  }
+  CK(cudaEventRecord(e1, s));
+  gsp::Ctrl fin;
+  CK(cudaMemcpyAsync(&fin, a.ctrl, sizeof(fin), cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  if (fin.final_buf == 1)
+    CK(cudaMemcpyAsync(colors_out, a.C[1], (size_t)n * 4, cudaMemcpyDeviceToDevice, s));
+  int32_t* dmax = (int32_t*)(ws + 3 * nb);  // reuse the counters
+  CK(cudaMemsetAsync(dmax, 0, 4, s));
+  k_max_color<<<reduce_grid(n), 256, 0, s>>>(colors_out, n, dmax);
+  int32_t mx = 0;
+  CK(cudaMemcpyAsync(&mx, dmax, 4, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  sgr_status status = SGR_OK;
+  if (fin.status == 1) {
+    set_error("sgr_color_gs: max_rounds (%d) reached", r.max_rounds);
+    status = SGR_ENOCONV;
+  }
+  if (stats) {
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, e0, e1);
+    stats->rounds = fin.rounds;
+    stats->num_colors = mx;
+    stats->vertices_processed = (int64_t)fin.verts_total;
+    stats->edges_scanned = (int64_t)fin.edges_total;
+    stats->entries_read = (int64_t)fin.edges_total;
+    stats->elapsed_ms = ms;
+    stats->launches = 4;
+    stats->color_bits = 32;
+    stats->grid_blocks = grid;
+    // per round: detection re-reads W's rows (id + color per entry), the first fits read
+    // them again; per member its id (list), row pair, two color words; the copies
+    stats->bytes_algorithmic = (int64_t)fin.edges_total * 16 + (int64_t)fin.verts_total * 40;
+  }
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  cudaFreeAsync(ws, s);
+  cudaStreamSynchronize(s);
+  return status;
+}
+}  // namespace sgr
+
+using namespace sgr;
+
 
 extern "C" {
 
@@ -862,6 +961,11 @@ sgr_status sgr_color_gs(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t subs
   const int64_t K = partition == 2 ? 1 : substeps;
   cudaStream_t s = r.stream;
   keep_pool_memory();
+  const char* hl = getenv("SGR_GS_HOSTLOOP");
+  if (partition != 2 && !(hl && hl[0] == '1'))
+    return r.tiebreak ? color_gs_persistent<1>(csr, n, nnz, K, partition, colors_out, stats, r)
+                      : color_gs_persistent<0>(csr, n, nnz, K, partition, colors_out, stats, r);
+  // host-driven rounds (the in-place mode; SGR_GS_HOSTLOOP=1 for the sub-step modes)
   // workspace: W[2] | T | flags | seg | tiles | counters | K counts / offsets / cursors
   const size_t nb = align_up((size_t)n * 4, 256);
   const int64_t tiles = (n + kCompactTile - 1) / kCompactTile;

@@ -172,4 +172,372 @@ static __global__ void k_gs_init(int64_t n, int32_t* __restrict__ wl, int32_t* _
   }
 }
 
+
+// =======================================================================================
+// Persistent K-sub-step rounds (one cooperative launch, one grid barrier per sub-step).
+//
+// Two color buffers alternate per sub-step: sub-step j reads Cur and writes its members'
+// new colors into Nxt, which before that equals the colors of one sub-step earlier — so the
+// same sub-step also copies the previous sub-step's members (the only vertices that changed
+// since) from Cur into Nxt. Nobody reads Nxt during the sub-step, so after the barrier Nxt
+// is exactly the colors every later sub-step must see (Jacobi inside a sub-step, the
+// earlier sub-steps' colors across them: reading C20).
+// Sub-step 0 of round R also detects the conflicts of round R-1 (Alg. 5 l.12-15) over all
+// of W_{R-1} against Cur (round R-1's final colors; Nxt is not read), pushing the losers
+// into round R's per-part lists, and assigns the part-0 members at once (same snapshot).
+// Lists: region j of a list array holds part j's members, low-degree ones from the front
+// (thread per vertex), the others from the back (warp per vertex), counts per part.
+namespace gsp {
+
+// Members of each part among all n vertices (the list regions' sizes).
+static __global__ void k_part_hist(int64_t n, int64_t K, int partition, int32_t* __restrict__ cnt) {
+  for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n;
+       v += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(cnt + gs_part(v, n, K, partition), 1);
+}
+
+constexpr int kSmallDeg = 64;  // thread-per-vertex first fit / detection up to this degree
+
+struct Ctrl {
+  uint32_t bar_count;
+  int32_t rounds;        // R: assignment rounds run
+  int32_t status;        // 1: max_rounds reached with W non-empty
+  int32_t final_buf;     // index of the color buffer holding the result
+  unsigned long long edges[2];  // per round parity: sum deg(W_R) (pushed members)
+  unsigned long long verts_total, edges_total;  // sum over rounds of |W_R|, sum deg(W_R)
+};
+
+struct Args {
+  const int64_t* row_ptr;
+  const int32_t* col_idx;
+  int32_t* C[2];
+  int32_t* L[2];
+  const int32_t* poff;   // K + 1 region offsets
+  int32_t* cnt;          // [2][K][2]: per list parity, part: small count, big count
+  Ctrl* ctrl;
+  int32_t* round_sizes;
+  int64_t* round_edges;
+  int64_t n;
+  int64_t K;
+  int32_t partition;
+  int32_t max_rounds;
+  int32_t round_cap;
+  int32_t tiebreak;
+};
+
+__device__ __forceinline__ int32_t* cnt_of(const Args& a, int par, int64_t j, int big) {
+  return a.cnt + ((int64_t)par * a.K + j) * 2 + big;
+}
+
+__device__ __forceinline__ void gsync(Ctrl* c, uint32_t& epoch) {
+  __syncthreads();
+  ++epoch;
+  if (threadIdx.x == 0) {
+    asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&c->bar_count) : "memory");
+    const uint32_t target = epoch * gridDim.x;
+    uint32_t v;
+    do {
+      asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(&c->bar_count) : "memory");
+      if ((int32_t)(v - target) < 0) __nanosleep(32);
+    } while ((int32_t)(v - target) < 0);
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(&c->bar_count) : "memory");
+  }
+  __syncthreads();
+}
+
+// 8-lane group per low-degree vertex (v < 0: idle group): lane gl gathers entries gl + 8u
+// (u < 8: all 64 at once); the group ORs its 64-bit color masks (bit c - 1 = color c; a
+// degree <= 64 row leaves a free color <= 65) and, with want_conf, ORs the conflict test.
+// Every listed entry counts, self-loops included (Alg. 5 l.5-6 literally, as O3).
+// All 32 lanes of the warp must call it. Returns the first fit.
+template <int TB>
+__device__ __forceinline__ int32_t group_scan(const Args& a, const int32_t* Cur, int32_t v, int64_t s,
+                                              int64_t e, int gl, unsigned gmask, bool want_conf,
+                                              bool& conf) {
+  const int32_t d = v >= 0 ? (int32_t)(e - s) : 0;
+  int32_t w[8], c[8];
+#pragma unroll
+  for (int u = 0; u < 8; ++u) w[u] = gl + 8 * u < d ? ld_ro(a.col_idx + s + gl + 8 * u) : -1;
+#pragma unroll
+  for (int u = 0; u < 8; ++u) c[u] = w[u] >= 0 ? __ldcg(Cur + w[u]) : 0;
+  const int32_t cv = (want_conf && v >= 0) ? __ldcg(Cur + v) : -1;
+  uint64_t m = 0;
+  bool cf = false;
+#pragma unroll
+  for (int u = 0; u < 8; ++u) {
+    const uint32_t ci = (uint32_t)(c[u] - 1);
+    m |= ci < 64u ? (1ull << ci) : 0ull;
+    cf |= w[u] >= 0 && c[u] == cv && lose<TB>(v, w[u]);
+  }
+#pragma unroll
+  for (int o = 4; o > 0; o >>= 1) m |= __shfl_xor_sync(0xffffffffu, m, o);
+  conf = (__ballot_sync(0xffffffffu, cf) & gmask) != 0u;
+  return ~m ? __ffsll((long long)~m) : 65;
+}
+
+// One warp per high-degree vertex: 8 entries per lane per batch (ids first, then all 8
+// gathers), so a long row keeps 256 loads in flight instead of one chain per lane.
+template <int TB>
+__device__ __forceinline__ bool warp_conflict(const Args& a, const int32_t* Cur, int32_t v, int64_t s,
+                                              int64_t e, int lane) {
+  const int32_t cv = __ldcg(Cur + v);
+  bool c = false;
+  for (int64_t q0 = s; q0 < e; q0 += 256) {
+    int32_t w[8], col[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int64_t q = q0 + 32 * u + lane;
+      w[u] = q < e ? ld_ro(a.col_idx + q) : -1;
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) col[u] = w[u] >= 0 ? __ldcg(Cur + w[u]) : -1;
+#pragma unroll
+    for (int u = 0; u < 8; ++u) c |= w[u] >= 0 && col[u] == cv && lose<TB>(v, w[u]);
+  }
+  return __any_sync(0xffffffffu, c);
+}
+
+// First fit of a high-degree vertex against Cur, one warp: 256-color windows (bit i of the
+// window word = color base + i + 1), rescanning the row per window, batches of 8 per lane.
+__device__ __forceinline__ int32_t warp_fit(const Args& a, const int32_t* Cur, int64_t s, int64_t e,
+                                           int lane) {
+  for (int32_t base = 0;; base += 256) {
+    uint64_t m0 = 0, m1 = 0, m2 = 0, m3 = 0;
+    for (int64_t q0 = s; q0 < e; q0 += 256) {
+      int32_t w[8], c[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const int64_t q = q0 + 32 * u + lane;
+        w[u] = q < e ? ld_ro(a.col_idx + q) : -1;
+      }
+#pragma unroll
+      for (int u = 0; u < 8; ++u) c[u] = w[u] >= 0 ? __ldcg(Cur + w[u]) : 0;
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const uint32_t idx = (uint32_t)(c[u] - base - 1);
+        const uint64_t bit = 1ull << (idx & 63u);
+        m0 |= idx < 64u ? bit : 0ull;
+        m1 |= idx - 64u < 64u ? bit : 0ull;
+        m2 |= idx - 128u < 64u ? bit : 0ull;
+        m3 |= idx - 192u < 64u ? bit : 0ull;
+      }
+    }
+    m0 = warp_or64(m0);
+    m1 = warp_or64(m1);
+    m2 = warp_or64(m2);
+    m3 = warp_or64(m3);
+    if (~m0) return base + __ffsll((long long)~m0);
+    if (~m1) return base + 64 + __ffsll((long long)~m1);
+    if (~m2) return base + 128 + __ffsll((long long)~m2);
+    if (~m3) return base + 192 + __ffsll((long long)~m3);
+  }
+}
+
+// Push v (degree d) into round list `par`, region of its part j: low-degree members from
+// the front, the others from the back. Warp-collective (all 32 lanes call; `pred` selects
+// the pushing lanes): lanes with the same (part, kind) share one atomicAdd (the callers
+// iterate parts in order, so a warp's lanes usually share both). Lists are unordered.
+__device__ __forceinline__ void push_warp(const Args& a, int par, int32_t v, int64_t d, bool pred) {
+  const int64_t j = pred ? gs_part(v, a.n, a.K, a.partition) : -1;
+  const int big = d > kSmallDeg ? 1 : 0;
+  const long long key = pred ? (long long)(2 * j + big) : -1ll;
+  const unsigned grp = __match_any_sync(0xffffffffu, key);
+  const int lane = threadIdx.x & 31;
+  const int lead = __ffs(grp) - 1;
+  int32_t o = 0;
+  if (pred && lane == lead) o = atomicAdd(cnt_of(a, par, j, big), __popc(grp));
+  o = __shfl_sync(0xffffffffu, o, lead) + __popc(grp & ((1u << lane) - 1u));
+  if (pred) {
+    if (!big) a.L[par][__ldg(a.poff + j) + o] = v;
+    else a.L[par][__ldg(a.poff + j + 1) - 1 - o] = v;
+  }
+}
+
+// The vertex at position p of the part-major order (part 0's vertices, then part 1's, ...):
+// blocked parts are contiguous id ranges, so p itself; strided part j holds j, j + K, ...
+__device__ __forceinline__ int32_t vertex_at(const Args& a, int64_t p) {
+  if (a.partition == 1) return (int32_t)p;
+  int64_t lo = 0, hi = a.K;  // largest j with poff[j] <= p
+  while (hi - lo > 1) {
+    const int64_t mid = (lo + hi) >> 1;
+    if (__ldg(a.poff + mid) <= p) lo = mid;
+    else hi = mid;
+  }
+  return (int32_t)(lo + a.K * (p - __ldg(a.poff + lo)));
+}
+
+template <int TB>
+__global__ void __launch_bounds__(256, 3) k_gs_persistent(Args a) {
+  const int lane = threadIdx.x & 31;
+  const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
+  const int64_t gw = tid >> 5, nw = nthr >> 5;
+  Ctrl* ctrl = a.ctrl;
+  const bool leader = blockIdx.x == 0 && threadIdx.x == 0;
+  uint32_t epoch = 0;
+  int cb = 0;   // Cur = C[cb]
+  int par = 0;  // W_{R-1}'s lists in L[par]; round R's are pushed into L[par ^ 1]
+  unsigned long long my_edges = 0;
+  for (int R = 1;; ++R) {
+    // ---------------- sub-step 0: detect round R-1 over W_{R-1}, assign part 0 ----------
+    const int32_t* Cur = a.C[cb];
+    int32_t* Nxt = a.C[cb ^ 1];
+    const int np = par ^ 1;  // round R's lists
+    const int g = lane >> 3, gl = lane & 7;
+    const unsigned gmask = 0xffu << (g * 8);
+    if (R == 1) {  // W_0 = V, everything "conflicts": round 1 starts with every vertex,
+                   // visited in part-major order so a warp's pushes share one atomic
+      for (int64_t b0 = tid - lane; b0 < a.n; b0 += nthr) {
+        const int64_t p = b0 + lane;
+        const bool ok = p < a.n;
+        const int32_t v = ok ? vertex_at(a, p) : 0;
+        const int64_t s = ok ? ld_ro(a.row_ptr + v) : 0, e = ok ? ld_ro(a.row_ptr + v + 1) : 0;
+        push_warp(a, np, v, e - s, ok);
+        my_edges += (unsigned long long)(e - s);
+      }
+    } else {
+      // small members of every part of W_{R-1}: an 8-lane group each; detection against
+      // Cur, the losers pushed, part-0 losers take their first fit from the same scan
+      for (int64_t j = 0; j < a.K; ++j) {
+        const int32_t base = __ldg(a.poff + j);
+        const int32_t ns = __ldcg(cnt_of(a, par, j, 0));
+        for (int64_t b0 = gw * 4; b0 < ns; b0 += nw * 4) {
+          const int64_t i = b0 + g;
+          const int32_t v = i < ns ? __ldcg(&a.L[par][base + i]) : -1;
+          const int64_t s = v >= 0 ? ld_ro(a.row_ptr + v) : 0, e = v >= 0 ? ld_ro(a.row_ptr + v + 1) : 0;
+          bool conf = false;
+          const int32_t tent = group_scan<TB>(a, Cur, v, s, e, gl, gmask, true, conf);
+          const bool lead = v >= 0 && gl == 0;
+          push_warp(a, np, v, e - s, lead && conf);
+          if (lead) {
+            if (!conf) {
+              if (a.K == 1) Nxt[v] = __ldcg(Cur + v);  // K = 1: W_{R-1} is the previous sub-step
+            } else {
+              my_edges += (unsigned long long)(e - s);
+              if (j == 0) Nxt[v] = tent;
+            }
+          }
+        }
+      }
+    }
+    // big members: warp per vertex (detection; part-0 ones also take their first fit)
+    for (int64_t j = 0; j < a.K; ++j) {
+      const int32_t top = __ldg(a.poff + j + 1);
+      const int32_t nbg = R == 1 ? 0 : __ldcg(cnt_of(a, par, j, 1));
+      for (int64_t i = gw; i < nbg; i += nw) {
+        const int32_t v = __ldcg(&a.L[par][top - 1 - i]);
+        const int64_t s = ld_ro(a.row_ptr + v), e = ld_ro(a.row_ptr + v + 1);
+        if (!warp_conflict<TB>(a, Cur, v, s, e, lane)) {
+          if (a.K == 1 && lane == 0) Nxt[v] = __ldcg(Cur + v);
+          continue;
+        }
+        push_warp(a, np, v, e - s, lane == 0);
+        if (lane == 0) my_edges += (unsigned long long)(e - s);
+        if (j == 0) {
+          const int32_t t = warp_fit(a, Cur, s, e, lane);
+          if (lane == 0) Nxt[v] = t;
+        }
+      }
+    }
+    // copy: the previous sub-step's members (W_{R-1} ∩ part K-1) into Nxt (K = 1: done above,
+    // where each member either takes its new color or keeps its old one)
+    if (R > 1 && a.K > 1) {
+      const int64_t j = a.K - 1;
+      const int32_t base = __ldg(a.poff + j), top = __ldg(a.poff + j + 1);
+      const int32_t ns = __ldcg(cnt_of(a, par, j, 0)), nbg = __ldcg(cnt_of(a, par, j, 1));
+      for (int64_t i = tid; i < ns + nbg; i += nthr) {
+        const int32_t u = i < ns ? __ldcg(&a.L[par][base + i]) : __ldcg(&a.L[par][top - 1 - (i - ns)]);
+        Nxt[u] = __ldcg(Cur + u);
+      }
+    }
+    block_add(my_edges, &ctrl->edges[np]);
+    my_edges = 0;
+    gsync(ctrl, epoch);
+    if (R == 1) {  // part-0 members of round 1 (all vertices conflict): their first fits
+      const int32_t base0 = __ldg(a.poff);
+      const int32_t ns0 = __ldcg(cnt_of(a, np, 0, 0));
+      for (int64_t b0 = gw * 4; b0 < ns0; b0 += nw * 4) {
+        const int64_t i = b0 + g;
+        const int32_t v = i < ns0 ? __ldcg(&a.L[np][base0 + i]) : -1;
+        const int64_t s = v >= 0 ? ld_ro(a.row_ptr + v) : 0, e = v >= 0 ? ld_ro(a.row_ptr + v + 1) : 0;
+        bool conf;
+        const int32_t tent = group_scan<TB>(a, Cur, v, s, e, gl, gmask, false, conf);
+        if (v >= 0 && gl == 0) Nxt[v] = tent;
+      }
+      const int32_t top = __ldg(a.poff + 1);
+      const int32_t nbg = __ldcg(cnt_of(a, np, 0, 1));
+      for (int64_t i = gw; i < nbg; i += nw) {
+        const int32_t v = __ldcg(&a.L[np][top - 1 - i]);
+        const int32_t t = warp_fit(a, Cur, ld_ro(a.row_ptr + v), ld_ro(a.row_ptr + v + 1), lane);
+        if (lane == 0) Nxt[v] = t;
+      }
+      gsync(ctrl, epoch);
+    }
+    // |W_R| and its edges; the previous parity's counts can be cleared for round R+1
+    int64_t wsz = 0;
+    for (int64_t j = 0; j < a.K; ++j) wsz += (int64_t)__ldcg(cnt_of(a, np, j, 0)) + __ldcg(cnt_of(a, np, j, 1));
+    if (wsz == 0) {  // W_R empty: round R-1 was the last; its final colors are in Cur
+      if (leader) {
+        ctrl->rounds = R - 1;
+        ctrl->final_buf = cb;
+      }
+      return;
+    }
+    if (R > a.max_rounds) {
+      if (leader) {
+        ctrl->rounds = R - 1;
+        ctrl->final_buf = cb;
+        ctrl->status = 1;
+      }
+      return;
+    }
+    if (leader) {
+      const unsigned long long ed = __ldcg(&ctrl->edges[np]);
+      ctrl->verts_total += (unsigned long long)wsz;
+      ctrl->edges_total += ed;
+      if (R - 1 < a.round_cap) {
+        if (a.round_sizes) a.round_sizes[R - 1] = (int32_t)wsz;
+        if (a.round_edges) a.round_edges[R - 1] = (int64_t)ed;
+      }
+    }
+    cb ^= 1;
+    // ---------------- sub-steps 1 .. K-1: assign part j, copy part j-1 ---------------
+    for (int64_t j = 1; j < a.K; ++j) {
+      const int32_t* Cj = a.C[cb];
+      int32_t* Nj = a.C[cb ^ 1];
+      const int32_t base = __ldg(a.poff + j), top = __ldg(a.poff + j + 1);
+      const int32_t ns = __ldcg(cnt_of(a, np, j, 0)), nbg = __ldcg(cnt_of(a, np, j, 1));
+      for (int64_t b0 = gw * 4; b0 < ns; b0 += nw * 4) {
+        const int64_t i = b0 + g;
+        const int32_t v = i < ns ? __ldcg(&a.L[np][base + i]) : -1;
+        const int64_t s = v >= 0 ? ld_ro(a.row_ptr + v) : 0, e = v >= 0 ? ld_ro(a.row_ptr + v + 1) : 0;
+        bool conf;
+        const int32_t tent = group_scan<TB>(a, Cj, v, s, e, gl, gmask, false, conf);
+        if (v >= 0 && gl == 0) Nj[v] = tent;
+      }
+      for (int64_t i = gw; i < nbg; i += nw) {
+        const int32_t v = __ldcg(&a.L[np][top - 1 - i]);
+        const int32_t t = warp_fit(a, Cj, ld_ro(a.row_ptr + v), ld_ro(a.row_ptr + v + 1), lane);
+        if (lane == 0) Nj[v] = t;
+      }
+      {  // copy part j-1's members (changed in the previous sub-step) into Nj
+        const int32_t pb = __ldg(a.poff + j - 1), pt = __ldg(a.poff + j);
+        const int32_t ps = __ldcg(cnt_of(a, np, j - 1, 0)), pg = __ldcg(cnt_of(a, np, j - 1, 1));
+        for (int64_t i = tid; i < ps + pg; i += nthr) {
+          const int32_t u = i < ps ? __ldcg(&a.L[np][pb + i]) : __ldcg(&a.L[np][pt - 1 - (i - ps)]);
+          Nj[u] = __ldcg(Cj + u);
+        }
+      }
+      gsync(ctrl, epoch);
+      cb ^= 1;
+    }
+    // round R's lists become W_R; clear the parity round R+1 pushes into, and its edges
+    if (tid < 2 * a.K) a.cnt[(int64_t)par * a.K * 2 + tid] = 0;
+    if (leader) ctrl->edges[par] = 0ull;
+    gsync(ctrl, epoch);
+    par = np;
+  }
+}
+
+}  // namespace gsp
 }  // namespace sgr

@@ -1,0 +1,4 @@
+#!/bin/bash
+cd $GRAFT_REPO_ROOT
+timeout 1200 python -m pytest tests/test_gpu_parity.py -m gpu -x -q -k "gs_" > gpurun_out/r2x_tests.log 2>&1; echo pytest=$? >> gpurun_out/r2x_tests.log
+timeout 900 python tools/gs_report.py --out gpurun_out/r2x_gs.jsonl > gpurun_out/r2x_gs.log 2>&1
