@@ -348,8 +348,8 @@ __device__ __forceinline__ void push_warp(const Args& a, int par, int32_t v, int
   if (pred && lane == lead) o = atomicAdd(cnt_of(a, par, j, big), __popc(grp));
   o = __shfl_sync(0xffffffffu, o, lead) + __popc(grp & ((1u << lane) - 1u));
   if (pred) {
-    if (!big) a.L[par][__ldg(a.poff + j) + o] = v;
-    else a.L[par][__ldg(a.poff + j + 1) - 1 - o] = v;
+    if (!big) (par ? a.L[1] : a.L[0])[__ldg(a.poff + j) + o] = v;
+    else (par ? a.L[1] : a.L[0])[__ldg(a.poff + j + 1) - 1 - o] = v;
   }
 }
 
@@ -380,8 +380,8 @@ __global__ void __launch_bounds__(256, 3) k_gs_persistent(Args a) {
   unsigned long long my_edges = 0;
   for (int R = 1;; ++R) {
     // ---------------- sub-step 0: detect round R-1 over W_{R-1}, assign part 0 ----------
-    const int32_t* Cur = a.C[cb];
-    int32_t* Nxt = a.C[cb ^ 1];
+    const int32_t* Cur = (cb ? a.C[1] : a.C[0]);
+    int32_t* Nxt = (cb ? a.C[0] : a.C[1]);
     const int np = par ^ 1;  // round R's lists
     const int g = lane >> 3, gl = lane & 7;
     const unsigned gmask = 0xffu << (g * 8);
@@ -403,7 +403,7 @@ __global__ void __launch_bounds__(256, 3) k_gs_persistent(Args a) {
         const int32_t ns = __ldcg(cnt_of(a, par, j, 0));
         for (int64_t b0 = gw * 4; b0 < ns; b0 += nw * 4) {
           const int64_t i = b0 + g;
-          const int32_t v = i < ns ? __ldcg(&a.L[par][base + i]) : -1;
+          const int32_t v = i < ns ? __ldcg(&(par ? a.L[1] : a.L[0])[base + i]) : -1;
           const int64_t s = v >= 0 ? ld_ro(a.row_ptr + v) : 0, e = v >= 0 ? ld_ro(a.row_ptr + v + 1) : 0;
           bool conf = false;
           const int32_t tent = group_scan<TB>(a, Cur, v, s, e, gl, gmask, true, conf);
@@ -425,7 +425,7 @@ __global__ void __launch_bounds__(256, 3) k_gs_persistent(Args a) {
       const int32_t top = __ldg(a.poff + j + 1);
       const int32_t nbg = R == 1 ? 0 : __ldcg(cnt_of(a, par, j, 1));
       for (int64_t i = gw; i < nbg; i += nw) {
-        const int32_t v = __ldcg(&a.L[par][top - 1 - i]);
+        const int32_t v = __ldcg(&(par ? a.L[1] : a.L[0])[top - 1 - i]);
         const int64_t s = ld_ro(a.row_ptr + v), e = ld_ro(a.row_ptr + v + 1);
         if (!warp_conflict<TB>(a, Cur, v, s, e, lane)) {
           if (a.K == 1 && lane == 0) Nxt[v] = __ldcg(Cur + v);
@@ -446,7 +446,7 @@ __global__ void __launch_bounds__(256, 3) k_gs_persistent(Args a) {
       const int32_t base = __ldg(a.poff + j), top = __ldg(a.poff + j + 1);
       const int32_t ns = __ldcg(cnt_of(a, par, j, 0)), nbg = __ldcg(cnt_of(a, par, j, 1));
       for (int64_t i = tid; i < ns + nbg; i += nthr) {
-        const int32_t u = i < ns ? __ldcg(&a.L[par][base + i]) : __ldcg(&a.L[par][top - 1 - (i - ns)]);
+        const int32_t u = i < ns ? __ldcg(&(par ? a.L[1] : a.L[0])[base + i]) : __ldcg(&(par ? a.L[1] : a.L[0])[top - 1 - (i - ns)]);
         Nxt[u] = __ldcg(Cur + u);
       }
     }
@@ -458,7 +458,7 @@ __global__ void __launch_bounds__(256, 3) k_gs_persistent(Args a) {
       const int32_t ns0 = __ldcg(cnt_of(a, np, 0, 0));
       for (int64_t b0 = gw * 4; b0 < ns0; b0 += nw * 4) {
         const int64_t i = b0 + g;
-        const int32_t v = i < ns0 ? __ldcg(&a.L[np][base0 + i]) : -1;
+        const int32_t v = i < ns0 ? __ldcg(&(np ? a.L[1] : a.L[0])[base0 + i]) : -1;
         const int64_t s = v >= 0 ? ld_ro(a.row_ptr + v) : 0, e = v >= 0 ? ld_ro(a.row_ptr + v + 1) : 0;
         bool conf;
         const int32_t tent = group_scan<TB>(a, Cur, v, s, e, gl, gmask, false, conf);
@@ -467,7 +467,7 @@ __global__ void __launch_bounds__(256, 3) k_gs_persistent(Args a) {
       const int32_t top = __ldg(a.poff + 1);
       const int32_t nbg = __ldcg(cnt_of(a, np, 0, 1));
       for (int64_t i = gw; i < nbg; i += nw) {
-        const int32_t v = __ldcg(&a.L[np][top - 1 - i]);
+        const int32_t v = __ldcg(&(np ? a.L[1] : a.L[0])[top - 1 - i]);
         const int32_t t = warp_fit(a, Cur, ld_ro(a.row_ptr + v), ld_ro(a.row_ptr + v + 1), lane);
         if (lane == 0) Nxt[v] = t;
       }
@@ -503,20 +503,20 @@ __global__ void __launch_bounds__(256, 3) k_gs_persistent(Args a) {
     cb ^= 1;
     // ---------------- sub-steps 1 .. K-1: assign part j, copy part j-1 ---------------
     for (int64_t j = 1; j < a.K; ++j) {
-      const int32_t* Cj = a.C[cb];
-      int32_t* Nj = a.C[cb ^ 1];
+      const int32_t* Cj = (cb ? a.C[1] : a.C[0]);
+      int32_t* Nj = (cb ? a.C[0] : a.C[1]);
       const int32_t base = __ldg(a.poff + j), top = __ldg(a.poff + j + 1);
       const int32_t ns = __ldcg(cnt_of(a, np, j, 0)), nbg = __ldcg(cnt_of(a, np, j, 1));
       for (int64_t b0 = gw * 4; b0 < ns; b0 += nw * 4) {
         const int64_t i = b0 + g;
-        const int32_t v = i < ns ? __ldcg(&a.L[np][base + i]) : -1;
+        const int32_t v = i < ns ? __ldcg(&(np ? a.L[1] : a.L[0])[base + i]) : -1;
         const int64_t s = v >= 0 ? ld_ro(a.row_ptr + v) : 0, e = v >= 0 ? ld_ro(a.row_ptr + v + 1) : 0;
         bool conf;
         const int32_t tent = group_scan<TB>(a, Cj, v, s, e, gl, gmask, false, conf);
         if (v >= 0 && gl == 0) Nj[v] = tent;
       }
       for (int64_t i = gw; i < nbg; i += nw) {
-        const int32_t v = __ldcg(&a.L[np][top - 1 - i]);
+        const int32_t v = __ldcg(&(np ? a.L[1] : a.L[0])[top - 1 - i]);
         const int32_t t = warp_fit(a, Cj, ld_ro(a.row_ptr + v), ld_ro(a.row_ptr + v + 1), lane);
         if (lane == 0) Nj[v] = t;
       }
@@ -524,7 +524,7 @@ __global__ void __launch_bounds__(256, 3) k_gs_persistent(Args a) {
         const int32_t pb = __ldg(a.poff + j - 1), pt = __ldg(a.poff + j);
         const int32_t ps = __ldcg(cnt_of(a, np, j - 1, 0)), pg = __ldcg(cnt_of(a, np, j - 1, 1));
         for (int64_t i = tid; i < ps + pg; i += nthr) {
-          const int32_t u = i < ps ? __ldcg(&a.L[np][pb + i]) : __ldcg(&a.L[np][pt - 1 - (i - ps)]);
+          const int32_t u = i < ps ? __ldcg(&(np ? a.L[1] : a.L[0])[pb + i]) : __ldcg(&(np ? a.L[1] : a.L[0])[pt - 1 - (i - ps)]);
           Nj[u] = __ldcg(Cj + u);
         }
       }

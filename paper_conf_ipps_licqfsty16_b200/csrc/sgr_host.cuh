@@ -81,6 +81,7 @@ inline void set_bitmaps(RoundArgs<C>& a, void* ws, const Layout& L, int64_t n) {
   const size_t bmb = align_up((size_t)((n + 31) / 32) * 4, 256);
   a.bm[0] = (uint32_t*)(b + L.off_bm);
   a.bm[1] = (uint32_t*)(b + L.off_bm + bmb);
+  if constexpr (packed<C>()) a.dcol = (int16_t*)a.adj[0];  // unused by the flat build
 }
 
 template <class C>

@@ -218,7 +218,8 @@ struct Ctrl {
   int32_t violations;
   uint32_t xbar;             // cross-part barrier counter (k_persistent_dist; other parts add)
   int32_t cmp_cnt[2];        // bitmap -> worklist compaction (dense -> sparse): bin cursors
-  int32_t pad[2];
+  int32_t dcol_bad;          // k_dense: some w - v does not fit 16 bits (dcol unusable)
+  int32_t pad;
   unsigned long long span_sum;  // F_1: sum over rows of (last - first entry) — row locality
   Counts ring[3];
   unsigned long long edges_acc[3][kBins];    // per ring slot: sum of deg(v) over the pass's
@@ -255,6 +256,8 @@ struct RoundArgs {
   int64_t* fin;               // finalize list: multi-chunk vertices of the pass
                               // (slot << 32 | buf << 31 | v)
   uint32_t* bm[2];            // worklist membership bitmaps (flat build's dense passes): W_k
+  int16_t* dcol;              // dense passes: w - v per CSR entry (aliases adj[0], which only
+                              // the hub build uses), nullptr when unavailable
                               // in bm[k & 1], bit v & 31 of word v >> 5
   Ctrl* ctrl;
   int64_t nnz;
@@ -1939,7 +1942,7 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, const C
 #define SGR_DENSE_SPAN 16  // dense passes only if the mean row width is below n / 16
 #endif
 
-template <int TB, bool Persist, class C>
+template <int TB, bool Persist, class C, bool D16>
 __device__ __forceinline__ void dense_body(const RoundArgs<C>& a, int k, const C* X, C* Y,
                                            uint8_t* wsm, unsigned long long (&edges)[kBins],
                                            unsigned long long (&entries)[kBins],
@@ -1961,23 +1964,29 @@ __device__ __forceinline__ void dense_body(const RoundArgs<C>& a, int k, const C
       const int64_t s = inr ? ldg_i64(a.row_ptr + v) : a.nnz;
       const int64_t e = inr ? ldg_i64(a.row_ptr + v + 1) : a.nnz;
       // the 32 rows are one contiguous segment: its 16-byte-aligned window (capped at the
-      // stage) by asynchronous 16-byte copies, all in flight at once, zero-filled past nnz
-      const int64_t seg0 = __shfl_sync(0xffffffffu, s, 0) & ~(int64_t)3;
+      // stage) by asynchronous 16-byte copies, all in flight at once, zero-filled past nnz.
+      // D16: the segment of dcol (2-byte w - v), half the bytes of col_idx's.
+      constexpr int kE = D16 ? 8 : 4;  // entries per 16-byte copy
+      const int64_t seg0 = __shfl_sync(0xffffffffu, s, 0) & ~(int64_t)(kE - 1);
       const int64_t seg1 = __shfl_sync(0xffffffffu, e, 31);
-      const int32_t nq = (int32_t)min((seg1 - seg0 + 3) >> 2, (int64_t)(kCap / 4));
-      const int32_t len = 4 * nq;  // staged entries [seg0, seg0 + len)
+      const int32_t nq = (int32_t)min((seg1 - seg0 + kE - 1) / kE, (int64_t)(kCap / 4));
+      const int32_t len = kE * nq;  // staged entries [seg0, seg0 + len)
       __syncwarp();
       for (int32_t q = lane; q < nq; q += 32) {
-        const int64_t p0 = seg0 + 4 * q;
-        const uint32_t bytes = (uint32_t)min((int64_t)16, (a.nnz - p0) * 4);
+        const int64_t p0 = seg0 + kE * q;
+        const uint32_t bytes = (uint32_t)min((int64_t)16, (a.nnz - p0) * (16 / kE));
+        const void* src = D16 ? (const void*)(a.dcol + p0) : (const void*)(a.col_idx + p0);
         asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_addr(stage + 4 * q)),
-                     "l"(a.col_idx + p0), "r"(bytes)
+                     "l"(src), "r"(bytes)
                      : "memory");
       }
       asm volatile("cp.async.commit_group;\n cp.async.wait_group 0;" ::: "memory");
       __syncwarp();
       const bool mem = (word >> lane) & 1u;
       bool conf = false;
+      const int16_t* st16 = reinterpret_cast<const int16_t*>(stage);
+      // staged entry i -> neighbour id
+      auto nb = [&](int32_t i) -> int32_t { return D16 ? v + (int32_t)st16[i] : stage[i]; };
       if (mem) {
         const int32_t xv = ldc<Persist>(X + v);
         const int32_t d = (int32_t)(e - s);
@@ -1986,13 +1995,13 @@ __device__ __forceinline__ void dense_body(const RoundArgs<C>& a, int k, const C
         if (d <= 32 && off + d <= len) {  // the whole row is staged: every gather at once
           int32_t c[32];
 #pragma unroll
-          for (int j = 0; j < 32; ++j) c[j] = j < d ? ldc<Persist>(X + stage[off + j]) : 0;
+          for (int j = 0; j < 32; ++j) c[j] = j < d ? ldc<Persist>(X + nb(off + j)) : 0;
           uint32_t m = 0;  // bit c - 1 = color c present (first fit <= 33)
 #pragma unroll
           for (int j = 0; j < 32; ++j) {
             const uint32_t ci = (uint32_t)(c[j] - 1);
             m |= ci < 32u ? (1u << ci) : 0u;
-            if (c[j] == xv && j < d) conf |= lose<TB>(v, stage[off + j]);
+            if (c[j] == xv && j < d) conf |= lose<TB>(v, nb(off + j));
           }
           tent = ~m ? __ffs(~m) : 33;
         } else {  // long or unstaged row: batches of 8, 4 x 64-bit masks (deg <= 256)
@@ -2002,7 +2011,7 @@ __device__ __forceinline__ void dense_body(const RoundArgs<C>& a, int k, const C
 #pragma unroll
             for (int u = 0; u < 8; ++u) {
               const int32_t q = off + j + u;
-              w[u] = j + u < d ? (q < len ? stage[q] : ld_row(a.col_idx + s + j + u)) : -1;
+              w[u] = j + u < d ? (q < len ? nb(q) : ld_row(a.col_idx + s + j + u)) : -1;
             }
 #pragma unroll
             for (int u = 0; u < 8; ++u) c[u] = w[u] >= 0 ? ldc<Persist>(X + w[u]) : 0;
@@ -2024,10 +2033,16 @@ __device__ __forceinline__ void dense_body(const RoundArgs<C>& a, int k, const C
           if (~m0) tent = __ffsll((long long)~m0);
         }
         put_y<C>(a, Y, k, v, conf ? cpack<C>(tent, k + 1, a) : cpack<C>(xv, k, a));
-        const int b = d <= a.small_max ? 0 : 1;
-        edges[b] += (unsigned long long)d;
-        entries[b] += (unsigned long long)d;
-        nxt[b] += conf ? 1 : 0;
+        // constant indices only: a runtime bin index would put the counters on the stack
+        const bool b0 = d <= a.small_max;
+        const unsigned long long d0 = b0 ? (unsigned long long)d : 0ull;
+        const unsigned long long d1 = b0 ? 0ull : (unsigned long long)d;
+        edges[0] += d0;
+        edges[1] += d1;
+        entries[0] += d0;
+        entries[1] += d1;
+        nxt[0] += (conf && b0) ? 1 : 0;
+        nxt[1] += (conf && !b0) ? 1 : 0;
       }
       out = __ballot_sync(0xffffffffu, mem && conf);
     }
@@ -2621,6 +2636,52 @@ __global__ void __launch_bounds__(kMaxThreads<C, Hub>, 1) k_persistent_dist(Roun
 // Dense passes pay only where consecutive vertices have neighbours close in id (meshes):
 // their thread-per-vertex gathers then share lines. 27-point stencil: mean row width ~2 N^2
 // = n / 52 at N = 104; on ER (mean width ~0.9 n) dense passes measured 6.3 -> 7.2 ms.
+#ifndef SGR_DENSE16
+#define SGR_DENSE16 1
+#endif
+// dcol[q] = col_idx[q] - v for every entry q of row v (16 bits; ctrl->dcol_bad if any does
+// not fit). A warp takes 32 consecutive rows (one contiguous segment: the flat build's rows
+// have <= 256 entries, so segment offsets fit 32 bits) and strides over its entries, 8 loads
+// per lane in flight, finding each entry's row by a 5-step binary search over the lanes' row
+// starts: reads and writes coalesced.
+template <class C>
+__device__ __forceinline__ void build_dcol(const RoundArgs<C>& a) {
+  const int lane = threadIdx.x & 31;
+  const int gw = (int)((blockIdx.x * blockDim.x + threadIdx.x) >> 5);
+  const int NW = (int)((gridDim.x * blockDim.x) >> 5);
+  const int nwords = (a.n + 31) >> 5;
+  bool bad = false;
+  for (int g = gw; g < nwords; g += NW) {
+    const int32_t v = (g << 5) + lane;
+    const int64_t S = ldg_i64(a.row_ptr + (g << 5));
+    const int64_t E = ldg_i64(a.row_ptr + min((g << 5) + 32, a.n));
+    const int32_t s = v < a.n ? (int32_t)(ldg_i64(a.row_ptr + v) - S) : INT32_MAX;
+    const int32_t len = (int32_t)(E - S);
+    for (int32_t i0 = 0; i0 < len; i0 += 256) {
+      int32_t w[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const int32_t i = i0 + 32 * u + lane;
+        w[u] = i < len ? ld_ro(a.col_idx + S + i) : 0;
+      }
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const int32_t i = i0 + 32 * u + lane;
+        int L = 0;
+#pragma unroll
+        for (int step = 16; step; step >>= 1)
+          if (__shfl_sync(0xffffffffu, s, L + step) <= i) L += step;
+        if (i < len) {
+          const int32_t d = w[u] - ((g << 5) + L);
+          bad |= d < -32768 || d > 32767;
+          a.dcol[S + i] = (int16_t)d;
+        }
+      }
+    }
+  }
+  if (__any_sync(0xffffffffu, bad) && lane == 0) atomicOr(&a.ctrl->dcol_bad, 1);
+}
+
 template <int TB, class C>
 __global__ void __launch_bounds__(kMaxThreads<C, false>, 1) k_dense(RoundArgs<C> a) {
   extern __shared__ __align__(16) uint8_t dsmem[];
@@ -2634,6 +2695,12 @@ __global__ void __launch_bounds__(kMaxThreads<C, false>, 1) k_dense(RoundArgs<C>
   const int max_rounds = ld_cg(&ctrl->max_rounds);
   const bool leader = blockIdx.x == gridDim.x - 1 && threadIdx.x == 0;
   int k = 2;
+  bool d16 = false;
+  if (SGR_DENSE16 && a.dcol != nullptr) {
+    build_dcol(a);  // once per coloring: ~1.5 col_idx worth of traffic, then half per pass
+    grid_sync(ctrl, epoch);
+    d16 = ld_cg(&ctrl->dcol_bad) == 0;
+  }
   for (;; ++k) {
     const Counts w = ld_counts(&ctrl->ring[rs(k)]);
     const bool dense = items_of(w) > 0 && !ld_cg(&ctrl->overflow) && k <= max_rounds &&
@@ -2644,7 +2711,8 @@ __global__ void __launch_bounds__(kMaxThreads<C, false>, 1) k_dense(RoundArgs<C>
     C* Y = sel(k & 1, a.col[0], a.col[1]);
     unsigned long long edges[kBins] = {0, 0, 0}, entries[kBins] = {0, 0, 0};
     int32_t nx[2] = {0, 0};
-    dense_body<TB, true, C>(a, k, X, Y, wsm, edges, entries, nx);
+    if (d16) dense_body<TB, true, C, true>(a, k, X, Y, wsm, edges, entries, nx);
+    else dense_body<TB, true, C, false>(a, k, X, Y, wsm, edges, entries, nx);
     block_add2(nx, &ctrl->ring[rs(k + 1)].t, &ctrl->ring[rs(k + 1)].m);
     block_add6(edges, entries, ctrl, k);
     grid_sync(ctrl, epoch);

@@ -691,13 +691,24 @@ def local_long_rows(nx, ny, every=997, width=120):
     return gen.from_edges(g.n, np.concatenate(e).astype(np.int64))
 
 
+def far_edges(N=40, gap=33000, every=3001):
+    """A 27-point stencil plus a few edges v -- v + gap with gap > 2^15 - 1: still local on
+    average (dense passes run) but some w - v does not fit the dense passes' 16-bit deltas
+    (dcol), so they must fall back to staging col_idx."""
+    g = gen.stencil3d(N, N, N, 27)
+    src = np.repeat(np.arange(g.n), np.diff(g.row_ptr))
+    extra = np.array([[v, v + gap] for v in range(0, g.n - gap, every)], np.int64)
+    return gen.from_edges(g.n, np.concatenate([np.stack([src, g.col_idx], 1), extra]))
+
+
 @pytest.mark.parametrize("maker", [
     lambda: gen.stencil3d(40, 40, 40, 27),
     lambda: gen.stencil3d(37, 35, 33, 7),
     lambda: gen.stencil2d(401, 299, 5),
     lambda: gen.stencil2d(250, 250, 9),
     lambda: local_long_rows(300, 301),
-], ids=["s27-40", "s7-odd", "s5-odd", "s9-250", "long-rows"])
+    lambda: far_edges(),
+], ids=["s27-40", "s7-odd", "s5-odd", "s9-250", "long-rows", "far-edges"])
 @pytest.mark.parametrize("tb", [LOW, PAP])
 def test_dense_passes_of_the_flat_build(maker, tb):
     """Graphs with local rows (mean row width < n/16) run their first rounds as dense passes
