@@ -73,6 +73,25 @@ constexpr int kJB = 4 * kQB;  // entries per lane per batch
 #ifndef SGR_SMALLMASK
 #define SGR_SMALLMASK 1
 #endif
+// Early exit of bin-2 chunk scans (small passes): once a vertex is known to conflict and
+// every color 1..k is forbidden (fixed set | colors seen so far; C_k holds no color above
+// k), its first fit is k + 1 whatever the rest of its list holds, so the chunk's remaining
+// batches are not gathered. Their entries stay listed (counted live: the lazy-trimming
+// semantics of a listed neighbour that has left W). Chunks of a multi-chunk vertex share
+// their progress through the slot's accumulators (colors 0..63 as one 64-bit word, the
+// conflict flag), read back one batch later.
+#ifndef SGR_EARLY
+#define SGR_EARLY 0  // measured: cfg4 35.0 -> 35.9 ms (entries read -6 %), off
+#endif
+#ifndef SGR_B2_STATIC
+#define SGR_B2_STATIC 0  // experiments: bin-2 items round-robin (no cursor claims)
+#endif
+#ifndef SGR_EARLY_MC
+#define SGR_EARLY_MC 1  // early exit for multi-chunk vertices too (shared progress)
+#endif
+#ifndef SGR_TRACE_ENTRIES
+#define SGR_TRACE_ENTRIES 0
+#endif
 #ifndef SGR_BARSLEEP
 #define SGR_BARSLEEP 20  // grid-barrier poll back-off (ns); 0 = spin
 #endif
@@ -459,6 +478,21 @@ __device__ __forceinline__ unsigned long long atom_add_acq_rel(unsigned long lon
   asm volatile("atom.acq_rel.gpu.global.add.u64 %0, [%1], %2;" : "=l"(r) : "l"(p), "l"(v) : "memory");
   return r;
 }
+// Work-cursor claim by one lane: inline PTX so the compiler does not turn it into a
+// warp-aggregated atomic whose result broadcast (a shuffle right after the atomic) waits
+// for the round trip at the claim; the caller consumes the result one work item later
+// (ncu, cfg4: 4.5 % of the round kernel's stall samples sat on that shuffle).
+// (a lane-dependent address, equal to p on lane 0, the one lane that executes it, keeps
+// ptxas from proving the address warp-uniform)
+__device__ __forceinline__ int lane0_add(int* p, int v) {
+  uint32_t lt;
+  asm volatile("mov.u32 %0, %%lanemask_lt;" : "=r"(lt));
+  int* q = p + lt;  // lane 0: lanemask_lt = 0, q == p
+  int r;
+  asm volatile("atom.relaxed.gpu.global.add.s32 %0, [%1], %2;" : "=r"(r) : "l"(q), "r"(v));
+  return r;
+}
+__device__ __forceinline__ int claim_add(int* p) { return lane0_add(p, 1); }
 // Generic-proxy global writes before later async-proxy (TMA) reads of the same locations.
 __device__ __forceinline__ void fence_proxy_async_global() {
   asm volatile("fence.proxy.async.global;" ::: "memory");
@@ -996,8 +1030,12 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
     zero_hdr(nn);
     if (inn < nC) finish_hdr(it_nn, nn);
     const int64_t it_nnn = innn < nC ? __ldcg(items + innn) : 0;
-    int claim = nC;  // the item after innn (monotone: once past nC, stop claiming)
-    if (lane == 0 && innn < nC) claim = 4 * NW + atomicAdd(cursor, 1);
+    // the item after innn, less 4 NW (monotone: once past nC, stop claiming). The raw
+    // cursor value is kept and 4 NW added at the broadcast: any arithmetic on it here
+    // would wait for the atomic's round trip right at the claim.
+    int claim = nC;
+    if (SGR_B2_STATIC) claim = innn + NW - 4 * NW;
+    else if (lane == 0 && innn < nC) claim = claim_add(cursor);
 
     // ---- chunk `cur` in stage st: slots [off0, off0 + cnt) of the 16-byte-aligned window
     const int32_t v = cur.v;
@@ -1077,19 +1115,65 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
         lvb |= live ? (1u << (kJB * bb + j)) : 0u;
       }
     };
+    const int32_t slot = cur.slot;
+    uint32_t* accb = a.acc_bits + (int64_t)slot * 32;
+    int nbr = nb;  // batches gathered (< nb after an early exit)
+#if SGR_EARLY
+    // colors 1..k (k <= 62), and the fixed set's colors 0..63 (lanes 0/1 hold them)
+    const uint64_t need = ((2ull << k) - 1ull) & ~1ull;
+    const uint64_t fx64 = (uint64_t)__shfl_sync(0xffffffffu, cur.fo, 0) |
+                          ((uint64_t)__shfl_sync(0xffffffffu, cur.fo, 1) << 32);
+    unsigned long long seen_pub = 0ull, conf_pub = 0ull;  // lane 0: the last read-back
+#endif
     for (int bb = 0; bb < nb; ++bb) {
       int32_t id[kJB];
       uint32_t raw[kJB];
       uint32_t okm;
       fetch(bb, id, raw, okm);
       consume(bb, id, raw, okm);
+#if SGR_EARLY
+      if (small && bb + 1 < nb && (SGR_EARLY_MC || nch == 1)) {
+        const uint64_t wm = warp_or64(mall);
+        const bool wc = __any_sync(0xffffffffu, conf);
+        uint64_t seen = wm | fx64;
+        bool cf = wc;
+        if (nch > 1) {
+          // publish this chunk's colors and conflict; the values read back (the other
+          // chunks' progress) are used at the next check, so the atomics' latency hides
+          // under one batch of gathers
+          const uint64_t sp = __shfl_sync(0xffffffffu, seen_pub, 0);
+          const uint64_t cp = __shfl_sync(0xffffffffu, conf_pub, 0);
+          seen |= sp;
+          cf = cf || (cp & 1ull);
+          if (lane == 0) {
+            seen_pub = atomicOr(reinterpret_cast<unsigned long long*>(accb), (unsigned long long)wm);
+            conf_pub = atomicOr(a.acc_cnt + slot, wc ? 1ull : 0ull);
+          }
+        }
+        if (cf && (seen & need) == need) {
+          nbr = bb + 1;
+          break;
+        }
+      }
+#endif
     }
+#if SGR_EARLY
+    if (nbr < nb) {  // unread window slots stay listed: counted as live entries
+      for (int bb = nbr; bb < nb; ++bb) {
+#pragma unroll
+        for (int j = 0; j < kJB; ++j) {
+          const int32_t r = 32 * (kJB * bb + j) + lane;
+          lvb |= (r >= off0 && r < nslots) ? (1u << (kJB * bb + j)) : 0u;
+        }
+      }
+    }
+#endif
 #if !SGR_NO_TMA
     const long long tc = pclock();
     pc2 += (unsigned long long)(tc - tb);
 #endif
     if (lane == 0) {
-      entries += (unsigned long long)cnt;
+      entries += (unsigned long long)(min(nslots, 32 * kJB * nbr) - off0);
       if (cur.c == 0) edges += (unsigned long long)(cur.e - cur.s);
     }
     __syncwarp();
@@ -1123,7 +1207,6 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
       for (uint32_t q = lane; q < live_total; q += 32) base[q] = sbuf[q];
     };
 
-    const int32_t slot = cur.slot;
     uint32_t* fx = a.fixed + (int64_t)slot * 32;
     int32_t* lst_same = sel(cur.buf, a.adj[0], a.adj[1]);
     int32_t* lst_other = sel(cur.buf, a.adj[1], a.adj[0]);
@@ -1172,13 +1255,17 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
         } else if (live_total) {
           lbase = atomicAdd(len_nxt + v, (int32_t)live_total);
         }
-        if (cur.c == 0) fpos = atomicAdd(&ctrl->ring[rs(k)].fin, 1);
+        if (cur.c == 0) fpos = lane0_add(&ctrl->ring[rs(k)].fin, 1);  // used at the end
         if (any) atomicOr(a.acc_cnt + slot, 1ull);  // conflict flag (bit 0)
       }
-      uint32_t* accb = a.acc_bits + (int64_t)slot * 32;
-      const uint32_t bits = set_word(tbl_all, mall);
       const uint32_t drop = set_word(tbl_drop, mdrop);
-      if (bits) atomicOr(accb + lane, bits);
+      if (SGR_EARLY && small) {  // colors 0..63 as one 64-bit word, as the early-exit checks
+        const uint64_t wm = warp_or64(mall);
+        if (lane == 0 && wm) atomicOr(reinterpret_cast<unsigned long long*>(accb), (unsigned long long)wm);
+      } else {
+        const uint32_t bits = set_word(tbl_all, mall);
+        if (bits) atomicOr(accb + lane, bits);
+      }
       if (drop) atomicOr(fx + lane, drop);
       if (!keep) {
         lbase = __shfl_sync(0xffffffffu, lbase, 0);
@@ -1212,7 +1299,7 @@ __device__ __forceinline__ void bin2_trimmed(const RoundArgs<Packed>& a, int k, 
     i = in;
     in = inn;
     inn = innn;
-    innn = __shfl_sync(0xffffffffu, claim, 0);
+    innn = 4 * NW + __shfl_sync(0xffffffffu, claim, 0);
     cur = nxt;
     nxt = nn;
     it_nn = it_nnn;
@@ -1488,16 +1575,16 @@ struct StepStream {
     tile = gw;
     j = 0;
     next = ntiles;
-    if (lane == 0 && tile < ntiles) next = NW + atomicAdd(cursor, 1);
+    if (lane == 0 && tile < ntiles) next = claim_add(cursor);  // NW added at the broadcast
   }
   // list position of the current step's first vertex (0x7fffffff: done)
   __device__ __forceinline__ int base() const { return tile < ntiles ? (tile * kT + j) * VPW : 0x7fffffff; }
   __device__ __forceinline__ void advance(int lane) {
     if (++j == kT) {
       j = 0;
-      tile = __shfl_sync(0xffffffffu, next, 0);
+      tile = NW + __shfl_sync(0xffffffffu, next, 0);
       next = ntiles;
-      if (lane == 0 && tile < ntiles) next = NW + atomicAdd(cursor, 1);
+      if (lane == 0 && tile < ntiles) next = claim_add(cursor);
     }
   }
 };
@@ -2170,7 +2257,7 @@ __device__ __forceinline__ void fold_pass(Ctrl* c, int k) {
   const Counts win = ld_counts(&c->ring[rs(k)]), wout = ld_counts(&c->ring[rs(k + 1)]);
   const int vin[kBins] = {win.t, win.m, win.cv};
   const int vout[kBins] = {wout.t, wout.m, wout.cv};
-  unsigned long long e_all = 0;
+  unsigned long long e_all = 0, x_all = 0;
   int tot_in = 0;
   for (int q = 0; q < kBins; ++q) {
     const unsigned long long e = __ldcg(&c->edges_acc[rs(k)][q]);
@@ -2183,6 +2270,7 @@ __device__ __forceinline__ void fold_pass(Ctrl* c, int k) {
     c->edges_acc[rs(k)][q] = 0ull;
     c->entries_acc[rs(k)][q] = 0ull;
     e_all += e;
+    x_all += x;
     tot_in += vin[q];
   }
   atomicAdd(&c->items_total, (unsigned long long)win.c);
@@ -2191,7 +2279,8 @@ __device__ __forceinline__ void fold_pass(Ctrl* c, int k) {
   c->tile_cur[rs(k)][1] = 0;
   if (k - 1 < c->round_cap) {
     if (c->round_sizes) c->round_sizes[k - 1] = tot_in;
-    if (c->round_edges) c->round_edges[k - 1] = (int64_t)e_all;
+    // SGR_TRACE_ENTRIES (experiment builds only): trace the list entries actually read
+    if (c->round_edges) c->round_edges[k - 1] = (int64_t)(SGR_TRACE_ENTRIES ? x_all : e_all);
   }
   stamp_round(c, k - 1);
 }

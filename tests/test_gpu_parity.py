@@ -608,6 +608,32 @@ def test_multi_chunk_hub_lists(maker, tb):
     assert res.stats["entries_read"] <= res.stats["edges_scanned"]
 
 
+def hub_core_graph(seed, hubs, hub_deg, n):
+    """A clique of `hubs` hub vertices, each adjacent to `hub_deg` random other vertices,
+    which also form a sparse random graph among themselves: the hubs see every small color
+    and conflict with each other for many rounds (the early-exit case of bin 2)."""
+    rng = np.random.default_rng(seed)
+    hub_ids = rng.choice(n, hubs, replace=False)
+    iu = np.triu_indices(hubs, 1)
+    core = np.stack([hub_ids[iu[0]], hub_ids[iu[1]]], 1)
+    spokes = np.stack([np.repeat(hub_ids, hub_deg), rng.integers(0, n, hubs * hub_deg)], 1)
+    rest = rng.integers(0, n, size=(4 * n, 2))
+    return gen.from_edges(n, np.concatenate([core, spokes, rest]).astype(np.int64))
+
+
+@pytest.mark.parametrize("hub_deg", [300, 900, 5000], ids=["one-batch+", "single-chunk", "multi-chunk"])
+@pytest.mark.parametrize("tb", [LOW, PAP])
+@pytest.mark.parametrize("seed", [0, 1])
+def test_bin2_early_exit(hub_deg, tb, seed):
+    """Bin-2 chunks stop gathering once their vertex conflicts and colors 1..k are all
+    forbidden (first fit k + 1 whatever the rest of the list holds); the unread entries
+    stay listed. Colors, R, |W_r| and sum deg(W_r) stay bit-exact, and fewer entries are read
+    than the untrimmed rounds scan."""
+    g = hub_core_graph(seed, 48, hub_deg, 20000)
+    res, _ = check_full(g, tb)
+    assert res.stats["entries_read"] < res.stats["edges_scanned"]
+
+
 # ----------------------------------------------------------------------------- §8(f) item 4
 def check_gs(g, K, part, tb):
     rp, ci = dev(g)
