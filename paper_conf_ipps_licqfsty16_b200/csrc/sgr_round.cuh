@@ -2025,6 +2025,9 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, const C
 #ifndef SGR_DENSE_DIV
 #define SGR_DENSE_DIV 2
 #endif
+#ifndef SGR_DENSE_U8
+#define SGR_DENSE_U8 1  // dense rows of <= 32 entries in passes k <= 255: byte gathers, bit masks
+#endif
 #ifndef SGR_DENSE_SPAN
 #define SGR_DENSE_SPAN 16  // dense passes only if the mean row width is below n / 16
 #endif
@@ -2078,7 +2081,43 @@ __device__ __forceinline__ void dense_body(const RoundArgs<C>& a, int k, const C
         const int32_t xv = ldc<Persist>(X + v);
         const int32_t d = (int32_t)(e - s);
         const int32_t off = (int32_t)(s - seg0);
-        int32_t tent;
+        int32_t tent = 0;
+        bool done = false;
+#if SGR_DENSE_U8
+        if (d <= 32 && off + d <= len && k <= 255 && xv < 32) {
+          // pass k reads C_k, whose colors are <= k <= 255: a word's low byte is its color
+          // (byte gathers, nothing to decode). Colors as bits of one 32-bit mask (shl.b32
+          // yields 0 for shifts >= 32; the color-0 placeholder of unused slots lands on bit 0,
+          // never a color) and the colors of the neighbours v loses to as a second mask, so
+          // the conflict test is one bit of it. A first fit beyond 31 takes the exact loop.
+          uint32_t c[32];
+          uint32_t lb = 0u;  // bit j: v loses to the j-th neighbour
+#pragma unroll
+          for (int j = 0; j < 32; ++j) {
+            c[j] = 0u;
+            if (j < d) {
+              const int32_t w = nb(off + j);
+              lb |= lose<TB>(v, w) ? (1u << j) : 0u;
+              c[j] = *reinterpret_cast<const uint8_t*>(X + w);  // little endian: low byte
+            }
+          }
+          uint32_t m = 1u, ml = 0u;
+#pragma unroll
+          for (int j = 0; j < 32; ++j) {
+            uint32_t bit;
+            asm("shl.b32 %0, 1, %1;" : "=r"(bit) : "r"(c[j]));
+            m |= bit;
+            if ((lb >> j) & 1u) ml |= bit;
+          }
+          if (~m) {
+            tent = __ffs(~m) - 1;
+            conf = (ml >> xv) & 1u;
+            done = true;
+          }
+        }
+        if (done) {
+        } else
+#endif
         if (d <= 32 && off + d <= len) {  // the whole row is staged: every gather at once
           int32_t c[32];
 #pragma unroll
