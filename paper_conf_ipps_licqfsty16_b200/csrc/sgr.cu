@@ -290,6 +290,7 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
   }
   const int grid = round_grid<TB, C>(persistent, B);
   const int grid_flat = persistent ? round_grid<TB, C, false>(true, B) : grid;
+  const int grid_flat_t0 = persistent ? round_grid<TB, C, false, true>(true, B) : grid;
   const int grid_dense = persistent && a.bm[0] ? dense_grid<TB, C>(B) : 0;
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
   sgr_status status = SGR_OK;
@@ -375,8 +376,12 @@ static sgr_status run_color(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t*
           cfg.dynamicSmemBytes = round_smem<C, false>(B);
           le = cudaLaunchKernelEx(&cfg, k_persistent<TB, C, false>, a);
         }
+        if (le == cudaSuccess) {  // flat build, thread-per-vertex bin 0 (flat_thread_bin0)
+          cfg.gridDim = dim3(grid_flat_t0);
+          le = cudaLaunchKernelEx(&cfg, k_persistent<TB, C, false, true>, a);
+        }
       });
-      launches += grid_dense > 0 ? 3 : 2;
+      launches += grid_dense > 0 ? 4 : 3;
       if (le != cudaSuccess) {
         status = cuda_fail(le, "cooperative launch of k_persistent", __LINE__);
         break;

@@ -146,7 +146,7 @@ template <class C, bool Hub = true>
 constexpr int round_max_block() { return kMaxThreads<C, Hub>; }
 
 // Blocks of the round kernels: as many as are co-resident (persistent: required).
-template <int TB, class C, bool Hub = true>
+template <int TB, class C, bool Hub = true, bool T0 = false>
 inline int round_grid(bool persistent, int B = kBlock) {
   // The > 48 KB dynamic shared memory opt-in is a per-device function attribute: one bit
   // per device (setting it twice from racing threads is harmless; the bit only skips the
@@ -159,7 +159,7 @@ inline int round_grid(bool persistent, int B = kBlock) {
     // the opt-in covers the largest block the build accepts
     const int smax = (int)round_smem<C, Hub>(round_max_block<C, Hub>());
     const cudaError_t e1 = cudaFuncSetAttribute(
-        k_persistent<TB, C, Hub>, cudaFuncAttributeMaxDynamicSharedMemorySize, smax);
+        k_persistent<TB, C, Hub, T0>, cudaFuncAttributeMaxDynamicSharedMemorySize, smax);
     const cudaError_t e2 = cudaFuncSetAttribute(
         k_round<TB, C, Hub>, cudaFuncAttributeMaxDynamicSharedMemorySize, smax);
     if (e1 == cudaSuccess && e2 == cudaSuccess && bit) attr_set.fetch_or(bit, std::memory_order_acq_rel);
@@ -167,7 +167,7 @@ inline int round_grid(bool persistent, int B = kBlock) {
   }
   int per_sm = 0;
   cudaError_t e = persistent
-      ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_persistent<TB, C, Hub>, B,
+      ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_persistent<TB, C, Hub, T0>, B,
                                                       round_smem<C, Hub>(B))
       : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_round<TB, C, Hub>, B,
                                                       round_smem<C, Hub>(B));

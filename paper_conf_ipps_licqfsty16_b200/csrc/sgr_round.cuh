@@ -107,6 +107,12 @@ constexpr int kJB = 4 * kQB;  // entries per lane per batch
 #ifndef SGR_BIN0_THREAD
 #define SGR_BIN0_THREAD 0  // bin 0: one thread per vertex (else 4-lane groups)
 #endif
+#ifndef SGR_DENSE_SPAN
+#define SGR_DENSE_SPAN 16  // dense passes only if the mean row width is below n / 16
+#endif
+#ifndef SGR_FLAT_B0T
+#define SGR_FLAT_B0T 1  // flat build, non-local rows: thread-per-vertex bin 0 (runtime choice)
+#endif
 
 namespace sgr {
 
@@ -1897,7 +1903,7 @@ __device__ __forceinline__ void bin1_tiled(const RoundArgs<C>& a, int k, const i
 // One fused pass F_k over all three bins; every warp of the grid calls it. Static
 // round-robin assignment (warp w takes items w, w + NW, ...), with the next item's list
 // entry and row offsets prefetched while the current one is processed.
-template <int TB, bool Persist, class C, bool Hub>
+template <int TB, bool Persist, class C, bool Hub, bool T0 = false>
 __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, const Counts& w,
                                            uint8_t* wsm,
                                            unsigned long long (&edges)[kBins],
@@ -1971,11 +1977,20 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, const C
           a, k, sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]),
           w.t, sel(p ^ 1, a.wl_t[0], a.wl_t[1]), &ctrl->ring[rs(k + 1)].t, X, Y,
           wsm, gw, NW, lane, edges[0], entries[0]);
-    else if constexpr (!Hub)
-      bin0_tiled<TB, Persist, C, Hub>(
-          a, k, sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]), w.t,
-          &ctrl->tile_cur[rs(k)][0], sel(p ^ 1, a.wl_t[0], a.wl_t[1]),
-          &ctrl->ring[rs(k + 1)].t, X, Y, wsm, gw, NW, lane, edges[0], entries[0]);
+    else if constexpr (!Hub) {
+      // T0 (a separate instantiation of the flat build, so the two bin-0 mappings do not
+      // share one register allocation): thread per vertex, a lane's whole row in flight
+      if constexpr (T0)
+        bin0_thread<TB, Persist, C, Hub>(
+            a, k, sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]),
+            w.t, sel(p ^ 1, a.wl_t[0], a.wl_t[1]), &ctrl->ring[rs(k + 1)].t, X, Y,
+            wsm, gw, NW, lane, edges[0], entries[0]);
+      else
+        bin0_tiled<TB, Persist, C, Hub>(
+            a, k, sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]), w.t,
+            &ctrl->tile_cur[rs(k)][0], sel(p ^ 1, a.wl_t[0], a.wl_t[1]),
+            &ctrl->ring[rs(k + 1)].t, X, Y, wsm, gw, NW, lane, edges[0], entries[0]);
+    }
     else
       bin0<TB, Persist, C, Hub>(
           a, k, sel(p, (const int32_t*)a.wl_t[0], (const int32_t*)a.wl_t[1]),
@@ -2027,9 +2042,6 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, const C
 #endif
 #ifndef SGR_DENSE_U8
 #define SGR_DENSE_U8 1  // dense rows of <= 32 entries in passes k <= 255: byte gathers, bit masks
-#endif
-#ifndef SGR_DENSE_SPAN
-#define SGR_DENSE_SPAN 16  // dense passes only if the mean row width is below n / 16
 #endif
 
 template <int TB, bool Persist, class C, bool D16>
@@ -2544,11 +2556,26 @@ __device__ __forceinline__ void grid_sync(Ctrl* ctrl, uint32_t& epoch) {
 // the totals while pass k runs. The host enqueues both builds; each returns at once unless
 // it is the right one for this coloring (Hub iff F_1 put a vertex into bin 2), so the
 // choice needs no host round trip.
-template <int TB, class C, bool Hub>
+// Flat build, bin-0 mapping: graphs with non-local rows (F_1's mean row width >= n / 16:
+// ER-like, the graphs that get no dense passes) and a color array beyond ~8 MB take the
+// thread-per-vertex instantiation (T0; cfg3 ER 2^24 -6 %): a lane's whole row in flight at
+// once covers the L2 latency of scattered gathers. Local rows keep the 4-lane groups, whose
+// gathers share lines (stencil +4 % with threads), as do small graphs whose colors stay
+// near (rmat-er s20 +5 %). Uniform over the grid; read after F_1 (same stream).
+template <class C>
+__device__ __forceinline__ bool flat_thread_bin0(const RoundArgs<C>& a) {
+  return SGR_FLAT_B0T && a.bm[0] != nullptr && a.n >= (1 << 22) &&
+         __ldcg(&a.ctrl->span_sum) > (unsigned long long)a.n * (unsigned long long)a.n / SGR_DENSE_SPAN;
+}
+
+template <int TB, class C, bool Hub, bool T0 = false>
 __global__ void __launch_bounds__(kMaxThreads<C, Hub>, 1) k_persistent(RoundArgs<C> a) {
   extern __shared__ __align__(16) uint8_t dsmem[];
   Ctrl* ctrl = a.ctrl;
   if ((ld_cg(&ctrl->big_count) != 0) != Hub) return;  // uniform across the grid
+  if constexpr (!Hub) {
+    if (flat_thread_bin0(a) != T0) return;  // the other flat instantiation runs
+  }
   if (!ld_cg(&ctrl->active)) return;                   // F_1 left W_2 empty
   uint8_t* wsm = warp_smem_init<C, Hub>(dsmem);
   uint32_t ph = 0;  // mbarrier phase bits of the warp's two TMA stages
@@ -2575,7 +2602,7 @@ __global__ void __launch_bounds__(kMaxThreads<C, Hub>, 1) k_persistent(RoundArgs
       break;
     }
     unsigned long long edges[kBins] = {0, 0, 0}, entries[kBins] = {0, 0, 0};
-    round_body<TB, true, C, Hub>(a, k, w, wsm, edges, entries, ph, cyc);
+    round_body<TB, true, C, Hub, T0>(a, k, w, wsm, edges, entries, ph, cyc);
     const long long t0 = pclock();
     block_add6(edges, entries, ctrl, k);
     const long long t1 = pclock();
