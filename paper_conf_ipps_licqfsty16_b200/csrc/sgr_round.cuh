@@ -110,6 +110,9 @@ constexpr int kJB = 4 * kQB;  // entries per lane per batch
 #ifndef SGR_DENSE_SPAN
 #define SGR_DENSE_SPAN 16  // dense passes only if the mean row width is below n / 16
 #endif
+#ifndef SGR_SMALL_U8
+#define SGR_SMALL_U8 1  // bin 0 (4-lane groups), passes k <= 255: byte gathers + shl masks
+#endif
 #ifndef SGR_FLAT_B0T
 #define SGR_FLAT_B0T 1  // flat build, non-local rows: thread-per-vertex bin 0 (runtime choice)
 #endif
@@ -374,6 +377,15 @@ template <bool Persist, bool Hub, class C>
 __device__ __forceinline__ int32_t ldc01(const C* p) {
   if constexpr (Persist && Hub && SGR_HUB01_CG) return cval<C>((uint32_t)__ldcg(p));
   else return cval<C>(ldraw<Persist>(p));
+}
+// The color as a byte: in passes k <= 255 every color of C_k is <= k, so a word's low byte
+// (little endian) is its color — no decode. Same cache path as ldc01.
+template <bool Persist, bool Hub, class C>
+__device__ __forceinline__ uint32_t ldc8(const C* p) {
+  const unsigned char* b = reinterpret_cast<const unsigned char*>(p);
+  if constexpr (Persist && ((Hub && SGR_HUB01_CG) || !SGR_GATHER_CA)) return (uint32_t)__ldcg(b);
+  else if constexpr (Persist) return (uint32_t)*b;
+  else return (uint32_t)__ldg(b);
 }
 
 template <class C>
@@ -1629,20 +1641,53 @@ __device__ __forceinline__ void bin0(const RoundArgs<C>& a, int k, const int32_t
     uint32_t lb = 0;
 #pragma unroll
     for (int u = 0; u < kK0; ++u) lb |= (w[u] >= 0 && lose<TB>(v, w[u])) ? (1u << u) : 0u;
-    int32_t c[kK0];
-#pragma unroll
-    for (int u = 0; u < kK0; ++u) c[u] = (w[u] >= 0) ? ldc01<Persist, Hub>(X + w[u]) : 0;
-    int32_t wn[kK0];
-    load_row(v1, s1, e1, wn);  // next vertex's row, in flight with the gathers above
     bool conf = false;
     uint32_t mask = 0;  // bit i = color i + 1 present (deg <= 32 => first fit <= 33)
+    int32_t wn[kK0];
+    if (SGR_SMALL_U8 && k <= 255) {
+      // byte gathers (ldc8) and a shl.b32 mask: colors >= 32 drop out, the placeholder 0
+      // lands on bit 0. Only a group with every color 1..31 present needs color 32: it
+      // redoes its scan exactly (rare).
+      uint32_t c8[kK0];
 #pragma unroll
-    for (int u = 0; u < kK0; ++u) {
-      mask |= ((uint32_t)(c[u] - 1) < 32u) ? (1u << (c[u] - 1)) : 0u;
-      conf |= (c[u] == xv) & ((lb >> u) & 1u);
+      for (int u = 0; u < kK0; ++u) c8[u] = (w[u] >= 0) ? ldc8<Persist, Hub>(X + w[u]) : 0u;
+      load_row(v1, s1, e1, wn);  // next vertex's row, in flight with the gathers above
+      uint32_t m = 0u;
+#pragma unroll
+      for (int u = 0; u < kK0; ++u) {
+        uint32_t bit;
+        asm("shl.b32 %0, 1, %1;" : "=r"(bit) : "r"(c8[u]));
+        m |= bit;
+        conf |= (c8[u] == (uint32_t)xv) & ((lb >> u) & 1u);
+      }
+#pragma unroll
+      for (int o = G / 2; o > 0; o >>= 1) m |= __shfl_xor_sync(0xffffffffu, m, o);
+      mask = m >> 1;
+      if (__any_sync(0xffffffffu, (mask & 0x7fffffffu) == 0x7fffffffu)) {
+        const bool full = (mask & 0x7fffffffu) == 0x7fffffffu;
+        uint32_t mx = 0u;
+#pragma unroll
+        for (int u = 0; u < kK0; ++u) {
+          const int32_t c = (full && w[u] >= 0) ? ldc01<Persist, Hub>(X + w[u]) : 0;
+          mx |= ((uint32_t)(c - 1) < 32u) ? (1u << (c - 1)) : 0u;
+        }
+#pragma unroll
+        for (int o = G / 2; o > 0; o >>= 1) mx |= __shfl_xor_sync(0xffffffffu, mx, o);
+        if (full) mask = mx;
+      }
+    } else {
+      int32_t c[kK0];
+#pragma unroll
+      for (int u = 0; u < kK0; ++u) c[u] = (w[u] >= 0) ? ldc01<Persist, Hub>(X + w[u]) : 0;
+      load_row(v1, s1, e1, wn);  // next vertex's row, in flight with the gathers above
+#pragma unroll
+      for (int u = 0; u < kK0; ++u) {
+        mask |= ((uint32_t)(c[u] - 1) < 32u) ? (1u << (c[u] - 1)) : 0u;
+        conf |= (c[u] == xv) & ((lb >> u) & 1u);
+      }
+#pragma unroll
+      for (int o = G / 2; o > 0; o >>= 1) mask |= __shfl_xor_sync(0xffffffffu, mask, o);
     }
-#pragma unroll
-    for (int o = G / 2; o > 0; o >>= 1) mask |= __shfl_xor_sync(0xffffffffu, mask, o);
     const bool any = (__ballot_sync(0xffffffffu, conf) & gmask) != 0u;
     if (v >= 0 && gl == 0) {
       const int32_t tent = ~mask ? __ffs(~mask) : 33;
@@ -1707,20 +1752,53 @@ __device__ __forceinline__ void bin0_tiled(const RoundArgs<C>& a, int k, const i
     uint32_t lb = 0;
 #pragma unroll
     for (int u = 0; u < kK0; ++u) lb |= (w[u] >= 0 && lose<TB>(v, w[u])) ? (1u << u) : 0u;
-    int32_t c[kK0];
-#pragma unroll
-    for (int u = 0; u < kK0; ++u) c[u] = (w[u] >= 0) ? ldc01<Persist, Hub>(X + w[u]) : 0;
-    int32_t wn[kK0];
-    load_row(v1, s1, e1, wn);  // next vertex's row, in flight with the gathers above
     bool conf = false;
     uint32_t mask = 0;  // bit i = color i + 1 present (deg <= 32 => first fit <= 33)
+    int32_t wn[kK0];
+    if (SGR_SMALL_U8 && k <= 255) {
+      // byte gathers (ldc8) and a shl.b32 mask: colors >= 32 drop out, the placeholder 0
+      // lands on bit 0. Only a group with every color 1..31 present needs color 32: it
+      // redoes its scan exactly (rare).
+      uint32_t c8[kK0];
 #pragma unroll
-    for (int u = 0; u < kK0; ++u) {
-      mask |= ((uint32_t)(c[u] - 1) < 32u) ? (1u << (c[u] - 1)) : 0u;
-      conf |= (c[u] == xv) & ((lb >> u) & 1u);
+      for (int u = 0; u < kK0; ++u) c8[u] = (w[u] >= 0) ? ldc8<Persist, Hub>(X + w[u]) : 0u;
+      load_row(v1, s1, e1, wn);  // next vertex's row, in flight with the gathers above
+      uint32_t m = 0u;
+#pragma unroll
+      for (int u = 0; u < kK0; ++u) {
+        uint32_t bit;
+        asm("shl.b32 %0, 1, %1;" : "=r"(bit) : "r"(c8[u]));
+        m |= bit;
+        conf |= (c8[u] == (uint32_t)xv) & ((lb >> u) & 1u);
+      }
+#pragma unroll
+      for (int o = G / 2; o > 0; o >>= 1) m |= __shfl_xor_sync(0xffffffffu, m, o);
+      mask = m >> 1;
+      if (__any_sync(0xffffffffu, (mask & 0x7fffffffu) == 0x7fffffffu)) {
+        const bool full = (mask & 0x7fffffffu) == 0x7fffffffu;
+        uint32_t mx = 0u;
+#pragma unroll
+        for (int u = 0; u < kK0; ++u) {
+          const int32_t c = (full && w[u] >= 0) ? ldc01<Persist, Hub>(X + w[u]) : 0;
+          mx |= ((uint32_t)(c - 1) < 32u) ? (1u << (c - 1)) : 0u;
+        }
+#pragma unroll
+        for (int o = G / 2; o > 0; o >>= 1) mx |= __shfl_xor_sync(0xffffffffu, mx, o);
+        if (full) mask = mx;
+      }
+    } else {
+      int32_t c[kK0];
+#pragma unroll
+      for (int u = 0; u < kK0; ++u) c[u] = (w[u] >= 0) ? ldc01<Persist, Hub>(X + w[u]) : 0;
+      load_row(v1, s1, e1, wn);  // next vertex's row, in flight with the gathers above
+#pragma unroll
+      for (int u = 0; u < kK0; ++u) {
+        mask |= ((uint32_t)(c[u] - 1) < 32u) ? (1u << (c[u] - 1)) : 0u;
+        conf |= (c[u] == xv) & ((lb >> u) & 1u);
+      }
+#pragma unroll
+      for (int o = G / 2; o > 0; o >>= 1) mask |= __shfl_xor_sync(0xffffffffu, mask, o);
     }
-#pragma unroll
-    for (int o = G / 2; o > 0; o >>= 1) mask |= __shfl_xor_sync(0xffffffffu, mask, o);
     const bool any = (__ballot_sync(0xffffffffu, conf) & gmask) != 0u;
     if (v >= 0 && gl == 0) {
       const int32_t tent = ~mask ? __ffs(~mask) : 33;
