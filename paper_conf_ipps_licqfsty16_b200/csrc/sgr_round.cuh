@@ -2116,7 +2116,10 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, const C
 #define SGR_DENSE 1
 #endif
 #ifndef SGR_DENSE_DIV
-#define SGR_DENSE_DIV 2
+#define SGR_DENSE_DIV 8  // n/2 before the byte-gather dense rows; n/3, n/4, n/8: 8.74, 8.70, 8.64 ms (cfg2)
+#endif
+#ifndef SGR_DENSE_PF
+#define SGR_DENSE_PF 1
 #endif
 #ifndef SGR_DENSE_U8
 #define SGR_DENSE_U8 1  // dense rows of <= 32 entries in passes k <= 255: byte gathers, bit masks
@@ -2135,14 +2138,32 @@ __device__ __forceinline__ void dense_body(const RoundArgs<C>& a, int k, const C
   int32_t* stage = reinterpret_cast<int32_t*>(wsm);  // the warp's tables + push buffer
   constexpr int kCap = WarpSmem<C, false>::kBytes / 4;
   const int nwords = (a.n + 31) >> 5;
+  // the next word's bitmap word and row offsets are loaded one word ahead (SGR_DENSE_PF):
+  // they head the word's dependency chain (offsets -> staged rows -> gathers)
+  auto ld_word = [&](int g, uint32_t& wd, int64_t& s, int64_t& e) {
+    wd = g < nwords ? __ldcg(bcur + g) : 0u;
+    const int32_t v = (g << 5) + lane;
+    const bool inr = g < nwords && v < a.n;
+    s = inr ? ldg_i64(a.row_ptr + v) : a.nnz;
+    e = inr ? ldg_i64(a.row_ptr + v + 1) : a.nnz;
+  };
+  uint32_t word_n = 0u;
+  int64_t s_n = 0, e_n = 0;
+  if (SGR_DENSE_PF) ld_word(gw, word_n, s_n, e_n);
   for (int g = gw; g < nwords; g += NW) {
-    const uint32_t word = __ldcg(bcur + g);
+    uint32_t word;
+    int64_t s, e;
+    if (SGR_DENSE_PF) {
+      word = word_n;
+      s = s_n;
+      e = e_n;
+      ld_word(g + NW, word_n, s_n, e_n);
+    } else {
+      ld_word(g, word, s, e);
+    }
     uint32_t out = 0u;
     if (word) {
       const int32_t v = (g << 5) + lane;
-      const bool inr = v < a.n;
-      const int64_t s = inr ? ldg_i64(a.row_ptr + v) : a.nnz;
-      const int64_t e = inr ? ldg_i64(a.row_ptr + v + 1) : a.nnz;
       // the 32 rows are one contiguous segment: its 16-byte-aligned window (capped at the
       // stage) by asynchronous 16-byte copies, all in flight at once, zero-filled past nnz.
       // D16: the segment of dcol (2-byte w - v), half the bytes of col_idx's.
