@@ -413,6 +413,22 @@ def test_full_size_configs_bit_exact(cfg):
 
 
 @pytest.mark.slow
+@pytest.mark.parametrize("maker", [
+    lambda: gen.er(1 << 22, 8 << 22, seed=5),
+    lambda: gen.rmat(22, 6, 0.25, 0.25, 0.25, seed=6),
+], ids=["er22", "rmat-er22"])
+@pytest.mark.parametrize("tb", [LOW, PAP])
+def test_flat_thread_bin0(maker, tb):
+    """Non-local rows and n >= 2^22: the flat build's thread-per-vertex instantiation
+    (k_persistent<..., T0>) against the oracle, both rules; the host loop (4-lane groups)
+    agrees too."""
+    g = maker()
+    res, _ = check_full(g, tb)
+    res_h = sgr.color(*dev(g), RULE[tb], loop_mode="host")
+    assert torch.equal(res_h.colors, res.colors)
+
+
+@pytest.mark.slow
 def test_nnz_beyond_2_31_full_size():
     """Row offsets past 2^31 (reading C17): cfg5's shape (R-MAT scale 27) with edge factor 9,
     nnz ~ 2.39e9 > 2^31 (cfg5 itself has 2,125,681,752 entries, just below 2^31), on one GPU
@@ -625,10 +641,11 @@ def hub_core_graph(seed, hubs, hub_deg, n):
 @pytest.mark.parametrize("tb", [LOW, PAP])
 @pytest.mark.parametrize("seed", [0, 1])
 def test_bin2_early_exit(hub_deg, tb, seed):
-    """Bin-2 chunks stop gathering once their vertex conflicts and colors 1..k are all
-    forbidden (first fit k + 1 whatever the rest of the list holds); the unread entries
-    stay listed. Colors, R, |W_r| and sum deg(W_r) stay bit-exact, and fewer entries are read
-    than the untrimmed rounds scan."""
+    """A clique of hubs whose rows span one batch, one chunk or several chunks, seeing every
+    small color: the trimmed bin-2 lists, the finalize merge and (in SGR_EARLY builds) the
+    chunk early exit — stop once the vertex conflicts and colors 1..k are all forbidden, the
+    unread entries staying listed — keep colors, R, |W_r| and sum deg(W_r) bit-exact, with
+    fewer entries read than the untrimmed rounds scan."""
     g = hub_core_graph(seed, 48, hub_deg, 20000)
     res, _ = check_full(g, tb)
     assert res.stats["entries_read"] < res.stats["edges_scanned"]
