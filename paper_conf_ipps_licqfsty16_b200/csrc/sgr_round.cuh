@@ -2118,6 +2118,9 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, const C
 #ifndef SGR_DENSE_DIV
 #define SGR_DENSE_DIV 8  // n/2 before the byte-gather dense rows; n/3, n/4, n/8: 8.74, 8.70, 8.64 ms (cfg2)
 #endif
+#ifndef SGR_DENSE_MAXT
+#define SGR_DENSE_MAXT 768  // k_dense launch bounds (768: 80 registers, 3 blocks of 256 / SM)
+#endif
 #ifndef SGR_DENSE_PF
 #define SGR_DENSE_PF 1
 #endif
@@ -2937,7 +2940,7 @@ __device__ __forceinline__ void build_dcol(const RoundArgs<C>& a) {
 }
 
 template <int TB, class C>
-__global__ void __launch_bounds__(kMaxThreads<C, false>, 1) k_dense(RoundArgs<C> a) {
+__global__ void __launch_bounds__(SGR_DENSE_MAXT, 1) k_dense(RoundArgs<C> a) {
   extern __shared__ __align__(16) uint8_t dsmem[];
   Ctrl* ctrl = a.ctrl;
   if (!SGR_DENSE || a.bm[0] == nullptr) return;
