@@ -117,6 +117,11 @@ typedef struct {
                             default contract: with unsorted rows and this flag 0 the
                             coloring can be improper). opts->validate reports unsorted rows
                             (bit 4) only when this flag is 0. */
+  int32_t flat_bin0;     /* test hook, graphs without rows of degree > bin_med_max (flat
+                            build, persistent loop): bin-0 mapping. 0 = automatic (one
+                            thread per vertex for non-local rows — mean row width >= n/16 —
+                            and n >= 2^22, else 4-lane groups), 1 = 4-lane groups, 2 = one
+                            thread per vertex. Never changes a result. */
 } sgr_opts;
 
 /* Kernel classes (stats->kernel_*): F_1, the fused round pass(es), loop control, final. */

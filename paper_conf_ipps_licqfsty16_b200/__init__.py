@@ -69,7 +69,7 @@ def make_opts(tiebreak="lowid", stream=None, max_rounds=0, loop_mode="auto", col
               bin_small_max=0, bin_med_max=0, validate=False, rounds_per_batch=0,
               profile=False, round_sizes=None, round_edges=None, round_cap=0,
               round_ms=None, color_cap=0, round_ns=None, block_size=0,
-              unsorted_rows=False) -> Opts:
+              unsorted_rows=False, flat_bin0=0) -> Opts:
     o = Opts()
     load().sgr_opts_default(ctypes.byref(o))
     o.tiebreak = _tb(tiebreak)
@@ -90,6 +90,7 @@ def make_opts(tiebreak="lowid", stream=None, max_rounds=0, loop_mode="auto", col
     o.round_ns = round_ns.data_ptr() if round_ns is not None else None
     o.block_size = int(block_size)
     o.unsorted_rows = int(bool(unsorted_rows))
+    o.flat_bin0 = int(flat_bin0)
     return o
 
 

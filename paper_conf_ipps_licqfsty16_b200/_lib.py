@@ -31,7 +31,8 @@ class Opts(ctypes.Structure):
                 ("validate", ctypes.c_int32), ("rounds_per_batch", ctypes.c_int32),
                 ("profile", ctypes.c_int32), ("round_ms", ctypes.c_void_p),
                 ("round_ns", ctypes.c_void_p), ("color_cap", ctypes.c_int32),
-                ("block_size", ctypes.c_int32), ("unsorted_rows", ctypes.c_int32)]
+                ("block_size", ctypes.c_int32), ("unsorted_rows", ctypes.c_int32),
+                ("flat_bin0", ctypes.c_int32)]
 
 
 class Stats(ctypes.Structure):

@@ -88,6 +88,7 @@ Resolved resolve_opts(const sgr_opts* o, int64_t n) {
                                                                          : (int32_t)kColorMask;
   r.block = o->block_size > 0 ? o->block_size : kBlock;
   r.sorted = o->unsorted_rows ? 0 : 1;
+  r.flat_bin0 = (o->flat_bin0 >= 0 && o->flat_bin0 <= 2) ? o->flat_bin0 : 0;
   return r;
 }
 

@@ -125,6 +125,7 @@ inline void build_args(RoundArgs<C>& a, const sgr_csr* csr, int64_t n, int64_t n
   a.small_max = r.small_max;
   a.med_max = r.med_max;
   a.color_cap = r.color_cap;
+  a.flat_bin0 = r.flat_bin0;
 }
 
 // Streaming per-vertex kernels (F_1, unpack, max): one thread per vertex up to 64 blocks

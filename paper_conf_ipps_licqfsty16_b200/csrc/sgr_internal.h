@@ -30,6 +30,7 @@ struct Resolved {
   int64_t* round_ns;
   int block;      // threads per block (opts->block_size; 0 -> 256)
   int sorted;     // rows sorted ascending (F_1 reads one entry per row); 0: whole rows
+  int flat_bin0;  // opts->flat_bin0 test hook: 0 auto, 1 groups, 2 thread per vertex
 };
 
 // Threads-per-block limits (opts->block_size): per-vertex kernels, and the fused round

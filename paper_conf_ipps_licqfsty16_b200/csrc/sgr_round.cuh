@@ -308,6 +308,7 @@ struct RoundArgs {
   // neighbour of v, i.e. replica q will ever read v's color; interior vertices (mask 0) are
   // written to the own replica only. nullptr: broadcast to every replica (> 8 parts).
   const uint8_t* rmask;
+  int32_t flat_bin0;          // opts->flat_bin0: 0 automatic, 1 4-lane groups, 2 thread per vertex
 };
 
 // This part's block group: the whole grid, or (multi-part launch) blocks
@@ -2118,6 +2119,9 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, const C
 #ifndef SGR_DENSE_DIV
 #define SGR_DENSE_DIV 8  // n/2 before the byte-gather dense rows; n/3, n/4, n/8: 8.74, 8.70, 8.64 ms (cfg2)
 #endif
+#ifndef SGR_DENSE_AHEAD
+#define SGR_DENSE_AHEAD 0  // under test
+#endif
 #ifndef SGR_DENSE_MAXT
 #define SGR_DENSE_MAXT 768  // k_dense launch bounds (768: 80 registers, 3 blocks of 256 / SM)
 #endif
@@ -2138,9 +2142,35 @@ __device__ __forceinline__ void dense_body(const RoundArgs<C>& a, int k, const C
   const int NW = (int)((gridDim.x * blockDim.x) >> 5);
   const uint32_t* bcur = a.bm[k & 1];
   uint32_t* bnxt = a.bm[(k + 1) & 1];
-  int32_t* stage = reinterpret_cast<int32_t*>(wsm);  // the warp's tables + push buffer
-  constexpr int kCap = WarpSmem<C, false>::kBytes / 4;
+  int32_t* stage0 = reinterpret_cast<int32_t*>(wsm);  // the warp's tables + push buffer
+  // D16 && SGR_DENSE_AHEAD: two half-size stages; the next word's rows are copied into the
+  // other half before this word is processed, so they land while its gathers run
+  constexpr bool kAh = D16 && SGR_DENSE_AHEAD;
+  constexpr int kCap = WarpSmem<C, false>::kBytes / 4 / (kAh ? 2 : 1);
+  constexpr int kE = D16 ? 8 : 4;  // entries per 16-byte copy
   const int nwords = (a.n + 31) >> 5;
+  // the 32 rows of a word are one contiguous segment: its 16-byte-aligned window (capped at
+  // the stage) by asynchronous 16-byte copies, all in flight at once, zero-filled past nnz.
+  // D16: the segment of dcol (2-byte w - v), half the bytes of col_idx's.
+  auto stage_rows = [&](int64_t s0, int64_t e0, int32_t* dst, int64_t& seg0, int32_t& len) {
+    seg0 = __shfl_sync(0xffffffffu, s0, 0) & ~(int64_t)(kE - 1);
+    const int64_t seg1 = __shfl_sync(0xffffffffu, e0, 31);
+    const int32_t nq = (int32_t)min((seg1 - seg0 + kE - 1) / kE, (int64_t)(kCap / 4));
+    len = kE * nq;  // staged entries [seg0, seg0 + len)
+    for (int32_t q = lane; q < nq; q += 32) {
+      const int64_t p0 = seg0 + kE * q;
+      const uint32_t bytes = (uint32_t)min((int64_t)16, (a.nnz - p0) * (16 / kE));
+      const void* src = D16 ? (const void*)(a.dcol + p0) : (const void*)(a.col_idx + p0);
+      asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_addr(dst + 4 * q)),
+                   "l"(src), "r"(bytes)
+                   : "memory");
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  int half = 0;          // kAh: half holding the current word's rows
+  bool ahead = false;    // kAh: they were staged while the previous word was processed
+  int64_t seg0_a = 0;
+  int32_t len_a = 0;
   // the next word's bitmap word and row offsets are loaded one word ahead (SGR_DENSE_PF):
   // they head the word's dependency chain (offsets -> staged rows -> gathers)
   auto ld_word = [&](int g, uint32_t& wd, int64_t& s, int64_t& e) {
@@ -2167,25 +2197,26 @@ __device__ __forceinline__ void dense_body(const RoundArgs<C>& a, int k, const C
     uint32_t out = 0u;
     if (word) {
       const int32_t v = (g << 5) + lane;
-      // the 32 rows are one contiguous segment: its 16-byte-aligned window (capped at the
-      // stage) by asynchronous 16-byte copies, all in flight at once, zero-filled past nnz.
-      // D16: the segment of dcol (2-byte w - v), half the bytes of col_idx's.
-      constexpr int kE = D16 ? 8 : 4;  // entries per 16-byte copy
-      const int64_t seg0 = __shfl_sync(0xffffffffu, s, 0) & ~(int64_t)(kE - 1);
-      const int64_t seg1 = __shfl_sync(0xffffffffu, e, 31);
-      const int32_t nq = (int32_t)min((seg1 - seg0 + kE - 1) / kE, (int64_t)(kCap / 4));
-      const int32_t len = kE * nq;  // staged entries [seg0, seg0 + len)
-      __syncwarp();
-      for (int32_t q = lane; q < nq; q += 32) {
-        const int64_t p0 = seg0 + kE * q;
-        const uint32_t bytes = (uint32_t)min((int64_t)16, (a.nnz - p0) * (16 / kE));
-        const void* src = D16 ? (const void*)(a.dcol + p0) : (const void*)(a.col_idx + p0);
-        asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_addr(stage + 4 * q)),
-                     "l"(src), "r"(bytes)
-                     : "memory");
+      int32_t* stage = stage0 + (kAh ? half * kCap : 0);
+      int64_t seg0;
+      int32_t len;
+      if (kAh && ahead) {
+        seg0 = seg0_a;
+        len = len_a;
+      } else {
+        __syncwarp();
+        stage_rows(s, e, stage, seg0, len);
       }
-      asm volatile("cp.async.commit_group;\n cp.async.wait_group 0;" ::: "memory");
+      ahead = false;
+      if (kAh && SGR_DENSE_PF && word_n) {  // the next word's rows into the other half
+        stage_rows(s_n, e_n, stage0 + (half ^ 1) * kCap, seg0_a, len_a);
+        ahead = true;
+        asm volatile("cp.async.wait_group 1;" ::: "memory");
+      } else {
+        asm volatile("cp.async.wait_group 0;" ::: "memory");
+      }
       __syncwarp();
+      half ^= kAh ? 1 : 0;
       const bool mem = (word >> lane) & 1u;
       bool conf = false;
       const int16_t* st16 = reinterpret_cast<const int16_t*>(stage);
@@ -2666,7 +2697,9 @@ __device__ __forceinline__ void grid_sync(Ctrl* ctrl, uint32_t& epoch) {
 // near (rmat-er s20 +5 %). Uniform over the grid; read after F_1 (same stream).
 template <class C>
 __device__ __forceinline__ bool flat_thread_bin0(const RoundArgs<C>& a) {
-  return SGR_FLAT_B0T && a.bm[0] != nullptr && a.n >= (1 << 22) &&
+  if (a.bm[0] == nullptr || a.flat_bin0 == 1) return false;
+  if (a.flat_bin0 == 2) return true;
+  return SGR_FLAT_B0T && a.n >= (1 << 22) &&
          __ldcg(&a.ctrl->span_sum) > (unsigned long long)a.n * (unsigned long long)a.n / SGR_DENSE_SPAN;
 }
 

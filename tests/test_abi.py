@@ -60,6 +60,7 @@ def test_host_entry_points_without_gpu():
     o = sgr._lib.Opts()
     lib.sgr_opts_default(ctypes.byref(o))
     assert o.tiebreak == 0 and o.loop_mode == 0
+    assert o.unsorted_rows == 0 and o.flat_bin0 == 0  # last fields: the struct sizes agree
     assert sgr.workspace_bytes(1000, 5000) > 4 * 4 * 1000  # Y, 2 thread lists, slots
     # invalid arguments are rejected before touching the device
     st = sgr._lib.Stats()

@@ -412,6 +412,26 @@ def test_full_size_configs_bit_exact(cfg):
     check_full(g, LOW)
 
 
+@pytest.mark.parametrize("seed", range(16))
+@pytest.mark.parametrize("tb", [LOW, PAP])
+@pytest.mark.parametrize("mapping", [1, 2])
+def test_flat_bin0_mappings_small(seed, tb, mapping):
+    """opts->flat_bin0 forces the flat build's bin-0 mapping (1: 4-lane groups, 2: the
+    thread-per-vertex instantiation) on small graphs of every family: same result."""
+    check_full(random_graph(seed, n=300), tb, flat_bin0=mapping)
+
+
+@pytest.mark.parametrize("maker", [
+    lambda: gen.stencil3d(24, 24, 24, 27),
+    lambda: gen.stencil2d(57, 31, 5),
+    lambda: gen.er(1 << 15, 8 << 15, seed=3),
+    lambda: gen.rmat(14, 10, 0.25, 0.25, 0.25, seed=2),
+], ids=["s27-24", "s5", "er15", "rmat-er14"])
+@pytest.mark.parametrize("tb", [LOW, PAP])
+def test_flat_bin0_thread_families(maker, tb):
+    check_full(maker(), tb, flat_bin0=2)
+
+
 @pytest.mark.slow
 @pytest.mark.parametrize("maker", [
     lambda: gen.er(1 << 22, 8 << 22, seed=5),

@@ -6,7 +6,7 @@
     compute-sanitizer --tool racecheck python tools/sanitize_run.py
 
 Covers: the persistent kernel (hub build with multi-chunk rows and TMA stages, flat build
-with dense and sparse passes), both color widths, the host loop (k_round, k_finalize),
+with dense and sparse passes, both bin-0 mappings of the flat build), both color widths, the host loop (k_round, k_finalize),
 the graph loop, the topology-driven kernels, the step entry points, the sub-step variants
 and the partitioned (multi-GPU protocol) path. Every result is checked against the oracle
 so a run that "passes" the sanitizer also colored correctly.
@@ -54,6 +54,11 @@ def main():
             for mode in ("persistent", "host", "graph"):
                 r = sgr.color(rp, ci, "lowid", color_bits=bits, loop_mode=mode)
                 check(f"{name} color bits={bits} {mode}", r.colors.cpu().numpy(), ref)
+        for mapping in (1, 2):  # flat build: 4-lane groups / thread-per-vertex instantiation
+            r = sgr.color(rp, ci, "lowid", flat_bin0=mapping)
+            check(f"{name} flat_bin0={mapping}", r.colors.cpu().numpy(), ref)
+        r = sgr.color(rp, ci, "paper", flat_bin0=2)
+        check(f"{name} flat_bin0=2 paper", r.colors.cpu().numpy(), oracle.jacobi(g, 1).colors)
         check(f"{name} topo", sgr.color_topo(rp, ci).colors.cpu().numpy(), ref)
         check(f"{name} partitioned P=3", sgr.color_partitioned(rp, ci, 3).colors.cpu().numpy(), ref)
         check(f"{name} gs K=4", sgr.color_gs(rp, ci, 4, "strided").colors.cpu().numpy(),
