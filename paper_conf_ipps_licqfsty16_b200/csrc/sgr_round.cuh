@@ -2122,6 +2122,9 @@ __device__ __forceinline__ void round_body(const RoundArgs<C>& a, int k, const C
 #ifndef SGR_DENSE_AHEAD
 #define SGR_DENSE_AHEAD 1  // next word staged ahead: cfg2 8.49 -> 8.17 ms
 #endif
+#ifndef SGR_DENSE_PF2
+#define SGR_DENSE_PF2 0  // offsets two words ahead: cfg2 8.18 -> 8.16 ms (noise), off
+#endif
 #ifndef SGR_DENSE_MAXT
 #define SGR_DENSE_MAXT 768  // k_dense launch bounds (768: 80 registers, 3 blocks of 256 / SM)
 #endif
@@ -2180,13 +2183,22 @@ __device__ __forceinline__ void dense_body(const RoundArgs<C>& a, int k, const C
     s = inr ? ldg_i64(a.row_ptr + v) : a.nnz;
     e = inr ? ldg_i64(a.row_ptr + v + 1) : a.nnz;
   };
-  uint32_t word_n = 0u;
-  int64_t s_n = 0, e_n = 0;
+  uint32_t word_n = 0u, word_nn = 0u;
+  int64_t s_n = 0, e_n = 0, s_nn = 0, e_nn = 0;
   if (SGR_DENSE_PF) ld_word(gw, word_n, s_n, e_n);
+  if (SGR_DENSE_PF2) ld_word(gw + NW, word_nn, s_nn, e_nn);
   for (int g = gw; g < nwords; g += NW) {
     uint32_t word;
     int64_t s, e;
-    if (SGR_DENSE_PF) {
+    if (SGR_DENSE_PF2) {  // offsets two words ahead: the next word's stage needs them now
+      word = word_n;
+      s = s_n;
+      e = e_n;
+      word_n = word_nn;
+      s_n = s_nn;
+      e_n = e_nn;
+      ld_word(g + 2 * NW, word_nn, s_nn, e_nn);
+    } else if (SGR_DENSE_PF) {
       word = word_n;
       s = s_n;
       e = e_n;
