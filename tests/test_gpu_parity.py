@@ -128,6 +128,25 @@ def test_complete_graphs_large_mex(k):
         assert res.colors.cpu().numpy().tolist() == list(range(1, k + 1))
 
 
+@pytest.mark.parametrize("k", [30, 31, 32])
+@pytest.mark.parametrize("apex_low", [False, True])
+@pytest.mark.parametrize("mapping", [0, 1, 2])
+def test_bin0_colors_beyond_31(k, apex_low, mapping):
+    """A K_k clique plus an apex adjacent to all of it: a row of <= 32 entries whose
+    neighbours end up colored 1..k, so the apex's first fit is k + 1 — past the 31 colors
+    the byte-gather bit masks of bin 0 hold (the exact rescan must take over), in both
+    bin-0 mappings of the flat build and both rules."""
+    n = k + 1
+    apex = 0 if apex_low else k
+    others = [v for v in range(n) if v != apex]
+    edges = [(others[i], others[j]) for i in range(k) for j in range(i + 1, k)]
+    edges += [(apex, v) for v in others]
+    g = gen.from_edges(n, np.asarray(edges, np.int64))
+    for tb in (LOW, PAP):
+        res, _ = check_full(g, tb, flat_bin0=mapping)
+        assert res.stats["num_colors"] == n
+
+
 @pytest.mark.parametrize("seed", range(8))
 def test_self_loops_and_duplicates(seed):
     g = random_graph(seed, n=200)
