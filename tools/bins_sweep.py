@@ -15,7 +15,7 @@ g = gen.config(cfg)
 rp = torch.from_numpy(g.row_ptr).cuda()
 ci = torch.from_numpy(g.col_idx).cuda()
 ref = sgr.color(rp, ci).colors.clone()
-for sm, mm in [(0, 0), (32, 128), (32, 64), (16, 256), (16, 64), (32, 512)]:
+for sm, mm in [(0, 0), (32, 128), (32, 192), (32, 96), (16, 256), (24, 256), (16, 128)]:
     ms = []
     for _ in range(4):
         r = sgr.color(rp, ci, bin_small_max=sm, bin_med_max=mm)
