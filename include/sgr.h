@@ -90,7 +90,8 @@ typedef struct {
                             full rows every round */
   int32_t bin_small_max; /* degree bins: d <= small -> 8 lanes/vertex, register mask (<= 62);
                             0 = 32 */
-  int32_t bin_med_max;   /* small < d <= med -> 8 lanes/vertex, smem table (<= 256); 0 = 256;
+  int32_t bin_med_max;   /* small < d <= med -> 8 lanes/vertex, smem table (<= 256); 0 = 256
+                            (128 when n <= 2^20);
                             d > med -> one warp per 1024-entry aligned chunk of the row */
   void* stream;          /* cudaStream_t; NULL = legacy default stream */
   int32_t* round_sizes;  /* optional DEVICE buffer: |W_r| for r = 1..R (R capped by cap) */

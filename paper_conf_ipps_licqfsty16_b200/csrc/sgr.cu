@@ -73,7 +73,11 @@ Resolved resolve_opts(const sgr_opts* o, int64_t n) {
                     ? o->loop_mode : SGR_LOOP_PERSISTENT;
   r.color_bits = o->color_bits == 32 ? 32 : 16;
   r.small_max = o->bin_small_max > 0 ? std::min(o->bin_small_max, kMaxSmall) : kMaxSmall;
-  r.med_max = o->bin_med_max > 0 ? std::min(o->bin_med_max, kMaxMed) : kMaxMed;
+  // default med_max: 256, or 128 on graphs of <= 2^20 vertices, where the shorter rows
+  // trimmed as bin-2 lists pay (profiles/r02_ncu_summary.md: R-MAT s16 -6.6 %, rmat-g s20
+  // -2.5 %; R-MAT s24 +0.2 % with 128, so large graphs keep 256)
+  r.med_max = o->bin_med_max > 0 ? std::min(o->bin_med_max, kMaxMed)
+                                 : (n <= (int64_t(1) << 20) ? 128 : kMaxMed);
   r.med_max = std::max(r.med_max, r.small_max);
   r.stream = (cudaStream_t)o->stream;
   r.round_sizes = o->round_sizes;
