@@ -451,6 +451,21 @@ def test_flat_bin0_thread_families(maker, tb):
     check_full(maker(), tb, flat_bin0=2)
 
 
+@pytest.mark.parametrize("maker", [
+    lambda: gen.stencil3d(24, 24, 24, 27),
+    lambda: gen.stencil2d(80, 61, 9),
+    lambda: gen.er(1 << 14, 8 << 14, seed=4),
+], ids=["s27-24", "s9", "er14"])
+@pytest.mark.parametrize("mapping", [1, 2])
+@pytest.mark.parametrize("B", [128, 256, 768])
+def test_flat_kernels_int32_words_and_block_sizes(maker, mapping, B):
+    """The flat build's kernels (dense passes with byte gathers of a word's low byte, both
+    bin-0 mappings) with plain int32 color words and other block sizes: same result."""
+    g = maker()
+    for tb in (LOW, PAP):
+        check_full(g, tb, flat_bin0=mapping, color_bits=32, block_size=B)
+
+
 @pytest.mark.slow
 @pytest.mark.parametrize("maker", [
     lambda: gen.er(1 << 22, 8 << 22, seed=5),
