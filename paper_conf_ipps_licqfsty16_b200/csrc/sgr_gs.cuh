@@ -333,6 +333,81 @@ __device__ __forceinline__ int32_t warp_fit(const Args& a, const int32_t* Cur, i
   }
 }
 
+// Huge members (degree > SGR_GS_HUGE): one BLOCK each — its warps take the row's 256-entry
+// tiles in turn (warp w: tiles w, w + nwb, ...), so a hub row is scanned by every warp of a
+// block instead of one (the sub-steps whose part holds a hub used to wait for one warp's
+// serial walk of it). Block-uniform; all threads of the block must call.
+#ifndef SGR_GS_HUGE
+#define SGR_GS_HUGE 2048
+#endif
+template <int TB>
+__device__ __forceinline__ bool block_conflict(const Args& a, const int32_t* Cur, int32_t v, int64_t s,
+                                               int64_t e) {
+  const int lane = threadIdx.x & 31, wi = threadIdx.x >> 5, nwb = blockDim.x >> 5;
+  const int32_t cv = __ldcg(Cur + v);
+  bool c = false;
+  for (int64_t q0 = s + 256 * (int64_t)wi; q0 < e; q0 += 256 * (int64_t)nwb) {
+    int32_t w[8], col[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int64_t q = q0 + 32 * u + lane;
+      w[u] = q < e ? ld_ro(a.col_idx + q) : -1;
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) col[u] = w[u] >= 0 ? __ldcg(Cur + w[u]) : -1;
+#pragma unroll
+    for (int u = 0; u < 8; ++u) c |= w[u] >= 0 && col[u] == cv && lose<TB>(v, w[u]);
+  }
+  return __syncthreads_or(c) != 0;
+}
+// First fit of a huge member, one block: 256-color windows as warp_fit, the warps' window
+// masks merged in shared memory (sm: 4 words, zero on entry and on return).
+__device__ __forceinline__ int32_t block_fit(const Args& a, const int32_t* Cur, int64_t s, int64_t e,
+                                            unsigned long long* sm) {
+  const int lane = threadIdx.x & 31, wi = threadIdx.x >> 5, nwb = blockDim.x >> 5;
+  for (int32_t base = 0;; base += 256) {
+    uint64_t m0 = 0, m1 = 0, m2 = 0, m3 = 0;
+    for (int64_t q0 = s + 256 * (int64_t)wi; q0 < e; q0 += 256 * (int64_t)nwb) {
+      int32_t w[8], c[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const int64_t q = q0 + 32 * u + lane;
+        w[u] = q < e ? ld_ro(a.col_idx + q) : -1;
+      }
+#pragma unroll
+      for (int u = 0; u < 8; ++u) c[u] = w[u] >= 0 ? __ldcg(Cur + w[u]) : 0;
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const uint32_t idx = (uint32_t)(c[u] - base - 1);
+        const uint64_t bit = 1ull << (idx & 63u);
+        m0 |= idx < 64u ? bit : 0ull;
+        m1 |= idx - 64u < 64u ? bit : 0ull;
+        m2 |= idx - 128u < 64u ? bit : 0ull;
+        m3 |= idx - 192u < 64u ? bit : 0ull;
+      }
+    }
+    m0 = warp_or64(m0);
+    m1 = warp_or64(m1);
+    m2 = warp_or64(m2);
+    m3 = warp_or64(m3);
+    if (lane == 0) {
+      if (m0) atomicOr(sm + 0, (unsigned long long)m0);
+      if (m1) atomicOr(sm + 1, (unsigned long long)m1);
+      if (m2) atomicOr(sm + 2, (unsigned long long)m2);
+      if (m3) atomicOr(sm + 3, (unsigned long long)m3);
+    }
+    __syncthreads();
+    const uint64_t t0 = sm[0], t1 = sm[1], t2 = sm[2], t3 = sm[3];
+    __syncthreads();  // every thread has read the merged masks before they are cleared
+    if (threadIdx.x < 4) sm[threadIdx.x] = 0ull;
+    __syncthreads();
+    if (~t0) return base + __ffsll((long long)~t0);
+    if (~t1) return base + 64 + __ffsll((long long)~t1);
+    if (~t2) return base + 128 + __ffsll((long long)~t2);
+    if (~t3) return base + 192 + __ffsll((long long)~t3);
+  }
+}
+
 // Push v (degree d) into round list `par`, region of its part j: low-degree members from
 // the front, the others from the back. Warp-collective (all 32 lanes call; `pred` selects
 // the pushing lanes): lanes with the same (part, kind) share one atomicAdd (the callers
@@ -368,6 +443,9 @@ __device__ __forceinline__ int32_t vertex_at(const Args& a, int64_t p) {
 
 template <int TB>
 __global__ void __launch_bounds__(256, 3) k_gs_persistent(Args a) {
+  __shared__ unsigned long long gs_sm[4];  // block_fit's merged window masks
+  if (threadIdx.x < 4) gs_sm[threadIdx.x] = 0ull;
+  __syncthreads();
   const int lane = threadIdx.x & 31;
   const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
@@ -420,6 +498,26 @@ __global__ void __launch_bounds__(256, 3) k_gs_persistent(Args a) {
         }
       }
     }
+    // huge members: block per vertex (detection; part-0 ones also take their first fit)
+    for (int64_t j = 0; j < a.K; ++j) {
+      const int32_t top = __ldg(a.poff + j + 1);
+      const int32_t nbg = R == 1 ? 0 : __ldcg(cnt_of(a, par, j, 1));
+      for (int64_t i = blockIdx.x; i < nbg; i += gridDim.x) {
+        const int32_t v = __ldcg(&(par ? a.L[1] : a.L[0])[top - 1 - i]);
+        const int64_t s = ld_ro(a.row_ptr + v), e = ld_ro(a.row_ptr + v + 1);
+        if (e - s <= SGR_GS_HUGE) continue;  // block-uniform
+        if (!block_conflict<TB>(a, Cur, v, s, e)) {
+          if (a.K == 1 && threadIdx.x == 0) Nxt[v] = __ldcg(Cur + v);
+          continue;
+        }
+        if (threadIdx.x < 32) push_warp(a, np, v, e - s, lane == 0);
+        if (threadIdx.x == 0) my_edges += (unsigned long long)(e - s);
+        if (j == 0) {
+          const int32_t t = block_fit(a, Cur, s, e, gs_sm);
+          if (threadIdx.x == 0) Nxt[v] = t;
+        }
+      }
+    }
     // big members: warp per vertex (detection; part-0 ones also take their first fit)
     for (int64_t j = 0; j < a.K; ++j) {
       const int32_t top = __ldg(a.poff + j + 1);
@@ -427,6 +525,7 @@ __global__ void __launch_bounds__(256, 3) k_gs_persistent(Args a) {
       for (int64_t i = gw; i < nbg; i += nw) {
         const int32_t v = __ldcg(&(par ? a.L[1] : a.L[0])[top - 1 - i]);
         const int64_t s = ld_ro(a.row_ptr + v), e = ld_ro(a.row_ptr + v + 1);
+        if (e - s > SGR_GS_HUGE) continue;  // the blocks took it
         if (!warp_conflict<TB>(a, Cur, v, s, e, lane)) {
           if (a.K == 1 && lane == 0) Nxt[v] = __ldcg(Cur + v);
           continue;
@@ -466,9 +565,18 @@ __global__ void __launch_bounds__(256, 3) k_gs_persistent(Args a) {
       }
       const int32_t top = __ldg(a.poff + 1);
       const int32_t nbg = __ldcg(cnt_of(a, np, 0, 1));
+      for (int64_t i = blockIdx.x; i < nbg; i += gridDim.x) {  // huge: block per vertex
+        const int32_t v = __ldcg(&(np ? a.L[1] : a.L[0])[top - 1 - i]);
+        const int64_t s = ld_ro(a.row_ptr + v), e = ld_ro(a.row_ptr + v + 1);
+        if (e - s <= SGR_GS_HUGE) continue;
+        const int32_t t = block_fit(a, Cur, s, e, gs_sm);
+        if (threadIdx.x == 0) Nxt[v] = t;
+      }
       for (int64_t i = gw; i < nbg; i += nw) {
         const int32_t v = __ldcg(&(np ? a.L[1] : a.L[0])[top - 1 - i]);
-        const int32_t t = warp_fit(a, Cur, ld_ro(a.row_ptr + v), ld_ro(a.row_ptr + v + 1), lane);
+        const int64_t s = ld_ro(a.row_ptr + v), e = ld_ro(a.row_ptr + v + 1);
+        if (e - s > SGR_GS_HUGE) continue;
+        const int32_t t = warp_fit(a, Cur, s, e, lane);
         if (lane == 0) Nxt[v] = t;
       }
       gsync(ctrl, epoch);
@@ -515,9 +623,18 @@ __global__ void __launch_bounds__(256, 3) k_gs_persistent(Args a) {
         const int32_t tent = group_scan<TB>(a, Cj, v, s, e, gl, gmask, false, conf);
         if (v >= 0 && gl == 0) Nj[v] = tent;
       }
+      for (int64_t i = blockIdx.x; i < nbg; i += gridDim.x) {  // huge: block per vertex
+        const int32_t v = __ldcg(&(np ? a.L[1] : a.L[0])[top - 1 - i]);
+        const int64_t s = ld_ro(a.row_ptr + v), e = ld_ro(a.row_ptr + v + 1);
+        if (e - s <= SGR_GS_HUGE) continue;
+        const int32_t t = block_fit(a, Cj, s, e, gs_sm);
+        if (threadIdx.x == 0) Nj[v] = t;
+      }
       for (int64_t i = gw; i < nbg; i += nw) {
         const int32_t v = __ldcg(&(np ? a.L[1] : a.L[0])[top - 1 - i]);
-        const int32_t t = warp_fit(a, Cj, ld_ro(a.row_ptr + v), ld_ro(a.row_ptr + v + 1), lane);
+        const int64_t s = ld_ro(a.row_ptr + v), e = ld_ro(a.row_ptr + v + 1);
+        if (e - s > SGR_GS_HUGE) continue;
+        const int32_t t = warp_fit(a, Cj, s, e, lane);
         if (lane == 0) Nj[v] = t;
       }
       {  // copy part j-1's members (changed in the previous sub-step) into Nj
