@@ -1012,6 +1012,7 @@ sgr_status sgr_color_gs(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t subs
   ++launches;
   int64_t len = n;
   int cur = 0;
+  int huge = -1;  // in-place mode: any row above SGR_GS_HUGE (unknown yet)
   while (len > 0) {
     if ((int64_t)sizes.size() >= r.max_rounds) {
       status = SGR_ENOCONV;
@@ -1021,7 +1022,19 @@ sgr_status sgr_color_gs(const sgr_csr* csr, int64_t n, int64_t nnz, int32_t subs
     sizes.push_back((int32_t)len);
     const int gw = grid_for(len, B / 32, B);
     if (partition == 2) {
-      k_gs_inplace<<<gw, B, 0, s>>>(csr->row_ptr, csr->col_idx, W[cur], len, colors_out, edges);
+      if (huge < 0) {  // once per call: is any row long enough for the block-level pass?
+        CK(cudaMemsetAsync(kcnt, 0, 4, s));
+        gsp::k_any_huge<<<grid_v, B, 0, s>>>(csr->row_ptr, n, kcnt);
+        int32_t h = 0;
+        CK(cudaMemcpyAsync(&h, kcnt, 4, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        huge = h;
+        ++launches;
+      }
+      if (huge)
+        gsp::k_gs_inplace<true><<<gw, B, 0, s>>>(csr->row_ptr, csr->col_idx, W[cur], len, colors_out, edges);
+      else
+        gsp::k_gs_inplace<false><<<gw, B, 0, s>>>(csr->row_ptr, csr->col_idx, W[cur], len, colors_out, edges);
       ++launches;
     } else {
       // the round's members split once into K contiguous sub-step segments

@@ -25,28 +25,6 @@ __device__ __forceinline__ int64_t gs_part(int64_t v, int64_t n, int64_t K, int 
                         : v % K;
 }
 
-// Paper-faithful in-place assignment (nondeterministic): one warp per listed vertex reads
-// its neighbours' colors from L2 (ld.global.cg: other warps' writes of this launch may or
-// may not be seen) and writes its first fit straight into C.
-static __global__ void __launch_bounds__(1024) k_gs_inplace(const int64_t* __restrict__ row_ptr,
-                                                            const int32_t* __restrict__ col_idx,
-                                                            const int32_t* __restrict__ wl, int64_t len,
-                                                            int32_t* C, unsigned long long* edges) {
-  const int lane = threadIdx.x & 31;
-  const int64_t wpb = blockDim.x >> 5;
-  unsigned long long my = 0;
-  for (int64_t i = (int64_t)blockIdx.x * wpb + (threadIdx.x >> 5); i < len;
-       i += (int64_t)gridDim.x * wpb) {
-    const int32_t v = __ldg(wl + i);
-    const int64_t s = ld_ro(row_ptr + v), e = ld_ro(row_ptr + v + 1);
-    const int32_t t = warp_first_fit_from<true>(col_idx, C, s, e, 0, lane);
-    if (lane == 0) {
-      __stcg(C + v, t);
-      my += (unsigned long long)(e - s);
-    }
-  }
-  block_add(my, edges);
-}
 
 // ---- bucketed sub-steps: each round's worklist is split once into its K sub-step
 // segments (a histogram, an exclusive scan and a scatter), so a sub-step touches only its
@@ -362,8 +340,8 @@ __device__ __forceinline__ bool block_conflict(const Args& a, const int32_t* Cur
 }
 // First fit of a huge member, one block: 256-color windows as warp_fit, the warps' window
 // masks merged in shared memory (sm: 4 words, zero on entry and on return).
-__device__ __forceinline__ int32_t block_fit(const Args& a, const int32_t* Cur, int64_t s, int64_t e,
-                                            unsigned long long* sm) {
+__device__ __forceinline__ int32_t block_fit(const int32_t* __restrict__ col_idx, const int32_t* Cur,
+                                            int64_t s, int64_t e, unsigned long long* sm) {
   const int lane = threadIdx.x & 31, wi = threadIdx.x >> 5, nwb = blockDim.x >> 5;
   for (int32_t base = 0;; base += 256) {
     uint64_t m0 = 0, m1 = 0, m2 = 0, m3 = 0;
@@ -372,7 +350,7 @@ __device__ __forceinline__ int32_t block_fit(const Args& a, const int32_t* Cur, 
 #pragma unroll
       for (int u = 0; u < 8; ++u) {
         const int64_t q = q0 + 32 * u + lane;
-        w[u] = q < e ? ld_ro(a.col_idx + q) : -1;
+        w[u] = q < e ? ld_ro(col_idx + q) : -1;
       }
 #pragma unroll
       for (int u = 0; u < 8; ++u) c[u] = w[u] >= 0 ? __ldcg(Cur + w[u]) : 0;
@@ -406,6 +384,80 @@ __device__ __forceinline__ int32_t block_fit(const Args& a, const int32_t* Cur, 
     if (~t2) return base + 128 + __ffsll((long long)~t2);
     if (~t3) return base + 192 + __ffsll((long long)~t3);
   }
+}
+
+// Paper-faithful in-place assignment (nondeterministic): one warp per listed vertex reads
+// its neighbours' colors from L2 (ld.global.cg: other warps' writes of this launch may or
+// may not be seen) and writes its first fit straight into C; vertices of degree
+// > SGR_GS_HUGE take a whole block (block_fit), as in the sub-step kernel.
+// Any row longer than SGR_GS_HUGE (selects the in-place kernel's instantiation once per call).
+static __global__ void k_any_huge(const int64_t* __restrict__ row_ptr, int64_t n, int32_t* flag) {
+  for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+    if (ld_ro(row_ptr + v + 1) - ld_ro(row_ptr + v) > SGR_GS_HUGE) *flag = 1;
+}
+
+template <bool Huge>
+static __global__ void __launch_bounds__(1024) k_gs_inplace(const int64_t* __restrict__ row_ptr,
+                                                            const int32_t* __restrict__ col_idx,
+                                                            const int32_t* __restrict__ wl, int64_t len,
+                                                            int32_t* C, unsigned long long* edges) {
+  if constexpr (!Huge) {  // no row above SGR_GS_HUGE: warps only, no block-level pass
+    const int lane = threadIdx.x & 31;
+    const int64_t wpb = blockDim.x >> 5;
+    unsigned long long my = 0;
+    for (int64_t i = (int64_t)blockIdx.x * wpb + (threadIdx.x >> 5); i < len;
+         i += (int64_t)gridDim.x * wpb) {
+      const int32_t v = __ldg(wl + i);
+      const int64_t s = ld_ro(row_ptr + v), e = ld_ro(row_ptr + v + 1);
+      const int32_t t = warp_first_fit_from<true>(col_idx, C, s, e, 0, lane);
+      if (lane == 0) {
+        __stcg(C + v, t);
+        my += (unsigned long long)(e - s);
+      }
+    }
+    block_add(my, edges);
+    return;
+  }
+  __shared__ unsigned long long sm[4];
+  __shared__ int32_t huge[64];  // this block's huge vertices (list positions)
+  __shared__ int32_t nhuge;
+  if (threadIdx.x < 4) sm[threadIdx.x] = 0ull;
+  if (threadIdx.x == 0) nhuge = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31;
+  const int64_t wpb = blockDim.x >> 5;
+  unsigned long long my = 0;
+  for (int64_t i = (int64_t)blockIdx.x * wpb + (threadIdx.x >> 5); i < len;
+       i += (int64_t)gridDim.x * wpb) {
+    const int32_t v = __ldg(wl + i);
+    const int64_t s = ld_ro(row_ptr + v), e = ld_ro(row_ptr + v + 1);
+    if (e - s > SGR_GS_HUGE) {  // deferred to the whole block (up to 64 per block)
+      int slot = 0;
+      if (lane == 0) slot = atomicAdd(&nhuge, 1);
+      slot = __shfl_sync(0xffffffffu, slot, 0);
+      if (slot < 64) {
+        if (lane == 0) huge[slot] = (int32_t)i;
+        continue;
+      }
+    }
+    const int32_t t = warp_first_fit_from<true>(col_idx, C, s, e, 0, lane);
+    if (lane == 0) {
+      __stcg(C + v, t);
+      my += (unsigned long long)(e - s);
+    }
+  }
+  __syncthreads();
+  const int32_t nh = min(nhuge, 64);
+  for (int32_t h = 0; h < nh; ++h) {  // huge vertices: the whole block each (block_fit)
+    const int32_t v = __ldg(wl + huge[h]);
+    const int64_t s = ld_ro(row_ptr + v), e = ld_ro(row_ptr + v + 1);
+    const int32_t t = block_fit(col_idx, C, s, e, sm);
+    if (threadIdx.x == 0) {
+      __stcg(C + v, t);
+      my += (unsigned long long)(e - s);
+    }
+  }
+  block_add(my, edges);
 }
 
 // Push v (degree d) into round list `par`, region of its part j: low-degree members from
@@ -513,7 +565,7 @@ __global__ void __launch_bounds__(256, 3) k_gs_persistent(Args a) {
         if (threadIdx.x < 32) push_warp(a, np, v, e - s, lane == 0);
         if (threadIdx.x == 0) my_edges += (unsigned long long)(e - s);
         if (j == 0) {
-          const int32_t t = block_fit(a, Cur, s, e, gs_sm);
+          const int32_t t = block_fit(a.col_idx, Cur, s, e, gs_sm);
           if (threadIdx.x == 0) Nxt[v] = t;
         }
       }
@@ -569,7 +621,7 @@ __global__ void __launch_bounds__(256, 3) k_gs_persistent(Args a) {
         const int32_t v = __ldcg(&(np ? a.L[1] : a.L[0])[top - 1 - i]);
         const int64_t s = ld_ro(a.row_ptr + v), e = ld_ro(a.row_ptr + v + 1);
         if (e - s <= SGR_GS_HUGE) continue;
-        const int32_t t = block_fit(a, Cur, s, e, gs_sm);
+        const int32_t t = block_fit(a.col_idx, Cur, s, e, gs_sm);
         if (threadIdx.x == 0) Nxt[v] = t;
       }
       for (int64_t i = gw; i < nbg; i += nw) {
@@ -627,7 +679,7 @@ __global__ void __launch_bounds__(256, 3) k_gs_persistent(Args a) {
         const int32_t v = __ldcg(&(np ? a.L[1] : a.L[0])[top - 1 - i]);
         const int64_t s = ld_ro(a.row_ptr + v), e = ld_ro(a.row_ptr + v + 1);
         if (e - s <= SGR_GS_HUGE) continue;
-        const int32_t t = block_fit(a, Cj, s, e, gs_sm);
+        const int32_t t = block_fit(a.col_idx, Cj, s, e, gs_sm);
         if (threadIdx.x == 0) Nj[v] = t;
       }
       for (int64_t i = gw; i < nbg; i += nw) {
